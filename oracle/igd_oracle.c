@@ -1,0 +1,371 @@
+/*
+ * igd_oracle.c -- TEST INFRASTRUCTURE ONLY.
+ *
+ * Plain, slow, single-threaded CPU oracle of iGUARD's race check (Kamath & Basu,
+ * SOSP'21, /root/reference/PAPER.md, cited as P:<line>), restated as a sequential
+ * shadow-memory replay of a fixed-order trace (readings A1-A30
+ * listed in DESIGN.md "Readings").
+ *
+ * Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference
+ * leg may load this library.  It shares no code, header, constant or helper with the
+ * CUDA path (paper_conf_sosp_kamathb21_b200/csrc): it has its own trace reader, its own
+ * kind/scope codes, its own hash constants.
+ *
+ * Algorithm, in the paper's order (Fig. 6):
+ *   synchronization events update the synchronization metadata (Fig. 5),
+ *   atomicCAS / atomicExch / fences drive lock inference (§6.3),
+ *   every load / store / atomic reads the word's memory metadata, runs the two-tier
+ *   check of Table 2 (P1..P6 then R1..R5, §6.4) and writes
+ *   the metadata back.
+ *
+ * Counters are exact u64 (reading A16) instead of the 6/8-bit fields of Fig. 4.
+ * Per-word state is exact (no tag aliasing, A18).
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+/* ---- trace encoding, read with the oracle's own reader ---------------- */
+enum { O_LD = 0, O_ST = 1, O_ATOM = 2, O_CAS = 3, O_EXCH = 4, O_FENCE = 5, O_SYNCWARP = 6,
+       O_SYNCTHREADS = 7, O_GRID = 8, O_CG_TILE = 9, O_CG_BLOCK = 10, O_CG_GRID = 11 };
+enum { S_NONE = 0, S_BLOCK = 1, S_DEVICE = 2, S_SYSTEM = 3 };
+enum { R_NONE = 0, R1 = 1, R2 = 2, R3 = 3, R4 = 4, R5 = 5 };
+
+typedef struct {
+    uint64_t addr;
+    uint32_t tid, kind, scope, mask;
+} o_event;
+
+/* little-endian decode of one 16-byte record: addr u64 | tk u32 | mask u32 */
+static int o_read_event(const uint8_t* p, o_event* e) {
+    uint64_t addr = 0;
+    uint32_t tk = 0, mask = 0;
+    for (int b = 0; b < 8; b++) addr |= (uint64_t)p[b] << (8 * b);
+    for (int b = 0; b < 4; b++) tk |= (uint32_t)p[8 + b] << (8 * b);
+    for (int b = 0; b < 4; b++) mask |= (uint32_t)p[12 + b] << (8 * b);
+    e->addr = addr;
+    e->tid = tk & 0xFFFFFFu;
+    e->kind = (tk >> 24) & 0xFu;
+    e->scope = (tk >> 28) & 0x3u;
+    e->mask = mask;
+    return (tk >> 30) == 0; /* bits 30-31 must be zero */
+}
+
+typedef struct {
+    uint64_t addr, cur, prev;
+    uint8_t type, cur_kind, prev_kind, pad[5];
+} o_report; /* 32 bytes, same field meaning as igd_report */
+
+/* ---- thread geometry (C.1) ---------------------------------- */
+typedef struct { uint32_t D, Wb, threads, blocks, warps; } o_geom;
+static uint32_t g_block(const o_geom* g, uint32_t t) { return t / g->D; }
+static uint32_t g_warp(const o_geom* g, uint32_t t) { return (t / g->D) * g->Wb + (t % g->D) / 32; }
+static uint32_t g_lane(const o_geom* g, uint32_t t) { return (t % g->D) % 32; }
+
+/* ---- lock tables (Fig. 7; §6.3) ------------------------------ */
+typedef struct { uint8_t valid, active, scope; uint32_t h18; } o_lock;
+typedef struct { o_lock e[3]; } o_table; /* "up to 3 separate locks" P:1083-1085 */
+
+/* reading A8: 18-bit address hash and the 2-way 16-bit Bloom summary */
+static uint32_t o_h18(uint64_t word) { return ((uint32_t)word * 0x9E3779B1u) >> 14; }
+static uint16_t o_bloom(uint32_t h) { return (uint16_t)((1u << (h & 15u)) | (1u << ((h >> 4) & 15u))); }
+
+/* activate: "sets the Active bit ... for all entries with matching or narrower scope" P:1076-1077 */
+static void o_activate(o_table* T, uint32_t s) {
+    for (int k = 0; k < 3; k++)
+        if (T->e[k].valid && T->e[k].scope <= s) T->e[k].active = 1;
+}
+/* held(t): OR of the Bloom bits of valid+active entries */
+static uint16_t o_held_of(const o_table* T) {
+    uint16_t b = 0;
+    for (int k = 0; k < 3; k++)
+        if (T->e[k].valid && T->e[k].active) b |= o_bloom(T->e[k].h18);
+    return b;
+}
+
+/* ---- shadow memory: one exact entry per 4-byte word (Fig. 4) ------------- */
+typedef struct {
+    uint64_t idx;                 /* trace index of the access */
+    uint32_t tid;                 /* full thread id (A19) */
+    uint32_t kind;
+    uint64_t sDEV, sANY, sWB, sBB; /* counters snapshotted at the access */
+} o_rec;
+
+typedef struct {
+    uint64_t word;
+    uint8_t used;                 /* hash slot occupied */
+    uint8_t valid, modified, atomic, ascope, devShared, blkShared;
+    uint16_t locks;               /* Bloom of the last accessor's held locks (A7) */
+    o_rec LA, LW;                 /* last accessor, last writer */
+} o_shadow;
+
+typedef struct {
+    o_shadow* slot;
+    uint64_t cap, count;
+} o_map;
+
+static uint64_t o_mix(uint64_t x) { /* slot spreading only; not semantic */
+    x ^= x >> 33; x *= 0xff51afd7ed558ccdULL; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ULL; x ^= x >> 33;
+    return x;
+}
+static int o_map_grow(o_map* m);
+static o_shadow* o_map_get(o_map* m, uint64_t word) {
+    if ((m->count + 1) * 4 > m->cap * 3)
+        if (!o_map_grow(m)) return NULL;
+    uint64_t i = o_mix(word) & (m->cap - 1);
+    while (m->slot[i].used && m->slot[i].word != word) i = (i + 1) & (m->cap - 1);
+    if (!m->slot[i].used) {
+        memset(&m->slot[i], 0, sizeof(o_shadow));
+        m->slot[i].used = 1;
+        m->slot[i].word = word;
+        m->count++;
+    }
+    return &m->slot[i];
+}
+static int o_map_grow(o_map* m) {
+    uint64_t ncap = m->cap ? m->cap * 2 : 1024;
+    o_shadow* ns = (o_shadow*)calloc(ncap, sizeof(o_shadow));
+    if (!ns) return 0;
+    for (uint64_t i = 0; i < m->cap; i++) {
+        if (!m->slot[i].used) continue;
+        uint64_t j = o_mix(m->slot[i].word) & (ncap - 1);
+        while (ns[j].used) j = (j + 1) & (ncap - 1);
+        ns[j] = m->slot[i];
+    }
+    free(m->slot);
+    m->slot = ns;
+    m->cap = ncap;
+    return 1;
+}
+
+/* address shard used by --addr-shard (C.7 5(b)); the hash is not semantic */
+static uint32_t o_fmix32(uint32_t h) {
+    h ^= h >> 16; h *= 0x85ebca6bu; h ^= h >> 13; h *= 0xc2b2ae35u; h ^= h >> 16;
+    return h;
+}
+
+/* return codes (same numeric meaning as include/igd.h, restated) */
+#define O_OK 0
+#define O_EINVAL (-1)
+#define O_ETRACE (-2)
+#define O_ENOMEM (-4)
+
+/* Field rules per kind. Returns 1 when the event is well-formed. */
+static int o_valid(const o_event* e, const o_geom* g) {
+    if (e->kind > O_CG_GRID) return 0;
+    if (e->tid >= g->threads) return 0;
+    uint32_t lanebit = 1u << g_lane(g, e->tid);
+    switch (e->kind) {
+    case O_LD: case O_ST:
+        return (e->mask & lanebit) && e->scope == S_NONE;
+    case O_ATOM: case O_CAS: case O_EXCH:
+        return (e->mask & lanebit) && e->scope != S_NONE;
+    case O_FENCE:
+        return e->addr == 0 && (e->mask & lanebit) && e->scope != S_NONE;
+    case O_SYNCWARP: case O_CG_TILE: case O_SYNCTHREADS: case O_CG_BLOCK:
+        return e->addr == 0 && e->scope == S_NONE;
+    case O_GRID: case O_CG_GRID:
+        return e->addr == 0 && e->scope == S_NONE && e->tid == 0;
+    }
+    return 0;
+}
+
+/*
+ * igdo_run: replay events[0..n) (16-byte records) of one kernel with grid geometry
+ * (n_blocks, block_dim).  Only words w with shard(w) == shard_k (of shard_K; K=1 means
+ * all) are shadow-checked; all synchronization and lock events are replayed regardless
+ * (C.7 5(b)).  Reports are written in ascending `cur` order (A21) to out[0..cap); the
+ * total is returned in *n_reports.  On an ill-formed event returns O_ETRACE and its index
+ * in *bad_index.
+ */
+int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,
+             uint32_t shard_k, uint32_t shard_K, o_report* out, uint64_t cap,
+             uint64_t* n_reports, uint64_t* bad_index) {
+    *n_reports = 0;
+    *bad_index = 0;
+    if (n_blocks == 0 || block_dim == 0) return O_EINVAL;
+    if ((uint64_t)n_blocks * block_dim > (1u << 24)) return O_EINVAL;
+    if (shard_K == 0 || shard_k >= shard_K) return O_EINVAL;
+
+    o_geom g;
+    g.D = block_dim;
+    g.Wb = (block_dim + 31) / 32;
+    g.blocks = n_blocks;
+    g.threads = n_blocks * block_dim;
+    g.warps = n_blocks * g.Wb;
+
+    /* validate everything first (the oracle applies the 8(b) rules independently) */
+    for (uint64_t i = 0; i < n; i++) {
+        o_event e;
+        int ok = o_read_event(events + 16 * i, &e);
+        if (!ok || !o_valid(&e, &g)) { *bad_index = i; return O_ETRACE; }
+    }
+
+    /* C.2 synchronization state: exact, unbounded counters */
+    uint64_t* devF = (uint64_t*)calloc(g.threads, sizeof(uint64_t));
+    uint64_t* anyF = (uint64_t*)calloc(g.threads, sizeof(uint64_t));
+    uint64_t* wbar = (uint64_t*)calloc(g.warps, sizeof(uint64_t));
+    uint64_t* bbar = (uint64_t*)calloc(g.blocks, sizeof(uint64_t));
+    uint64_t G = 0;
+    o_table* wt = (o_table*)calloc(g.warps, sizeof(o_table));
+    o_table* tt = (o_table*)calloc(g.threads, sizeof(o_table));
+    uint8_t* isThread = (uint8_t*)calloc(g.warps, 1);
+    uint8_t* touched = (uint8_t*)calloc(g.warps, 1); /* warps whose tables were ever filled */
+    uint32_t* touched_list = (uint32_t*)calloc(g.warps, sizeof(uint32_t));
+    uint32_t n_touched = 0;
+    o_map map = {0, 0, 0};
+    int rc = O_OK;
+    if (!devF || !anyF || !wbar || !bbar || !wt || !tt || !isThread || !touched || !touched_list) {
+        rc = O_ENOMEM;
+        goto done;
+    }
+
+#define DEV(t) (devF[t] + G)
+#define ANY(t) (anyF[t] + G)
+#define WB(w) (wbar[w])
+#define BB(b) (bbar[b] + G)
+#define TABLE(t) (isThread[g_warp(&g, t)] ? &tt[t] : &wt[g_warp(&g, t)])
+
+    for (uint64_t i = 0; i < n; i++) {
+        o_event e;
+        o_read_event(events + 16 * i, &e);
+        uint32_t k = e.kind, c = e.tid;
+        uint32_t s = (e.scope == S_SYSTEM) ? S_DEVICE : e.scope; /* A12: SYSTEM == DEVICE */
+        /* CG syncs are their constituents (A15) */
+        if (k == O_CG_TILE) k = O_SYNCWARP;
+        if (k == O_CG_BLOCK) k = O_SYNCTHREADS;
+        if (k == O_CG_GRID) k = O_GRID;
+
+        /* ---- Step 1: synchronization metadata (Fig. 5) ---- */
+        if (k == O_FENCE) {
+            if (s >= S_DEVICE) devF[c]++;  /* DevFenceId (Fig. 5b) */
+            anyF[c]++;                     /* any fence changes DevFenceID or BlkFenceID */
+            o_activate(TABLE(c), s);       /* activateLocks(scope) P:1076-1077 */
+            continue;
+        }
+        if (k == O_SYNCWARP) { wbar[g_warp(&g, c)]++; continue; } /* A14: mask ignored */
+        if (k == O_SYNCTHREADS) { bbar[g_block(&g, c)]++; continue; } /* Fig. 5a; A13 */
+        if (k == O_GRID) {
+            /* A15: a device fence by every thread (incl. lock activation) + a barrier for
+               every block; implemented through the G term of DEV/ANY/BB */
+            G++;
+            for (uint32_t q = 0; q < n_touched; q++) {
+                uint32_t w = touched_list[q];
+                o_activate(&wt[w], S_DEVICE);
+                uint32_t b = w / g.Wb, wi = w % g.Wb;
+                for (uint32_t l = 0; l < 32; l++) {
+                    uint32_t off = wi * 32 + l;
+                    if (off >= g.D) break;
+                    o_activate(&tt[b * g.D + off], S_DEVICE);
+                }
+            }
+            continue;
+        }
+
+        /* ---- Step 3: an access (LD/ST/ATOM/CAS/EXCH) ---- */
+        int isWrite = (k != O_LD);                                /* atomics are stores */
+        int isAtomic = (k == O_ATOM || k == O_CAS || k == O_EXCH);
+        uint64_t word = e.addr >> 2;                              /* 4-byte granularity */
+        uint32_t w_c = g_warp(&g, c), b_c = g_block(&g, c);
+        uint16_t L = o_held_of(TABLE(c));                        /* 3.1: before own update (A11) */
+
+        int owned = (shard_K == 1) || ((o_fmix32((uint32_t)word ^ (uint32_t)(word >> 32)) % shard_K) == shard_k);
+        if (owned) {
+            o_shadow* S = o_map_get(&map, word);
+            if (!S) { rc = O_ENOMEM; goto done; }
+            if (!S->valid) goto writeback;                        /* P1: first access */
+
+            /* sharing flags vs the last accessor, sticky (A5) */
+            {
+                uint32_t la = S->LA.tid;
+                if (g_block(&g, la) != b_c) S->devShared = 1;
+                else if (g_warp(&g, la) != w_c) S->blkShared = 1;
+            }
+            if (k == O_LD && !S->modified) goto writeback;        /* P2: no write (A25) */
+
+            {
+                const o_rec* md = (k == O_LD) ? &S->LW : &S->LA; /* Table 2 definitions */
+                uint32_t p = md->tid;
+                uint32_t w_p = g_warp(&g, p), b_p = g_block(&g, p);
+                /* preliminary checks (reading A4: md.* = relation between md and curr) */
+                int P3 = (p == c);
+                int P4 = (w_p == w_c) && (WB(w_c) != md->sWB || (e.mask >> g_lane(&g, p)) & 1u);
+                int P5 = (b_p == b_c) && (BB(b_c) != md->sBB);
+                int P6 = S->atomic && isAtomic && (b_p == b_c || S->ascope == S_DEVICE);
+                if (P3 || P4 || P5 || P6) goto writeback;
+
+                /* race checks in order; first true is reported */
+                int noAny = (ANY(p) == md->sANY);   /* A1: md's thread has not fenced since */
+                int noDev = (DEV(p) == md->sDEV);
+                int type = R_NONE;
+                if (S->atomic && S->ascope == S_BLOCK && g_block(&g, S->LW.tid) != b_c) type = R1;
+                else if (w_p == w_c && noAny && !S->devShared && !S->blkShared) type = R2;
+                else if (b_p == b_c && noAny && !S->devShared) type = R3;
+                else if (b_p != b_c && noDev) type = R4;
+                else if ((S->locks | L) != 0 && (S->locks & L) == 0) type = R5; /* A3, A7 */
+                if (type != R_NONE) {
+                    if (*n_reports < cap) {
+                        o_report* r = &out[*n_reports];
+                        memset(r, 0, sizeof(*r));
+                        r->addr = word << 2;
+                        r->cur = i;
+                        r->prev = md->idx;
+                        r->type = (uint8_t)type;
+                        r->cur_kind = (uint8_t)e.kind;
+                        r->prev_kind = (uint8_t)md->kind;
+                    }
+                    (*n_reports)++;
+                }
+            }
+        writeback: /* Fig. 6 "Race -> Writeback": always done (A11) */
+            {
+                o_rec r;
+                r.idx = i; r.tid = c; r.kind = e.kind;
+                r.sDEV = DEV(c); r.sANY = ANY(c); r.sWB = WB(w_c); r.sBB = BB(b_c);
+                S->valid = 1;
+                S->LA = r;
+                S->locks = L;
+                if (isWrite) { S->modified = 1; S->LW = r; }
+                if (isAtomic) { S->atomic = 1; S->ascope = (uint8_t)s; }
+            }
+        }
+
+        /* ---- Step 4: lock-table update for CAS / EXCH, after the check (A9-A11) ---- */
+        if (k == O_CAS || k == O_EXCH) {
+            uint32_t h = o_h18(word);
+            if (k == O_CAS) {
+                /* isThread: more than one lane executes the CAS together */
+                if (!isThread[w_c] && __builtin_popcount(e.mask) > 1) isThread[w_c] = 1;
+                if (!touched[w_c]) { touched[w_c] = 1; touched_list[n_touched++] = w_c; }
+                o_table* T = TABLE(c);
+                int present = 0;
+                for (int q = 0; q < 3; q++)
+                    if (T->e[q].valid && T->e[q].h18 == h && T->e[q].scope == s) present = 1;
+                if (!present) {
+                    for (int q = 0; q < 3; q++) {
+                        if (!T->e[q].valid) {
+                            T->e[q].valid = 1; T->e[q].active = 0;
+                            T->e[q].scope = (uint8_t)s; T->e[q].h18 = h;
+                            break;
+                        }
+                    } /* full table: the insert is dropped (A9) */
+                }
+            } else {
+                /* atomicExch unsets Valid of entries matching hash and scope */
+                o_table* T = TABLE(c);
+                for (int q = 0; q < 3; q++)
+                    if (T->e[q].valid && T->e[q].h18 == h && T->e[q].scope == s) {
+                        T->e[q].valid = 0; T->e[q].active = 0;
+                    }
+            }
+        }
+    }
+
+done:
+    free(devF); free(anyF); free(wbar); free(bbar); free(wt); free(tt);
+    free(isThread); free(touched); free(touched_list); free(map.slot);
+    return rc;
+}
+
+/* Exported constants so the Python side can check it loaded this library. */
+int igdo_version(void) { return 1; }

@@ -1,0 +1,96 @@
+"""Mutation check of the pins: each plausible one-line mistake in the oracle (a dropped term,
+a wrong sign or index, a swapped operand) must be caught by the golden fixtures or by the
+from-scratch brute force.  Builds mutated copies of oracle/igd_oracle.c with gcc."""
+import ctypes
+import os
+import subprocess
+import tempfile
+
+import numpy as np
+import pytest
+
+import tracegen as tg
+from golden_io import all_golden, full_tuples, parse
+from pins import bf_scratch
+
+SRC = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "oracle", "igd_oracle.c")
+REPORT = np.dtype([("addr", "<u8"), ("cur", "<u8"), ("prev", "<u8"), ("type", "u1"),
+                   ("cur_kind", "u1"), ("prev_kind", "u1"), ("pad", "u1", (5,))])
+
+MUTANTS = {
+    "noAny_uses_current_thread": ("int noAny = (ANY(p) == md->sANY);", "int noAny = (ANY(c) == md->sANY);"),
+    "noDev_uses_any": ("int noDev = (DEV(p) == md->sDEV);", "int noDev = (ANY(p) == md->sDEV);"),
+    "md_always_last_accessor": ("(k == O_LD) ? &S->LW : &S->LA", "&S->LA"),
+    "P4_drops_mask_clause": ("|| (e.mask >> g_lane(&g, p)) & 1u", "|| 0"),
+    "P4_mask_uses_current_lane": ("(e.mask >> g_lane(&g, p))", "(e.mask >> g_lane(&g, c))"),
+    "P5_drops_barrier": ("(BB(b_c) != md->sBB)", "1"),
+    "P6_drops_scope": ("|| S->ascope == S_DEVICE)", ")"),
+    "R1_uses_md_block": ("g_block(&g, S->LW.tid) != b_c", "b_p != b_c"),
+    "R2_drops_blkShared": ("&& !S->devShared && !S->blkShared) type = R2", "&& !S->devShared) type = R2"),
+    "R3_drops_devShared": ("noAny && !S->devShared) type = R3", "noAny) type = R3"),
+    "R5_or_instead_of_and": ("(S->locks & L) == 0", "(S->locks | L) == 0"),
+    "devShared_not_sticky": ("if (g_block(&g, la) != b_c) S->devShared = 1;", "S->devShared = 0; if (g_block(&g, la) != b_c) S->devShared = 1;"),
+    "blkShared_not_sticky": ("else if (g_warp(&g, la) != w_c) S->blkShared = 1;", "else { S->blkShared = (g_warp(&g, la) != w_c); }"),
+    "P2_for_stores_too": ("if (k == O_LD && !S->modified)", "if (!S->modified)"),
+    "locks_field_last_writer": ("S->locks = L;", "if (isWrite) S->locks = L;"),
+    "block_fence_counts_dev": ("if (s >= S_DEVICE) devF[c]++;", "devF[c]++;"),
+    "activate_wider_scope": ("T->e[k].scope <= s", "T->e[k].scope >= s"),
+    "isThread_never": ("__builtin_popcount(e.mask) > 1", "__builtin_popcount(e.mask) > 32"),
+    "exch_ignores_scope": ("T->e[q].h18 == h && T->e[q].scope == s) {", "T->e[q].h18 == h) {"),
+    "grid_no_lock_activation": ("o_activate(&wt[w], S_DEVICE);", ";"),
+    "grid_not_barrier": ("#define BB(b) (bbar[b] + G)", "#define BB(b) (bbar[b])"),
+    "system_not_device": ("(e.scope == S_SYSTEM) ? S_DEVICE : e.scope", "e.scope"),
+    "ascope_first_atomic": ("if (isAtomic) { S->atomic = 1; S->ascope = (uint8_t)s; }",
+                            "if (isAtomic) { if (!S->atomic) S->ascope = (uint8_t)s; S->atomic = 1; }"),
+    "check_after_lock_update": ("uint16_t L = o_held_of(TABLE(c));", "uint16_t L = o_held_of(TABLE(c)) | (k == O_CAS ? o_bloom(o_h18(e.addr >> 2)) : 0);"),
+    "bloom_single_bit": ("| (1u << ((h >> 4) & 15u))", ""),
+}
+
+
+def _build(mutant_src, d):
+    c = os.path.join(d, "m.c")
+    so = os.path.join(d, "m.so")
+    with open(c, "w") as f:
+        f.write(mutant_src)
+    subprocess.check_call(["gcc", "-O1", "-std=c11", "-w", "-fPIC", "-shared", "-o", so, c])
+    lib = ctypes.CDLL(so)
+    lib.igdo_run.restype = ctypes.c_int
+    lib.igdo_run.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                             ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
+                             ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
+    return lib
+
+
+def _run(lib, ev, nb, bd):
+    cap = 4096
+    out = np.zeros(cap, REPORT)
+    nrep, bad = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    rc = lib.igdo_run(ev.ctypes.data if len(ev) else None, len(ev), nb, bd, 0, 1, out.ctypes.data, cap,
+                      ctypes.byref(nrep), ctypes.byref(bad))
+    assert rc == 0
+    return full_tuples(out[: nrep.value])
+
+
+def _caught(lib):
+    for path in all_golden():
+        ev, nb, bd, exp = parse(path)
+        if [r[:4] for r in _run(lib, ev, nb, bd)] != exp:
+            return "golden:" + os.path.basename(path)
+    w_lock = [12, 10, 6, 10, 8, 12, 2, 2, 1, 1, 1, 1]
+    for seed in range(300):
+        rng = np.random.default_rng(seed)
+        kw = {"weights": w_lock, "lock_words": 5 + seed % 40, "p_lock_data": 0.2} if seed % 2 else {}
+        ev, nb, bd = tg.random_trace(seed, int(rng.integers(20, 160)), n_words=int(rng.integers(1, 10)), **kw)
+        if _run(lib, ev, nb, bd) != bf_scratch(ev, nb, bd):
+            return f"bruteforce seed {seed}"
+    return None
+
+
+@pytest.mark.parametrize("name", sorted(MUTANTS))
+def test_mutant_is_caught(name):
+    src = open(SRC).read()
+    old, new = MUTANTS[name]
+    assert src.count(old) >= 1, f"mutation anchor vanished: {old!r}"
+    with tempfile.TemporaryDirectory() as d:
+        lib = _build(src.replace(old, new, 1), d)
+        assert _caught(lib) is not None, f"mutant {name} survived every pin"

@@ -1,0 +1,187 @@
+"""Seeded synthetic trace generators -- shared INPUT module (no race-check arithmetic).
+
+This package only *produces* traces in the 16-byte ``igd_event`` format of
+include/igd.h; it never evaluates the race rules.  Both the oracle
+(tests) and the CUDA path (tests, bench) consume what it produces.  The generator
+families C1..C5 live in the C library ``tracegen/igdgen.c`` and are
+wrapped by :mod:`tracegen.families`; this module holds the format, a hand-written trace
+builder used by the golden fixtures and a small random-trace fuzzer.
+
+Each family also returns an *injection ledger*: the races it deliberately planted
+(which events, which rule was intended).  The ledger records generator intent, written
+down when the injection is emitted; tests use it as an independent pin of the oracle.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+EVENT_DTYPE = np.dtype([("addr", "<u8"), ("tk", "<u4"), ("mask", "<u4")])
+assert EVENT_DTYPE.itemsize == 16
+
+REPORT_DTYPE = np.dtype([("addr", "<u8"), ("cur", "<u8"), ("prev", "<u8"), ("type", "u1"),
+                         ("cur_kind", "u1"), ("prev_kind", "u1"), ("pad", "u1", (5,))])
+assert REPORT_DTYPE.itemsize == 32
+
+# kind codes
+LD, ST, ATOM, CAS, EXCH, FENCE, SYNCWARP, SYNCTHREADS, GRID_SYNC = range(9)
+CG_TILE_SYNC, CG_BLOCK_SYNC, CG_GRID_SYNC = 9, 10, 11
+KIND_NAMES = ["LD", "ST", "ATOM", "CAS", "EXCH", "FENCE", "SYNCWARP", "SYNCTHREADS", "GRID_SYNC",
+              "CG_TILE_SYNC", "CG_BLOCK_SYNC", "CG_GRID_SYNC"]
+# scope codes
+NONE, BLOCK, DEVICE, SYSTEM = 0, 1, 2, 3
+SCOPE_NAMES = ["NONE", "BLOCK", "DEVICE", "SYSTEM"]
+
+
+def pack_tk(tid, kind, scope):
+    return (np.asarray(tid, np.uint32) | (np.asarray(kind, np.uint32) << 24)
+            | (np.asarray(scope, np.uint32) << 28)).astype(np.uint32)
+
+
+def unpack(events):
+    """Split an EVENT_DTYPE array into (addr, tid, kind, scope, mask) numpy arrays."""
+    tk = events["tk"]
+    return (events["addr"], tk & 0xFFFFFF, (tk >> 24) & 0xF, (tk >> 28) & 0x3, events["mask"])
+
+
+class Geometry:
+    """Grid geometry of the traced kernel."""
+
+    def __init__(self, n_blocks: int, block_dim: int):
+        self.n_blocks = int(n_blocks)
+        self.block_dim = int(block_dim)
+        self.wpb = (self.block_dim + 31) // 32
+
+    @property
+    def threads(self):
+        return self.n_blocks * self.block_dim
+
+    def lane(self, t):
+        return (t % self.block_dim) % 32
+
+    def warp(self, t):
+        return (t // self.block_dim) * self.wpb + (t % self.block_dim) // 32
+
+    def block(self, t):
+        return t // self.block_dim
+
+
+class TraceBuilder:
+    """Append events one by one (hand-written traces: golden fixtures, unit tests).
+
+    ``mask`` defaults to the single lane of ``tid``.  Word-level helpers take a *word*
+    number and store the byte address ``word << 2``.
+    """
+
+    def __init__(self, n_blocks: int, block_dim: int):
+        self.geom = Geometry(n_blocks, block_dim)
+        self.rows = []
+
+    def _lanebit(self, tid):
+        return 1 << self.geom.lane(tid)
+
+    def ev(self, kind, tid, word=0, scope=NONE, mask=None, addr=None):
+        if mask is None:
+            mask = self._lanebit(tid)
+        if addr is None:
+            addr = int(word) << 2
+        self.rows.append((int(addr), int(tid), int(kind), int(scope), int(mask) & 0xFFFFFFFF))
+        return len(self.rows) - 1
+
+    def ld(self, tid, word, mask=None):
+        return self.ev(LD, tid, word, NONE, mask)
+
+    def st(self, tid, word, mask=None):
+        return self.ev(ST, tid, word, NONE, mask)
+
+    def atom(self, tid, word, scope=DEVICE, mask=None):
+        return self.ev(ATOM, tid, word, scope, mask)
+
+    def cas(self, tid, word, scope=DEVICE, mask=None):
+        return self.ev(CAS, tid, word, scope, mask)
+
+    def exch(self, tid, word, scope=DEVICE, mask=None):
+        return self.ev(EXCH, tid, word, scope, mask)
+
+    def fence(self, tid, scope=DEVICE, mask=None):
+        return self.ev(FENCE, tid, 0, scope, mask)
+
+    def syncwarp(self, tid, mask=0xFFFFFFFF):
+        return self.ev(SYNCWARP, tid, 0, NONE, mask)
+
+    def syncthreads(self, block):
+        return self.ev(SYNCTHREADS, block * self.geom.block_dim, 0, NONE, 0xFFFFFFFF)
+
+    def grid_sync(self):
+        return self.ev(GRID_SYNC, 0, 0, NONE, 0xFFFFFFFF)
+
+    def events(self):
+        out = np.zeros(len(self.rows), EVENT_DTYPE)
+        if self.rows:
+            a = np.array(self.rows, dtype=np.uint64)
+            out["addr"] = a[:, 0]
+            out["tk"] = pack_tk(a[:, 1].astype(np.uint32), a[:, 2].astype(np.uint32),
+                                a[:, 3].astype(np.uint32))
+            out["mask"] = a[:, 4].astype(np.uint32)
+        return out
+
+
+def random_trace(seed: int, n: int, n_blocks: int = None, block_dim: int = None, n_words: int = 16,
+                 weights=None, max_uses_per_word: int = 0, lock_words: int = 2, p_lock_data: float = 0.0):
+    """Arbitrary event sequence for fuzzing.
+
+    Geometry is 1-3 blocks x {32,64,96} threads unless given.  Kinds are drawn with
+    weights, scopes at random, masks random but containing the lane.  With
+    ``max_uses_per_word`` > 0 every data word is accessed at most that many times
+    (the pairwise evaluator needs 2).  ``p_lock_data`` sends that fraction of LD/ST/ATOM to
+    the lock words.  Returns (events, n_blocks, block_dim).
+    """
+    rng = np.random.default_rng(seed)
+    if n_blocks is None:
+        n_blocks = int(rng.integers(1, 4))
+    if block_dim is None:
+        block_dim = int(rng.choice([32, 64, 96]))
+    g = Geometry(n_blocks, block_dim)
+    kinds = np.arange(12)
+    if weights is None:
+        weights = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    w = np.asarray(weights, float)
+    w = w / w.sum()
+    b = TraceBuilder(n_blocks, block_dim)
+    uses = {}
+    next_fresh = 1000
+    for _ in range(n):
+        k = int(rng.choice(kinds, p=w))
+        t = int(rng.integers(0, g.threads))
+        lane = g.lane(t)
+        mask = (int(rng.integers(0, 1 << 32)) | (1 << lane)) & 0xFFFFFFFF
+        if rng.random() < 0.5:
+            mask = 1 << lane
+        if k in (LD, ST, ATOM):
+            if max_uses_per_word:
+                # pick a word that still has budget, else a fresh one
+                cands = [x for x, u in uses.items() if u < max_uses_per_word]
+                if cands and rng.random() < 0.6:
+                    word = int(rng.choice(cands))
+                else:
+                    word = next_fresh
+                    next_fresh += 1
+                uses[word] = uses.get(word, 0) + 1
+            elif p_lock_data and rng.random() < p_lock_data:
+                word = 500 + int(rng.integers(0, lock_words))   # plain access to a lock word
+            else:
+                word = int(rng.integers(0, n_words))
+            scope = NONE if k in (LD, ST) else int(rng.integers(1, 4))
+            b.ev(k, t, word, scope, mask)
+        elif k in (CAS, EXCH):
+            # lock words live in their own range; their own accesses are atomics
+            word = 500 + int(rng.integers(0, lock_words))
+            b.ev(k, t, word, int(rng.integers(1, 4)), mask)
+        elif k == FENCE:
+            b.ev(FENCE, t, 0, int(rng.integers(1, 4)), mask)
+        elif k in (SYNCWARP, CG_TILE_SYNC):
+            b.ev(k, t, 0, NONE, mask)
+        elif k in (SYNCTHREADS, CG_BLOCK_SYNC):
+            b.ev(k, t, 0, NONE, 0xFFFFFFFF)
+        else:
+            b.ev(k, 0, 0, NONE, 0xFFFFFFFF)
+    return b.events(), n_blocks, block_dim
