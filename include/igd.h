@@ -1,0 +1,166 @@
+/*
+ * igd.h -- C ABI of libigd, the B200-native race check of iGUARD (Kamath & Basu, SOSP'21),
+ * restated as deterministic replay of a fixed-order trace.  PAPER.md lines are cited P:<n>.
+ *
+ * The operation (§6.2-§6.4): for every load/store/atomic of a kernel, compare it
+ * with the last writer (loads) or last accessor (stores/atomics) of the same 4-byte word
+ * (P:1097-1099), skip it if one of the preliminary checks P1-P6 holds, and otherwise
+ * report the first of the race conditions R1-R5 that holds (Table 2, P:1093-1151;
+ * "checked in the order given in the table").  Synchronization metadata
+ * comes from fences, __syncwarp, __syncthreads and grid syncs (Fig. 5); locks are
+ * inferred from atomicCAS + fence / atomicExch (§6.3).  Cooperative-group syncs
+ * are checked through their constituents.  Readings where the paper is
+ * silent are listed in DESIGN.md ("Readings", A1-A30); they bind this library.
+ *
+ * All arithmetic is integer; results are a deterministic function of the trace.
+ * No C++ types cross this ABI; every call returns an int status (IGD_OK = 0, < 0 = error)
+ * except igd_ctx_destroy / igd_strerror.  Nothing throws.  One context per stream;
+ * contexts are not thread-safe.
+ */
+#ifndef IGD_H
+#define IGD_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes --------------------------------------------------------------- */
+#define IGD_OK 0
+#define IGD_EINVAL (-1)  /* bad argument or geometry (threads must be 1..2^24) */
+#define IGD_ETRACE (-2)  /* an event violates the field rules below; see igd_bad_event() */
+#define IGD_ETOOBIG (-3) /* n_events >= 2^32-1, or the accessed word range spans >= 2^32 words */
+#define IGD_ENOMEM (-4)  /* device allocation failed */
+#define IGD_ECUDA (-5)   /* a CUDA runtime call failed; see igd_last_error() */
+#define IGD_ENCCL (-6)   /* reserved for the multi-GPU exchange */
+#define IGD_ESTATE (-7)  /* call out of order (e.g. igd_detect before igd_trace_load) */
+
+/* ---- trace event: 16 bytes, little-endian, arrays 16-byte aligned ---------------- */
+typedef struct {
+    uint64_t addr; /* accesses: byte address, checked at the 4-byte word addr>>2;
+                      synchronization events: 0 */
+    uint32_t tk;   /* bits [0,24) tid = global linear thread id; [24,28) kind; [28,30) scope;
+                      [30,32) must be 0 */
+    uint32_t mask; /* active mask of the warp instruction the event belongs to (P4, P:1115-1119;
+                      isThread inference); SYNCWARP: member lanes (ignored) */
+} igd_event;
+
+/* kind (tk bits 24..27) */
+#define IGD_LD 0
+#define IGD_ST 1
+#define IGD_ATOM 2         /* any other atomic RMW / atomic load or store */
+#define IGD_CAS 3          /* atomicCAS: also a lock-acquire candidate */
+#define IGD_EXCH 4         /* atomicExch: also a lock release */
+#define IGD_FENCE 5        /* __threadfence{_block,,_system} (Fig. 5b) */
+#define IGD_SYNCWARP 6     /* __syncwarp */
+#define IGD_SYNCTHREADS 7  /* __syncthreads (Fig. 5a) */
+#define IGD_GRID_SYNC 8    /* grid-wide barrier: device fence by every thread + barrier (reading A15) */
+#define IGD_CG_TILE_SYNC 9 /* == SYNCWARP */
+#define IGD_CG_BLOCK_SYNC 10 /* == SYNCTHREADS */
+#define IGD_CG_GRID_SYNC 11  /* == GRID_SYNC */
+/* scope (tk bits 28..29) */
+#define IGD_SCOPE_NONE 0
+#define IGD_SCOPE_BLOCK 1
+#define IGD_SCOPE_DEVICE 2
+#define IGD_SCOPE_SYSTEM 3 /* treated as DEVICE: the paper ignores system scope */
+
+/*
+ * Field rules (violations -> IGD_ETRACE, first offending index via igd_bad_event):
+ *   LD, ST            : tid < threads, mask contains lane(tid), scope NONE
+ *   ATOM, CAS, EXCH   : tid < threads, mask contains lane(tid), scope BLOCK/DEVICE/SYSTEM
+ *   FENCE             : addr 0, tid < threads, mask contains lane(tid), scope != NONE
+ *   SYNCWARP, CG_TILE : addr 0, tid = any thread of the warp (< threads), scope NONE
+ *   SYNCTHREADS, CG_BLOCK : addr 0, tid = any thread of the block (< threads), scope NONE
+ *   GRID_SYNC, CG_GRID: addr 0, tid 0, scope NONE
+ *   kind > 11 or tk bits 30..31 set: invalid.
+ * Geometry: block(t) = t / block_dim, warps per block
+ * Wb = ceil(block_dim/32), warp(t) = block(t)*Wb + (t % block_dim)/32,
+ * lane(t) = (t % block_dim) % 32.
+ * Conventions: the trace order is the execution order; per-lane events of one warp
+ * instruction are contiguous in ascending lane order; one SYNCTHREADS per (block, barrier
+ * instance), one SYNCWARP per (warp, instance), one GRID_SYNC per instance.
+ */
+
+typedef struct {
+    uint32_t n_blocks, block_dim; /* geometry of the traced kernel */
+    uint64_t n_events_total;      /* global trace length (all ranks) */
+    uint64_t first_event;         /* global index of events[0] on this rank (0 on one GPU) */
+    uint64_t n_events;            /* events in this buffer */
+    uint32_t flags;               /* IGD_TRACE_DEVICE_PTR: `events` is a device pointer */
+} igd_trace_desc;
+#define IGD_TRACE_DEVICE_PTR 1u
+
+/* ---- report: 32 bytes ------------------------------------------------------------ */
+typedef struct {
+    uint64_t addr;    /* byte address of the racy 4-byte word (word << 2) */
+    uint64_t cur;     /* global index of the access at which the race is declared */
+    uint64_t prev;    /* global index of md: the last writer for a load, else the last accessor */
+    uint8_t type;     /* 1 R1 scoped atomic, 2 R2 intra-warp (ITS), 3 R3 intra-block,
+                         4 R4 inter-block, 5 R5 missing lock (Table 2) */
+    uint8_t cur_kind, prev_kind; /* igd kinds of the two accesses */
+    uint8_t pad[5];
+} igd_report;
+#define IGD_R1 1
+#define IGD_R2 2
+#define IGD_R3 3
+#define IGD_R4 4
+#define IGD_R5 5
+
+/* Device allocator callbacks (e.g. a shim over torch's caching allocator).  May be NULL,
+   then cudaMallocAsync / cudaFreeAsync on the context stream are used. */
+typedef void* (*igd_alloc_fn)(size_t bytes, void* stream, void* user);
+typedef void (*igd_free_fn)(void* p, void* stream, void* user);
+
+typedef struct igd_ctx igd_ctx; /* opaque; owns every device buffer it allocates */
+
+/* Create a context on `cuda_device`, issuing all work on `cuda_stream` (a cudaStream_t;
+   NULL = the legacy default stream).  nranks must be 1 in this build (multi-GPU sharding
+   is driven from the host binding; IGD_EINVAL otherwise).  nccl_unique_id is ignored when
+   nranks == 1 and may be NULL. */
+int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks, int rank,
+                   const uint8_t* nccl_unique_id, igd_alloc_fn alloc_fn, igd_free_fn free_fn,
+                   void* alloc_user);
+
+/* Attach a trace.  Host `events` (flags without IGD_TRACE_DEVICE_PTR) are copied to device
+   memory owned by the context, asynchronously on the context stream from the caller's
+   buffer; the call synchronizes the stream before returning, so the caller may free the
+   buffer afterwards.  Device `events` are BORROWED: they must stay valid and unmodified until
+   igd_detect returns.  Returns IGD_EINVAL on bad geometry / desc, IGD_ETOOBIG when
+   n_events >= 2^32 - 1.  Field validation happens in igd_detect. */
+int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* events);
+
+/* Run the race check over the attached trace.  On success *n_reports_global holds the number
+   of reports; the reports stay in context-owned device memory until the next igd_detect or
+   igd_ctx_destroy.  Returns IGD_ETRACE (igd_bad_event gives the index) on an ill-formed
+   event, IGD_ETOOBIG if the accessed words span >= 2^32 words.  flags: 0. */
+int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
+
+/* Copy min(cap, total) reports, ascending by `cur` (at most one report per access, so the
+   order is total), to host memory `host_out`; *n_written = number copied. */
+int igd_reports(igd_ctx* ctx, igd_report* host_out, uint64_t cap, uint64_t* n_written);
+
+/* Device pointer to the report array of the last igd_detect (context-owned; same order). */
+int igd_reports_device(igd_ctx* ctx, const igd_report** dev_ptr, uint64_t* n);
+
+/* Index of the first invalid event found by the last igd_detect (valid after IGD_ETRACE). */
+uint64_t igd_bad_event(const igd_ctx* ctx);
+
+/* Per-stage device timings (milliseconds, CUDA events on the context stream) of the last
+   igd_detect when IGD_DETECT_TIMING was passed; stage order: see igd_stage_name. */
+#define IGD_DETECT_TIMING 1u
+#define IGD_N_STAGES 8
+int igd_stage_times(const igd_ctx* ctx, float* ms_out /* [IGD_N_STAGES] */);
+const char* igd_stage_name(int stage);
+
+/* Number of kernel launches the last igd_detect issued (evidence for gpu_launches). */
+uint64_t igd_last_launch_count(const igd_ctx* ctx);
+
+void igd_ctx_destroy(igd_ctx* ctx);
+const char* igd_strerror(int code);
+const char* igd_last_error(const igd_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* IGD_H */

@@ -1,0 +1,575 @@
+// igd.cu -- host orchestration of the race-check pipeline and the C ABI of include/igd.h.
+//
+// Pipeline (one stream, kernels in csrc/*.cuh):
+//   a1+a2+a4  ingest::k_ingest      validate, compact accesses / sync records, digit histograms
+//   a2        rsort::k_onesweep     stable radix sort of sync records by entity
+//             syncx::k_csr_offsets  CSR offsets of the per-entity timestamp lists
+//   a3        syncx::k_lock_infer   per-warp lock-table replay -> held-lock change points
+//   a5        rsort::k_onesweep     stable radix sort of accesses by word (trace order kept)
+//   a6        check::k_check        segmented shadow-metadata scan + Table 2 check
+//   a7        report sort by `cur`  canonical order
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+
+#include "check.cuh"
+#include "common.cuh"
+#include "ingest.cuh"
+#include "sort.cuh"
+#include "sync.cuh"
+
+namespace {
+
+struct Buf {
+    void* p = nullptr;
+    size_t cap = 0;
+};
+
+enum Stage { S_INGEST = 0, S_SYNC_SORT, S_TABLES, S_ACC_SORT, S_CHECK, S_REPORT, S_HOST, S_TOTAL };
+const char* kStageNames[IGD_N_STAGES] = {"ingest", "sync_sort", "epoch_lock_tables", "access_sort",
+                                         "check", "report_sort", "host_sync", "total"};
+
+}  // namespace
+
+struct igd_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    igd_alloc_fn afn = nullptr;
+    igd_free_fn ffn = nullptr;
+    void* auser = nullptr;
+    std::string err;
+
+    igd_trace_desc desc{};
+    const igd_event* events = nullptr;
+    bool loaded = false;
+    Buf owned_events;
+
+    Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
+    Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
+    Buf off, sw, wcnt, tcnt, wpts, tpts;
+    Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
+    u64 sync_cap = 0;
+    u64 rep_cap = 0;
+    u64 n_reports = 0;
+    u64 bad_event = 0;
+    u64 launches = 0;
+
+    // pinned host mirrors
+    u64* h_stats = nullptr;  // 8
+    u32* h_hist = nullptr;   // 2 x 1024 (+ report hist 1024)
+    u64* h_small = nullptr;  // 8
+
+    bool timing = false;
+    cudaEvent_t ev[IGD_N_STAGES + 1];
+    float stage_ms[IGD_N_STAGES];
+};
+
+#define CK(call)                                                                               \
+    do {                                                                                       \
+        cudaError_t e_ = (call);                                                               \
+        if (e_ != cudaSuccess) {                                                               \
+            ctx->err = std::string(#call) + ": " + cudaGetErrorString(e_);                     \
+            return e_ == cudaErrorMemoryAllocation ? IGD_ENOMEM : IGD_ECUDA;                   \
+        }                                                                                      \
+    } while (0)
+#define RET(x)                   \
+    do {                         \
+        int r_ = (x);            \
+        if (r_ != IGD_OK) return r_; \
+    } while (0)
+
+static int buf_free(igd_ctx* ctx, Buf& b) {
+    if (b.p) {
+        if (ctx->ffn) ctx->ffn(b.p, (void*)ctx->stream, ctx->auser);
+        else CK(cudaFreeAsync(b.p, ctx->stream));
+    }
+    b.p = nullptr;
+    b.cap = 0;
+    return IGD_OK;
+}
+
+static int ensure(igd_ctx* ctx, Buf& b, size_t bytes) {
+    if (bytes == 0) bytes = 16;
+    if (b.cap >= bytes) return IGD_OK;
+    RET(buf_free(ctx, b));
+    size_t want = bytes + bytes / 8;  // some headroom for growing traces
+    void* p = nullptr;
+    if (ctx->afn) {
+        p = ctx->afn(want, (void*)ctx->stream, ctx->auser);
+        if (!p) {
+            ctx->err = "allocator callback returned NULL for " + std::to_string(want) + " bytes";
+            return IGD_ENOMEM;
+        }
+    } else {
+        cudaError_t e = cudaMallocAsync(&p, want, ctx->stream);
+        if (e != cudaSuccess) {
+            ctx->err = std::string("cudaMallocAsync: ") + cudaGetErrorString(e);
+            (void)cudaGetLastError();
+            return IGD_ENOMEM;
+        }
+    }
+    b.p = p;
+    b.cap = want;
+    return IGD_OK;
+}
+
+template <class T>
+static T* P_(Buf& b) {
+    return reinterpret_cast<T*>(b.p);
+}
+
+static u32 bits_needed(u64 maxval) {
+    u32 b = 0;
+    while (b < 64 && (maxval >> b)) b++;
+    return b;
+}
+
+static void geo_init(Geo& g, u32 nb, u32 bd) {
+    g.D = bd;
+    g.Wb = (bd + 31) / 32;
+    g.B = nb;
+    g.T = nb * bd;
+    g.W = nb * g.Wb;
+    g.fd.init(bd);
+}
+
+static int sm_count(igd_ctx* ctx) {
+    int v = 148;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, ctx->device);
+    return v;
+}
+
+static void mark(igd_ctx* ctx, int stage) {
+    if (ctx->timing) cudaEventRecord(ctx->ev[stage], ctx->stream);
+}
+
+// Stable LSD radix sort of n (key, value) pairs in buffers k[cur], v[cur]; h_hist is the host
+// copy of the 4x256 digit histogram (device copy d_hist).  Digits above max_bits and digits
+// with one occupied bin are skipped.  Returns the buffer index holding the result.
+static int radix_sort(igd_ctx* ctx, Buf* k, Buf* v, u64 n, const u32* d_hist, const u32* h_hist, u32 max_bits,
+                      int* out_cur) {
+    int cur = 0;
+    *out_cur = 0;
+    if (n <= 1) return IGD_OK;
+    rsort::k_digit_base<<<4, rsort::RADIX, 0, ctx->stream>>>(d_hist, P_<u32>(ctx->base));
+    ctx->launches++;
+    const u64 tiles = (n + rsort::TILE - 1) / rsort::TILE;
+    RET(ensure(ctx, ctx->status, tiles * rsort::RADIX * sizeof(u64)));
+    for (u32 p = 0; p < 4; p++) {
+        if (p * 8 >= max_bits) break;
+        bool trivial = false;
+        for (int d = 0; d < 256; d++)
+            if (h_hist[p * 256 + d] == n) trivial = true;
+        if (trivial) continue;
+        CK(cudaMemsetAsync(ctx->status.p, 0, tiles * rsort::RADIX * sizeof(u64), ctx->stream));
+        CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
+        rsort::PassParams pp;
+        pp.kin = P_<u32>(k[cur]);
+        pp.vin = P_<u32>(v[cur]);
+        pp.kout = P_<u32>(k[cur ^ 1]);
+        pp.vout = P_<u32>(v[cur ^ 1]);
+        pp.n = (u32)n;
+        pp.shift = p * 8;
+        pp.digit_base = P_<u32>(ctx->base) + p * 256;
+        pp.status = P_<u64>(ctx->status);
+        pp.tile_ctr = P_<u32>(ctx->ctr);
+        rsort::k_onesweep<<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        cur ^= 1;
+    }
+    *out_cur = cur;
+    return IGD_OK;
+}
+
+static int scan_excl(igd_ctx* ctx, u32* data, u64 n) {
+    const u64 per = (u64)syncx::SCAN_THREADS * syncx::SCAN_ITEMS;
+    const u64 tiles = (n + per - 1) / per;
+    RET(ensure(ctx, ctx->status, tiles * sizeof(u64)));
+    CK(cudaMemsetAsync(ctx->status.p, 0, tiles * sizeof(u64), ctx->stream));
+    CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
+    syncx::k_scan_excl<<<(unsigned)tiles, syncx::SCAN_THREADS, 0, ctx->stream>>>(data, data, (u32)n, P_<u64>(ctx->status),
+                                                                                 P_<u32>(ctx->ctr));
+    ctx->launches++;
+    CK(cudaGetLastError());
+    return IGD_OK;
+}
+
+static int detect_impl(igd_ctx* ctx, u64* n_out) {
+    const igd_trace_desc& D = ctx->desc;
+    const u64 n = D.n_events;
+    ctx->n_reports = 0;
+    ctx->bad_event = 0;
+    ctx->launches = 0;
+    *n_out = 0;
+    mark(ctx, 0);
+    if (n == 0) {
+        for (int s = 1; s <= IGD_N_STAGES; s++) mark(ctx, s);
+        return IGD_OK;
+    }
+    Geo g;
+    geo_init(g, D.n_blocks, D.block_dim);
+    KeySpace ks;
+    ks.init(g);
+    const int sms = sm_count(ctx);
+
+    // ---------------- a1 + a2 + a4: ingest ----------------
+    const u64 in_tiles = (n + ingest::TILE - 1) / ingest::TILE;
+    if (ctx->sync_cap == 0) ctx->sync_cap = n / 4 + 4096;
+    RET(ensure(ctx, ctx->stats, 8 * sizeof(u64)));
+    RET(ensure(ctx, ctx->hist, 3 * 1024 * sizeof(u32)));
+    RET(ensure(ctx, ctx->base, 4 * 256 * sizeof(u32)));
+    RET(ensure(ctx, ctx->ctr, 64));
+    RET(ensure(ctx, ctx->st_in_a, in_tiles * sizeof(u64)));
+    RET(ensure(ctx, ctx->st_in_s, in_tiles * sizeof(u64)));
+    for (int b = 0; b < 2; b++) {
+        RET(ensure(ctx, ctx->acc_k[b], n * sizeof(u32)));
+        RET(ensure(ctx, ctx->acc_v[b], n * sizeof(u32)));
+    }
+    for (int attempt = 0;; attempt++) {
+        for (int b = 0; b < 2; b++) {
+            RET(ensure(ctx, ctx->syn_k[b], ctx->sync_cap * sizeof(u32)));
+            RET(ensure(ctx, ctx->syn_v[b], ctx->sync_cap * sizeof(u32)));
+        }
+        u64 init[8] = {~0ull, 0, ~0ull, 0, 0, 0, 0, 0};
+        memcpy(ctx->h_small, init, sizeof(init));
+        CK(cudaMemcpyAsync(ctx->stats.p, ctx->h_small, sizeof(init), cudaMemcpyHostToDevice, ctx->stream));
+        CK(cudaMemsetAsync(ctx->hist.p, 0, 2 * 1024 * sizeof(u32), ctx->stream));
+        CK(cudaMemsetAsync(ctx->st_in_a.p, 0, in_tiles * sizeof(u64), ctx->stream));
+        CK(cudaMemsetAsync(ctx->st_in_s.p, 0, in_tiles * sizeof(u64), ctx->stream));
+        CK(cudaMemsetAsync(ctx->ctr.p, 0, sizeof(u32), ctx->stream));
+        ingest::Params ip;
+        ip.ev = ctx->events;
+        ip.n = n;
+        ip.g = g;
+        ip.ks = ks;
+        ip.acc_key = P_<u32>(ctx->acc_k[0]);
+        ip.acc_val = P_<u32>(ctx->acc_v[0]);
+        ip.sync_key = P_<u32>(ctx->syn_k[0]);
+        ip.sync_val = P_<u32>(ctx->syn_v[0]);
+        ip.sync_cap = ctx->sync_cap;
+        ip.st_acc = P_<u64>(ctx->st_in_a);
+        ip.st_sync = P_<u64>(ctx->st_in_s);
+        ip.tile_ctr = P_<u32>(ctx->ctr);
+        ip.hist_acc = P_<u32>(ctx->hist);
+        ip.hist_sync = P_<u32>(ctx->hist) + 1024;
+        ip.stats = P_<u64>(ctx->stats);
+        ip.n_tiles = (u32)in_tiles;
+        int occ = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ingest::k_ingest, ingest::THREADS, 0);
+        u64 grid = (u64)sms * (occ > 0 ? occ : 1);
+        if (grid > in_tiles) grid = in_tiles;
+        ingest::k_ingest<<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(ctx->h_stats, ctx->stats.p, 8 * sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 2 * 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        if (ctx->h_stats[2] != ~0ull) {
+            ctx->bad_event = ctx->h_stats[2];
+            ctx->err = "invalid event at index " + std::to_string(ctx->bad_event);
+            return IGD_ETRACE;
+        }
+        if (ctx->h_stats[4] <= ctx->sync_cap) break;
+        ctx->sync_cap = ctx->h_stats[4] + ctx->h_stats[4] / 8 + 4096;  // rare: rerun with room
+        if (attempt > 2) return IGD_ECUDA;
+    }
+    mark(ctx, 1);
+    const u64 n_acc = ctx->h_stats[3], n_sync = ctx->h_stats[4], n_lock = ctx->h_stats[5];
+    if (n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32)) {
+        ctx->err = "accessed word range spans >= 2^32 words";
+        return IGD_ETOOBIG;
+    }
+    if (n_sync >= 0xFFFFFFFFull) return IGD_ETOOBIG;
+    u32 h_hist_acc[1024], h_hist_sync[1024];
+    memcpy(h_hist_acc, ctx->h_hist, sizeof(h_hist_acc));
+    memcpy(h_hist_sync, ctx->h_hist + 1024, sizeof(h_hist_sync));
+
+    // ---------------- a2: sync records sorted by entity, CSR offsets ----------------
+    int scur = 0;
+    RET(radix_sort(ctx, ctx->syn_k, ctx->syn_v, n_sync, P_<u32>(ctx->hist) + 1024, h_hist_sync, bits_needed(ks.E),
+                   &scur));
+    mark(ctx, 2);
+    RET(ensure(ctx, ctx->off, ((u64)ks.E + 2) * sizeof(u32)));
+    {
+        u64 work = (u64)ks.E + 1;
+        unsigned blocks = (unsigned)std::min<u64>((work + 255) / 256, (u64)sms * 16);
+        syncx::k_csr_offsets<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->syn_k[scur]), (u32)n_sync, ks.E,
+                                                             P_<u32>(ctx->off));
+        ctx->launches++;
+        CK(cudaGetLastError());
+    }
+    // ---------------- a3: lock inference ----------------
+    syncx::LockView lv;
+    memset(&lv, 0, sizeof(lv));
+    if (n_lock > 0) {
+        RET(ensure(ctx, ctx->sw, (u64)g.W * sizeof(u32)));
+        RET(ensure(ctx, ctx->wcnt, ((u64)g.W + 1) * sizeof(u32)));
+        RET(ensure(ctx, ctx->tcnt, ((u64)g.T + 1) * sizeof(u32)));
+        CK(cudaMemsetAsync(ctx->wcnt.p, 0, ((u64)g.W + 1) * sizeof(u32), ctx->stream));
+        CK(cudaMemsetAsync(ctx->tcnt.p, 0, ((u64)g.T + 1) * sizeof(u32), ctx->stream));
+        syncx::LockParams lp;
+        lp.ev = ctx->events;
+        lp.g = g;
+        lp.ks = ks;
+        lp.off = P_<u32>(ctx->off);
+        lp.sts = P_<u32>(ctx->syn_v[scur]);
+        lp.switch_ts = P_<u32>(ctx->sw);
+        lp.wcnt = P_<u32>(ctx->wcnt);
+        lp.tcnt = P_<u32>(ctx->tcnt);
+        lp.woff = nullptr;
+        lp.toff = nullptr;
+        lp.wpts = nullptr;
+        lp.tpts = nullptr;
+        const unsigned lblocks = (unsigned)(((u64)g.W * 32 + 255) / 256);
+        syncx::k_lock_infer<false><<<lblocks, 256, 0, ctx->stream>>>(lp);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        RET(scan_excl(ctx, P_<u32>(ctx->wcnt), (u64)g.W + 1));
+        RET(scan_excl(ctx, P_<u32>(ctx->tcnt), (u64)g.T + 1));
+        u32 tot[2];
+        CK(cudaMemcpyAsync(&tot[0], P_<u32>(ctx->wcnt) + g.W, sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaMemcpyAsync(&tot[1], P_<u32>(ctx->tcnt) + g.T, sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        RET(ensure(ctx, ctx->wpts, ((u64)tot[0] + 1) * sizeof(u64)));
+        RET(ensure(ctx, ctx->tpts, ((u64)tot[1] + 1) * sizeof(u64)));
+        lp.woff = P_<u32>(ctx->wcnt);
+        lp.toff = P_<u32>(ctx->tcnt);
+        lp.wpts = P_<u64>(ctx->wpts);
+        lp.tpts = P_<u64>(ctx->tpts);
+        syncx::k_lock_infer<true><<<lblocks, 256, 0, ctx->stream>>>(lp);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        lv.off = P_<u32>(ctx->off);
+        lv.lock_key0 = ks.lock;
+        lv.switch_ts = P_<u32>(ctx->sw);
+        lv.woff = P_<u32>(ctx->wcnt);
+        lv.toff = P_<u32>(ctx->tcnt);
+        lv.wpts = P_<u64>(ctx->wpts);
+        lv.tpts = P_<u64>(ctx->tpts);
+        lv.any = 1;
+    }
+    mark(ctx, 3);
+    // ---------------- a5: accesses sorted by word, stable ----------------
+    int acur = 0;
+    RET(radix_sort(ctx, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur));
+    mark(ctx, 4);
+    // ---------------- a6: segmented shadow pass + check ----------------
+    if (ctx->rep_cap == 0) ctx->rep_cap = 1 << 20;
+    u64 n_rep = 0;
+    if (n_acc > 0) {
+        const u64 tiles = (n_acc + check::TILE - 1) / check::TILE;
+        for (int attempt = 0;; attempt++) {
+            RET(ensure(ctx, ctx->rep_raw, ctx->rep_cap * sizeof(igd_report)));
+            RET(ensure(ctx, ctx->rep_ctr, sizeof(u64)));
+            RET(ensure(ctx, ctx->status, tiles * sizeof(u64)));
+            CK(cudaMemsetAsync(ctx->status.p, 0, tiles * sizeof(u64), ctx->stream));
+            CK(cudaMemsetAsync(ctx->ctr.p, 0, sizeof(u32), ctx->stream));
+            CK(cudaMemsetAsync(ctx->rep_ctr.p, 0, sizeof(u64), ctx->stream));
+            check::Params cp;
+            cp.key = P_<u32>(ctx->acc_k[acur]);
+            cp.val = P_<u32>(ctx->acc_v[acur]);
+            cp.n = (u32)n_acc;
+            cp.ev = ctx->events;
+            cp.g = g;
+            cp.ks = ks;
+            cp.off = P_<u32>(ctx->off);
+            cp.sts = P_<u32>(ctx->syn_v[scur]);
+            cp.lv = lv;
+            cp.status = P_<u64>(ctx->status);
+            cp.tile_ctr = P_<u32>(ctx->ctr);
+            cp.rep = P_<igd_report>(ctx->rep_raw);
+            cp.rep_cap = ctx->rep_cap;
+            cp.rep_ctr = P_<unsigned long long>(ctx->rep_ctr);
+            cp.first_event = 0;
+            check::k_check<<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+            ctx->launches++;
+            CK(cudaGetLastError());
+            CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
+            CK(cudaStreamSynchronize(ctx->stream));
+            n_rep = ctx->h_small[0];
+            if (n_rep <= ctx->rep_cap) break;
+            ctx->rep_cap = n_rep + n_rep / 8;
+            if (attempt > 2) return IGD_ECUDA;
+        }
+    }
+    mark(ctx, 5);
+    // ---------------- a7: canonical order (ascending cur) ----------------
+    RET(ensure(ctx, ctx->rep_out, (n_rep ? n_rep : 1) * sizeof(igd_report)));
+    if (n_rep == 1) {
+        CK(cudaMemcpyAsync(ctx->rep_out.p, ctx->rep_raw.p, sizeof(igd_report), cudaMemcpyDeviceToDevice, ctx->stream));
+    } else if (n_rep > 1) {
+        for (int b = 0; b < 2; b++) {
+            RET(ensure(ctx, ctx->rep_k[b], n_rep * sizeof(u32)));
+            RET(ensure(ctx, ctx->rep_v[b], n_rep * sizeof(u32)));
+        }
+        RET(ensure(ctx, ctx->rep_hist, 1024 * sizeof(u32)));
+        unsigned blocks = (unsigned)std::min<u64>((n_rep + 255) / 256, (u64)sms * 8);
+        check::k_report_keys<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw), (u32)n_rep, 0,
+                                                            P_<u32>(ctx->rep_k[0]), P_<u32>(ctx->rep_v[0]));
+        CK(cudaMemsetAsync(ctx->rep_hist.p, 0, 1024 * sizeof(u32), ctx->stream));
+        rsort::k_hist4<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->rep_k[0]), n_rep, P_<u32>(ctx->rep_hist));
+        ctx->launches += 2;
+        CK(cudaMemcpyAsync(ctx->h_hist + 2048, ctx->rep_hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost,
+                           ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        u32 hh[1024];
+        memcpy(hh, ctx->h_hist + 2048, sizeof(hh));
+        int rcur = 0;
+        RET(radix_sort(ctx, ctx->rep_k, ctx->rep_v, n_rep, P_<u32>(ctx->rep_hist), hh, bits_needed(n - 1), &rcur));
+        check::k_report_gather<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw), P_<u32>(ctx->rep_v[rcur]),
+                                                               (u32)n_rep, P_<igd_report>(ctx->rep_out));
+        ctx->launches++;
+        CK(cudaGetLastError());
+    }
+    mark(ctx, 6);
+    CK(cudaStreamSynchronize(ctx->stream));
+    mark(ctx, 7);
+    mark(ctx, 8);
+    ctx->n_reports = n_rep;
+    *n_out = n_rep;
+    return IGD_OK;
+}
+
+// ================================ C ABI =====================================================
+extern "C" {
+
+int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks, int rank,
+                   const uint8_t* nccl_unique_id, igd_alloc_fn alloc_fn, igd_free_fn free_fn, void* alloc_user) {
+    (void)nccl_unique_id;
+    if (!out) return IGD_EINVAL;
+    *out = nullptr;
+    if (nranks != 1 || rank != 0) return IGD_EINVAL;
+    if ((alloc_fn == nullptr) != (free_fn == nullptr)) return IGD_EINVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
+        (void)cudaGetLastError();
+        return IGD_ECUDA;
+    }
+    if (cudaSetDevice(cuda_device) != cudaSuccess) return IGD_ECUDA;
+    igd_ctx* ctx = new igd_ctx();
+    ctx->device = cuda_device;
+    ctx->stream = (cudaStream_t)cuda_stream;
+    ctx->afn = alloc_fn;
+    ctx->ffn = free_fn;
+    ctx->auser = alloc_user;
+    if (cudaMallocHost(&ctx->h_stats, 8 * sizeof(u64)) != cudaSuccess ||
+        cudaMallocHost(&ctx->h_hist, 3 * 1024 * sizeof(u32)) != cudaSuccess ||
+        cudaMallocHost(&ctx->h_small, 8 * sizeof(u64)) != cudaSuccess) {
+        delete ctx;
+        return IGD_ENOMEM;
+    }
+    for (int i = 0; i <= IGD_N_STAGES; i++) cudaEventCreate(&ctx->ev[i]);
+    for (int i = 0; i < IGD_N_STAGES; i++) ctx->stage_ms[i] = 0.f;
+    *out = ctx;
+    return IGD_OK;
+}
+
+int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* events) {
+    if (!ctx || !desc) return IGD_EINVAL;
+    if (desc->n_blocks == 0 || desc->block_dim == 0) return IGD_EINVAL;
+    if ((u64)desc->n_blocks * desc->block_dim > (1ull << 24)) return IGD_EINVAL;
+    if (desc->n_events >= 0xFFFFFFFFull) return IGD_ETOOBIG;
+    if (desc->n_events > 0 && !events) return IGD_EINVAL;
+    if (desc->first_event != 0 || (desc->n_events_total != 0 && desc->n_events_total != desc->n_events)) {
+        ctx->err = "single-rank build: first_event must be 0 and n_events_total == n_events";
+        return IGD_EINVAL;
+    }
+    cudaSetDevice(ctx->device);
+    ctx->desc = *desc;
+    ctx->loaded = false;
+    if (desc->flags & IGD_TRACE_DEVICE_PTR) {
+        ctx->events = events;
+    } else {
+        const size_t bytes = desc->n_events * sizeof(igd_event);
+        RET(ensure(ctx, ctx->owned_events, bytes));
+        if (bytes) CK(cudaMemcpyAsync(ctx->owned_events.p, events, bytes, cudaMemcpyHostToDevice, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        ctx->events = P_<igd_event>(ctx->owned_events);
+    }
+    ctx->loaded = true;
+    return IGD_OK;
+}
+
+int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
+    if (!ctx || !n_reports_global) return IGD_EINVAL;
+    if (!ctx->loaded) return IGD_ESTATE;
+    cudaSetDevice(ctx->device);
+    ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
+    int rc = detect_impl(ctx, n_reports_global);
+    if (rc == IGD_OK && ctx->timing) {
+        cudaEventSynchronize(ctx->ev[8]);
+        for (int s = 0; s < IGD_N_STAGES - 1; s++) cudaEventElapsedTime(&ctx->stage_ms[s], ctx->ev[s], ctx->ev[s + 1]);
+        cudaEventElapsedTime(&ctx->stage_ms[IGD_N_STAGES - 1], ctx->ev[0], ctx->ev[7]);
+    }
+    return rc;
+}
+
+int igd_reports(igd_ctx* ctx, igd_report* host_out, uint64_t cap, uint64_t* n_written) {
+    if (!ctx || !n_written || (cap > 0 && !host_out)) return IGD_EINVAL;
+    u64 k = ctx->n_reports < cap ? ctx->n_reports : cap;
+    *n_written = k;
+    if (k) {
+        CK(cudaMemcpyAsync(host_out, ctx->rep_out.p, k * sizeof(igd_report), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+    }
+    return IGD_OK;
+}
+
+int igd_reports_device(igd_ctx* ctx, const igd_report** dev_ptr, uint64_t* n) {
+    if (!ctx || !dev_ptr || !n) return IGD_EINVAL;
+    *dev_ptr = P_<igd_report>(ctx->rep_out);
+    *n = ctx->n_reports;
+    return IGD_OK;
+}
+
+uint64_t igd_bad_event(const igd_ctx* ctx) { return ctx ? ctx->bad_event : 0; }
+
+int igd_stage_times(const igd_ctx* ctx, float* ms_out) {
+    if (!ctx || !ms_out) return IGD_EINVAL;
+    for (int i = 0; i < IGD_N_STAGES; i++) ms_out[i] = ctx->stage_ms[i];
+    return IGD_OK;
+}
+
+const char* igd_stage_name(int stage) {
+    return (stage >= 0 && stage < IGD_N_STAGES) ? kStageNames[stage] : "?";
+}
+
+uint64_t igd_last_launch_count(const igd_ctx* ctx) { return ctx ? ctx->launches : 0; }
+
+void igd_ctx_destroy(igd_ctx* ctx) {
+    if (!ctx) return;
+    cudaSetDevice(ctx->device);
+    Buf* all[] = {&ctx->owned_events, &ctx->acc_k[0], &ctx->acc_k[1], &ctx->acc_v[0], &ctx->acc_v[1],
+                  &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
+                  &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
+                  &ctx->ctr,          &ctx->off,      &ctx->sw,       &ctx->wcnt,     &ctx->tcnt,
+                  &ctx->wpts,         &ctx->tpts,     &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
+                  &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist};
+    for (Buf* b : all) buf_free(ctx, *b);
+    cudaStreamSynchronize(ctx->stream);
+    cudaFreeHost(ctx->h_stats);
+    cudaFreeHost(ctx->h_hist);
+    cudaFreeHost(ctx->h_small);
+    for (int i = 0; i <= IGD_N_STAGES; i++) cudaEventDestroy(ctx->ev[i]);
+    delete ctx;
+}
+
+const char* igd_strerror(int code) {
+    switch (code) {
+        case IGD_OK: return "ok";
+        case IGD_EINVAL: return "invalid argument or geometry";
+        case IGD_ETRACE: return "ill-formed trace event";
+        case IGD_ETOOBIG: return "trace too large for the 32-bit index path";
+        case IGD_ENOMEM: return "device out of memory";
+        case IGD_ECUDA: return "CUDA error";
+        case IGD_ENCCL: return "NCCL error";
+        case IGD_ESTATE: return "call out of order";
+        default: return "unknown error";
+    }
+}
+
+const char* igd_last_error(const igd_ctx* ctx) { return ctx ? ctx->err.c_str() : ""; }
+
+}  // extern "C"

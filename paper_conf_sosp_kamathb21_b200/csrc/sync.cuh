@@ -1,0 +1,300 @@
+// sync.cuh -- a2 epoch tables and a3 lock inference.
+//
+// a2: after the stable sort of synchronization records by entity key, offsets[e] is the first
+//     record of entity e (CSR).  The per-entity timestamp lists replace the paper's bounded
+//     per-thread / per-warp / per-block counters (Fig. 4, Fig. 5) by exact
+//     "was there a sync of this entity in (a, b)?" queries (reading A16).
+// a3: per-warp lock-table state machine of §6.3: atomicCAS inserts an 18-bit
+//     address hash (Valid, not Active), a fence of matching-or-wider scope activates entries,
+//     atomicExch invalidates the entry with the same hash and scope, a CAS executed by more
+//     than one lane switches the warp to per-thread tables for good, a grid sync
+//     is a device fence by every thread (reading A15).  One CUDA warp replays one traced warp,
+//     lane l owning thread l's per-thread table; it emits change points (ts, bloom) of the
+//     held-lock Bloom summary so the check can ask "locks of thread c just before
+//     event i" with one binary search.
+#pragma once
+#include "common.cuh"
+
+namespace syncx {
+
+// offsets[e] = lower_bound(keys, e) for e in [0, E]
+__global__ void k_csr_offsets(const u32* __restrict__ keys, u32 n, u32 E, u32* __restrict__ off) {
+    for (u64 e = (u64)blockIdx.x * blockDim.x + threadIdx.x; e <= E; e += (u64)gridDim.x * blockDim.x) {
+        u32 lo = 0, hi = n;
+        while (lo < hi) {
+            u32 mid = (lo + hi) >> 1;
+            if (__ldg(keys + mid) < (u32)e) lo = mid + 1;
+            else hi = mid;
+        }
+        off[e] = lo;
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Lock tables.  An entry is packed in a u32: bit 31 valid, bit 30 active, bits 28..29 scope,
+// bits 0..17 the 18-bit hash.
+__device__ __forceinline__ u32 le_valid(u32 e) { return e >> 31; }
+__device__ __forceinline__ u32 le_active(u32 e) { return (e >> 30) & 1u; }
+__device__ __forceinline__ u32 le_scope(u32 e) { return (e >> 28) & 3u; }
+__device__ __forceinline__ u32 le_hash(u32 e) { return e & 0x3FFFFu; }
+
+struct Table {
+    u32 e[3];
+    __device__ __forceinline__ void clear() { e[0] = e[1] = e[2] = 0; }
+    // "sets the Active bit ... for all entries with matching or narrower scope"
+    __device__ __forceinline__ void activate(u32 s) {
+#pragma unroll
+        for (int k = 0; k < 3; k++)
+            if (le_valid(e[k]) && le_scope(e[k]) <= s) e[k] |= (1u << 30);
+    }
+    // insert on atomicCAS (readings A9): dedup (hash, scope), lowest free slot,
+    // dropped when full
+    __device__ __forceinline__ void insert(u32 h, u32 s) {
+#pragma unroll
+        for (int k = 0; k < 3; k++)
+            if (le_valid(e[k]) && le_hash(e[k]) == h && le_scope(e[k]) == s) return;
+#pragma unroll
+        for (int k = 0; k < 3; k++)
+            if (!le_valid(e[k])) {
+                e[k] = (1u << 31) | (s << 28) | h;
+                return;
+            }
+    }
+    // remove on atomicExch: "Valid bit of any entry matching the address hash and scope is unset"
+    __device__ __forceinline__ void remove(u32 h, u32 s) {
+#pragma unroll
+        for (int k = 0; k < 3; k++)
+            if (le_valid(e[k]) && le_hash(e[k]) == h && le_scope(e[k]) == s) e[k] = 0;
+    }
+    __device__ __forceinline__ u32 held() const {
+        u32 b = 0;
+#pragma unroll
+        for (int k = 0; k < 3; k++)
+            if (le_valid(e[k]) && le_active(e[k])) b |= lock_bloom(le_hash(e[k]));
+        return b;
+    }
+};
+
+struct LockParams {
+    const igd_event* ev;
+    Geo g;
+    KeySpace ks;
+    const u32* off;       // CSR offsets of sync records
+    const u32* sts;       // sorted sync timestamps
+    u32* switch_ts;       // [W] isThread switch time (NONE = never)
+    u32* wcnt;            // [W+1] warp change-point counts (pass 0) -> offsets after scan
+    u32* tcnt;            // [T+1] thread change-point counts
+    const u32* woff;      // [W+1] (pass 1)
+    const u32* toff;      // [T+1] (pass 1)
+    u64* wpts;            // warp change points  (ts << 16 | bloom)
+    u64* tpts;            // thread change points
+};
+
+// One warp per traced warp.  WRITE = false: count change points; true: write them.
+template <bool WRITE>
+__global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
+    const u32 lane = threadIdx.x & 31u;
+    const u32 w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (w >= P.g.W) return;
+    const KeySpace ks = P.ks;
+    u32 lk_lo = P.off[ks.lock + w];
+    const u32 lk_hi = P.off[ks.lock + w + 1];
+    if (lk_lo == lk_hi) {
+        if (!WRITE && lane == 0) {
+            P.wcnt[w] = 0;
+            P.switch_ts[w] = IGD_NONE32;
+        }
+        if (!WRITE) {
+            // thread counts of this warp's lanes
+            u32 b = w / P.g.Wb, wi = w - b * P.g.Wb;
+            u32 off = wi * 32 + lane;
+            if (off < P.g.D) P.tcnt[b * P.g.D + off] = 0;
+        }
+        return;
+    }
+    const u32 b = w / P.g.Wb, wi = w - b * P.g.Wb;
+    const u32 my_off = wi * 32 + lane;
+    const bool has_thread = my_off < P.g.D;
+    const u32 my_t = b * P.g.D + my_off;
+    u32 f_lo = 0, f_hi = 0;
+    if (has_thread) {
+        f_lo = P.off[ks.any + my_t];
+        f_hi = P.off[ks.any + my_t + 1];
+    }
+    u32 g_lo = P.off[ks.grid], g_hi = P.off[ks.grid + 1];
+
+    Table wt, tt;
+    wt.clear();
+    tt.clear();
+    bool isThread = false;
+    u32 sw = IGD_NONE32;
+    u32 held_w = 0, held_t = 0;
+    u32 nw = 0, nt = 0;
+    u32 wout = WRITE ? P.woff[w] : 0;
+    u32 tout = (WRITE && has_thread) ? P.toff[my_t] : 0;
+
+    u32 my_next = (f_lo < f_hi) ? __ldg(P.sts + f_lo) : IGD_NONE32;
+    u32 lk_next = __ldg(P.sts + lk_lo);
+    u32 g_next = (g_lo < g_hi) ? __ldg(P.sts + g_lo) : IGD_NONE32;
+    while (true) {
+        const u32 f_min = __reduce_min_sync(IGD_FULL, my_next);
+        const u32 ts = min(f_min, min(lk_next, g_next));
+        if (ts == IGD_NONE32) break;
+        if (ts == g_next) {
+            // grid sync: every thread fences at device scope (A15)
+            wt.activate(IGD_SCOPE_DEVICE);
+            tt.activate(IGD_SCOPE_DEVICE);
+            g_lo++;
+            g_next = (g_lo < g_hi) ? __ldg(P.sts + g_lo) : IGD_NONE32;
+        } else if (ts == lk_next) {
+            const uint4 e = ld_event(P.ev, ts);
+            const u32 kind = ev_kind(e), s = norm_scope(ev_scope(e));
+            const u32 h = lock_h18(ev_addr(e) >> 2);
+            const u32 el = P.g.lane(ev_tid(e));
+            if (kind == IGD_CAS) {
+                if (!isThread && __popc(e.w) > 1) {
+                    isThread = true;
+                    sw = ts;
+                }
+                if (isThread) {
+                    if (lane == el) tt.insert(h, s);
+                } else {
+                    wt.insert(h, s);
+                }
+            } else {  // EXCH
+                if (isThread) {
+                    if (lane == el) tt.remove(h, s);
+                } else {
+                    wt.remove(h, s);
+                }
+            }
+            lk_lo++;
+            lk_next = (lk_lo < lk_hi) ? __ldg(P.sts + lk_lo) : IGD_NONE32;
+        } else {
+            // a fence by the lane whose next fence is ts
+            const u32 owner = __ffs(__ballot_sync(IGD_FULL, my_next == ts)) - 1;
+            u32 s = 0;
+            if (lane == owner) {
+                s = norm_scope(ev_scope(ld_event(P.ev, ts)));
+                f_lo++;
+                my_next = (f_lo < f_hi) ? __ldg(P.sts + f_lo) : IGD_NONE32;
+            }
+            s = __shfl_sync(IGD_FULL, s, owner);
+            if (isThread) {
+                if (lane == owner) tt.activate(s);
+            } else {
+                wt.activate(s);
+            }
+        }
+        // change points
+        if (!isThread) {
+            const u32 hw = wt.held();
+            if (hw != held_w) {
+                if (WRITE && lane == 0) P.wpts[wout + nw] = ((u64)ts << 16) | hw;
+                nw++;
+                held_w = hw;
+            }
+        } else {
+            const u32 ht = tt.held();
+            if (ht != held_t) {
+                if (WRITE && has_thread) P.tpts[tout + nt] = ((u64)ts << 16) | ht;
+                nt++;
+                held_t = ht;
+            }
+        }
+    }
+    if (!WRITE) {
+        if (lane == 0) {
+            P.wcnt[w] = nw;
+            P.switch_ts[w] = sw;
+        }
+        if (has_thread) P.tcnt[my_t] = nt;
+    }
+}
+
+// held-lock Bloom of thread c just before event i (the check's L(c, i))
+struct LockView {
+    const u32* off;
+    u32 lock_key0;
+    const u32* switch_ts;
+    const u32* woff;
+    const u32* toff;
+    const u64* wpts;
+    const u64* tpts;
+    u32 any;  // 0 when the trace has no CAS/EXCH at all
+};
+
+__device__ __forceinline__ u32 last_before(const u64* __restrict__ pts, u32 lo, u32 hi, u32 i) {
+    // last entry with ts < i
+    u32 L = lo, H = hi;
+    while (L < H) {
+        u32 mid = (L + H) >> 1;
+        if ((u32)(__ldg(pts + mid) >> 16) < i) L = mid + 1;
+        else H = mid;
+    }
+    return (L > lo) ? (u32)(__ldg(pts + L - 1) & 0xFFFFu) : 0u;
+}
+
+__device__ __forceinline__ u32 held_before(const LockView& V, const Geo& g, u32 c, u32 i) {
+    if (!V.any) return 0;
+    const u32 w = g.warp(c);
+    if (__ldg(V.off + V.lock_key0 + w) == __ldg(V.off + V.lock_key0 + w + 1)) return 0;
+    const u32 sw = __ldg(V.switch_ts + w);
+    if (sw != IGD_NONE32 && i > sw) return last_before(V.tpts, __ldg(V.toff + c), __ldg(V.toff + c + 1), i);
+    return last_before(V.wpts, __ldg(V.woff + w), __ldg(V.woff + w + 1), i);
+}
+
+// ---------------------------------------------------------------------------------------------
+// Exclusive scan of u32 counts (in place allowed), chained look-back. n includes the sentinel.
+constexpr int SCAN_THREADS = 256;
+constexpr int SCAN_ITEMS = 8;
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan_excl(const u32* in, u32* out, u32 n, u64* status,
+                                                          u32* tile_ctr) {
+    __shared__ u32 s_tile;
+    __shared__ u32 s_wsum[SCAN_THREADS / 32];
+    __shared__ u64 s_base;
+    const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
+    if (t == 0) s_tile = atomicAdd(tile_ctr, 1u);
+    __syncthreads();
+    const u32 tile = s_tile;
+    const u64 base = (u64)tile * SCAN_THREADS * SCAN_ITEMS + (u64)t * SCAN_ITEMS;
+    u32 v[SCAN_ITEMS];
+    u32 sum = 0;
+#pragma unroll
+    for (int j = 0; j < SCAN_ITEMS; j++) {
+        v[j] = (base + j < n) ? in[base + j] : 0;
+        sum += v[j];
+    }
+    u32 inc = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        u32 x = __shfl_up_sync(IGD_FULL, inc, o);
+        if (lane >= (u32)o) inc += x;
+    }
+    if (lane == 31) s_wsum[warp] = inc;
+    __syncthreads();
+    u32 wpre = 0, total = 0;
+#pragma unroll
+    for (int w = 0; w < SCAN_THREADS / 32; w++) {
+        if ((u32)w < warp) wpre += s_wsum[w];
+        total += s_wsum[w];
+    }
+    if (warp == 0) {
+        if (lane == 0) st_relaxed(&status[tile], (tile == 0 ? ST_INC : ST_AGG) | total);
+        u64 b = 0;
+        if (tile > 0) {
+            b = lookback_sum_warp(status, tile);
+            if (lane == 0) st_relaxed(&status[tile], ST_INC | (b + total));
+        }
+        if (lane == 0) s_base = b;
+    }
+    __syncthreads();
+    u32 run = (u32)s_base + wpre + inc - sum;
+#pragma unroll
+    for (int j = 0; j < SCAN_ITEMS; j++) {
+        if (base + j < n) out[base + j] = run;
+        run += v[j];
+    }
+}
+
+}  // namespace syncx

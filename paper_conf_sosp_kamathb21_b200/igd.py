@@ -1,0 +1,219 @@
+"""ctypes binding of libigd (include/igd.h): argument marshalling only.
+
+Functions keep the C names (``igd_ctx_create``, ``igd_trace_load``, ``igd_detect``,
+``igd_reports``, ``igd_ctx_destroy``, ``igd_strerror``).  :class:`Detector` wires them to
+PyTorch for device memory (caching-allocator callbacks) and the current CUDA stream.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from . import _build
+
+EVENT_DTYPE = np.dtype([("addr", "<u8"), ("tk", "<u4"), ("mask", "<u4")])
+REPORT_DTYPE = np.dtype([("addr", "<u8"), ("cur", "<u8"), ("prev", "<u8"), ("type", "u1"),
+                         ("cur_kind", "u1"), ("prev_kind", "u1"), ("pad", "u1", (5,))])
+IGD_OK, IGD_EINVAL, IGD_ETRACE, IGD_ETOOBIG, IGD_ENOMEM, IGD_ECUDA, IGD_ENCCL, IGD_ESTATE = 0, -1, -2, -3, -4, -5, -6, -7
+IGD_TRACE_DEVICE_PTR = 1
+IGD_DETECT_TIMING = 1
+IGD_N_STAGES = 8
+
+
+class igd_trace_desc(ctypes.Structure):
+    _fields_ = [("n_blocks", ctypes.c_uint32), ("block_dim", ctypes.c_uint32),
+                ("n_events_total", ctypes.c_uint64), ("first_event", ctypes.c_uint64),
+                ("n_events", ctypes.c_uint64), ("flags", ctypes.c_uint32)]
+
+
+ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+
+_lib = None
+
+
+def lib_path() -> str:
+    return _build.LIB
+
+
+def load_library(build_if_missing: bool = True):
+    """Load libigd.so (building it with nvcc first if it is missing or stale)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if build_if_missing and _build.needs_build():
+        _build.build()
+    if not os.path.exists(_build.LIB):
+        raise ImportError(f"libigd.so not built at {_build.LIB}")
+    lib = ctypes.CDLL(_build.LIB)
+    vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+    lib.igd_ctx_create.argtypes = [ctypes.POINTER(vp), i32, vp, i32, i32, vp, ALLOC_FN, FREE_FN, vp]
+    lib.igd_ctx_create.restype = i32
+    lib.igd_trace_load.argtypes = [vp, ctypes.POINTER(igd_trace_desc), vp]
+    lib.igd_trace_load.restype = i32
+    lib.igd_detect.argtypes = [vp, u32, ctypes.POINTER(u64)]
+    lib.igd_detect.restype = i32
+    lib.igd_reports.argtypes = [vp, vp, u64, ctypes.POINTER(u64)]
+    lib.igd_reports.restype = i32
+    lib.igd_reports_device.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(u64)]
+    lib.igd_reports_device.restype = i32
+    lib.igd_bad_event.argtypes = [vp]
+    lib.igd_bad_event.restype = u64
+    lib.igd_stage_times.argtypes = [vp, ctypes.POINTER(ctypes.c_float)]
+    lib.igd_stage_times.restype = i32
+    lib.igd_stage_name.argtypes = [i32]
+    lib.igd_stage_name.restype = ctypes.c_char_p
+    lib.igd_last_launch_count.argtypes = [vp]
+    lib.igd_last_launch_count.restype = u64
+    lib.igd_ctx_destroy.argtypes = [vp]
+    lib.igd_ctx_destroy.restype = None
+    lib.igd_strerror.argtypes = [i32]
+    lib.igd_strerror.restype = ctypes.c_char_p
+    lib.igd_last_error.argtypes = [vp]
+    lib.igd_last_error.restype = ctypes.c_char_p
+    _lib = lib
+    return lib
+
+
+class IgdError(RuntimeError):
+    def __init__(self, code: int, msg: str = "", bad_index=None):
+        super().__init__(f"igd error {code} ({igd_strerror(code)}): {msg}")
+        self.code = code
+        self.bad_index = bad_index
+
+
+# ---- thin same-name wrappers ---------------------------------------------------------------
+def igd_strerror(code: int) -> str:
+    return load_library().igd_strerror(code).decode()
+
+
+def igd_ctx_create(cuda_device: int, cuda_stream: int, alloc_fn=None, free_fn=None, nranks: int = 1,
+                   rank: int = 0):
+    lib = load_library()
+    ctx = ctypes.c_void_p()
+    rc = lib.igd_ctx_create(ctypes.byref(ctx), cuda_device, ctypes.c_void_p(cuda_stream), nranks, rank, None,
+                            alloc_fn or ALLOC_FN(), free_fn or FREE_FN(), None)
+    if rc != IGD_OK:
+        raise IgdError(rc, "igd_ctx_create")
+    return ctx
+
+
+def igd_trace_load(ctx, n_blocks: int, block_dim: int, events_ptr: int, n_events: int, device_ptr: bool):
+    lib = load_library()
+    d = igd_trace_desc(n_blocks, block_dim, n_events, 0, n_events, IGD_TRACE_DEVICE_PTR if device_ptr else 0)
+    rc = lib.igd_trace_load(ctx, ctypes.byref(d), ctypes.c_void_p(events_ptr or None))
+    if rc != IGD_OK:
+        raise IgdError(rc, lib.igd_last_error(ctx).decode())
+
+
+def igd_detect(ctx, flags: int = 0) -> int:
+    lib = load_library()
+    n = ctypes.c_uint64(0)
+    rc = lib.igd_detect(ctx, flags, ctypes.byref(n))
+    if rc != IGD_OK:
+        bad = lib.igd_bad_event(ctx) if rc == IGD_ETRACE else None
+        raise IgdError(rc, lib.igd_last_error(ctx).decode(), bad)
+    return int(n.value)
+
+
+def igd_reports(ctx, cap: int) -> np.ndarray:
+    lib = load_library()
+    out = np.zeros(cap, REPORT_DTYPE)
+    n = ctypes.c_uint64(0)
+    rc = lib.igd_reports(ctx, out.ctypes.data if cap else None, cap, ctypes.byref(n))
+    if rc != IGD_OK:
+        raise IgdError(rc, lib.igd_last_error(ctx).decode())
+    return out[: n.value]
+
+
+def igd_ctx_destroy(ctx) -> None:
+    load_library().igd_ctx_destroy(ctx)
+
+
+# ---- torch plumbing ------------------------------------------------------------------------
+class Detector:
+    """One libigd context on a CUDA device, using torch's caching allocator and stream.
+
+    ``load`` accepts a host numpy EVENT_DTYPE array (copied by the library) or a CUDA
+    tensor of the same bytes (borrowed: kept alive here until the next load)."""
+
+    def __init__(self, device: int = 0, stream=None):
+        import torch
+
+        if not torch.cuda.is_available():
+            raise RuntimeError("libigd needs a CUDA device; there is no CPU fallback")
+        self._torch = torch
+        self.device = device
+        self.stream = stream if stream is not None else torch.cuda.current_stream(device)
+        dev = device
+
+        def _alloc(nbytes, stream, user):
+            try:
+                return torch.cuda.caching_allocator_alloc(int(nbytes), dev, stream or 0)
+            except Exception:  # noqa: BLE001 -- reported to the library as NULL (IGD_ENOMEM)
+                return None
+
+        def _free(p, stream, user):
+            torch.cuda.caching_allocator_delete(p)
+
+        self._afn = ALLOC_FN(_alloc)
+        self._ffn = FREE_FN(_free)
+        self.ctx = igd_ctx_create(device, self.stream.cuda_stream, self._afn, self._ffn)
+        self._borrowed = None
+        self.n_reports = 0
+
+    def load(self, events, n_blocks: int, block_dim: int):
+        torch = self._torch
+        if isinstance(events, torch.Tensor):
+            assert events.is_cuda and events.is_contiguous() and events.numel() * events.element_size() % 16 == 0
+            n = events.numel() * events.element_size() // 16
+            self._borrowed = events
+            igd_trace_load(self.ctx, n_blocks, block_dim, events.data_ptr() if n else 0, n, True)
+        else:
+            ev = np.ascontiguousarray(events)
+            assert ev.dtype.itemsize == 16
+            self._borrowed = None
+            igd_trace_load(self.ctx, n_blocks, block_dim, ev.ctypes.data if len(ev) else 0, len(ev), False)
+
+    def detect(self, timing: bool = False) -> int:
+        self.n_reports = igd_detect(self.ctx, IGD_DETECT_TIMING if timing else 0)
+        return self.n_reports
+
+    def reports(self) -> np.ndarray:
+        return igd_reports(self.ctx, self.n_reports)
+
+    def stage_times(self) -> dict:
+        lib = load_library()
+        arr = (ctypes.c_float * IGD_N_STAGES)()
+        lib.igd_stage_times(self.ctx, arr)
+        return {lib.igd_stage_name(i).decode(): float(arr[i]) for i in range(IGD_N_STAGES)}
+
+    def launch_count(self) -> int:
+        return int(load_library().igd_last_launch_count(self.ctx))
+
+    def close(self):
+        if self.ctx is not None:
+            igd_ctx_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+def detect(events, n_blocks: int, block_dim: int, device: int = 0) -> np.ndarray:
+    """One-shot convenience: load, detect, fetch reports (ascending ``cur``)."""
+    with Detector(device) as d:
+        d.load(events, n_blocks, block_dim)
+        d.detect()
+        return d.reports()

@@ -1,0 +1,160 @@
+"""GPU parity: libigd (CUDA, through the C ABI) vs the CPU oracle, element by element on the
+same seeded traces.  Bar: identical report arrays (bit-exact integers; A29: no tie-breaks)."""
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import tracegen as tg
+from golden_io import all_golden, full_tuples, parse, report_tuples
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def det():
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    d = igd.Detector(0)
+    yield d
+    d.close()
+
+
+def gpu_run(det, ev, nb, bd):
+    det.load(ev, nb, bd)
+    det.detect()
+    return det.reports()
+
+
+def assert_same(det, ev, nb, bd, what=""):
+    want = oracle.run(ev, nb, bd)
+    got = gpu_run(det, ev, nb, bd)
+    assert len(got) == len(want), f"{what}: {len(got)} GPU reports vs {len(want)} oracle"
+    assert np.array_equal(got, want), f"{what}: first diff at {np.nonzero(got != want)[0][:5]}"
+    return len(want)
+
+
+@pytest.mark.parametrize("path", all_golden(), ids=[os.path.basename(p) for p in all_golden()])
+def test_golden(det, path):
+    ev, nb, bd, expects = parse(path)
+    got = gpu_run(det, ev, nb, bd)
+    assert report_tuples(got) == expects
+    assert full_tuples(got) == full_tuples(oracle.run(ev, nb, bd))
+
+
+def test_empty(det):
+    assert len(gpu_run(det, tg.TraceBuilder(2, 64).events(), 2, 64)) == 0
+
+
+@pytest.mark.parametrize("batch", range(4))
+def test_random_small(det, batch):
+    for seed in range(batch * 250, (batch + 1) * 250):
+        rng = np.random.default_rng(seed)
+        kw = {}
+        if seed % 3 == 0:
+            kw = dict(weights=[12, 10, 6, 10, 8, 12, 2, 2, 1, 1, 1, 1], lock_words=3 + seed % 30, p_lock_data=0.2)
+        ev, nb, bd = tg.random_trace(seed, int(rng.integers(1, 300)), n_words=int(rng.integers(1, 20)), **kw)
+        assert_same(det, ev, nb, bd, f"seed {seed}")
+
+
+@pytest.mark.parametrize("seed,n,words,nb,bd", [
+    (1, 20_000, 50, 3, 96),        # few words -> segments spanning many tiles
+    (2, 100_000, 5_000, 8, 256),
+    (3, 300_000, 1, 4, 64),        # one hot word: a single segment across ~300 tiles
+    (4, 200_000, 70_000, 16, 128),
+    (5, 150_000, 3, 1, 32),
+])
+def test_random_multi_tile(det, seed, n, words, nb, bd):
+    w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    ev, nb, bd = _fast_random(seed, n, words, nb, bd, w)
+    assert_same(det, ev, nb, bd, f"seed {seed}")
+
+
+def _fast_random(seed, n, n_words, nb, bd, weights, lock_words=8):
+    """Vectorised arbitrary-event generator (same distribution family as tg.random_trace)."""
+    rng = np.random.default_rng(seed)
+    T = nb * bd
+    w = np.asarray(weights, float)
+    kind = rng.choice(12, size=n, p=w / w.sum()).astype(np.uint32)
+    tid = rng.integers(0, T, n).astype(np.uint32)
+    lane = (tid % bd) % 32
+    lb = (np.uint32(1) << lane).astype(np.uint32)
+    mask = np.where(rng.random(n) < 0.5, lb, rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32) | lb)
+    scope = rng.integers(1, 4, n).astype(np.uint32)
+    word = rng.integers(0, n_words, n).astype(np.uint64)
+    lockw = (500_000 + rng.integers(0, lock_words, n)).astype(np.uint64)
+    is_lock = (kind == tg.CAS) | (kind == tg.EXCH)
+    word = np.where(is_lock, lockw, word)
+    plain = (kind == tg.LD) | (kind == tg.ST)
+    sync_noscope = (kind >= tg.SYNCWARP)
+    scope = np.where(plain | sync_noscope, 0, scope).astype(np.uint32)
+    addr = np.where(kind <= tg.EXCH, word << np.uint64(2), 0).astype(np.uint64)
+    grid = (kind == tg.GRID_SYNC) | (kind == tg.CG_GRID_SYNC)
+    tid = np.where(grid, 0, tid).astype(np.uint32)
+    mask = np.where(kind >= tg.SYNCTHREADS, 0xFFFFFFFF, mask).astype(np.uint32)
+    ev = np.zeros(n, tg.EVENT_DTYPE)
+    ev["addr"] = addr
+    ev["tk"] = tg.pack_tk(tid, kind, scope)
+    ev["mask"] = mask
+    return ev, nb, bd
+
+
+def test_lock_heavy_multi_tile(det):
+    w = [12, 10, 6, 10, 8, 12, 2, 2, 1, 1, 1, 1]
+    ev, nb, bd = _fast_random(11, 120_000, 300, 4, 64, w, lock_words=40)
+    assert assert_same(det, ev, nb, bd, "lock heavy") > 0
+
+
+def test_sparse_high_addresses(det):
+    # 45-bit virtual addresses, span < 2^32 words: the 32-bit key path is exact
+    ev, nb, bd = _fast_random(12, 50_000, 2_000, 2, 64, [20, 18, 10, 0, 0, 8, 3, 3, 1, 1, 1, 1])
+    acc = (ev["tk"] >> 24) & 0xF <= 4
+    ev["addr"][acc] += np.uint64(0x7F3A_0000_0000)
+    assert_same(det, ev, nb, bd, "high VA")
+
+
+def test_word_span_too_big(det):
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    b = tg.TraceBuilder(1, 32)
+    b.st(0, 1)
+    b.st(0, 1 + (1 << 32))
+    det.load(b.events(), 1, 32)
+    with pytest.raises(igd.IgdError) as ei:
+        det.detect()
+    assert ei.value.code == igd.igd.IGD_ETOOBIG
+
+
+@pytest.mark.parametrize("bad_at", [0, 5000, 99_999])
+def test_invalid_event_index_matches_oracle(det, bad_at):
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    ev, nb, bd = _fast_random(13, 100_000, 100, 2, 64, [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1])
+    ev["tk"][bad_at] = tg.pack_tk(0, 13, 0)
+    ev["tk"][min(bad_at + 7, len(ev) - 1)] = tg.pack_tk(0, 14, 0)
+    with pytest.raises(oracle.OracleError) as eo:
+        oracle.run(ev, nb, bd)
+    det.load(ev, nb, bd)
+    with pytest.raises(igd.IgdError) as eg:
+        det.detect()
+    assert eg.value.code == igd.igd.IGD_ETRACE and eg.value.bad_index == eo.value.bad_index == bad_at
+
+
+def test_device_pointer_borrowed(det):
+    import torch
+
+    ev, nb, bd = _fast_random(14, 30_000, 500, 2, 96, [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1])
+    t = torch.from_numpy(ev.view(np.uint8).copy()).cuda()
+    det.load(t, nb, bd)
+    det.detect()
+    assert np.array_equal(det.reports(), oracle.run(ev, nb, bd))
+
+
+def test_repeat_detect_is_deterministic(det):
+    ev, nb, bd = _fast_random(15, 60_000, 50, 4, 64, [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1])
+    det.load(ev, nb, bd)
+    det.detect()
+    a = det.reports()
+    det.detect()
+    assert np.array_equal(a, det.reports())
