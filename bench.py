@@ -1,0 +1,310 @@
+#!/usr/bin/env python
+"""bench.py -- G events race-checked/s on B200 (BASELINE.json metric).
+
+One step = one ``igd_detect`` over the whole synthetic trace of the workload: ingest +
+validation, sync-epoch tables, lock inference, radix sort by word, segmented shadow check,
+report compaction and canonical ordering (every SURVEY 8(a) row).  The trace is resident in
+HBM when the timed region starts (``value``); ``e2e`` repeats the measurement through the C
+ABI with HOST buffers (H2D of the trace and D2H of the reports inside the timed region).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl igd|reference]
+
+The default workload is C5 (4x10^9 events over 2^30 words; BASELINE.json configs[4], the
+configuration the metric is quoted on at 1/2/4/8 GPUs).  Inputs (64 GB) are far larger than
+L2 (126 MB), so no L2 flush is needed between steps.  ``cpu_baseline`` times the CPU oracle
+(single thread) on a bounded prefix of the same trace; ``--impl reference`` times only the
+oracle.  Data is synthetic (tracegen, seed 0x16D0000 + k).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "G events race-checked/s at 1/2/4/8 B200; achieved HBM GB/s vs peak"
+CONFIGS = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.proc = None
+            return
+        self.t = threading.Thread(target=self._read, daemon=True)
+        self.t.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 9:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows for k in range(4) if r[5 + k].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except (OSError, KeyError, ValueError):
+        return 6650.0, "fallback"
+
+
+def oracle_baseline(ev, nb, bd, budget_s=15.0):
+    """Time the CPU oracle (as it stands, single-threaded) on a bounded prefix of the trace."""
+    import oracle
+
+    n = min(len(ev), 2_000_000)
+    t0 = time.perf_counter()
+    oracle.run(ev[:n], nb, bd)
+    dt = time.perf_counter() - t0
+    rate = n / dt
+    n2 = int(min(len(ev), max(n, rate * budget_s)))
+    if n2 > n:
+        t0 = time.perf_counter()
+        oracle.run(ev[:n2], nb, bd)
+        dt = time.perf_counter() - t0
+        n = n2
+    return n, dt
+
+
+def run_reference(args, fam, rank, world):
+    """--impl reference: the CPU oracle, timed as it stands on the host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    import tracegen.families as F
+    import oracle
+
+    plan = F.Plan(fam)
+    # each step checks a bounded prefix sample of the workload so the run ends in minutes
+    sample = min(plan.n_events, args.oracle_events or 12_000_000)
+    ev = plan.fill(0, sample)
+    nb, bd, n_total = plan.n_blocks, plan.block_dim, plan.n_events
+    plan.close()
+    for _ in range(args.warmup):
+        oracle.run(ev[: min(sample, 1_000_000)], nb, bd)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.run(ev, nb, bd)
+        times.append(time.perf_counter() - t0)
+    t = sum(times) / len(times)
+    value = sample / t / 1e9
+    sample_desc = f"first {sample} of {n_total} events of {F.FAMILY_NAMES[fam]} (single-threaded oracle)"
+    line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic", "impl": "reference",
+            "config": {"workload": F.FAMILY_NAMES[fam], "events": n_total, "sample_events": sample,
+                       "n_blocks": nb, "block_dim": bd},
+            "cpu_baseline": {"value": value, "unit": "G events/s", "cores": 1, "kind": "oracle",
+                             "sample": sample_desc},
+            "e2e": {"value": value, "unit": "G events/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C5", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="igd", choices=["igd", "reference"])
+    ap.add_argument("--events", type=int, default=0, help="override the trace length (testing)")
+    ap.add_argument("--oracle-events", type=int, default=0)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer run (profiling)")
+    ap.add_argument("--threads", type=int, default=0, help="generator threads (0 = all cores)")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    fam = CONFIGS[args.config]
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, fam, rank, world)
+
+    import torch
+    import torch.distributed as dist
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import tracegen.families as F
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    # ---------------- workload ----------------
+    t0 = time.time()
+    plan = F.Plan(fam, args.events or None)
+    n, nb, bd = plan.n_events, plan.n_blocks, plan.block_dim
+    host = np.empty(n, igd.EVENT_DTYPE)
+    plan.fill(out=host, threads=args.threads)
+    ledger_n = len(plan.ledger())
+    plan.close()
+    log(f"[bench] {F.FAMILY_NAMES[fam]}: {n} events, {nb}x{bd} threads, generated in {time.time() - t0:.1f}s")
+    cudart = torch.cuda.cudart()
+    pinned = cudart.cudaHostRegister(host.ctypes.data, host.nbytes, 0) == 0
+    dev = torch.empty(host.nbytes, dtype=torch.uint8, device="cuda")
+    dev.copy_(torch.from_numpy(host.view(np.uint8)), non_blocking=False)
+    torch.cuda.synchronize()
+
+    det = igd.Detector(local)
+    stream = det.stream
+    det.load(dev, nb, bd)
+    for _ in range(args.warmup):
+        nrep = det.detect()
+    # ---------------- timed region (device-resident trace) ----------------
+    clocks = ClockSampler(local)
+    clocks.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    kstats = {}
+    launches = 0
+    e0.record(stream)
+    for _ in range(args.steps):
+        nrep = det.detect(timing=True)
+        launches += det.launch_count()
+        for k, (cnt, ms, b) in det.kernel_stats().items():
+            c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
+            kstats[k] = (c0 + cnt, m0 + ms, b0 + b)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    if world > 1:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = n * world / (ms / 1e3) / 1e9
+    reports = det.reports()
+    stages = det.stage_times()
+
+    # ---------------- roofline of the dominant kernel class ----------------
+    peak, peak_kind = peaks()
+    dom = max(kstats, key=lambda k: kstats[k][1])
+    cnt, kms, kbytes = kstats[dom]
+    achieved = kbytes / (kms / 1e3) / 1e9 if kms > 0 else 0.0
+    total_alg = sum(v[2] for v in kstats.values()) / args.steps
+    path_gbs = total_alg / (ms / 1e3) / 1e9
+    f_acc = None
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "peak_source": peak_kind, "traffic": None,
+                "launches_per_step": cnt / args.steps, "ms_per_launch": kms / max(cnt, 1),
+                "alg_bytes_per_launch": kbytes / max(cnt, 1)}
+    breakdown = {k: {"launches": v[0] // args.steps, "ms": v[1] / args.steps,
+                     "alg_GBps": (v[2] / (v[1] / 1e3) / 1e9) if v[1] > 0 else None}
+                 for k, v in kstats.items() if v[0]}
+
+    # ---------------- end to end through the C ABI with host buffers ----------------
+    del dev
+    det.load(np.zeros(0, igd.EVENT_DTYPE), nb, bd)  # drop the borrowed pointer
+    torch.cuda.empty_cache()
+    e2e_times = []
+    h2d = host.nbytes
+    d2h = 0
+    nr, out = nrep, reports
+    for s in range(0 if args.no_e2e else args.e2e_steps + 1):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        det.load(host, nb, bd)           # H2D copy of the trace inside the library
+        nr = det.detect()
+        out = det.reports()              # D2H of the reports
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        d2h = out.nbytes + 8
+        if s > 0:                        # first pass allocates the owned trace buffer
+            e2e_times.append(dt)
+    e2e_s = sum(e2e_times) / len(e2e_times) if e2e_times else float("inf")
+    if world > 1:
+        t = torch.tensor([e2e_s], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = float(t.item())
+    e2e = {"value": n * world / e2e_s / 1e9, "unit": "G events/s", "h2d_bytes_per_step": h2d,
+           "d2h_bytes_per_step": d2h, "ms_per_step": e2e_s * 1e3, "pinned_host": bool(pinned)}
+    assert nr == nrep and np.array_equal(out, reports), "e2e and device-resident runs disagree"
+    det.close()
+
+    # ---------------- CPU oracle baseline (rank 0, N=1) ----------------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        sn, sdt = oracle_baseline(host, nb, bd)
+        cpu = {"value": sn / sdt / 1e9, "unit": "G events/s", "cores": 1, "kind": "oracle",
+               "sample": f"first {sn} events of {F.FAMILY_NAMES[fam]} ({sdt:.1f}s, single-threaded C oracle)"}
+    if pinned:
+        cudart.cudaHostUnregister(host.ctypes.data)
+
+    kinds = np.bincount(((host["tk"] >> 24) & 0xF).astype(np.int64), minlength=12)
+    f_acc = float(kinds[:5].sum()) / max(n, 1)
+    b_alg = 16 + 32 * f_acc  # read the event + read/write a 16-B metadata entry per access
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
+                           "f_acc": f_acc, "reports": int(nrep), "ledger_reports": ledger_n,
+                           "l2": "inputs larger than L2 (no flush)",
+                           "parallelism": f"{world} GPU(s), one process per GPU"},
+                "roofline": roofline,
+                "path": {"alg_bytes_per_event_B_alg": b_alg, "alg_GBps_B_alg": value * b_alg,
+                         "frac_B_alg": value * b_alg / peak, "kernel_alg_GBps": path_gbs,
+                         "stages_ms": stages, "kernels": breakdown},
+                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -156,6 +156,14 @@ const char* igd_stage_name(int stage);
 /* Number of kernel launches the last igd_detect issued (evidence for gpu_launches). */
 uint64_t igd_last_launch_count(const igd_ctx* ctx);
 
+/* Per kernel class (0..IGD_N_KCLASS-1: ingest, sort_sync, csr_offsets, lock_infer, sort_access,
+   check, report, misc) of the last igd_detect run with IGD_DETECT_TIMING: launch count, summed
+   device time (CUDA events on the context stream around each launch) and the algorithmic bytes
+   those launches must move.  Any output pointer may be NULL. */
+#define IGD_N_KCLASS 8
+int igd_kernel_stats(const igd_ctx* ctx, int kclass, const char** name, uint32_t* launches, float* ms,
+                     double* alg_bytes);
+
 void igd_ctx_destroy(igd_ctx* ctx);
 const char* igd_strerror(int code);
 const char* igd_last_error(const igd_ctx* ctx);

@@ -21,12 +21,17 @@
 
 namespace {
 
+enum KClass { KC_INGEST = 0, KC_SORT_SYNC, KC_CSR, KC_LOCK, KC_SORT_ACC, KC_CHECK, KC_REPORT, KC_MISC };
+
 struct Buf {
     void* p = nullptr;
     size_t cap = 0;
 };
 
 enum Stage { S_INGEST = 0, S_SYNC_SORT, S_TABLES, S_ACC_SORT, S_CHECK, S_REPORT, S_HOST, S_TOTAL };
+const char* kClassNames[IGD_N_KCLASS] = {"ingest", "sort_sync", "csr_offsets", "lock_infer",
+                                         "sort_access", "check", "report", "misc"};
+constexpr int kMaxTimed = 128;
 const char* kStageNames[IGD_N_STAGES] = {"ingest", "sync_sort", "epoch_lock_tables", "access_sort",
                                          "check", "report_sort", "host_sync", "total"};
 
@@ -63,6 +68,32 @@ struct igd_ctx {
     bool timing = false;
     cudaEvent_t ev[IGD_N_STAGES + 1];
     float stage_ms[IGD_N_STAGES];
+    // per-launch timing (IGD_DETECT_TIMING): events around every kernel launch
+    cudaEvent_t kev[2 * kMaxTimed];
+    int kcls[kMaxTimed];
+    double kbytes[kMaxTimed];
+    int nk = 0;
+    float cls_ms[IGD_N_KCLASS];
+    uint32_t cls_n[IGD_N_KCLASS];
+    double cls_bytes[IGD_N_KCLASS];
+};
+
+// Launch bracket: records CUDA events on the context stream around one kernel launch.
+struct KTimer {
+    igd_ctx* ctx;
+    int slot;
+    KTimer(igd_ctx* c, int cls, double alg_bytes) : ctx(c), slot(-1) {
+        c->launches++;
+        if (c->timing && c->nk < kMaxTimed) {
+            slot = c->nk++;
+            c->kcls[slot] = cls;
+            c->kbytes[slot] = alg_bytes;
+            cudaEventRecord(c->kev[2 * slot], c->stream);
+        }
+    }
+    ~KTimer() {
+        if (slot >= 0) cudaEventRecord(ctx->kev[2 * slot + 1], ctx->stream);
+    }
 };
 
 #define CK(call)                                                                               \
@@ -93,7 +124,7 @@ static int ensure(igd_ctx* ctx, Buf& b, size_t bytes) {
     if (bytes == 0) bytes = 16;
     if (b.cap >= bytes) return IGD_OK;
     RET(buf_free(ctx, b));
-    size_t want = bytes + bytes / 8;  // some headroom for growing traces
+    size_t want = bytes < (1ull << 30) ? bytes + bytes / 8 : bytes;  // headroom for small buffers only
     void* p = nullptr;
     if (ctx->afn) {
         p = ctx->afn(want, (void*)ctx->stream, ctx->auser);
@@ -147,13 +178,15 @@ static void mark(igd_ctx* ctx, int stage) {
 // Stable LSD radix sort of n (key, value) pairs in buffers k[cur], v[cur]; h_hist is the host
 // copy of the 4x256 digit histogram (device copy d_hist).  Digits above max_bits and digits
 // with one occupied bin are skipped.  Returns the buffer index holding the result.
-static int radix_sort(igd_ctx* ctx, Buf* k, Buf* v, u64 n, const u32* d_hist, const u32* h_hist, u32 max_bits,
-                      int* out_cur) {
+static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d_hist, const u32* h_hist,
+                      u32 max_bits, int* out_cur) {
     int cur = 0;
     *out_cur = 0;
     if (n <= 1) return IGD_OK;
-    rsort::k_digit_base<<<4, rsort::RADIX, 0, ctx->stream>>>(d_hist, P_<u32>(ctx->base));
-    ctx->launches++;
+    {
+        KTimer kt(ctx, KC_MISC, 0);
+        rsort::k_digit_base<<<4, rsort::RADIX, 0, ctx->stream>>>(d_hist, P_<u32>(ctx->base));
+    }
     const u64 tiles = (n + rsort::TILE - 1) / rsort::TILE;
     RET(ensure(ctx, ctx->status, tiles * rsort::RADIX * sizeof(u64)));
     for (u32 p = 0; p < 4; p++) {
@@ -174,8 +207,10 @@ static int radix_sort(igd_ctx* ctx, Buf* k, Buf* v, u64 n, const u32* d_hist, co
         pp.digit_base = P_<u32>(ctx->base) + p * 256;
         pp.status = P_<u64>(ctx->status);
         pp.tile_ctr = P_<u32>(ctx->ctr);
-        rsort::k_onesweep<<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
-        ctx->launches++;
+        {
+            KTimer kt(ctx, cls, 16.0 * (double)n);  // read + write 4 B key and 4 B value
+            rsort::k_onesweep<<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
+        }
         CK(cudaGetLastError());
         cur ^= 1;
     }
@@ -189,9 +224,12 @@ static int scan_excl(igd_ctx* ctx, u32* data, u64 n) {
     RET(ensure(ctx, ctx->status, tiles * sizeof(u64)));
     CK(cudaMemsetAsync(ctx->status.p, 0, tiles * sizeof(u64), ctx->stream));
     CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
-    syncx::k_scan_excl<<<(unsigned)tiles, syncx::SCAN_THREADS, 0, ctx->stream>>>(data, data, (u32)n, P_<u64>(ctx->status),
-                                                                                 P_<u32>(ctx->ctr));
-    ctx->launches++;
+    {
+        KTimer kt(ctx, KC_LOCK, 8.0 * (double)n);
+        syncx::k_scan_excl<<<(unsigned)tiles, syncx::SCAN_THREADS, 0, ctx->stream>>>(data, data, (u32)n,
+                                                                                     P_<u64>(ctx->status),
+                                                                                     P_<u32>(ctx->ctr));
+    }
     CK(cudaGetLastError());
     return IGD_OK;
 }
@@ -202,6 +240,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     ctx->n_reports = 0;
     ctx->bad_event = 0;
     ctx->launches = 0;
+    ctx->nk = 0;
     *n_out = 0;
     mark(ctx, 0);
     if (n == 0) {
@@ -216,7 +255,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
 
     // ---------------- a1 + a2 + a4: ingest ----------------
     const u64 in_tiles = (n + ingest::TILE - 1) / ingest::TILE;
-    if (ctx->sync_cap == 0) ctx->sync_cap = n / 4 + 4096;
+    if (ctx->sync_cap == 0) ctx->sync_cap = n / 16 + 4096;  // grown and re-run on overflow
     RET(ensure(ctx, ctx->stats, 8 * sizeof(u64)));
     RET(ensure(ctx, ctx->hist, 3 * 1024 * sizeof(u32)));
     RET(ensure(ctx, ctx->base, 4 * 256 * sizeof(u32)));
@@ -260,8 +299,12 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ingest::k_ingest, ingest::THREADS, 0);
         u64 grid = (u64)sms * (occ > 0 ? occ : 1);
         if (grid > in_tiles) grid = in_tiles;
-        ingest::k_ingest<<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
-        ctx->launches++;
+        {
+            // algorithmic bytes: the events read once + the records written (known after the
+            // launch; the estimate uses the previous call's counts, fixed up below)
+            KTimer kt(ctx, KC_INGEST, 16.0 * (double)n);
+            ingest::k_ingest<<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+        }
         CK(cudaGetLastError());
         CK(cudaMemcpyAsync(ctx->h_stats, ctx->stats.p, 8 * sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 2 * 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
@@ -277,6 +320,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     }
     mark(ctx, 1);
     const u64 n_acc = ctx->h_stats[3], n_sync = ctx->h_stats[4], n_lock = ctx->h_stats[5];
+    for (int q = 0; q < ctx->nk; q++)  // events read + (key, value) records written
+        if (ctx->kcls[q] == KC_INGEST) ctx->kbytes[q] = 16.0 * (double)n + 8.0 * (double)(n_acc + n_sync);
     if (n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32)) {
         ctx->err = "accessed word range spans >= 2^32 words";
         return IGD_ETOOBIG;
@@ -288,16 +333,16 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
 
     // ---------------- a2: sync records sorted by entity, CSR offsets ----------------
     int scur = 0;
-    RET(radix_sort(ctx, ctx->syn_k, ctx->syn_v, n_sync, P_<u32>(ctx->hist) + 1024, h_hist_sync, bits_needed(ks.E),
-                   &scur));
+    RET(radix_sort(ctx, KC_SORT_SYNC, ctx->syn_k, ctx->syn_v, n_sync, P_<u32>(ctx->hist) + 1024, h_hist_sync,
+                   bits_needed(ks.E), &scur));
     mark(ctx, 2);
     RET(ensure(ctx, ctx->off, ((u64)ks.E + 2) * sizeof(u32)));
     {
         u64 work = (u64)ks.E + 1;
         unsigned blocks = (unsigned)std::min<u64>((work + 255) / 256, (u64)sms * 16);
+        KTimer kt(ctx, KC_CSR, 4.0 * (double)work);
         syncx::k_csr_offsets<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->syn_k[scur]), (u32)n_sync, ks.E,
                                                              P_<u32>(ctx->off));
-        ctx->launches++;
         CK(cudaGetLastError());
     }
     // ---------------- a3: lock inference ----------------
@@ -323,8 +368,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lp.wpts = nullptr;
         lp.tpts = nullptr;
         const unsigned lblocks = (unsigned)(((u64)g.W * 32 + 255) / 256);
-        syncx::k_lock_infer<false><<<lblocks, 256, 0, ctx->stream>>>(lp);
-        ctx->launches++;
+        {
+            KTimer kt(ctx, KC_LOCK, 0);
+            syncx::k_lock_infer<false><<<lblocks, 256, 0, ctx->stream>>>(lp);
+        }
         CK(cudaGetLastError());
         RET(scan_excl(ctx, P_<u32>(ctx->wcnt), (u64)g.W + 1));
         RET(scan_excl(ctx, P_<u32>(ctx->tcnt), (u64)g.T + 1));
@@ -338,8 +385,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lp.toff = P_<u32>(ctx->tcnt);
         lp.wpts = P_<u64>(ctx->wpts);
         lp.tpts = P_<u64>(ctx->tpts);
-        syncx::k_lock_infer<true><<<lblocks, 256, 0, ctx->stream>>>(lp);
-        ctx->launches++;
+        {
+            KTimer kt(ctx, KC_LOCK, 0);
+            syncx::k_lock_infer<true><<<lblocks, 256, 0, ctx->stream>>>(lp);
+        }
         CK(cudaGetLastError());
         lv.off = P_<u32>(ctx->off);
         lv.lock_key0 = ks.lock;
@@ -353,7 +402,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     mark(ctx, 3);
     // ---------------- a5: accesses sorted by word, stable ----------------
     int acur = 0;
-    RET(radix_sort(ctx, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur));
+    RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur));
     mark(ctx, 4);
     // ---------------- a6: segmented shadow pass + check ----------------
     if (ctx->rep_cap == 0) ctx->rep_cap = 1 << 20;
@@ -383,8 +432,11 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.rep_cap = ctx->rep_cap;
             cp.rep_ctr = P_<unsigned long long>(ctx->rep_ctr);
             cp.first_event = 0;
-            check::k_check<<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
-            ctx->launches++;
+            {
+                // 4 B key + 4 B value streamed, one 16-B event gathered per access
+                KTimer kt(ctx, KC_CHECK, 24.0 * (double)n_acc);
+                check::k_check<<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+            }
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
             CK(cudaStreamSynchronize(ctx->stream));
@@ -406,21 +458,30 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         }
         RET(ensure(ctx, ctx->rep_hist, 1024 * sizeof(u32)));
         unsigned blocks = (unsigned)std::min<u64>((n_rep + 255) / 256, (u64)sms * 8);
-        check::k_report_keys<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw), (u32)n_rep, 0,
-                                                            P_<u32>(ctx->rep_k[0]), P_<u32>(ctx->rep_v[0]));
+        {
+            KTimer kt(ctx, KC_REPORT, 40.0 * (double)n_rep);
+            check::k_report_keys<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw), (u32)n_rep, 0,
+                                                                P_<u32>(ctx->rep_k[0]), P_<u32>(ctx->rep_v[0]));
+        }
         CK(cudaMemsetAsync(ctx->rep_hist.p, 0, 1024 * sizeof(u32), ctx->stream));
-        rsort::k_hist4<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->rep_k[0]), n_rep, P_<u32>(ctx->rep_hist));
-        ctx->launches += 2;
+        {
+            KTimer kt(ctx, KC_REPORT, 4.0 * (double)n_rep);
+            rsort::k_hist4<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->rep_k[0]), n_rep, P_<u32>(ctx->rep_hist));
+        }
         CK(cudaMemcpyAsync(ctx->h_hist + 2048, ctx->rep_hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost,
                            ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
         u32 hh[1024];
         memcpy(hh, ctx->h_hist + 2048, sizeof(hh));
         int rcur = 0;
-        RET(radix_sort(ctx, ctx->rep_k, ctx->rep_v, n_rep, P_<u32>(ctx->rep_hist), hh, bits_needed(n - 1), &rcur));
-        check::k_report_gather<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw), P_<u32>(ctx->rep_v[rcur]),
-                                                               (u32)n_rep, P_<igd_report>(ctx->rep_out));
-        ctx->launches++;
+        RET(radix_sort(ctx, KC_REPORT, ctx->rep_k, ctx->rep_v, n_rep, P_<u32>(ctx->rep_hist), hh, bits_needed(n - 1),
+                       &rcur));
+        {
+            KTimer kt(ctx, KC_REPORT, 68.0 * (double)n_rep);
+            check::k_report_gather<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw),
+                                                                   P_<u32>(ctx->rep_v[rcur]), (u32)n_rep,
+                                                                   P_<igd_report>(ctx->rep_out));
+        }
         CK(cudaGetLastError());
     }
     mark(ctx, 6);
@@ -461,7 +522,13 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
         return IGD_ENOMEM;
     }
     for (int i = 0; i <= IGD_N_STAGES; i++) cudaEventCreate(&ctx->ev[i]);
+    for (int i = 0; i < 2 * kMaxTimed; i++) cudaEventCreate(&ctx->kev[i]);
     for (int i = 0; i < IGD_N_STAGES; i++) ctx->stage_ms[i] = 0.f;
+    for (int i = 0; i < IGD_N_KCLASS; i++) {
+        ctx->cls_ms[i] = 0.f;
+        ctx->cls_n[i] = 0;
+        ctx->cls_bytes[i] = 0;
+    }
     *out = ctx;
     return IGD_OK;
 }
@@ -502,6 +569,18 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
         cudaEventSynchronize(ctx->ev[8]);
         for (int s = 0; s < IGD_N_STAGES - 1; s++) cudaEventElapsedTime(&ctx->stage_ms[s], ctx->ev[s], ctx->ev[s + 1]);
         cudaEventElapsedTime(&ctx->stage_ms[IGD_N_STAGES - 1], ctx->ev[0], ctx->ev[7]);
+        for (int i = 0; i < IGD_N_KCLASS; i++) {
+            ctx->cls_ms[i] = 0.f;
+            ctx->cls_n[i] = 0;
+            ctx->cls_bytes[i] = 0;
+        }
+        for (int q = 0; q < ctx->nk; q++) {
+            float ms = 0.f;
+            cudaEventElapsedTime(&ms, ctx->kev[2 * q], ctx->kev[2 * q + 1]);
+            ctx->cls_ms[ctx->kcls[q]] += ms;
+            ctx->cls_n[ctx->kcls[q]] += 1;
+            ctx->cls_bytes[ctx->kcls[q]] += ctx->kbytes[q];
+        }
     }
     return rc;
 }
@@ -538,6 +617,16 @@ const char* igd_stage_name(int stage) {
 
 uint64_t igd_last_launch_count(const igd_ctx* ctx) { return ctx ? ctx->launches : 0; }
 
+int igd_kernel_stats(const igd_ctx* ctx, int kclass, const char** name, uint32_t* launches, float* ms,
+                     double* alg_bytes) {
+    if (!ctx || kclass < 0 || kclass >= IGD_N_KCLASS) return IGD_EINVAL;
+    if (name) *name = kClassNames[kclass];
+    if (launches) *launches = ctx->cls_n[kclass];
+    if (ms) *ms = ctx->cls_ms[kclass];
+    if (alg_bytes) *alg_bytes = ctx->cls_bytes[kclass];
+    return IGD_OK;
+}
+
 void igd_ctx_destroy(igd_ctx* ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->device);
@@ -553,6 +642,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
     cudaFreeHost(ctx->h_hist);
     cudaFreeHost(ctx->h_small);
     for (int i = 0; i <= IGD_N_STAGES; i++) cudaEventDestroy(ctx->ev[i]);
+    for (int i = 0; i < 2 * kMaxTimed; i++) cudaEventDestroy(ctx->kev[i]);
     delete ctx;
 }
 

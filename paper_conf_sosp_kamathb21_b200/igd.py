@@ -20,6 +20,7 @@ IGD_OK, IGD_EINVAL, IGD_ETRACE, IGD_ETOOBIG, IGD_ENOMEM, IGD_ECUDA, IGD_ENCCL, I
 IGD_TRACE_DEVICE_PTR = 1
 IGD_DETECT_TIMING = 1
 IGD_N_STAGES = 8
+IGD_N_KCLASS = 8
 
 
 class igd_trace_desc(ctypes.Structure):
@@ -67,6 +68,9 @@ def load_library(build_if_missing: bool = True):
     lib.igd_stage_name.restype = ctypes.c_char_p
     lib.igd_last_launch_count.argtypes = [vp]
     lib.igd_last_launch_count.restype = u64
+    lib.igd_kernel_stats.argtypes = [vp, i32, ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(u32),
+                                     ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_double)]
+    lib.igd_kernel_stats.restype = i32
     lib.igd_ctx_destroy.argtypes = [vp]
     lib.igd_ctx_destroy.restype = None
     lib.igd_strerror.argtypes = [i32]
@@ -189,6 +193,16 @@ class Detector:
         arr = (ctypes.c_float * IGD_N_STAGES)()
         lib.igd_stage_times(self.ctx, arr)
         return {lib.igd_stage_name(i).decode(): float(arr[i]) for i in range(IGD_N_STAGES)}
+
+    def kernel_stats(self) -> dict:
+        """{class: (launches, ms, algorithmic bytes)} of the last detect(timing=True)."""
+        lib = load_library()
+        out = {}
+        for k in range(IGD_N_KCLASS):
+            nm, n, ms, b = ctypes.c_char_p(), ctypes.c_uint32(), ctypes.c_float(), ctypes.c_double()
+            lib.igd_kernel_stats(self.ctx, k, ctypes.byref(nm), ctypes.byref(n), ctypes.byref(ms), ctypes.byref(b))
+            out[nm.value.decode()] = (int(n.value), float(ms.value), float(b.value))
+        return out
 
     def launch_count(self) -> int:
         return int(load_library().igd_last_launch_count(self.ctx))
