@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include "../../include/igd.h"
+#include "../../include/igd_debug.h"
 
 typedef uint32_t u32;
 typedef uint64_t u64;

@@ -56,6 +56,7 @@ struct igd_ctx {
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
+    int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any (IGD_SORT_MODE)
     u64 n_reports = 0;
     u64 bad_event = 0;
     u64 launches = 0;
@@ -183,6 +184,7 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
     int cur = 0;
     *out_cur = 0;
     if (n <= 1) return IGD_OK;
+    if (n > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;  // 32-bit tile indexing
     {
         KTimer kt(ctx, KC_MISC, 0);
         rsort::k_digit_base<<<4, rsort::RADIX, 0, ctx->stream>>>(d_hist, P_<u32>(ctx->base));
@@ -209,7 +211,10 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         pp.tile_ctr = P_<u32>(ctx->ctr);
         {
             KTimer kt(ctx, cls, 16.0 * (double)n);  // read + write 4 B key and 4 B value
-            rsort::k_onesweep<<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
+            if (ctx->sort_mode == 0)
+                rsort::k_onesweep<0><<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
+            else
+                rsort::k_onesweep<1><<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
         }
         CK(cudaGetLastError());
         cur ^= 1;
@@ -515,6 +520,7 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     ctx->afn = alloc_fn;
     ctx->ffn = free_fn;
     ctx->auser = alloc_user;
+    if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = atoi(m) == 0 ? 0 : 1;
     if (cudaMallocHost(&ctx->h_stats, 8 * sizeof(u64)) != cudaSuccess ||
         cudaMallocHost(&ctx->h_hist, 3 * 1024 * sizeof(u32)) != cudaSuccess ||
         cudaMallocHost(&ctx->h_small, 8 * sizeof(u64)) != cudaSuccess) {
@@ -537,7 +543,7 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
     if (!ctx || !desc) return IGD_EINVAL;
     if (desc->n_blocks == 0 || desc->block_dim == 0) return IGD_EINVAL;
     if ((u64)desc->n_blocks * desc->block_dim > (1ull << 24)) return IGD_EINVAL;
-    if (desc->n_events >= 0xFFFFFFFFull) return IGD_ETOOBIG;
+    if (desc->n_events > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;
     if (desc->n_events > 0 && !events) return IGD_EINVAL;
     if (desc->first_event != 0 || (desc->n_events_total != 0 && desc->n_events_total != desc->n_events)) {
         ctx->err = "single-rank build: first_event must be 0 and n_events_total == n_events";
@@ -661,5 +667,45 @@ const char* igd_strerror(int code) {
 }
 
 const char* igd_last_error(const igd_ctx* ctx) { return ctx ? ctx->err.c_str() : ""; }
+
+// ---- stage-level test / micro-benchmark hooks (include/igd_debug.h) ----
+int igd_debug_radix_sort(igd_ctx* ctx, uint32_t* d_keys, uint32_t* d_vals, uint64_t n, uint32_t max_bits, int mode,
+                         float* ms) {
+    if (!ctx || n >= 0xFFFFFFFFull || (n && (!d_keys || !d_vals))) return IGD_EINVAL;
+    cudaSetDevice(ctx->device);
+    ctx->sort_mode = mode == 0 ? 0 : 1;
+    for (int b = 0; b < 2; b++) {
+        RET(ensure(ctx, ctx->acc_k[b], n * sizeof(u32)));
+        RET(ensure(ctx, ctx->acc_v[b], n * sizeof(u32)));
+    }
+    RET(ensure(ctx, ctx->hist, 3 * 1024 * sizeof(u32)));
+    RET(ensure(ctx, ctx->base, 4 * 256 * sizeof(u32)));
+    RET(ensure(ctx, ctx->ctr, 64));
+    CK(cudaMemcpyAsync(ctx->acc_k[0].p, d_keys, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->acc_v[0].p, d_vals, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
+    CK(cudaMemsetAsync(ctx->hist.p, 0, 1024 * sizeof(u32), ctx->stream));
+    const int sms = sm_count(ctx);
+    rsort::k_hist4<<<sms * 8, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[0]), n, P_<u32>(ctx->hist));
+    CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    u32 hh[1024];
+    memcpy(hh, ctx->h_hist, sizeof(hh));
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    cudaEventRecord(a, ctx->stream);
+    int cur = 0;
+    int rc = radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n, P_<u32>(ctx->hist), hh, max_bits, &cur);
+    cudaEventRecord(b, ctx->stream);
+    cudaEventSynchronize(b);
+    if (ms) cudaEventElapsedTime(ms, a, b);
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    if (rc != IGD_OK) return rc;
+    CK(cudaMemcpyAsync(d_keys, ctx->acc_k[cur].p, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
+    CK(cudaMemcpyAsync(d_vals, ctx->acc_v[cur].p, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return IGD_OK;
+}
 
 }  // extern "C"

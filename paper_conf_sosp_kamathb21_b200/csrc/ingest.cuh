@@ -6,10 +6,13 @@
 //     order (stable chained-scan compaction with decoupled look-back),
 //   * compacts synchronization events into (entity key, timestamp) records (KeySpace), also in
 //     trace order, so a stable sort by entity gives per-entity timestamp lists,
-//   * builds the 4 x 8-bit digit histograms of both record streams for the radix sorts,
+//   * builds the 4 x 8-bit digit histograms of both record streams for the radix sorts
+//     (warp-uniform digits -- the common case for the high digits -- cost one shared atomic
+//     per warp instead of 32 conflicting ones),
 //   * reduces min / max accessed word (the 32-bit key is injective iff max - min < 2^32).
-// Persistent CTAs (one per SM slot) pull 4096-event tiles from an atomic counter, so tiles are
-// scheduled in order (forward progress for look-back) and histograms are flushed once per CTA.
+// Persistent CTAs pull 2048-event tiles from an atomic counter, so tiles are scheduled in order
+// (forward progress for look-back) and histograms are flushed once per CTA.  Each event is
+// decoded once into 4 registers; the raw 16 bytes are not kept.
 #pragma once
 #include "common.cuh"
 
@@ -17,7 +20,7 @@ namespace ingest {
 
 constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
-constexpr int ITEMS = 16;
+constexpr int ITEMS = 8;
 constexpr int TILE = THREADS * ITEMS;
 
 struct Params {
@@ -39,34 +42,29 @@ struct Params {
     u32 n_tiles;
 };
 
-// Field rules (include/igd.h).  Returns the number of access records (0/1) and sync records
-// (0..2) this event produces, or -1 if invalid.
-struct Decoded {
-    u32 ok, acc, nsync;
-    u32 key;          // access key
-    u32 skey0, skey1; // sync record keys
+// Decoded event: flags bit 0 = access, bits 1..2 = number of sync records, bit 3 = CAS/EXCH,
+// bit 4 = invalid; key = access key; s0, s1 = sync record keys.
+struct Dec {
+    u32 flags, key, s0, s1;
 };
 
-__device__ __forceinline__ Decoded decode(const uint4& e, const Geo& g, const KeySpace& ks) {
-    Decoded d;
-    d.ok = 1;
-    d.acc = 0;
-    d.nsync = 0;
+__device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpace& ks) {
+    Dec d;
+    d.flags = 0;
     d.key = 0;
-    d.skey0 = d.skey1 = 0;
+    d.s0 = d.s1 = 0;
     const u32 tid = ev_tid(e), kind = ev_kind(e), scope = ev_scope(e);
-    const u64 addr = ev_addr(e);
-    const bool hib = (e.z >> 30) != 0;
+    const bool addr0 = (e.x | e.y) == 0;
     const bool tid_ok = tid < g.T;
     u32 b = 0, w = 0, lanebit = 0;
     if (tid_ok) {
         b = g.block(tid);
-        u32 off = tid - b * g.D;
+        const u32 off = tid - b * g.D;
         w = b * g.Wb + (off >> 5);
         lanebit = 1u << (off & 31u);
     }
     const bool inmask = (e.w & lanebit) != 0;
-    bool ok = !hib && tid_ok && kind <= IGD_CG_GRID_SYNC;
+    bool ok = (e.z >> 30) == 0 && tid_ok && kind <= IGD_CG_GRID_SYNC;
     if (ok) {
         switch (kind) {
             case IGD_LD:
@@ -79,56 +77,70 @@ __device__ __forceinline__ Decoded decode(const uint4& e, const Geo& g, const Ke
                 ok = inmask && scope != IGD_SCOPE_NONE;
                 break;
             case IGD_FENCE:
-                ok = addr == 0 && inmask && scope != IGD_SCOPE_NONE;
+                ok = addr0 && inmask && scope != IGD_SCOPE_NONE;
                 break;
             case IGD_SYNCWARP:
             case IGD_CG_TILE_SYNC:
             case IGD_SYNCTHREADS:
             case IGD_CG_BLOCK_SYNC:
-                ok = addr == 0 && scope == IGD_SCOPE_NONE;
+                ok = addr0 && scope == IGD_SCOPE_NONE;
                 break;
             default:  // GRID_SYNC, CG_GRID_SYNC
-                ok = addr == 0 && scope == IGD_SCOPE_NONE && tid == 0;
+                ok = addr0 && scope == IGD_SCOPE_NONE && tid == 0;
                 break;
         }
     }
     if (!ok) {
-        d.ok = 0;
+        d.flags = 16;
         return d;
     }
     if (kind <= IGD_EXCH) {
-        d.acc = 1;
-        d.key = (u32)(addr >> 2);
+        d.key = (e.x >> 2) | (e.y << 30);  // low 32 bits of the word addr >> 2
+        d.flags = 1;
         if (kind == IGD_CAS || kind == IGD_EXCH) {
-            d.nsync = 1;
-            d.skey0 = ks.lock + w;
+            d.flags |= (1u << 1) | 8u;
+            d.s0 = ks.lock + w;
         }
     } else if (kind == IGD_FENCE) {
-        d.skey0 = ks.any + tid;
-        d.nsync = 1;
+        d.s0 = ks.any + tid;
         if (norm_scope(scope) == IGD_SCOPE_DEVICE) {
-            d.skey1 = ks.dev + tid;
-            d.nsync = 2;
+            d.s1 = ks.dev + tid;
+            d.flags = 2u << 1;
+        } else {
+            d.flags = 1u << 1;
         }
     } else if (kind == IGD_SYNCWARP || kind == IGD_CG_TILE_SYNC) {
-        d.skey0 = ks.wb + w;
-        d.nsync = 1;
+        d.s0 = ks.wb + w;
+        d.flags = 1u << 1;
     } else if (kind == IGD_SYNCTHREADS || kind == IGD_CG_BLOCK_SYNC) {
-        d.skey0 = ks.bb + b;
-        d.nsync = 1;
+        d.s0 = ks.bb + b;
+        d.flags = 1u << 1;
     } else {
-        d.skey0 = ks.grid;
-        d.nsync = 1;
+        d.s0 = ks.grid;
+        d.flags = 1u << 1;
     }
     return d;
 }
 
-__global__ void __launch_bounds__(THREADS) k_ingest(Params P) {
+// Histogram update of one 8-bit digit for the lanes in `active`: one shared atomic when all
+// active lanes agree on the digit, else one per lane.
+__device__ __forceinline__ void hist_add(u32* h, u32 digit, bool on, u32 lane) {
+    const u32 active = __ballot_sync(IGD_FULL, on);
+    if (!active) return;
+    const u32 src = __ffs(active) - 1;
+    const u32 first = __shfl_sync(IGD_FULL, digit, src);
+    if (__all_sync(IGD_FULL, !on || digit == first)) {
+        if (lane == src) atomicAdd(&h[first], __popc(active));
+    } else if (on) {
+        atomicAdd(&h[digit], 1u);
+    }
+}
+
+__global__ void __launch_bounds__(THREADS, 3) k_ingest(Params P) {
     __shared__ u32 s_hacc[4][256];
     __shared__ u32 s_hsync[4][256];
     __shared__ u32 s_wtot[ITEMS][WARPS];  // packed (acc | nsync << 16) per (item, warp)
-    __shared__ u32 s_woff_acc[ITEMS][WARPS];
-    __shared__ u32 s_woff_sync[ITEMS][WARPS];
+    __shared__ u32 s_woff[ITEMS][WARPS];  // packed exclusive offsets (acc | sync << 16)
     __shared__ u64 s_base_acc, s_base_sync;
     __shared__ u32 s_tile;
 
@@ -138,7 +150,7 @@ __global__ void __launch_bounds__(THREADS) k_ingest(Params P) {
         (&s_hsync[0][0])[i] = 0;
     }
     u64 wmin = ~0ull, wmax = 0, bad = ~0ull;
-    u64 cnt_acc = 0, cnt_sync = 0, cnt_lock = 0;
+    u32 cnt_acc = 0, cnt_sync = 0, cnt_lock = 0;
     const Geo g = P.g;
     const KeySpace ks = P.ks;
 
@@ -150,52 +162,51 @@ __global__ void __launch_bounds__(THREADS) k_ingest(Params P) {
         if (tile >= P.n_tiles) break;
         const u64 base = (u64)tile * TILE;
 
-        uint4 e[ITEMS];
+        Dec dv[ITEMS];
+        {
+            uint4 e[ITEMS];
 #pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            u64 i = base + (u64)j * THREADS + tid;
-            e[j] = (i < P.n) ? ld_event_stream(P.ev, i) : make_uint4(0, 0, 0, 0);
+            for (int j = 0; j < ITEMS; j++) {
+                const u64 i = base + (u64)j * THREADS + tid;
+                e[j] = (i < P.n) ? ld_event_stream(P.ev, i) : make_uint4(0, 0, 0, 0);
+            }
+#pragma unroll
+            for (int j = 0; j < ITEMS; j++) {
+                const u64 i = base + (u64)j * THREADS + tid;
+                if (i < P.n) {
+                    dv[j] = decode(e[j], g, ks);
+                    if (dv[j].flags & 1u) {
+                        const u64 word = ev_addr(e[j]) >> 2;
+                        wmin = min(wmin, word);
+                        wmax = max(wmax, word);
+                    }
+                } else {
+                    dv[j].flags = 0;
+                    dv[j].key = dv[j].s0 = dv[j].s1 = 0;
+                }
+            }
         }
-        // counts per item, warp-scanned
         u32 excl[ITEMS];
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
-            u64 i = base + (u64)j * THREADS + tid;
-            u32 v = 0;
-            if (i < P.n) {
-                Decoded d = decode(e[j], g, ks);
-                if (!d.ok) {
-                    bad = min(bad, i);
-                } else {
-                    v = d.acc | (d.nsync << 16);
-                    if (d.acc) {
-                        u64 word = ev_addr(e[j]) >> 2;
-                        wmin = min(wmin, word);
-                        wmax = max(wmax, word);
-                        atomicAdd(&s_hacc[0][d.key & 255u], 1u);
-                        atomicAdd(&s_hacc[1][(d.key >> 8) & 255u], 1u);
-                        atomicAdd(&s_hacc[2][(d.key >> 16) & 255u], 1u);
-                        atomicAdd(&s_hacc[3][d.key >> 24], 1u);
-                    }
-                    if (d.nsync) {
-                        atomicAdd(&s_hsync[0][d.skey0 & 255u], 1u);
-                        atomicAdd(&s_hsync[1][(d.skey0 >> 8) & 255u], 1u);
-                        atomicAdd(&s_hsync[2][(d.skey0 >> 16) & 255u], 1u);
-                        atomicAdd(&s_hsync[3][d.skey0 >> 24], 1u);
-                    }
-                    if (d.nsync == 2) {
-                        atomicAdd(&s_hsync[0][d.skey1 & 255u], 1u);
-                        atomicAdd(&s_hsync[1][(d.skey1 >> 8) & 255u], 1u);
-                        atomicAdd(&s_hsync[2][(d.skey1 >> 16) & 255u], 1u);
-                        atomicAdd(&s_hsync[3][d.skey1 >> 24], 1u);
-                    }
-                    cnt_lock += (d.acc && d.nsync) ? 1 : 0;
-                }
+            const u32 f = dv[j].flags;
+            if (f & 16u) bad = min(bad, base + (u64)j * THREADS + tid);
+            const bool acc = (f & 1u) != 0;
+            const u32 ns = (f >> 1) & 3u;
+#pragma unroll
+            for (int p = 0; p < 4; p++) hist_add(s_hacc[p], (dv[j].key >> (8 * p)) & 255u, acc, lane);
+            if (__any_sync(IGD_FULL, ns != 0)) {
+#pragma unroll
+                for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s0 >> (8 * p)) & 255u, ns != 0, lane);
+#pragma unroll
+                for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s1 >> (8 * p)) & 255u, ns == 2, lane);
             }
+            cnt_lock += (f >> 3) & 1u;
+            const u32 v = (acc ? 1u : 0u) | (ns << 16);
             u32 inc = v;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
-                u32 t = __shfl_up_sync(IGD_FULL, inc, o);
+                const u32 t = __shfl_up_sync(IGD_FULL, inc, o);
                 if (lane >= (u32)o) inc += t;
             }
             excl[j] = inc - v;
@@ -204,23 +215,20 @@ __global__ void __launch_bounds__(THREADS) k_ingest(Params P) {
         __syncthreads();
         // scan the ITEMS x WARPS totals in (item, warp) order; warp 0 does it
         if (warp == 0) {
-            constexpr int PER = ITEMS * WARPS / 32;  // 4
+            constexpr int PER = ITEMS * WARPS / 32;  // 2
+            u32 vv[PER];
             u32 la = 0, ls = 0;
-            u32 va[PER], vs[PER];
 #pragma unroll
             for (int q = 0; q < PER; q++) {
-                int idx = lane * PER + q;
-                u32 t = (&s_wtot[0][0])[idx];
-                va[q] = t & 0xFFFFu;
-                vs[q] = t >> 16;
-                la += va[q];
-                ls += vs[q];
+                vv[q] = (&s_wtot[0][0])[lane * PER + q];
+                la += vv[q] & 0xFFFFu;
+                ls += vv[q] >> 16;
             }
             u32 ia = la, is = ls;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
-                u32 ta = __shfl_up_sync(IGD_FULL, ia, o);
-                u32 ts = __shfl_up_sync(IGD_FULL, is, o);
+                const u32 ta = __shfl_up_sync(IGD_FULL, ia, o);
+                const u32 ts = __shfl_up_sync(IGD_FULL, is, o);
                 if (lane >= (u32)o) {
                     ia += ta;
                     is += ts;
@@ -229,23 +237,15 @@ __global__ void __launch_bounds__(THREADS) k_ingest(Params P) {
             u32 ea = ia - la, es = is - ls;
 #pragma unroll
             for (int q = 0; q < PER; q++) {
-                int idx = lane * PER + q;
-                (&s_woff_acc[0][0])[idx] = ea;
-                (&s_woff_sync[0][0])[idx] = es;
-                ea += va[q];
-                es += vs[q];
+                (&s_woff[0][0])[lane * PER + q] = ea | (es << 16);
+                ea += vv[q] & 0xFFFFu;
+                es += vv[q] >> 16;
             }
             const u32 tot_a = __shfl_sync(IGD_FULL, ia, 31);
             const u32 tot_s = __shfl_sync(IGD_FULL, is, 31);
-            // publish aggregates, look back
             if (lane == 0) {
-                if (tile == 0) {
-                    st_relaxed(&P.st_acc[0], ST_INC | tot_a);
-                    st_relaxed(&P.st_sync[0], ST_INC | tot_s);
-                } else {
-                    st_relaxed(&P.st_acc[tile], ST_AGG | tot_a);
-                    st_relaxed(&P.st_sync[tile], ST_AGG | tot_s);
-                }
+                st_relaxed(&P.st_acc[tile], (tile == 0 ? ST_INC : ST_AGG) | tot_a);
+                st_relaxed(&P.st_sync[tile], (tile == 0 ? ST_INC : ST_AGG) | tot_s);
             }
             u64 ba = 0, bs = 0;
             if (tile > 0) {
@@ -265,55 +265,55 @@ __global__ void __launch_bounds__(THREADS) k_ingest(Params P) {
         const u64 ba = s_base_acc, bs = s_base_sync;
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
-            u64 i = base + (u64)j * THREADS + tid;
-            if (i >= P.n) continue;
-            Decoded d = decode(e[j], g, ks);
-            if (!d.ok) continue;
-            u32 ex = excl[j];
-            if (d.acc) {
-                u64 pos = ba + s_woff_acc[j][warp] + (ex & 0xFFFFu);
-                P.acc_key[pos] = d.key;
-                P.acc_val[pos] = (u32)i;
+            const u32 f = dv[j].flags;
+            const u32 wo = s_woff[j][warp];
+            const u32 ex = excl[j];
+            if (f & 1u) {
+                const u64 pos = ba + (wo & 0xFFFFu) + (ex & 0xFFFFu);
+                P.acc_key[pos] = dv[j].key;
+                P.acc_val[pos] = (u32)(base + (u64)j * THREADS + tid);
+                cnt_acc++;
             }
-            if (d.nsync) {
-                u64 pos = bs + s_woff_sync[j][warp] + (ex >> 16);
-                if (pos + d.nsync <= P.sync_cap) {
-                    P.sync_key[pos] = d.skey0;
-                    P.sync_val[pos] = (u32)i;
+            const u32 ns = (f >> 1) & 3u;
+            if (ns) {
+                const u64 pos = bs + (wo >> 16) + (ex >> 16);
+                const u32 ts = (u32)(base + (u64)j * THREADS + tid);
+                if (pos + ns <= P.sync_cap) {
+                    P.sync_key[pos] = dv[j].s0;
+                    P.sync_val[pos] = ts;
+                    if (ns == 2) {
+                        P.sync_key[pos + 1] = dv[j].s1;
+                        P.sync_val[pos + 1] = ts;
+                    }
                 }
-                if (d.nsync == 2 && pos + 2 <= P.sync_cap) {
-                    P.sync_key[pos + 1] = d.skey1;
-                    P.sync_val[pos + 1] = (u32)i;
-                }
-                cnt_sync += d.nsync;
+                cnt_sync += ns;
             }
-            cnt_acc += d.acc;
         }
     }
     // flush per-CTA results
     for (int i = tid; i < 4 * 256; i += THREADS) {
-        u32 a = (&s_hacc[0][0])[i];
+        const u32 a = (&s_hacc[0][0])[i];
         if (a) atomicAdd(&P.hist_acc[i], a);
-        u32 s = (&s_hsync[0][0])[i];
+        const u32 s = (&s_hsync[0][0])[i];
         if (s) atomicAdd(&P.hist_sync[i], s);
     }
-    // reduce min/max/bad/counts
+    u64 ca = cnt_acc, cs = cnt_sync, cl = cnt_lock;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         wmin = min(wmin, __shfl_xor_sync(IGD_FULL, wmin, o));
         wmax = max(wmax, __shfl_xor_sync(IGD_FULL, wmax, o));
         bad = min(bad, __shfl_xor_sync(IGD_FULL, bad, o));
-        cnt_acc += __shfl_xor_sync(IGD_FULL, cnt_acc, o);
-        cnt_sync += __shfl_xor_sync(IGD_FULL, cnt_sync, o);
-        cnt_lock += __shfl_xor_sync(IGD_FULL, cnt_lock, o);
+        ca += __shfl_xor_sync(IGD_FULL, ca, o);
+        cs += __shfl_xor_sync(IGD_FULL, cs, o);
+        cl += __shfl_xor_sync(IGD_FULL, cl, o);
     }
     if (lane == 0) {
         if (wmin != ~0ull) atomicMin((unsigned long long*)&P.stats[0], (unsigned long long)wmin);
-        if (cnt_acc) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
+        if (ca) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
         if (bad != ~0ull) atomicMin((unsigned long long*)&P.stats[2], (unsigned long long)bad);
-        if (cnt_acc) atomicAdd((unsigned long long*)&P.stats[3], (unsigned long long)cnt_acc);
-        if (cnt_sync) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cnt_sync);
-        if (cnt_lock) atomicAdd((unsigned long long*)&P.stats[5], (unsigned long long)cnt_lock);
+        if (ca) atomicAdd((unsigned long long*)&P.stats[3], (unsigned long long)ca);
+        if (cs) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cs);
+        if (cl) atomicAdd((unsigned long long*)&P.stats[5], (unsigned long long)cl);
     }
 }
 

@@ -6,6 +6,12 @@
 // look-back) + (earlier warps of the tile) + (earlier items / lanes of the warp), i.e. its
 // input order.  Sorting accesses that arrive in trace order therefore yields (word, time)
 // order, the order the per-word shadow replay needs (SURVEY 8(c) C.3 "equivalent formulation").
+//
+// Per tile: keys are loaded (coalesced, warp-striped), ranked with a warp multisplit (eight
+// ballots give the mask of lanes holding the same digit -- no MATCH/MIO traffic), the tile's
+// digit counts are published and looked back, keys are reordered through shared memory and
+// written out in digit runs; values follow with the same ranks through the same buffer, so a
+// thread never holds keys and values at once (register budget -> 3-4 CTAs per SM).
 #pragma once
 #include "common.cuh"
 
@@ -65,12 +71,30 @@ struct PassParams {
     u32* tile_ctr;          // zeroed
 };
 
-__global__ void __launch_bounds__(THREADS) k_onesweep(PassParams P) {
+// Mask of the lanes (within vmask) whose 8-bit digit equals this lane's.
+template <int MODE>
+__device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
+    if (MODE == 0) {
+        return __match_any_sync(IGD_FULL, d) & vmask;
+    } else {
+        u32 peers = vmask;
+#pragma unroll
+        for (int b = 0; b < 8; b++) {
+            const u32 bit = (d >> b) & 1u;
+            const u32 bal = __ballot_sync(IGD_FULL, bit);
+            peers &= bit ? bal : ~bal;
+        }
+        return peers;
+    }
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
     __shared__ u32 s_whist[WARPS][RADIX];
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
-    __shared__ u32 s_keys[TILE];
-    __shared__ u32 s_vals[TILE];
+    __shared__ u32 s_buf[TILE];
+    __shared__ uint8_t s_dig[TILE];
     __shared__ u32 s_tile;
     __shared__ u32 s_wsum[WARPS];
 
@@ -79,45 +103,38 @@ __global__ void __launch_bounds__(THREADS) k_onesweep(PassParams P) {
     for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_whist[0][0])[i] = 0;
     __syncthreads();
     const u32 tile = s_tile;
-    const u64 base = (u64)tile * TILE;
-    const u64 wbase = base + (u64)warp * 32 * ITEMS;
+    const u32 base = tile * TILE;  // n <= 2^32 - 2^13 (checked by the host)
+    const u32 wbase = base + warp * 32 * ITEMS;
+    const u32 shift = P.shift;
+    const bool full = (u64)base + TILE <= P.n;
 
-    u32 key[ITEMS], val[ITEMS], rank[ITEMS];
+    u32 key[ITEMS];
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
-        u64 i = wbase + (u64)j * 32 + lane;
-        if (i < P.n) {
-            key[j] = __ldcs(P.kin + i);
-            val[j] = __ldcs(P.vin + i);
-        } else {
-            key[j] = 0;
-            val[j] = 0;
-        }
+        const u32 i = wbase + j * 32 + lane;
+        key[j] = (full || i < P.n) ? __ldcs(P.kin + i) : 0u;
     }
+    u32 rank[ITEMS];
     const u32 lt = lanemask_lt();
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
-        u64 i = wbase + (u64)j * 32 + lane;
-        bool valid = i < P.n;
-        u32 vmask = __ballot_sync(IGD_FULL, valid);
-        u32 r = 0;
-        if (valid) {
-            u32 d = (key[j] >> P.shift) & 255u;
-            u32 peers = __match_any_sync(vmask, d);
-            u32 leader = __ffs(peers) - 1;
-            u32 old = 0;
-            if (lane == leader) {
-                old = s_whist[warp][d];
-                s_whist[warp][d] = old + __popc(peers);
-            }
-            old = __shfl_sync(peers, old, leader);
-            r = old + __popc(peers & lt);
+        const bool valid = full || wbase + j * 32 + lane < P.n;
+        const u32 vmask = full ? IGD_FULL : __ballot_sync(IGD_FULL, valid);
+        const u32 d = (key[j] >> shift) & 255u;
+        // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set
+        const u32 peers = peers_of<MODE>(valid ? d : (0x100u | lane), vmask);
+        const u32 leader = __ffs(peers) - 1;
+        u32 old = 0;
+        if (lane == leader && valid) {
+            old = s_whist[warp][d];
+            s_whist[warp][d] = old + __popc(peers);
         }
-        rank[j] = r;
+        old = __shfl_sync(IGD_FULL, old, leader & 31u);
+        rank[j] = old + __popc(peers & lt);
         __syncwarp();
     }
     __syncthreads();
-    // per digit: exclusive over warps, tile count
+    // per digit: exclusive over warps, tile count, publish
     u32 cnt;
     {
         const u32 d = t;  // THREADS == RADIX
@@ -129,12 +146,7 @@ __global__ void __launch_bounds__(THREADS) k_onesweep(PassParams P) {
             sum += c;
         }
         cnt = sum;
-        u64* st = P.status + (u64)tile * RADIX + d;
-        if (tile == 0) {
-            st_relaxed(st, ST_INC | cnt);
-        } else {
-            st_relaxed(st, ST_AGG | cnt);
-        }
+        st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
     }
     // block exclusive scan of cnt over digits
     {
@@ -172,26 +184,44 @@ __global__ void __launch_bounds__(THREADS) k_onesweep(PassParams P) {
         s_gbase[d] = P.digit_base[d] + (u32)excl;
     }
     __syncthreads();
-    // local reorder through shared memory
+    // keys: reorder through shared memory (rank[] becomes the tile position), then write
+    // digit runs; the digit of every tile position is kept for the value pass
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
-        u64 i = wbase + (u64)j * 32 + lane;
-        if (i < P.n) {
-            u32 d = (key[j] >> P.shift) & 255u;
-            u32 pos = s_tile_excl[d] + s_whist[warp][d] + rank[j];
-            s_keys[pos] = key[j];
-            s_vals[pos] = val[j];
-        }
+        const u32 d = (key[j] >> shift) & 255u;
+        rank[j] += s_tile_excl[d] + s_whist[warp][d];
+        if (full || wbase + j * 32 + lane < P.n) s_buf[rank[j]] = key[j];
     }
     __syncthreads();
-    const u32 tile_n = (u32)min((u64)TILE, (u64)P.n - base);
-#pragma unroll 4
-    for (u32 i = t; i < tile_n; i += THREADS) {
-        u32 k = s_keys[i];
-        u32 d = (k >> P.shift) & 255u;
-        u32 out = s_gbase[d] + (i - s_tile_excl[d]);
-        __stcs(P.kout + out, k);
-        __stcs(P.vout + out, s_vals[i]);
+    const u32 tile_n = full ? (u32)TILE : P.n - base;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const u32 i = t + k * THREADS;
+        if (i < tile_n) {
+            const u32 kk = s_buf[i];
+            const u32 d = (kk >> shift) & 255u;
+            s_dig[i] = (uint8_t)d;
+            __stcs(P.kout + s_gbase[d] + (i - s_tile_excl[d]), kk);
+        }
+    }
+    // values: same permutation through the same buffer
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++) {
+        const u32 i = wbase + j * 32 + lane;
+        key[j] = (full || i < P.n) ? __ldcs(P.vin + i) : 0u;  // key[] now holds values
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++)
+        if (full || wbase + j * 32 + lane < P.n) s_buf[rank[j]] = key[j];
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const u32 i = t + k * THREADS;
+        if (i < tile_n) {
+            const u32 d = s_dig[i];
+            __stcs(P.vout + s_gbase[d] + (i - s_tile_excl[d]), s_buf[i]);
+        }
     }
 }
 

@@ -159,8 +159,13 @@ class Detector:
             except Exception:  # noqa: BLE001 -- reported to the library as NULL (IGD_ENOMEM)
                 return None
 
+        cdelete = torch.cuda.caching_allocator_delete  # bound now: survives interpreter teardown
+
         def _free(p, stream, user):
-            torch.cuda.caching_allocator_delete(p)
+            try:
+                cdelete(p)
+            except Exception:  # noqa: BLE001 -- process exit: the driver reclaims the memory
+                pass
 
         self._afn = ALLOC_FN(_alloc)
         self._ffn = FREE_FN(_free)
