@@ -9,11 +9,18 @@
 //   Atomic/Scope = any atomic before j / scope of the last one       (reading A6)
 //   DevShared / BlkShared = OR of adjacent-pair predicates up to j   (A5)
 //   Locks      = held-lock Bloom of LA at LA's time                  (A7)
-// The scans run per tile (256 threads x 4 accesses) and across tiles with decoupled look-back;
-// a tile that contains a segment head publishes its inclusive state immediately, so only
-// tiles inside one long (hot-word) segment ever wait.  The synchronization-counter comparisons
-// of Table 2 become interval queries on the a2 CSR lists ("did md's thread fence in
-// (md.idx, i)?", reading A1), lock sets come from the a3 change points.
+//
+// Two phases per 1024-access tile (256 threads x 4 consecutive accesses):
+//  1. streaming: coalesced key/index loads, one 16-byte event gather per access, thread-local
+//     + warp-shuffle + block scans of the packed shadow state, decoupled look-back across tiles
+//     (a tile containing a segment head publishes its inclusive state at once, so only tiles
+//     inside one long hot-word segment wait), then the checks that need no synchronization
+//     history: P1, P2, P3, P6 and P4's lockstep clause.
+//  2. the accesses still undecided are queued in shared memory and processed densely by the
+//     whole CTA: P4 (syncwarp), P5, R1..R5.  The synchronization-counter comparisons of Table 2
+//     become interval queries on the a2 lists ("did md's thread fence in (md.idx, i)?", reading
+//     A1), answered by a per-list descriptor {lo, hi, first, last} and interpolation-guided
+//     32-byte probes (two dependent loads for the periodic lists of real kernels).
 #pragma once
 #include "common.cuh"
 #include "sync.cuh"
@@ -21,10 +28,11 @@
 namespace check {
 
 constexpr int THREADS = 256;
+constexpr int WARPS = THREADS / 32;
 constexpr int ITEMS = 4;
 constexpr int TILE = THREADS * ITEMS;
 
-// Packed scan state (39 bits): [31:0] lastW position (NONE = 0xFFFFFFFF), [33:32] scope of the
+// Packed scan state (37 bits): [31:0] lastW position (NONE = 0xFFFFFFFF), [33:32] scope of the
 // last atomic (0 none, 1 block, 2 device), [34] devShared, [35] blkShared, [36] segment head seen.
 __device__ __forceinline__ u64 st_make(u32 lastW, u32 as, u32 dev, u32 blk, u32 head) {
     return (u64)lastW | ((u64)as << 32) | ((u64)dev << 34) | ((u64)blk << 35) | ((u64)head << 36);
@@ -39,20 +47,90 @@ __device__ __forceinline__ u32 st_head(u64 s) { return (u32)(s >> 36) & 1u; }
 // a then b (b later): segmented "last-of" / OR combine
 __device__ __forceinline__ u64 combine(u64 a, u64 b) {
     if (st_head(b)) return b;
-    u32 lw = st_lastW(b) != IGD_NONE32 ? st_lastW(b) : st_lastW(a);
-    u32 as = st_as(b) ? st_as(b) : st_as(a);
+    const u32 lw = st_lastW(b) != IGD_NONE32 ? st_lastW(b) : st_lastW(a);
+    const u32 as = st_as(b) ? st_as(b) : st_as(a);
     return st_make(lw, as, st_dev(a) | st_dev(b), st_blk(a) | st_blk(b), st_head(a));
+}
+
+// List descriptors: desc[e] = {lo, hi, ts[lo], ts[hi-1]} of entity e's timestamp list.
+__global__ void k_list_desc(const u32* __restrict__ off, const u32* __restrict__ ts, u32 E, uint4* __restrict__ desc) {
+    for (u64 e = (u64)blockIdx.x * blockDim.x + threadIdx.x; e < E; e += (u64)gridDim.x * blockDim.x) {
+        const u32 lo = off[e], hi = off[e + 1];
+        desc[e] = make_uint4(lo, hi, lo < hi ? ts[lo] : 0u, lo < hi ? ts[hi - 1] : 0u);
+    }
+}
+
+// Optional event counters (igd_debug_check_stats): a debug aid, off unless enabled.
+__device__ int g_chk_stats_on;
+__device__ unsigned long long g_chk_stats[16];
+#define CSTAT(k)                                                \
+    do {                                                        \
+        if (g_chk_stats_on) atomicAdd(&g_chk_stats[k], 1ull);   \
+    } while (0)
+
+// Is there an element x of entity e's list with a < x < b ?
+__device__ __noinline__ bool q_between(const uint4* __restrict__ desc, const u32* __restrict__ ts, u32 e, u32 a,
+                                       u32 b) {
+    const uint4 d = __ldg(desc + e);
+    CSTAT(7);
+    if (d.x == d.y || d.w <= a) {  // empty, or every element <= a
+        CSTAT(8);
+        return false;
+    }
+    if (d.z > a) {  // the first element is the first one > a
+        CSTAT(8);
+        return d.z < b;
+    }
+    // first <= a < last: the successor of a lies in [lo, hi]; guess its position by
+    // interpolation and probe aligned 32-byte sectors (8 timestamps) around the guess
+    u32 lo = d.x + 1, hi = d.y - 1;
+    // single-precision guess (a hint only: it is clamped and verified by the probes)
+    u32 g = d.x + 1 + (u32)(__fdividef((float)(a - d.z), (float)(d.w - d.z)) * (float)(d.y - 1 - d.x));
+    g = min(max(g, lo), hi);
+#pragma unroll 1
+    for (int probe = 0; probe < 3 && lo < hi; probe++) {
+        g = min(max(g, lo), hi);  // the probe always covers a position of [lo, hi]
+        const u32 g0 = g & ~7u;
+        const uint4* p = reinterpret_cast<const uint4*>(ts + g0);
+        const uint4 v0 = __ldg(p), v1 = __ldg(p + 1);
+        const u32 s0 = max(g0, lo), s1 = min(g0 + 8, hi + 1);  // probed positions inside [lo, hi]
+        const u32 lem = (u32)(v0.x <= a) | ((u32)(v0.y <= a) << 1) | ((u32)(v0.z <= a) << 2) |
+                        ((u32)(v0.w <= a) << 3) | ((u32)(v1.x <= a) << 4) | ((u32)(v1.y <= a) << 5) |
+                        ((u32)(v1.z <= a) << 6) | ((u32)(v1.w <= a) << 7);
+        const u32 rng = ((1u << (s1 - g0)) - 1u) & ~((1u << (s0 - g0)) - 1u);
+        const u32 le = __popc(lem & rng);
+        if (le == s1 - s0) {          // all <= a: successor after the probe
+            lo = s1;
+            g = s1;
+        } else if (le == 0) {         // all > a: successor is s0 or before
+            hi = s0;
+            g = s0 > 8 ? s0 - 8 : 0;
+        } else {                      // successor inside the probe (L1-resident)
+            CSTAT(9);
+            return __ldg(ts + s0 + le) < b;
+        }
+    }
+    CSTAT(10);
+    while (lo < hi) {
+        const u32 mid = (lo + hi) >> 1;
+        if (__ldg(ts + mid) <= a) lo = mid + 1;
+        else hi = mid;
+    }
+    return __ldg(ts + lo) < b;
 }
 
 struct Params {
     const u32* key;  // sorted word keys
-    const u32* val;  // sorted trace indices
+    const u64* val;  // sorted (trace index | tk << 32)
     u32 n;           // number of accesses
     const igd_event* ev;
     Geo g;
     KeySpace ks;
-    const u32* off;  // sync CSR offsets
-    const u32* sts;  // sync timestamps
+    const uint4* desc;  // per-entity list descriptors
+    const u32* gtab;    // grid-sync bucket table: first grid-list index at or after bucket start
+    u32 gshift;         // bucket = t >> gshift
+    u32 glo, ghi;       // the grid list inside sts
+    const u32* sts;     // sync timestamps (sorted by entity, then time)
     syncx::LockView lv;
     u64* status;     // [n_tiles] zeroed
     u32* tile_ctr;   // zeroed
@@ -62,216 +140,317 @@ struct Params {
     u64 first_event; // global index offset (multi-rank)
 };
 
-__device__ __forceinline__ bool sync_between(const Params& P, u32 key, u32 a, u32 b) {
-    const u32 lo = __ldg(P.off + key), hi = __ldg(P.off + key + 1);
-    if (lo == hi) return false;
-    return between(P.sts, lo, hi, a, b);
+// Grid-sync bucket table: gtab[b] = index of the first grid sync with timestamp >= b << shift.
+// The grid list is global and short, so "a grid sync in (a, b)?" -- the most frequent query of
+// P5 / R2..R4 -- becomes one L2-resident table load plus a step or two along the list.
+__global__ void k_grid_table(const u32* __restrict__ ts, u32 glo, u32 ghi, u32 shift, u32 nb, u32* __restrict__ gtab) {
+    for (u64 b = (u64)blockIdx.x * blockDim.x + threadIdx.x; b < nb; b += (u64)gridDim.x * blockDim.x) {
+        const u64 start = b << shift;
+        u32 lo = glo, hi = ghi;
+        while (lo < hi) {
+            const u32 mid = (lo + hi) >> 1;
+            if ((u64)ts[mid] < start) lo = mid + 1;
+            else hi = mid;
+        }
+        gtab[b] = lo;
+    }
 }
 
-__global__ void __launch_bounds__(THREADS) k_check(Params P) {
+template <class PP>
+__device__ __forceinline__ bool q_grid(const PP& P, u32 a, u32 b) {
+    if (P.glo == P.ghi) return false;
+    u32 x = __ldg(P.gtab + ((a + 1) >> P.gshift));  // first grid sync at or after a's bucket
+#pragma unroll 1
+    for (int step = 0; x < P.ghi; step++, x++) {
+        const u32 v = __ldg(P.sts + x);
+        if (v > a) return v < b;
+        if (step == 8) return q_between(P.desc, P.sts, P.ks.grid, a, b);  // dense grid syncs
+    }
+    return false;
+}
+
+// queue entry flags
+#define QF_SAME_W 1u
+#define QF_SAME_B 2u
+#define QF_DEV 4u
+#define QF_BLK 8u
+#define QF_R1 16u
+
+__global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
     __shared__ u32 s_tile;
-    __shared__ u64 s_wagg[THREADS / 32];
+    __shared__ u64 s_wagg[WARPS];
     __shared__ u64 s_prefix;
+    __shared__ u32 s_ready;
+    __shared__ u32 s_qn;
+    // queue of undecided accesses (SoA)
+    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_la[TILE], q_lt[TILE];
+
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
-    if (t == 0) s_tile = atomicAdd(P.tile_ctr, 1u);
+    if (t == 0) {
+        s_tile = atomicAdd(P.tile_ctr, 1u);
+        s_qn = 0;
+        s_ready = 0;
+    }
     __syncthreads();
     const u32 tile = s_tile;
-    const u64 first = (u64)tile * TILE + (u64)t * ITEMS;
+    const u32 first = tile * TILE + t * ITEMS;  // n <= 2^32 - 2^13
     const Geo g = P.g;
 
-    u32 K[ITEMS], V[ITEMS];
+    // K: word key, V: trace index, Z: the event's tk word (tid | kind | scope), carried by the sort
+    u32 K[ITEMS], V[ITEMS], Z[ITEMS];
     if (first + ITEMS <= P.n) {
-        uint4 k4 = __ldcs(reinterpret_cast<const uint4*>(P.key + first));
-        uint4 v4 = __ldcs(reinterpret_cast<const uint4*>(P.val + first));
+        const uint4 k4 = __ldcs(reinterpret_cast<const uint4*>(P.key + first));
+        const uint4 v01 = __ldcs(reinterpret_cast<const uint4*>(P.val + first));
+        const uint4 v23 = __ldcs(reinterpret_cast<const uint4*>(P.val + first + 2));
         K[0] = k4.x; K[1] = k4.y; K[2] = k4.z; K[3] = k4.w;
-        V[0] = v4.x; V[1] = v4.y; V[2] = v4.z; V[3] = v4.w;
+        V[0] = v01.x; Z[0] = v01.y; V[1] = v01.z; Z[1] = v01.w;
+        V[2] = v23.x; Z[2] = v23.y; V[3] = v23.z; Z[3] = v23.w;
     } else {
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
+            const u64 v = (first + j < P.n) ? P.val[first + j] : 0ull;
             K[j] = (first + j < P.n) ? P.key[first + j] : 0;
-            V[j] = (first + j < P.n) ? P.val[first + j] : 0;
+            V[j] = (u32)v;
+            Z[j] = (u32)(v >> 32);
         }
     }
-    uint4 E[ITEMS];
-#pragma unroll
-    for (int j = 0; j < ITEMS; j++) E[j] = (first + j < P.n) ? ld_event(P.ev, V[j]) : make_uint4(0, 0, 0, 0);
 
-    // previous element (first - 1): from the neighbour lane, lane 0 reads it
+    // previous element (first - 1): from the neighbour lane; lane 0 reads it
     u32 pK = __shfl_up_sync(IGD_FULL, K[ITEMS - 1], 1);
     u32 pV = __shfl_up_sync(IGD_FULL, V[ITEMS - 1], 1);
-    u32 pZ = __shfl_up_sync(IGD_FULL, E[ITEMS - 1].z, 1);
-    bool has_prev = first > 0;
-    if (lane == 0 && has_prev && first - 1 < P.n) {
-        pK = P.key[first - 1];
-        pV = P.val[first - 1];
-        pZ = ld_event(P.ev, pV).z;
+    u32 pZ = __shfl_up_sync(IGD_FULL, Z[ITEMS - 1], 1);
+    if (lane == 0 && first > 0 && first - 1 < P.n) {
+        pK = __ldg(P.key + first - 1);
+        const u64 v = __ldg(reinterpret_cast<const unsigned long long*>(P.val) + first - 1);
+        pV = (u32)v;
+        pZ = (u32)(v >> 32);
     }
 
-    // per-element scan contributions
+    // per-access scan contributions
     u64 contrib[ITEMS];
-    u32 prevTid = pZ & 0xFFFFFFu;
-    u32 prevKey = pK;
-    bool prevValid = has_prev;
+    {
+        u32 prevTid = pZ & 0xFFFFFFu, prevKey = pK;
+        bool prevValid = first > 0;
 #pragma unroll
-    for (int j = 0; j < ITEMS; j++) {
-        const bool inr = first + j < P.n;
-        const u32 c = ev_tid(E[j]);
-        const u32 kind = ev_kind(E[j]);
-        const bool head = !prevValid || prevKey != K[j];
-        u32 dev = 0, blk = 0;
-        if (!head) {
-            u32 bp = g.block(prevTid), bc = g.block(c);
-            if (bp != bc) dev = 1;
-            else if (g.warp(prevTid) != g.warp(c)) blk = 1;
+        for (int j = 0; j < ITEMS; j++) {
+            const bool inr = first + j < P.n;
+            const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
+            const bool head = !prevValid || prevKey != K[j];
+            u32 dev = 0, blk = 0;
+            if (!head) {
+                const u32 bp = g.block(prevTid), bc = g.block(c);
+                if (bp != bc) dev = 1;
+                else if (g.warp(prevTid) != g.warp(c)) blk = 1;
+            }
+            const u32 lw = kind != IGD_LD ? first + j : IGD_NONE32;
+            const u32 as = (kind >= IGD_ATOM && kind <= IGD_EXCH) ? norm_scope((Z[j] >> 28) & 3u) : 0u;
+            contrib[j] = inr ? st_make(lw, as, dev, blk, head ? 1u : 0u) : ST_IDENTITY;
+            prevTid = c;
+            prevKey = K[j];
+            prevValid = true;
         }
-        u32 lw = (inr && kind != IGD_LD) ? (u32)(first + j) : IGD_NONE32;
-        u32 as = (inr && kind >= IGD_ATOM && kind <= IGD_EXCH) ? norm_scope(ev_scope(E[j])) : 0u;
-        contrib[j] = inr ? st_make(lw, as, dev, blk, head ? 1u : 0u) : st_make(IGD_NONE32, 0, 0, 0, 0);
-        prevTid = c;
-        prevKey = K[j];
-        prevValid = true;
     }
-    // thread aggregate
     u64 agg = contrib[0];
 #pragma unroll
     for (int j = 1; j < ITEMS; j++) agg = combine(agg, contrib[j]);
-    // warp inclusive scan
     u64 inc = agg;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        u64 x = __shfl_up_sync(IGD_FULL, inc, o);
+        const u64 x = __shfl_up_sync(IGD_FULL, inc, o);
         if (lane >= (u32)o) inc = combine(x, inc);
     }
     if (lane == 31) s_wagg[warp] = inc;
     u64 wexcl = __shfl_up_sync(IGD_FULL, inc, 1);
     if (lane == 0) wexcl = ST_IDENTITY;
     __syncthreads();
-    if (warp == 0) {
-        // scan warp aggregates (8) -> tile aggregate, look back
+    // Tile-relative state.  Only accesses of the segment that continues from the previous tile
+    // (no head before them in this tile) need the look-back prefix; warp 0 lane 0 computes it
+    // while every other access proceeds.
+    if (t == 0) {
         u64 tagg = s_wagg[0];
 #pragma unroll
-        for (int w = 1; w < THREADS / 32; w++) tagg = combine(tagg, s_wagg[w]);
+        for (int w = 1; w < WARPS; w++) tagg = combine(tagg, s_wagg[w]);
         u64 prefix = ST_IDENTITY;
-        if (tile == 0 || st_head(tagg)) {
-            if (lane == 0) st_relaxed(&P.status[tile], ST_INC | tagg);
-            // the tile prefix is still needed for the elements before the first head
-        } else {
-            if (lane == 0) st_relaxed(&P.status[tile], ST_AGG | tagg);
-        }
+        st_relaxed(&P.status[tile], ((tile == 0 || st_head(tagg)) ? ST_INC : ST_AGG) | tagg);
         if (tile > 0) {
-            // walk back: combine predecessors until an inclusive status or a head-containing aggregate
-            if (lane == 0) {
-                long tt = (long)tile - 1;
-                u64 acc = ST_IDENTITY;
-                bool have = false;
-                while (tt >= 0) {
-                    u64 s;
-                    do {
-                        s = ld_relaxed(&P.status[tt]);
-                    } while ((s >> 62) == 0);
-                    u64 v = s & ST_VAL_MASK;
-                    acc = have ? combine(v, acc) : v;
-                    have = true;
-                    if ((s >> 62) == 2 || st_head(v)) break;
-                    tt--;
-                }
-                prefix = acc;
-                if (!st_head(tagg)) st_relaxed(&P.status[tile], ST_INC | combine(prefix, tagg));
+            // combine predecessors back to an inclusive status or a head-containing aggregate
+            long tt = (long)tile - 1;
+            u64 acc = ST_IDENTITY;
+            bool have = false;
+            while (tt >= 0) {
+                u64 s;
+                do {
+                    s = ld_relaxed(&P.status[tt]);
+                } while ((s >> 62) == 0);
+                const u64 v = s & ST_VAL_MASK;
+                acc = have ? combine(v, acc) : v;
+                have = true;
+                if ((s >> 62) == 2 || st_head(v)) break;
+                tt--;
             }
+            prefix = acc;
+            if (!st_head(tagg)) st_relaxed(&P.status[tile], ST_INC | combine(prefix, tagg));
         }
-        if (lane == 0) s_prefix = prefix;
+        s_prefix = prefix;
+        __threadfence_block();
+        *(volatile u32*)&s_ready = 1u;
     }
-    __syncthreads();
-    u64 wpre = ST_IDENTITY;
-    for (u32 w = 0; w < warp; w++) wpre = (w == 0) ? s_wagg[0] : combine(wpre, s_wagg[w]);
-    u64 run = combine(combine(s_prefix, wpre), wexcl);  // state before this thread's first element
+    u64 run = ST_IDENTITY;
+    for (u32 w = 0; w < warp; w++) run = combine(run, s_wagg[w]);
+    run = combine(run, wexcl);  // tile-relative shadow state before this thread's first access
 
-    // evaluate each access
+    // ---- phase 1: history-free checks; queue the rest ----
     u32 laIdx = pV, laTid = pZ & 0xFFFFFFu, laKind = (pZ >> 24) & 0xFu;
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
-        const bool inr = first + j < P.n;
-        const u64 before = run;
+        u64 before = run;
         run = combine(run, contrib[j]);
+        if (!st_head(before) && first + j < P.n && !st_head(contrib[j])) {
+            // continues the previous tile's segment: wait for the look-back prefix
+            CSTAT(12);
+            while (*(volatile u32*)&s_ready == 0u) __nanosleep(64);
+            before = combine(*(volatile u64*)&s_prefix, before);
+        }
         const u32 i = V[j];
-        const u32 c = ev_tid(E[j]), kind = ev_kind(E[j]);
-        if (inr && !st_head(contrib[j])) {
+        const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
+        bool queue = false;
+        u32 mdIdx = laIdx, p = laTid, mdKind = laKind, flags = 0;
+        const unsigned long long* val64 = reinterpret_cast<const unsigned long long*>(P.val);
+        if (first + j < P.n && !st_head(contrib[j])) {
             const u32 lastW = st_lastW(before), as = st_as(before);
-            const u32 dev = st_dev(before) | st_dev(contrib[j]);
-            const u32 blk = st_blk(before) | st_blk(contrib[j]);
+            CSTAT(0);
             do {
-                if (kind == IGD_LD && lastW == IGD_NONE32) break;  // P2
-                u32 mdIdx, p, mdKind;
-                if (kind == IGD_LD && lastW != (u32)(first + j - 1)) {
-                    mdIdx = __ldg(P.val + lastW);
-                    uint4 me = ld_event(P.ev, mdIdx);
-                    p = ev_tid(me);
-                    mdKind = ev_kind(me);
-                } else {
-                    mdIdx = laIdx;
-                    p = laTid;
-                    mdKind = laKind;
+                if (kind == IGD_LD && lastW == IGD_NONE32) {  // P2: never written
+                    CSTAT(1);
+                    break;
                 }
-                if (p == c) break;  // P3
+                if (kind == IGD_LD && lastW != first + j - 1) {  // md = last writer, further back
+                    CSTAT(13);
+                    const u64 mv = __ldg(val64 + lastW);
+                    mdIdx = (u32)mv;
+                    p = (u32)(mv >> 32) & 0xFFFFFFu;
+                    mdKind = (u32)(mv >> 56) & 0xFu;
+                }
+                if (p == c) {  // P3: program order
+                    CSTAT(2);
+                    break;
+                }
                 const bool isA = kind >= IGD_ATOM && kind <= IGD_EXCH;
-                const u32 bp = g.block(p), bc = g.block(c);
-                const bool same_b = bp == bc;
-                if (as && isA && (same_b || as == IGD_SCOPE_DEVICE)) break;  // P6
-                const u32 wp = g.warp(p), wc = g.warp(c);
-                const bool same_w = wp == wc;
-                if (same_w && ((E[j].w >> g.lane(p)) & 1u)) break;                      // P4 (lockstep)
-                if (same_w && sync_between(P, P.ks.wb + wc, mdIdx, i)) break;           // P4 (syncwarp)
-                bool grid = false, grid_known = false;
-                if (same_b) {
-                    if (sync_between(P, P.ks.bb + bc, mdIdx, i)) break;                 // P5
-                    grid = sync_between(P, P.ks.grid, mdIdx, i);
-                    grid_known = true;
-                    if (grid) break;                                                    // P5 (grid)
+                const u32 bc = g.block(c);
+                const bool same_b = g.block(p) == bc;
+                if (as && isA && (same_b || as == IGD_SCOPE_DEVICE)) {  // P6
+                    CSTAT(3);
+                    break;
                 }
-                u32 type = 0;
-                if (as == IGD_SCOPE_BLOCK) {  // R1
-                    u32 lwTid = (lastW == (u32)(first + j - 1)) ? laTid : ev_tid(ld_event(P.ev, __ldg(P.val + lastW)));
-                    if (g.block(lwTid) != bc) type = IGD_R1;
+                const bool same_w = same_b && g.warp(p) == g.warp(c);
+                // P4, lockstep clause: md's lane is in this instruction's active mask.  The sort
+                // carries two mask summaries in tk bits 31 (full warp) and 30 (own lane only); the
+                // mask itself is gathered only for other partial masks
+                if (same_w && !(Z[j] >> 30)) CSTAT(5);
+                if (same_w && ((Z[j] >> 31) ||
+                               (!((Z[j] >> 30) & 1u) && ((ld_event(P.ev, i).w >> g.lane(p)) & 1u)))) {
+                    CSTAT(4);
+                    break;
                 }
-                if (!type) {
-                    if (!grid_known) grid = sync_between(P, P.ks.grid, mdIdx, i);
-                    if (same_b) {
-                        // R2 (same warp, no sharing) then R3 (same block, no DevShared); both
-                        // need md's thread not to have fenced since md (A1, A30)
-                        if (!dev) {
-                            bool noAny = !grid && !sync_between(P, P.ks.any + p, mdIdx, i);
-                            if (noAny) type = (same_w && !blk) ? IGD_R2 : IGD_R3;
-                        }
-                    } else {
-                        bool noDev = !grid && !sync_between(P, P.ks.dev + p, mdIdx, i);
-                        if (noDev) type = IGD_R4;  // R4: other block, no device fence by md's thread
-                    }
+                flags = (same_w ? QF_SAME_W : 0u) | (same_b ? QF_SAME_B : 0u) |
+                        ((st_dev(before) | st_dev(contrib[j])) ? QF_DEV : 0u) |
+                        ((st_blk(before) | st_blk(contrib[j])) ? QF_BLK : 0u);
+                if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
+                    u32 lwTid = p;
+                    if (kind != IGD_LD && lastW != first + j - 1)
+                        lwTid = (u32)(__ldg(val64 + lastW) >> 32) & 0xFFFFFFu;
+                    if (g.block(lwTid) != bc) flags |= QF_R1;
                 }
-                if (!type) {
-                    const u32 L = syncx::held_before(P.lv, g, c, i);
-                    const u32 locks = syncx::held_before(P.lv, g, laTid, laIdx);
-                    if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
-                }
-                if (type) {
-                    unsigned long long slot = atomicAdd(P.rep_ctr, 1ull);
-                    if (slot < P.rep_cap) {
-                        igd_report r;
-                        r.addr = (ev_addr(E[j]) >> 2) << 2;
-                        r.cur = P.first_event + i;
-                        r.prev = P.first_event + mdIdx;
-                        r.type = (uint8_t)type;
-                        r.cur_kind = (uint8_t)kind;
-                        r.prev_kind = (uint8_t)mdKind;
-                        for (int q = 0; q < 5; q++) r.pad[q] = 0;
-                        P.rep[slot] = r;
-                    }
-                }
+                queue = true;
+                CSTAT(6);
             } while (0);
+        }
+        const u32 qmask = __ballot_sync(IGD_FULL, queue);
+        if (qmask) {
+            u32 qbase = 0;
+            if (lane == 0) qbase = atomicAdd(&s_qn, __popc(qmask));
+            qbase = __shfl_sync(IGD_FULL, qbase, 0);
+            if (queue) {
+                const u32 q = qbase + __popc(qmask & lanemask_lt());
+                q_i[q] = i;
+                q_md[q] = mdIdx;
+                q_c[q] = c | (flags << 24);
+                q_p[q] = p | (kind << 24) | (mdKind << 28);
+                q_la[q] = laIdx;
+                q_lt[q] = laTid;
+            }
         }
         laIdx = i;
         laTid = c;
         laKind = kind;
     }
+    __syncthreads();
+    // ---- phase 2: the queued accesses, densely over the CTA ----
+    const u32 qn = s_qn;
+    const KeySpace ks = P.ks;
+    for (u32 q = t; q < qn; q += THREADS) {
+        const u32 i = q_i[q], mdIdx = q_md[q];
+        const u32 c = q_c[q] & 0xFFFFFFu, flags = q_c[q] >> 24;
+        const u32 p = q_p[q] & 0xFFFFFFu;
+        const bool same_w = flags & QF_SAME_W, same_b = flags & QF_SAME_B;
+        if (same_w && q_between(P.desc, P.sts, ks.wb + g.warp(c), mdIdx, i)) continue;  // P4: syncwarp
+        const bool grid = q_grid(P, mdIdx, i);
+        if (same_b && (grid || q_between(P.desc, P.sts, ks.bb + g.block(c), mdIdx, i))) continue;  // P5
+        u32 type = (flags & QF_R1) ? IGD_R1 : 0u;
+        if (!type) {
+            if (same_b) {
+                // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread must
+                // not have fenced since md (A1, A30)
+                if (!(flags & QF_DEV) && !grid && !q_between(P.desc, P.sts, ks.any + p, mdIdx, i))
+                    type = (same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3;
+            } else if (!grid && !q_between(P.desc, P.sts, ks.dev + p, mdIdx, i)) {
+                type = IGD_R4;  // R4: other block, no device fence by md's thread
+            }
+        }
+        if (!type && P.lv.any) {  // R5: lock sets of the last accessor and of this access
+            const u32 L = syncx::held_before(P.lv, g, c, i);
+            const u32 locks = syncx::held_before(P.lv, g, q_lt[q], q_la[q]);
+            if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
+        }
+        if (type) {
+            CSTAT(11);
+            const unsigned long long slot = atomicAdd(P.rep_ctr, 1ull);
+            if (slot < P.rep_cap) {
+                igd_report r;
+                r.addr = (ev_addr(ld_event(P.ev, i)) >> 2) << 2;
+                r.cur = P.first_event + i;
+                r.prev = P.first_event + mdIdx;
+                r.type = (uint8_t)type;
+                r.cur_kind = (uint8_t)((q_p[q] >> 24) & 0xFu);
+                r.prev_kind = (uint8_t)(q_p[q] >> 28);
+                for (int z = 0; z < 5; z++) r.pad[z] = 0;
+                P.rep[slot] = r;
+            }
+        }
+    }
+}
+
+// Micro-benchmark probe: stream the sorted keys / indices and gather each access's event,
+// nothing else (the memory floor of phase 1).
+__global__ void k_gather_probe(const u32* __restrict__ key, const u64* __restrict__ val, u32 n,
+                               const igd_event* __restrict__ ev, u32* __restrict__ sink, int gather) {
+    u32 acc = 0;
+    for (u32 k = (blockIdx.x * blockDim.x + threadIdx.x) * 4; k < n; k += gridDim.x * blockDim.x * 4) {
+        if (k + 4 <= n) {
+            const uint4 k4 = __ldcs(reinterpret_cast<const uint4*>(key + k));
+            const uint4 va = __ldcs(reinterpret_cast<const uint4*>(val + k));
+            const uint4 vb = __ldcs(reinterpret_cast<const uint4*>(val + k + 2));
+            acc ^= k4.x ^ k4.y ^ k4.z ^ k4.w;
+            if (gather) {
+                const uint4 e0 = ld_event(ev, va.x), e1 = ld_event(ev, va.z), e2 = ld_event(ev, vb.x),
+                            e3 = ld_event(ev, vb.z);
+                acc ^= e0.z ^ e1.z ^ e2.z ^ e3.z;
+            } else {
+                acc ^= va.x ^ va.y ^ vb.z ^ vb.w;
+            }
+        }
+    }
+    if (acc == 0x12345678u) sink[0] = acc;
 }
 
 // reports: key = cur (u32 trace index) for the canonical-order sort

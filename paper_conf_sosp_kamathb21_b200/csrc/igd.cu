@@ -52,11 +52,13 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
-    Buf off, sw, wcnt, tcnt, wpts, tpts;
+    Buf off, ldesc, gtab, sw, wcnt, tcnt, wpts, tpts;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
     int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any (IGD_SORT_MODE)
+    int last_acur = 0;  // buffer holding the sorted accesses of the last igd_detect (debug hooks)
+    u64 last_nacc = 0;
     u64 n_reports = 0;
     u64 bad_event = 0;
     u64 launches = 0;
@@ -180,7 +182,7 @@ static void mark(igd_ctx* ctx, int stage) {
 // copy of the 4x256 digit histogram (device copy d_hist).  Digits above max_bits and digits
 // with one occupied bin are skipped.  Returns the buffer index holding the result.
 static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d_hist, const u32* h_hist,
-                      u32 max_bits, int* out_cur) {
+                      u32 max_bits, int* out_cur, int vbytes = 4) {
     int cur = 0;
     *out_cur = 0;
     if (n <= 1) return IGD_OK;
@@ -201,20 +203,24 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
         rsort::PassParams pp;
         pp.kin = P_<u32>(k[cur]);
-        pp.vin = P_<u32>(v[cur]);
+        pp.vin = v[cur].p;
         pp.kout = P_<u32>(k[cur ^ 1]);
-        pp.vout = P_<u32>(v[cur ^ 1]);
+        pp.vout = v[cur ^ 1].p;
         pp.n = (u32)n;
         pp.shift = p * 8;
         pp.digit_base = P_<u32>(ctx->base) + p * 256;
         pp.status = P_<u64>(ctx->status);
         pp.tile_ctr = P_<u32>(ctx->ctr);
         {
-            KTimer kt(ctx, cls, 16.0 * (double)n);  // read + write 4 B key and 4 B value
-            if (ctx->sort_mode == 0)
-                rsort::k_onesweep<0><<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
-            else
-                rsort::k_onesweep<1><<<(unsigned)tiles, rsort::THREADS, 0, ctx->stream>>>(pp);
+            KTimer kt(ctx, cls, 2.0 * (4 + vbytes) * (double)n);  // read + write 4 B key and the value
+            const unsigned gb = (unsigned)tiles;
+            if (vbytes == 8) {
+                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u64><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
+                else rsort::k_onesweep<1, u64><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
+            } else {
+                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u32><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
+                else rsort::k_onesweep<1, u32><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
+            }
         }
         CK(cudaGetLastError());
         cur ^= 1;
@@ -260,73 +266,76 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
 
     // ---------------- a1 + a2 + a4: ingest ----------------
     const u64 in_tiles = (n + ingest::TILE - 1) / ingest::TILE;
-    if (ctx->sync_cap == 0) ctx->sync_cap = n / 16 + 4096;  // grown and re-run on overflow
     RET(ensure(ctx, ctx->stats, 8 * sizeof(u64)));
     RET(ensure(ctx, ctx->hist, 3 * 1024 * sizeof(u32)));
     RET(ensure(ctx, ctx->base, 4 * 256 * sizeof(u32)));
     RET(ensure(ctx, ctx->ctr, 64));
-    RET(ensure(ctx, ctx->st_in_a, in_tiles * sizeof(u64)));
-    RET(ensure(ctx, ctx->st_in_s, in_tiles * sizeof(u64)));
+    RET(ensure(ctx, ctx->st_in_a, (in_tiles + 1) * sizeof(u32)));
+    RET(ensure(ctx, ctx->st_in_s, (in_tiles + 1) * sizeof(u32)));
     for (int b = 0; b < 2; b++) {
         RET(ensure(ctx, ctx->acc_k[b], n * sizeof(u32)));
-        RET(ensure(ctx, ctx->acc_v[b], n * sizeof(u32)));
+        RET(ensure(ctx, ctx->acc_v[b], n * sizeof(u64)));  // (trace index, tk) per access
     }
-    for (int attempt = 0;; attempt++) {
-        for (int b = 0; b < 2; b++) {
-            RET(ensure(ctx, ctx->syn_k[b], ctx->sync_cap * sizeof(u32)));
-            RET(ensure(ctx, ctx->syn_v[b], ctx->sync_cap * sizeof(u32)));
-        }
-        u64 init[8] = {~0ull, 0, ~0ull, 0, 0, 0, 0, 0};
-        memcpy(ctx->h_small, init, sizeof(init));
-        CK(cudaMemcpyAsync(ctx->stats.p, ctx->h_small, sizeof(init), cudaMemcpyHostToDevice, ctx->stream));
-        CK(cudaMemsetAsync(ctx->hist.p, 0, 2 * 1024 * sizeof(u32), ctx->stream));
-        CK(cudaMemsetAsync(ctx->st_in_a.p, 0, in_tiles * sizeof(u64), ctx->stream));
-        CK(cudaMemsetAsync(ctx->st_in_s.p, 0, in_tiles * sizeof(u64), ctx->stream));
-        CK(cudaMemsetAsync(ctx->ctr.p, 0, sizeof(u32), ctx->stream));
-        ingest::Params ip;
-        ip.ev = ctx->events;
-        ip.n = n;
-        ip.g = g;
-        ip.ks = ks;
-        ip.acc_key = P_<u32>(ctx->acc_k[0]);
-        ip.acc_val = P_<u32>(ctx->acc_v[0]);
-        ip.sync_key = P_<u32>(ctx->syn_k[0]);
-        ip.sync_val = P_<u32>(ctx->syn_v[0]);
-        ip.sync_cap = ctx->sync_cap;
-        ip.st_acc = P_<u64>(ctx->st_in_a);
-        ip.st_sync = P_<u64>(ctx->st_in_s);
-        ip.tile_ctr = P_<u32>(ctx->ctr);
-        ip.hist_acc = P_<u32>(ctx->hist);
-        ip.hist_sync = P_<u32>(ctx->hist) + 1024;
-        ip.stats = P_<u64>(ctx->stats);
-        ip.n_tiles = (u32)in_tiles;
-        int occ = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ingest::k_ingest, ingest::THREADS, 0);
-        u64 grid = (u64)sms * (occ > 0 ? occ : 1);
-        if (grid > in_tiles) grid = in_tiles;
-        {
-            // algorithmic bytes: the events read once + the records written (known after the
-            // launch; the estimate uses the previous call's counts, fixed up below)
-            KTimer kt(ctx, KC_INGEST, 16.0 * (double)n);
-            ingest::k_ingest<<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
-        }
-        CK(cudaGetLastError());
-        CK(cudaMemcpyAsync(ctx->h_stats, ctx->stats.p, 8 * sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
-        CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 2 * 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
-        CK(cudaStreamSynchronize(ctx->stream));
-        if (ctx->h_stats[2] != ~0ull) {
-            ctx->bad_event = ctx->h_stats[2];
-            ctx->err = "invalid event at index " + std::to_string(ctx->bad_event);
-            return IGD_ETRACE;
-        }
-        if (ctx->h_stats[4] <= ctx->sync_cap) break;
-        ctx->sync_cap = ctx->h_stats[4] + ctx->h_stats[4] / 8 + 4096;  // rare: rerun with room
-        if (attempt > 2) return IGD_ECUDA;
+    u64 init[8] = {~0ull, 0, ~0ull, 0, 0, 0, 0, 0};
+    memcpy(ctx->h_small, init, sizeof(init));
+    CK(cudaMemcpyAsync(ctx->stats.p, ctx->h_small, sizeof(init), cudaMemcpyHostToDevice, ctx->stream));
+    CK(cudaMemsetAsync(ctx->hist.p, 0, 2 * 1024 * sizeof(u32), ctx->stream));
+    CK(cudaMemsetAsync(ctx->st_in_a.p, 0, (in_tiles + 1) * sizeof(u32), ctx->stream));
+    CK(cudaMemsetAsync(ctx->st_in_s.p, 0, (in_tiles + 1) * sizeof(u32), ctx->stream));
+    ingest::Params ip;
+    ip.ev = ctx->events;
+    ip.n = n;
+    ip.g = g;
+    ip.ks = ks;
+    ip.tile_acc = P_<u32>(ctx->st_in_a);
+    ip.tile_sync = P_<u32>(ctx->st_in_s);
+    ip.hist_acc = P_<u32>(ctx->hist);
+    ip.hist_sync = P_<u32>(ctx->hist) + 1024;
+    ip.stats = P_<u64>(ctx->stats);
+    ip.n_tiles = (u32)in_tiles;
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ingest::k_ingest<0>, ingest::THREADS, 0);
+    const u64 grid = std::min<u64>((u64)sms * (occ > 0 ? occ : 1), in_tiles);
+    {
+        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n);  // pass 0 reads every event
+        ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
     }
+    CK(cudaGetLastError());
+    RET(scan_excl(ctx, P_<u32>(ctx->st_in_a), in_tiles + 1));
+    RET(scan_excl(ctx, P_<u32>(ctx->st_in_s), in_tiles + 1));
+    CK(cudaMemcpyAsync(ctx->h_stats, ctx->stats.p, 8 * sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 2 * 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(&ctx->h_small[0], P_<u32>(ctx->st_in_a) + in_tiles, sizeof(u32), cudaMemcpyDeviceToHost,
+                       ctx->stream));
+    CK(cudaMemcpyAsync(&ctx->h_small[1], P_<u32>(ctx->st_in_s) + in_tiles, sizeof(u32), cudaMemcpyDeviceToHost,
+                       ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (ctx->h_stats[2] != ~0ull) {
+        ctx->bad_event = ctx->h_stats[2];
+        ctx->err = "invalid event at index " + std::to_string(ctx->bad_event);
+        return IGD_ETRACE;
+    }
+    const u64 n_acc = ctx->h_small[0] & 0xFFFFFFFFull, n_sync = ctx->h_stats[4];
+    const u64 n_lock = ctx->h_stats[5];
+    if (n_sync + 64 > 0xFFFFFFFFull) return IGD_ETOOBIG;  // 32-bit record positions
+    if (ctx->sync_cap < n_sync) ctx->sync_cap = n_sync + n_sync / 8 + 4096;
+    for (int b = 0; b < 2; b++) {
+        // +64 entries: the check's 32-byte timestamp probes may read past the last list
+        RET(ensure(ctx, ctx->syn_k[b], (ctx->sync_cap + 64) * sizeof(u32)));
+        RET(ensure(ctx, ctx->syn_v[b], (ctx->sync_cap + 64) * sizeof(u32)));
+    }
+    ip.acc_key = P_<u32>(ctx->acc_k[0]);
+    ip.acc_val = P_<u64>(ctx->acc_v[0]);
+    ip.sync_key = P_<u32>(ctx->syn_k[0]);
+    ip.sync_val = P_<u32>(ctx->syn_v[0]);
+    ip.sync_cap = ctx->sync_cap;
+    {
+        // pass 1 re-reads the events and writes the (key, value) records
+        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
+        ingest::k_ingest<1><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+    }
+    CK(cudaGetLastError());
     mark(ctx, 1);
-    const u64 n_acc = ctx->h_stats[3], n_sync = ctx->h_stats[4], n_lock = ctx->h_stats[5];
-    for (int q = 0; q < ctx->nk; q++)  // events read + (key, value) records written
-        if (ctx->kcls[q] == KC_INGEST) ctx->kbytes[q] = 16.0 * (double)n + 8.0 * (double)(n_acc + n_sync);
     if (n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32)) {
         ctx->err = "accessed word range spans >= 2^32 words";
         return IGD_ETOOBIG;
@@ -348,6 +357,28 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         KTimer kt(ctx, KC_CSR, 4.0 * (double)work);
         syncx::k_csr_offsets<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->syn_k[scur]), (u32)n_sync, ks.E,
                                                              P_<u32>(ctx->off));
+        CK(cudaGetLastError());
+    }
+    RET(ensure(ctx, ctx->ldesc, ((u64)ks.E + 1) * sizeof(uint4)));
+    {
+        unsigned blocks = (unsigned)std::min<u64>(((u64)ks.E + 255) / 256, (u64)sms * 16);
+        KTimer kt(ctx, KC_CSR, 24.0 * (double)ks.E);
+        check::k_list_desc<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->off), P_<u32>(ctx->syn_v[scur]), ks.E,
+                                                           P_<uint4>(ctx->ldesc));
+        CK(cudaGetLastError());
+    }
+    // grid-sync bucket table (<= 2^22 buckets, L2-resident)
+    u32 glims[2] = {0, 0};
+    CK(cudaMemcpyAsync(glims, P_<u32>(ctx->off) + ks.grid, 2 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    const u32 gshift = std::max<u32>(8, bits_needed(n) > 22 ? bits_needed(n) - 22 : 0);
+    const u32 gnb = (u32)((n >> gshift) + 2);
+    RET(ensure(ctx, ctx->gtab, (u64)gnb * sizeof(u32)));
+    if (glims[1] > glims[0]) {
+        unsigned blocks = (unsigned)std::min<u64>((gnb + 255) / 256, (u64)sms * 16);
+        KTimer kt(ctx, KC_CSR, 4.0 * (double)gnb);
+        check::k_grid_table<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->syn_v[scur]), glims[0], glims[1], gshift,
+                                                            gnb, P_<u32>(ctx->gtab));
         CK(cudaGetLastError());
     }
     // ---------------- a3: lock inference ----------------
@@ -407,7 +438,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     mark(ctx, 3);
     // ---------------- a5: accesses sorted by word, stable ----------------
     int acur = 0;
-    RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur));
+    RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur, 8));
+    ctx->last_acur = acur;
+    ctx->last_nacc = n_acc;
     mark(ctx, 4);
     // ---------------- a6: segmented shadow pass + check ----------------
     if (ctx->rep_cap == 0) ctx->rep_cap = 1 << 20;
@@ -423,12 +456,16 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             CK(cudaMemsetAsync(ctx->rep_ctr.p, 0, sizeof(u64), ctx->stream));
             check::Params cp;
             cp.key = P_<u32>(ctx->acc_k[acur]);
-            cp.val = P_<u32>(ctx->acc_v[acur]);
+            cp.val = P_<u64>(ctx->acc_v[acur]);
             cp.n = (u32)n_acc;
             cp.ev = ctx->events;
             cp.g = g;
             cp.ks = ks;
-            cp.off = P_<u32>(ctx->off);
+            cp.desc = P_<uint4>(ctx->ldesc);
+            cp.gtab = P_<u32>(ctx->gtab);
+            cp.gshift = gshift;
+            cp.glo = glims[0];
+            cp.ghi = glims[1];
             cp.sts = P_<u32>(ctx->syn_v[scur]);
             cp.lv = lv;
             cp.status = P_<u64>(ctx->status);
@@ -439,7 +476,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.first_event = 0;
             {
                 // 4 B key + 4 B value streamed, one 16-B event gathered per access
-                KTimer kt(ctx, KC_CHECK, 24.0 * (double)n_acc);
+                KTimer kt(ctx, KC_CHECK, 12.0 * (double)n_acc);  // 4 B key + 8 B (index, tk) streamed
                 check::k_check<<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
             }
             CK(cudaGetLastError());
@@ -639,7 +676,8 @@ void igd_ctx_destroy(igd_ctx* ctx) {
     Buf* all[] = {&ctx->owned_events, &ctx->acc_k[0], &ctx->acc_k[1], &ctx->acc_v[0], &ctx->acc_v[1],
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
                   &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
-                  &ctx->ctr,          &ctx->off,      &ctx->sw,       &ctx->wcnt,     &ctx->tcnt,
+                  &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->sw,       &ctx->wcnt,
+                  &ctx->tcnt,
                   &ctx->wpts,         &ctx->tpts,     &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist};
     for (Buf* b : all) buf_free(ctx, *b);
@@ -669,6 +707,37 @@ const char* igd_strerror(int code) {
 const char* igd_last_error(const igd_ctx* ctx) { return ctx ? ctx->err.c_str() : ""; }
 
 // ---- stage-level test / micro-benchmark hooks (include/igd_debug.h) ----
+int igd_debug_check_stats(igd_ctx* ctx, int enable, uint64_t* out16) {
+    if (!ctx) return IGD_EINVAL;
+    cudaSetDevice(ctx->device);
+    if (out16) CK(cudaMemcpyFromSymbol(out16, check::g_chk_stats, 16 * sizeof(u64)));
+    const unsigned long long zero[16] = {0};
+    CK(cudaMemcpyToSymbol(check::g_chk_stats, zero, sizeof(zero)));
+    CK(cudaMemcpyToSymbol(check::g_chk_stats_on, &enable, sizeof(int)));
+    return IGD_OK;
+}
+
+int igd_debug_gather_probe(igd_ctx* ctx, int gather, float* ms) {
+    if (!ctx || !ctx->loaded || ctx->last_nacc == 0) return IGD_ESTATE;
+    cudaSetDevice(ctx->device);
+    RET(ensure(ctx, ctx->ctr, 64));
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    const int sms = sm_count(ctx);
+    cudaEventRecord(a, ctx->stream);
+    check::k_gather_probe<<<sms * 8, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[ctx->last_acur]),
+                                                          P_<u64>(ctx->acc_v[ctx->last_acur]), (u32)ctx->last_nacc,
+                                                          ctx->events, P_<u32>(ctx->ctr), gather);
+    cudaEventRecord(b, ctx->stream);
+    cudaEventSynchronize(b);
+    if (ms) cudaEventElapsedTime(ms, a, b);
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    CK(cudaGetLastError());
+    return IGD_OK;
+}
+
 int igd_debug_radix_sort(igd_ctx* ctx, uint32_t* d_keys, uint32_t* d_vals, uint64_t n, uint32_t max_bits, int mode,
                          float* ms) {
     if (!ctx || n >= 0xFFFFFFFFull || (n && (!d_keys || !d_vals))) return IGD_EINVAL;

@@ -1,18 +1,17 @@
-// ingest.cuh -- a1 + a2 extraction + a4 key build, fused into one streaming pass over the trace.
+// ingest.cuh -- a1 + a2 extraction + a4 key build: streaming passes over the trace.
 //
-// One read of every 16-byte event:
+// Per 16-byte event:
 //   * validates the field rules of include/igd.h (first bad index -> atomicMin),
-//   * compacts accesses into (key = low 32 bits of the word, value = event index), in trace
-//     order (stable chained-scan compaction with decoupled look-back),
+//   * compacts accesses into (key = low 32 bits of the word, value = event index | tk << 32),
+//     in trace order (stable compaction: per-tile counts, a scan, then positioned writes),
 //   * compacts synchronization events into (entity key, timestamp) records (KeySpace), also in
 //     trace order, so a stable sort by entity gives per-entity timestamp lists,
 //   * builds the 4 x 8-bit digit histograms of both record streams for the radix sorts
 //     (warp-uniform digits -- the common case for the high digits -- cost one shared atomic
 //     per warp instead of 32 conflicting ones),
 //   * reduces min / max accessed word (the 32-bit key is injective iff max - min < 2^32).
-// Persistent CTAs pull 2048-event tiles from an atomic counter, so tiles are scheduled in order
-// (forward progress for look-back) and histograms are flushed once per CTA.  Each event is
-// decoded once into 4 registers; the raw 16 bytes are not kept.
+// Persistent CTAs stride over 2048-event tiles; histograms are flushed once per CTA.  Each event
+// is decoded into 5 registers; the raw 16 bytes are not kept.
 #pragma once
 #include "common.cuh"
 
@@ -29,13 +28,12 @@ struct Params {
     Geo g;
     KeySpace ks;
     u32* acc_key;
-    u32* acc_val;
+    u64* acc_val;  // trace index | tk << 32 (the check then needs no event gather)
     u32* sync_key;
     u32* sync_val;
     u64 sync_cap;  // records beyond capacity are counted, not written (host re-runs)
-    u64* st_acc;   // [n_tiles]
-    u64* st_sync;  // [n_tiles]
-    u32* tile_ctr;
+    u32* tile_acc;   // [n_tiles + 1] pass 0: access records per tile; scanned to bases
+    u32* tile_sync;  // [n_tiles + 1] pass 0: sync records per tile; scanned to bases
     u32* hist_acc;   // [4][256]
     u32* hist_sync;  // [4][256]
     u64* stats;      // [0] min word, [1] max word, [2] bad index, [3] n_acc, [4] n_sync, [5] n_lock
@@ -45,7 +43,7 @@ struct Params {
 // Decoded event: flags bit 0 = access, bits 1..2 = number of sync records, bit 3 = CAS/EXCH,
 // bit 4 = invalid; key = access key; s0, s1 = sync record keys.
 struct Dec {
-    u32 flags, key, s0, s1;
+    u32 flags, key, s0, s1, tk;
 };
 
 __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpace& ks) {
@@ -53,6 +51,7 @@ __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpa
     d.flags = 0;
     d.key = 0;
     d.s0 = d.s1 = 0;
+    d.tk = e.z;
     const u32 tid = ev_tid(e), kind = ev_kind(e), scope = ev_scope(e);
     const bool addr0 = (e.x | e.y) == 0;
     const bool tid_ok = tid < g.T;
@@ -97,6 +96,9 @@ __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpa
     if (kind <= IGD_EXCH) {
         d.key = (e.x >> 2) | (e.y << 30);  // low 32 bits of the word addr >> 2
         d.flags = 1;
+        // mask summaries for the check's lockstep clause (tk bits 30..31 are zero in the trace):
+        // bit 31 = full warp, bit 30 = only the issuing lane
+        d.tk |= (e.w == IGD_FULL ? (1u << 31) : 0u) | (e.w == lanebit ? (1u << 30) : 0u);
         if (kind == IGD_CAS || kind == IGD_EXCH) {
             d.flags |= (1u << 1) | 8u;
             d.s0 = ks.lock + w;
@@ -136,32 +138,32 @@ __device__ __forceinline__ void hist_add(u32* h, u32 digit, bool on, u32 lane) {
     }
 }
 
-__global__ void __launch_bounds__(THREADS, 3) k_ingest(Params P) {
-    __shared__ u32 s_hacc[4][256];
-    __shared__ u32 s_hsync[4][256];
+// Pass 0 (count): per tile, the number of access records and sync records; digit histograms,
+// min / max word, first invalid event.  Pass 1 (write): the same decode, positions from the
+// scanned per-tile counts plus warp scans inside the tile.  Two reads of the trace instead of
+// one, but every tile is independent: no look-back chain across 2M tiles (which bounded the
+// single-pass variant at ~40 G events/s on B200).
+template <int PASS>
+__global__ void __launch_bounds__(THREADS, 2) k_ingest(Params P) {
+    __shared__ u32 s_hacc[PASS == 0 ? 4 : 1][256];
+    __shared__ u32 s_hsync[PASS == 0 ? 4 : 1][256];
     __shared__ u32 s_wtot[ITEMS][WARPS];  // packed (acc | nsync << 16) per (item, warp)
     __shared__ u32 s_woff[ITEMS][WARPS];  // packed exclusive offsets (acc | sync << 16)
-    __shared__ u64 s_base_acc, s_base_sync;
-    __shared__ u32 s_tile;
 
     const u32 tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
-    for (int i = tid; i < 4 * 256; i += THREADS) {
-        (&s_hacc[0][0])[i] = 0;
-        (&s_hsync[0][0])[i] = 0;
-    }
+    if (PASS == 0)
+        for (int i = tid; i < 4 * 256; i += THREADS) {
+            (&s_hacc[0][0])[i] = 0;
+            (&s_hsync[0][0])[i] = 0;
+        }
     u64 wmin = ~0ull, wmax = 0, bad = ~0ull;
-    u32 cnt_acc = 0, cnt_sync = 0, cnt_lock = 0;
+    u32 cnt_lock = 0;
+    u64 cta_sync = 0;  // thread 0 of pass 0: sync records of this CTA's tiles (64-bit total)
     const Geo g = P.g;
     const KeySpace ks = P.ks;
 
-    while (true) {
-        __syncthreads();
-        if (tid == 0) s_tile = atomicAdd(P.tile_ctr, 1u);
-        __syncthreads();
-        const u32 tile = s_tile;
-        if (tile >= P.n_tiles) break;
+    for (u32 tile = blockIdx.x; tile < P.n_tiles; tile += gridDim.x) {
         const u64 base = (u64)tile * TILE;
-
         Dec dv[ITEMS];
         {
             uint4 e[ITEMS];
@@ -175,42 +177,64 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest(Params P) {
                 const u64 i = base + (u64)j * THREADS + tid;
                 if (i < P.n) {
                     dv[j] = decode(e[j], g, ks);
-                    if (dv[j].flags & 1u) {
+                    if (PASS == 0 && (dv[j].flags & 1u)) {
                         const u64 word = ev_addr(e[j]) >> 2;
                         wmin = min(wmin, word);
                         wmax = max(wmax, word);
                     }
                 } else {
                     dv[j].flags = 0;
-                    dv[j].key = dv[j].s0 = dv[j].s1 = 0;
+                    dv[j].key = dv[j].s0 = dv[j].s1 = dv[j].tk = 0;
                 }
             }
         }
         u32 excl[ITEMS];
+        u32 wsum = 0;  // PASS 0: packed warp totals summed over items
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
             const u32 f = dv[j].flags;
-            if (f & 16u) bad = min(bad, base + (u64)j * THREADS + tid);
             const bool acc = (f & 1u) != 0;
             const u32 ns = (f >> 1) & 3u;
-#pragma unroll
-            for (int p = 0; p < 4; p++) hist_add(s_hacc[p], (dv[j].key >> (8 * p)) & 255u, acc, lane);
-            if (__any_sync(IGD_FULL, ns != 0)) {
-#pragma unroll
-                for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s0 >> (8 * p)) & 255u, ns != 0, lane);
-#pragma unroll
-                for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s1 >> (8 * p)) & 255u, ns == 2, lane);
-            }
-            cnt_lock += (f >> 3) & 1u;
             const u32 v = (acc ? 1u : 0u) | (ns << 16);
-            u32 inc = v;
+            if (PASS == 0) {
+                if (f & 16u) bad = min(bad, base + (u64)j * THREADS + tid);
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const u32 t = __shfl_up_sync(IGD_FULL, inc, o);
-                if (lane >= (u32)o) inc += t;
+                for (int p = 0; p < 4; p++) hist_add(s_hacc[p], (dv[j].key >> (8 * p)) & 255u, acc, lane);
+                if (__any_sync(IGD_FULL, ns != 0)) {
+#pragma unroll
+                    for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s0 >> (8 * p)) & 255u, ns != 0, lane);
+#pragma unroll
+                    for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s1 >> (8 * p)) & 255u, ns == 2, lane);
+                }
+                cnt_lock += (f >> 3) & 1u;
+                wsum += __reduce_add_sync(IGD_FULL, v);
+            } else {
+                u32 inc = v;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const u32 t = __shfl_up_sync(IGD_FULL, inc, o);
+                    if (lane >= (u32)o) inc += t;
+                }
+                excl[j] = inc - v;
+                if (lane == 31) s_wtot[j][warp] = inc;
             }
-            excl[j] = inc - v;
-            if (lane == 31) s_wtot[j][warp] = inc;
+        }
+        if (PASS == 0) {
+            // per-tile totals: one packed word per warp, summed by warp 0
+            if (lane == 0) s_wtot[0][warp] = wsum;
+            __syncthreads();
+            if (warp == 0) {
+                const u32 x = lane < WARPS ? s_wtot[0][lane] : 0u;
+                const u32 ta = __reduce_add_sync(IGD_FULL, x & 0xFFFFu);
+                const u32 ts = __reduce_add_sync(IGD_FULL, x >> 16);
+                if (lane == 0) {
+                    P.tile_acc[tile] = ta;
+                    P.tile_sync[tile] = ts;
+                    cta_sync += ts;
+                }
+            }
+            __syncthreads();
+            continue;
         }
         __syncthreads();
         // scan the ITEMS x WARPS totals in (item, warp) order; warp 0 does it
@@ -241,28 +265,9 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest(Params P) {
                 ea += vv[q] & 0xFFFFu;
                 es += vv[q] >> 16;
             }
-            const u32 tot_a = __shfl_sync(IGD_FULL, ia, 31);
-            const u32 tot_s = __shfl_sync(IGD_FULL, is, 31);
-            if (lane == 0) {
-                st_relaxed(&P.st_acc[tile], (tile == 0 ? ST_INC : ST_AGG) | tot_a);
-                st_relaxed(&P.st_sync[tile], (tile == 0 ? ST_INC : ST_AGG) | tot_s);
-            }
-            u64 ba = 0, bs = 0;
-            if (tile > 0) {
-                ba = lookback_sum_warp(P.st_acc, tile);
-                bs = lookback_sum_warp(P.st_sync, tile);
-                if (lane == 0) {
-                    st_relaxed(&P.st_acc[tile], ST_INC | (ba + tot_a));
-                    st_relaxed(&P.st_sync[tile], ST_INC | (bs + tot_s));
-                }
-            }
-            if (lane == 0) {
-                s_base_acc = ba;
-                s_base_sync = bs;
-            }
         }
         __syncthreads();
-        const u64 ba = s_base_acc, bs = s_base_sync;
+        const u64 ba = P.tile_acc[tile], bs = P.tile_sync[tile];  // exclusive tile bases (scanned)
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
             const u32 f = dv[j].flags;
@@ -271,8 +276,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest(Params P) {
             if (f & 1u) {
                 const u64 pos = ba + (wo & 0xFFFFu) + (ex & 0xFFFFu);
                 P.acc_key[pos] = dv[j].key;
-                P.acc_val[pos] = (u32)(base + (u64)j * THREADS + tid);
-                cnt_acc++;
+                P.acc_val[pos] = (base + (u64)j * THREADS + tid) | ((u64)dv[j].tk << 32);
             }
             const u32 ns = (f >> 1) & 3u;
             if (ns) {
@@ -286,35 +290,34 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest(Params P) {
                         P.sync_val[pos + 1] = ts;
                     }
                 }
-                cnt_sync += ns;
             }
         }
+        __syncthreads();  // s_woff / s_wtot reuse by the next tile
     }
+    if (PASS != 0) return;
     // flush per-CTA results
+    __syncthreads();
     for (int i = tid; i < 4 * 256; i += THREADS) {
         const u32 a = (&s_hacc[0][0])[i];
         if (a) atomicAdd(&P.hist_acc[i], a);
         const u32 s = (&s_hsync[0][0])[i];
         if (s) atomicAdd(&P.hist_sync[i], s);
     }
-    u64 ca = cnt_acc, cs = cnt_sync, cl = cnt_lock;
+    u64 cl = cnt_lock;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         wmin = min(wmin, __shfl_xor_sync(IGD_FULL, wmin, o));
         wmax = max(wmax, __shfl_xor_sync(IGD_FULL, wmax, o));
         bad = min(bad, __shfl_xor_sync(IGD_FULL, bad, o));
-        ca += __shfl_xor_sync(IGD_FULL, ca, o);
-        cs += __shfl_xor_sync(IGD_FULL, cs, o);
         cl += __shfl_xor_sync(IGD_FULL, cl, o);
     }
     if (lane == 0) {
         if (wmin != ~0ull) atomicMin((unsigned long long*)&P.stats[0], (unsigned long long)wmin);
-        if (ca) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
+        if (wmin != ~0ull) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
         if (bad != ~0ull) atomicMin((unsigned long long*)&P.stats[2], (unsigned long long)bad);
-        if (ca) atomicAdd((unsigned long long*)&P.stats[3], (unsigned long long)ca);
-        if (cs) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cs);
         if (cl) atomicAdd((unsigned long long*)&P.stats[5], (unsigned long long)cl);
     }
+    if (tid == 0 && cta_sync) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cta_sync);
 }
 
 }  // namespace ingest

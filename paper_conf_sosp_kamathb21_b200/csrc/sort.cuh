@@ -61,9 +61,9 @@ __global__ void k_hist4(const u32* __restrict__ keys, u64 n, u32* __restrict__ h
 
 struct PassParams {
     const u32* kin;
-    const u32* vin;
+    const void* vin;  // u32 or u64 values (template VT)
     u32* kout;
-    u32* vout;
+    void* vout;
     u32 n;
     u32 shift;
     const u32* digit_base;  // [256] exclusive global offsets of this pass's digits
@@ -88,12 +88,16 @@ __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     }
 }
 
-template <int MODE>
+template <int MODE, typename VT>
 __global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
     __shared__ u32 s_whist[WARPS][RADIX];
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
-    __shared__ u32 s_buf[TILE];
+    __shared__ __align__(16) unsigned char s_raw[TILE * sizeof(VT)];  // keys, then values
+    u32* s_buf = reinterpret_cast<u32*>(s_raw);
+    VT* s_vbuf = reinterpret_cast<VT*>(s_raw);
+    const VT* vin = reinterpret_cast<const VT*>(P.vin);
+    VT* vout = reinterpret_cast<VT*>(P.vout);
     __shared__ uint8_t s_dig[TILE];
     __shared__ u32 s_tile;
     __shared__ u32 s_wsum[WARPS];
@@ -205,22 +209,23 @@ __global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
         }
     }
     // values: same permutation through the same buffer
+    VT val[ITEMS];
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
         const u32 i = wbase + j * 32 + lane;
-        key[j] = (full || i < P.n) ? __ldcs(P.vin + i) : 0u;  // key[] now holds values
+        val[j] = (full || i < P.n) ? __ldcs(vin + i) : (VT)0;
     }
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < ITEMS; j++)
-        if (full || wbase + j * 32 + lane < P.n) s_buf[rank[j]] = key[j];
+        if (full || wbase + j * 32 + lane < P.n) s_vbuf[rank[j]] = val[j];
     __syncthreads();
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const u32 i = t + k * THREADS;
         if (i < tile_n) {
             const u32 d = s_dig[i];
-            __stcs(P.vout + s_gbase[d] + (i - s_tile_excl[d]), s_buf[i]);
+            __stcs(vout + s_gbase[d] + (i - s_tile_excl[d]), s_vbuf[i]);
         }
     }
 }

@@ -158,3 +158,20 @@ def test_repeat_detect_is_deterministic(det):
     a = det.reports()
     det.detect()
     assert np.array_equal(a, det.reports())
+
+
+@pytest.mark.parametrize("seed", [21, 22])
+def test_long_irregular_sync_lists(det, seed):
+    # few entities with long, bursty synchronization lists: exercises the interpolation probes
+    # and their binary-search fallback in every direction
+    rng = np.random.default_rng(seed)
+    n = 400_000
+    w = np.array([20, 18, 10, 2, 2, 14, 12, 8, 1, 2, 2, 1], float)
+    ev, nb, bd = _fast_random(seed, n, 40, 2, 64, w)
+    # make the sync events bursty: shuffle blocks of the trace so syncs cluster
+    kind = (ev["tk"] >> 24) & 0xF
+    sync = kind >= 5
+    burst = (np.arange(n) // 5000) % 3 == 0
+    drop = sync & ~burst & (rng.random(n) < 0.9)
+    ev = ev[~drop]
+    assert_same(det, ev, nb, bd, f"bursty {seed}")
