@@ -138,6 +138,7 @@ struct Params {
     u64 rep_cap;
     unsigned long long* rep_ctr;
     u64 first_event; // global index offset (multi-rank)
+    int debug_stop;  // profiling only (IGD_CHECK_STOP): 1 = stop after the scans, 2 = after phase 1
 };
 
 // Grid-sync bucket table: gtab[b] = index of the first grid sync with timestamp >= b << shift.
@@ -299,6 +300,10 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
     for (u32 w = 0; w < warp; w++) run = combine(run, s_wagg[w]);
     run = combine(run, wexcl);  // tile-relative shadow state before this thread's first access
 
+    if (P.debug_stop == 1) {
+        if (run == 0x123456789ull) P.rep_ctr[1] = run;  // keep the scans alive
+        return;
+    }
     // ---- phase 1: history-free checks; queue the rest ----
     u32 laIdx = pV, laTid = pZ & 0xFFFFFFu, laKind = (pZ >> 24) & 0xFu;
 #pragma unroll
@@ -385,6 +390,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
         laKind = kind;
     }
     __syncthreads();
+    if (P.debug_stop == 2) return;
     // ---- phase 2: the queued accesses, densely over the CTA ----
     const u32 qn = s_qn;
     const KeySpace ks = P.ks;

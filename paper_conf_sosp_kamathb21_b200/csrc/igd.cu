@@ -57,6 +57,7 @@ struct igd_ctx {
     u64 sync_cap = 0;
     u64 rep_cap = 0;
     int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any (IGD_SORT_MODE)
+    int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
     int last_acur = 0;  // buffer holding the sorted accesses of the last igd_detect (debug hooks)
     u64 last_nacc = 0;
     u64 n_reports = 0;
@@ -214,12 +215,13 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         {
             KTimer kt(ctx, cls, 2.0 * (4 + vbytes) * (double)n);  // read + write 4 B key and the value
             const unsigned gb = (unsigned)tiles;
+            const size_t s8 = rsort::onesweep_smem<u64>(), s4 = rsort::onesweep_smem<u32>();
             if (vbytes == 8) {
-                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u64><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
-                else rsort::k_onesweep<1, u64><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
+                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u64><<<gb, rsort::THREADS, s8, ctx->stream>>>(pp);
+                else rsort::k_onesweep<1, u64><<<gb, rsort::THREADS, s8, ctx->stream>>>(pp);
             } else {
-                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u32><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
-                else rsort::k_onesweep<1, u32><<<gb, rsort::THREADS, 0, ctx->stream>>>(pp);
+                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u32><<<gb, rsort::THREADS, s4, ctx->stream>>>(pp);
+                else rsort::k_onesweep<1, u32><<<gb, rsort::THREADS, s4, ctx->stream>>>(pp);
             }
         }
         CK(cudaGetLastError());
@@ -474,6 +476,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.rep_cap = ctx->rep_cap;
             cp.rep_ctr = P_<unsigned long long>(ctx->rep_ctr);
             cp.first_event = 0;
+            cp.debug_stop = ctx->check_stop;
             {
                 // 4 B key + 4 B value streamed, one 16-B event gathered per access
                 KTimer kt(ctx, KC_CHECK, 12.0 * (double)n_acc);  // 4 B key + 8 B (index, tk) streamed
@@ -558,6 +561,15 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     ctx->ffn = free_fn;
     ctx->auser = alloc_user;
     if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = atoi(m) == 0 ? 0 : 1;
+    if (const char* m = getenv("IGD_CHECK_STOP")) ctx->check_stop = atoi(m);
+    cudaFuncSetAttribute(rsort::k_onesweep<0, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<u64>());
+    cudaFuncSetAttribute(rsort::k_onesweep<1, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<u64>());
+    cudaFuncSetAttribute(rsort::k_onesweep<0, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<u32>());
+    cudaFuncSetAttribute(rsort::k_onesweep<1, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<u32>());
     if (cudaMallocHost(&ctx->h_stats, 8 * sizeof(u64)) != cudaSuccess ||
         cudaMallocHost(&ctx->h_hist, 3 * 1024 * sizeof(u32)) != cudaSuccess ||
         cudaMallocHost(&ctx->h_small, 8 * sizeof(u64)) != cudaSuccess) {

@@ -88,35 +88,63 @@ __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     }
 }
 
+// Dynamic shared memory of k_onesweep<MODE, VT>: staged keys, staged values, digit per position.
+template <typename VT>
+constexpr size_t onesweep_smem() {
+    return (size_t)TILE * sizeof(u32) + (size_t)TILE * sizeof(VT) + TILE;
+}
+
 template <int MODE, typename VT>
 __global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
     __shared__ u32 s_whist[WARPS][RADIX];
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
-    __shared__ __align__(16) unsigned char s_raw[TILE * sizeof(VT)];  // keys, then values
-    u32* s_buf = reinterpret_cast<u32*>(s_raw);
-    VT* s_vbuf = reinterpret_cast<VT*>(s_raw);
-    const VT* vin = reinterpret_cast<const VT*>(P.vin);
-    VT* vout = reinterpret_cast<VT*>(P.vout);
-    __shared__ uint8_t s_dig[TILE];
     __shared__ u32 s_tile;
     __shared__ u32 s_wsum[WARPS];
+    __shared__ __align__(8) u64 s_mbar[2];
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    u32* s_k = reinterpret_cast<u32*>(s_dyn);                         // keys in, then keys out
+    VT* s_v = reinterpret_cast<VT*>(s_dyn + TILE * sizeof(u32));      // values in, then values out
+    uint8_t* s_dig = s_dyn + TILE * sizeof(u32) + TILE * sizeof(VT);  // digit of each output position
+    const VT* vin = reinterpret_cast<const VT*>(P.vin);
+    VT* vout = reinterpret_cast<VT*>(P.vout);
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
-    if (t == 0) s_tile = atomicAdd(P.tile_ctr, 1u);
+    if (t == 0) {
+        // tile id, then TMA bulk copies of the tile's keys and values into shared memory: the
+        // value copy lands while the keys are ranked
+        const u32 tile = atomicAdd(P.tile_ctr, 1u);
+        s_tile = tile;
+        const u64 base = (u64)tile * TILE;
+        if (base + TILE <= P.n) {
+            mbar_init(&s_mbar[0], 1);
+            mbar_init(&s_mbar[1], 1);
+            mbar_expect_tx(&s_mbar[0], TILE * sizeof(u32));
+            bulk_g2s(s_k, P.kin + base, TILE * sizeof(u32), &s_mbar[0]);
+            mbar_expect_tx(&s_mbar[1], TILE * sizeof(VT));
+            bulk_g2s(s_v, vin + base, TILE * sizeof(VT), &s_mbar[1]);
+        }
+    }
     for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_whist[0][0])[i] = 0;
     __syncthreads();
     const u32 tile = s_tile;
     const u32 base = tile * TILE;  // n <= 2^32 - 2^13 (checked by the host)
-    const u32 wbase = base + warp * 32 * ITEMS;
+    const u32 wofs = warp * 32 * ITEMS;
+    const u32 wbase = base + wofs;
     const u32 shift = P.shift;
     const bool full = (u64)base + TILE <= P.n;
 
     u32 key[ITEMS];
+    if (full) {
+        mbar_wait(&s_mbar[0], 0);
 #pragma unroll
-    for (int j = 0; j < ITEMS; j++) {
-        const u32 i = wbase + j * 32 + lane;
-        key[j] = (full || i < P.n) ? __ldcs(P.kin + i) : 0u;
+        for (int j = 0; j < ITEMS; j++) key[j] = s_k[wofs + j * 32 + lane];
+    } else {
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const u32 i = wbase + j * 32 + lane;
+            key[j] = i < P.n ? __ldcs(P.kin + i) : 0u;
+        }
     }
     u32 rank[ITEMS];
     const u32 lt = lanemask_lt();
@@ -188,13 +216,12 @@ __global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
         s_gbase[d] = P.digit_base[d] + (u32)excl;
     }
     __syncthreads();
-    // keys: reorder through shared memory (rank[] becomes the tile position), then write
-    // digit runs; the digit of every tile position is kept for the value pass
+    // keys: reorder in shared memory (rank[] becomes the tile position), write digit runs
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
         const u32 d = (key[j] >> shift) & 255u;
         rank[j] += s_tile_excl[d] + s_whist[warp][d];
-        if (full || wbase + j * 32 + lane < P.n) s_buf[rank[j]] = key[j];
+        if (full || wbase + j * 32 + lane < P.n) s_k[rank[j]] = key[j];
     }
     __syncthreads();
     const u32 tile_n = full ? (u32)TILE : P.n - base;
@@ -202,30 +229,36 @@ __global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
     for (int k = 0; k < ITEMS; k++) {
         const u32 i = t + k * THREADS;
         if (i < tile_n) {
-            const u32 kk = s_buf[i];
+            const u32 kk = s_k[i];
             const u32 d = (kk >> shift) & 255u;
             s_dig[i] = (uint8_t)d;
             __stcs(P.kout + s_gbase[d] + (i - s_tile_excl[d]), kk);
         }
     }
-    // values: same permutation through the same buffer
+    // values: same permutation, in place through the staged buffer
     VT val[ITEMS];
+    if (full) {
+        mbar_wait(&s_mbar[1], 0);
 #pragma unroll
-    for (int j = 0; j < ITEMS; j++) {
-        const u32 i = wbase + j * 32 + lane;
-        val[j] = (full || i < P.n) ? __ldcs(vin + i) : (VT)0;
+        for (int j = 0; j < ITEMS; j++) val[j] = s_v[wofs + j * 32 + lane];
+    } else {
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const u32 i = wbase + j * 32 + lane;
+            val[j] = i < P.n ? __ldcs(vin + i) : (VT)0;
+        }
     }
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < ITEMS; j++)
-        if (full || wbase + j * 32 + lane < P.n) s_vbuf[rank[j]] = val[j];
+        if (full || wbase + j * 32 + lane < P.n) s_v[rank[j]] = val[j];
     __syncthreads();
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const u32 i = t + k * THREADS;
         if (i < tile_n) {
             const u32 d = s_dig[i];
-            __stcs(vout + s_gbase[d] + (i - s_tile_excl[d]), s_vbuf[i]);
+            __stcs(vout + s_gbase[d] + (i - s_tile_excl[d]), s_v[i]);
         }
     }
 }
