@@ -337,6 +337,14 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         ingest::k_ingest<1><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
     }
     CK(cudaGetLastError());
+    if (n_acc > 0) {
+        KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digit histograms
+        const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
+        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[0]), (u32)n_acc, P_<u32>(ctx->hist));
+    }
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
     mark(ctx, 1);
     if (n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32)) {
         ctx->err = "accessed word range spans >= 2^32 words";

@@ -198,8 +198,7 @@ __global__ void __launch_bounds__(THREADS, 2) k_ingest(Params P) {
             const u32 v = (acc ? 1u : 0u) | (ns << 16);
             if (PASS == 0) {
                 if (f & 16u) bad = min(bad, base + (u64)j * THREADS + tid);
-#pragma unroll
-                for (int p = 0; p < 4; p++) hist_add(s_hacc[p], (dv[j].key >> (8 * p)) & 255u, acc, lane);
+                // (access-key digit histograms: k_hist_keys over the compacted keys)
                 if (__any_sync(IGD_FULL, ns != 0)) {
 #pragma unroll
                     for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s0 >> (8 * p)) & 255u, ns != 0, lane);
@@ -318,6 +317,36 @@ __global__ void __launch_bounds__(THREADS, 2) k_ingest(Params P) {
         if (cl) atomicAdd((unsigned long long*)&P.stats[5], (unsigned long long)cl);
     }
     if (tid == 0 && cta_sync) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cta_sync);
+}
+
+// Digit histograms (4 x 8-bit) of the compacted access keys: a light, high-occupancy pass over
+// 4 bytes per access, with warp-uniform digits aggregated into one shared atomic.
+__global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys, u32 n, u32* __restrict__ hist) {
+    __shared__ u32 s[4][256];
+    const u32 lane = threadIdx.x & 31u;
+    for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&s[0][0])[i] = 0;
+    __syncthreads();
+    const u32 n4 = n / 4;
+    for (u32 q = blockIdx.x * blockDim.x + threadIdx.x; q - lane < n4; q += gridDim.x * blockDim.x) {
+        const bool in = q < n4;
+        const uint4 k4 = in ? __ldcs(reinterpret_cast<const uint4*>(keys) + q) : make_uint4(0, 0, 0, 0);
+        const u32 kk[4] = {k4.x, k4.y, k4.z, k4.w};
+#pragma unroll
+        for (int e = 0; e < 4; e++)
+#pragma unroll
+            for (int p = 0; p < 4; p++) hist_add(s[p], (kk[e] >> (8 * p)) & 255u, in, lane);
+    }
+    if (blockIdx.x == 0)  // the n % 4 tail
+        for (u32 i = n4 * 4 + threadIdx.x; i < n; i += blockDim.x) {
+            const u32 k = keys[i];
+#pragma unroll
+            for (int p = 0; p < 4; p++) atomicAdd(&s[p][(k >> (8 * p)) & 255u], 1u);
+        }
+    __syncthreads();
+    for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) {
+        const u32 v = (&s[0][0])[i];
+        if (v) atomicAdd(&hist[i], v);
+    }
 }
 
 }  // namespace ingest
