@@ -136,6 +136,35 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
    event, IGD_ETOOBIG if the accessed words span >= 2^32 words.  flags: 0. */
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
 
+/* ---- multi-GPU sharding, driven by the host over torch.distributed / NCCL ----
+   Each rank loads its contiguous chunk with igd_trace_load (desc.first_event = global index of
+   events[0], desc.n_events_total = global length).  Words are hash-sharded:
+   owner(word) = fmix32(low 32 bits of word) % nranks (murmur3 finalizer).
+
+   Stage 1, igd_shard_prepare: partitions the chunk.  counts[o] = access records destined to rank o;
+   *n_sync_stream = synchronization-stream events (FENCE, SYNCWARP, SYNCTHREADS, GRID_SYNC, the CG
+   kinds, CAS, EXCH); *bad_event = first invalid GLOBAL index (~0 if none; the caller reduces it over
+   ranks and must not continue if any rank has one); word_minmax = min / max accessed word of the chunk
+   (the caller reduces them; the global span must be < 2^32 words).  Returns IGD_OK even when
+   *bad_event is set.
+   igd_shard_buffers: device pointers (context-owned, valid until the next prepare) to the records
+   (uint4 {low 32 bits of the word, global index, tk, active mask}, grouped by owner in rank order,
+   trace order inside a group), the sync-stream global indices (u32) and events (16 B).
+   Exchange (caller): all-to-all of the record groups; all-gather of the sync streams concatenated
+   in rank order (= trace order).
+
+   Stage 2, igd_shard_detect: checks the words this rank owns.  d_records = the records received from
+   all ranks concatenated in source-rank order; d_sync_idx / d_sync_events = the global sync stream;
+   min_word = global minimum accessed word.  Device pointers are borrowed for the call.  Reports (global
+   indices) are read with igd_reports / igd_reports_device; the union over ranks is the single-GPU
+   report set (address-shard invariance).  flags: IGD_DETECT_TIMING or 0. */
+int igd_shard_prepare(igd_ctx* ctx, uint32_t nranks, uint64_t* counts, uint64_t* n_sync_stream,
+                      uint64_t* bad_event, uint64_t* word_minmax);
+int igd_shard_buffers(igd_ctx* ctx, void** d_records, void** d_sync_idx, void** d_sync_events);
+int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, const uint32_t* d_sync_idx,
+                     const void* d_sync_events, uint64_t n_sync_stream, uint64_t min_word, uint32_t flags,
+                     uint64_t* n_reports);
+
 /* Copy min(cap, total) reports, ascending by `cur` (at most one report per access, so the
    order is total), to host memory `host_out`; *n_written = number copied. */
 int igd_reports(igd_ctx* ctx, igd_report* host_out, uint64_t cap, uint64_t* n_written);

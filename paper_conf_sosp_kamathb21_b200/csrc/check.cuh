@@ -121,7 +121,8 @@ __device__ __noinline__ bool q_between(const uint4* __restrict__ desc, const u32
 
 struct Params {
     const u32* key;  // sorted word keys
-    const u64* val;  // sorted (trace index | tk << 32)
+    const void* val; // sorted payload: u64 (index | tk << 32), or uint4 {index, tk, mask, 0} (MV)
+    u64 wbase;       // smallest accessed word (reports rebuild the 64-bit word from the key)
     u32 n;           // number of accesses
     const igd_event* ev;
     Geo g;
@@ -177,6 +178,30 @@ __device__ __forceinline__ bool q_grid(const PP& P, u32 a, u32 b) {
 #define QF_BLK 8u
 #define QF_R1 16u
 
+// Sorted payload of one access: single GPU = u64 (trace index | tk << 32), the active mask is
+// gathered from the trace when needed; sharded = uint4 {index, tk, mask, 0} (the events of
+// other ranks are not resident).
+struct Acc {
+    u32 idx, tk, mask;
+};
+template <bool MV>
+__device__ __forceinline__ Acc acc_at(const void* val, u32 k) {
+    Acc a;
+    if (MV) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(val) + k);
+        a.idx = v.x;
+        a.tk = v.y;
+        a.mask = v.z;
+    } else {
+        const unsigned long long v = __ldg(reinterpret_cast<const unsigned long long*>(val) + k);
+        a.idx = (u32)v;
+        a.tk = (u32)(v >> 32);
+        a.mask = 0;
+    }
+    return a;
+}
+
+template <bool MV>
 __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
     __shared__ u32 s_tile;
     __shared__ u64 s_wagg[WARPS];
@@ -184,7 +209,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
     __shared__ u32 s_ready;
     __shared__ u32 s_qn;
     // queue of undecided accesses (SoA)
-    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_la[TILE], q_lt[TILE];
+    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_la[TILE], q_lt[TILE], q_k[TILE];
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     if (t == 0) {
@@ -198,21 +223,25 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
     const Geo g = P.g;
 
     // K: word key, V: trace index, Z: the event's tk word (tid | kind | scope), carried by the sort
-    u32 K[ITEMS], V[ITEMS], Z[ITEMS];
-    if (first + ITEMS <= P.n) {
+    u32 K[ITEMS], V[ITEMS], Z[ITEMS], M[ITEMS];
+    if (!MV && first + ITEMS <= P.n) {
         const uint4 k4 = __ldcs(reinterpret_cast<const uint4*>(P.key + first));
-        const uint4 v01 = __ldcs(reinterpret_cast<const uint4*>(P.val + first));
-        const uint4 v23 = __ldcs(reinterpret_cast<const uint4*>(P.val + first + 2));
+        const uint4 v01 = __ldcs(reinterpret_cast<const uint4*>(P.val) + first / 2);
+        const uint4 v23 = __ldcs(reinterpret_cast<const uint4*>(P.val) + first / 2 + 1);
         K[0] = k4.x; K[1] = k4.y; K[2] = k4.z; K[3] = k4.w;
         V[0] = v01.x; Z[0] = v01.y; V[1] = v01.z; Z[1] = v01.w;
         V[2] = v23.x; Z[2] = v23.y; V[3] = v23.z; Z[3] = v23.w;
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) M[j] = 0;
     } else {
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
-            const u64 v = (first + j < P.n) ? P.val[first + j] : 0ull;
-            K[j] = (first + j < P.n) ? P.key[first + j] : 0;
-            V[j] = (u32)v;
-            Z[j] = (u32)(v >> 32);
+            const bool in = first + j < P.n;
+            const Acc a = in ? acc_at<MV>(P.val, first + j) : Acc{0, 0, 0};
+            K[j] = in ? P.key[first + j] : 0;
+            V[j] = a.idx;
+            Z[j] = a.tk;
+            M[j] = a.mask;
         }
     }
 
@@ -222,9 +251,9 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
     u32 pZ = __shfl_up_sync(IGD_FULL, Z[ITEMS - 1], 1);
     if (lane == 0 && first > 0 && first - 1 < P.n) {
         pK = __ldg(P.key + first - 1);
-        const u64 v = __ldg(reinterpret_cast<const unsigned long long*>(P.val) + first - 1);
-        pV = (u32)v;
-        pZ = (u32)(v >> 32);
+        const Acc a = acc_at<MV>(P.val, first - 1);
+        pV = a.idx;
+        pZ = a.tk;
     }
 
     // per-access scan contributions
@@ -320,7 +349,6 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
         const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
         bool queue = false;
         u32 mdIdx = laIdx, p = laTid, mdKind = laKind, flags = 0;
-        const unsigned long long* val64 = reinterpret_cast<const unsigned long long*>(P.val);
         if (first + j < P.n && !st_head(contrib[j])) {
             const u32 lastW = st_lastW(before), as = st_as(before);
             CSTAT(0);
@@ -331,10 +359,10 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
                 }
                 if (kind == IGD_LD && lastW != first + j - 1) {  // md = last writer, further back
                     CSTAT(13);
-                    const u64 mv = __ldg(val64 + lastW);
-                    mdIdx = (u32)mv;
-                    p = (u32)(mv >> 32) & 0xFFFFFFu;
-                    mdKind = (u32)(mv >> 56) & 0xFu;
+                    const Acc mv = acc_at<MV>(P.val, lastW);
+                    mdIdx = mv.idx;
+                    p = mv.tk & 0xFFFFFFu;
+                    mdKind = (mv.tk >> 24) & 0xFu;
                 }
                 if (p == c) {  // P3: program order
                     CSTAT(2);
@@ -353,7 +381,8 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
                 // mask itself is gathered only for other partial masks
                 if (same_w && !(Z[j] >> 30)) CSTAT(5);
                 if (same_w && ((Z[j] >> 31) ||
-                               (!((Z[j] >> 30) & 1u) && ((ld_event(P.ev, i).w >> g.lane(p)) & 1u)))) {
+                               (!((Z[j] >> 30) & 1u) &&
+                                (((MV ? M[j] : ld_event(P.ev, i).w) >> g.lane(p)) & 1u)))) {
                     CSTAT(4);
                     break;
                 }
@@ -363,7 +392,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
                 if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
                     u32 lwTid = p;
                     if (kind != IGD_LD && lastW != first + j - 1)
-                        lwTid = (u32)(__ldg(val64 + lastW) >> 32) & 0xFFFFFFu;
+                        lwTid = acc_at<MV>(P.val, lastW).tk & 0xFFFFFFu;
                     if (g.block(lwTid) != bc) flags |= QF_R1;
                 }
                 queue = true;
@@ -383,6 +412,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
                 q_p[q] = p | (kind << 24) | (mdKind << 28);
                 q_la[q] = laIdx;
                 q_lt[q] = laTid;
+                q_k[q] = K[j];
             }
         }
         laIdx = i;
@@ -423,7 +453,8 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
             const unsigned long long slot = atomicAdd(P.rep_ctr, 1ull);
             if (slot < P.rep_cap) {
                 igd_report r;
-                r.addr = (ev_addr(ld_event(P.ev, i)) >> 2) << 2;
+                // full word from the 32-bit key: the accessed words span < 2^32 from wbase
+                r.addr = (P.wbase + (u32)(q_k[q] - (u32)P.wbase)) << 2;
                 r.cur = P.first_event + i;
                 r.prev = P.first_event + mdIdx;
                 r.type = (uint8_t)type;

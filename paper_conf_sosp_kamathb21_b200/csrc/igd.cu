@@ -17,7 +17,9 @@
 #include "common.cuh"
 #include "ingest.cuh"
 #include "sort.cuh"
+#include "shard.cuh"
 #include "sync.cuh"
+#include <vector>
 
 namespace {
 
@@ -58,6 +60,15 @@ struct igd_ctx {
     u64 rep_cap = 0;
     int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any (IGD_SORT_MODE)
     int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
+    // sharded mode: stage-1 outputs, stage-2 inputs
+    bool shard = false;
+    Buf sh_cnt, sh_obase, sh_send, sh_sidx_buf, sh_sev_buf;
+    u64 sh_send_n = 0, sh_sync_n = 0;
+    const void* sh_rec = nullptr;
+    u64 sh_nrec = 0;
+    const u32* sh_sidx = nullptr;
+    const void* sh_sev = nullptr;
+    u64 sh_ns = 0, sh_wbase = 0, sh_ntotal = 0;
     int last_acur = 0;  // buffer holding the sorted accesses of the last igd_detect (debug hooks)
     u64 last_nacc = 0;
     u64 n_reports = 0;
@@ -216,7 +227,11 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
             KTimer kt(ctx, cls, 2.0 * (4 + vbytes) * (double)n);  // read + write 4 B key and the value
             const unsigned gb = (unsigned)tiles;
             const size_t s8 = rsort::onesweep_smem<u64>(), s4 = rsort::onesweep_smem<u32>();
-            if (vbytes == 8) {
+            if (vbytes == 16) {
+                const size_t s16 = rsort::onesweep_smem<uint4>();
+                if (ctx->sort_mode == 0) rsort::k_onesweep<0, uint4><<<gb, rsort::THREADS, s16, ctx->stream>>>(pp);
+                else rsort::k_onesweep<1, uint4><<<gb, rsort::THREADS, s16, ctx->stream>>>(pp);
+            } else if (vbytes == 8) {
                 if (ctx->sort_mode == 0) rsort::k_onesweep<0, u64><<<gb, rsort::THREADS, s8, ctx->stream>>>(pp);
                 else rsort::k_onesweep<1, u64><<<gb, rsort::THREADS, s8, ctx->stream>>>(pp);
             } else {
@@ -247,16 +262,22 @@ static int scan_excl(igd_ctx* ctx, u32* data, u64 n) {
     return IGD_OK;
 }
 
+// The pipeline.  Single GPU: the trace is `ctx->events`.  Sharded (ctx->shard): the
+// synchronization side runs over the all-gathered sync stream (global timestamps in sh_sidx),
+// the access side over the records this rank received in the all-to-all.
 static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const igd_trace_desc& D = ctx->desc;
-    const u64 n = D.n_events;
+    const bool SH = ctx->shard;
+    const u64 n = SH ? ctx->sh_ntotal : D.n_events;               // timestamp domain [0, n)
+    const igd_event* src_ev = SH ? (const igd_event*)ctx->sh_sev : ctx->events;
+    const u64 n_src = SH ? ctx->sh_ns : D.n_events;                // events the ingest reads
     ctx->n_reports = 0;
     ctx->bad_event = 0;
     ctx->launches = 0;
     ctx->nk = 0;
     *n_out = 0;
     mark(ctx, 0);
-    if (n == 0) {
+    if (n == 0 || (n_src == 0 && (!SH || ctx->sh_nrec == 0))) {
         for (int s = 1; s <= IGD_N_STAGES; s++) mark(ctx, s);
         return IGD_OK;
     }
@@ -267,16 +288,18 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const int sms = sm_count(ctx);
 
     // ---------------- a1 + a2 + a4: ingest ----------------
-    const u64 in_tiles = (n + ingest::TILE - 1) / ingest::TILE;
+    const u64 in_tiles = (n_src + ingest::TILE - 1) / ingest::TILE;
     RET(ensure(ctx, ctx->stats, 8 * sizeof(u64)));
     RET(ensure(ctx, ctx->hist, 3 * 1024 * sizeof(u32)));
     RET(ensure(ctx, ctx->base, 4 * 256 * sizeof(u32)));
     RET(ensure(ctx, ctx->ctr, 64));
     RET(ensure(ctx, ctx->st_in_a, (in_tiles + 1) * sizeof(u32)));
     RET(ensure(ctx, ctx->st_in_s, (in_tiles + 1) * sizeof(u32)));
+    const u64 acc_cap = SH ? ctx->sh_nrec : D.n_events;
+    const int vbytes = SH ? 16 : 8;  // sorted payload: (index | tk) or {index, tk, mask, 0}
     for (int b = 0; b < 2; b++) {
-        RET(ensure(ctx, ctx->acc_k[b], n * sizeof(u32)));
-        RET(ensure(ctx, ctx->acc_v[b], n * sizeof(u64)));  // (trace index, tk) per access
+        RET(ensure(ctx, ctx->acc_k[b], acc_cap * sizeof(u32)));
+        RET(ensure(ctx, ctx->acc_v[b], acc_cap * vbytes));
     }
     u64 init[8] = {~0ull, 0, ~0ull, 0, 0, 0, 0, 0};
     memcpy(ctx->h_small, init, sizeof(init));
@@ -285,10 +308,12 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     CK(cudaMemsetAsync(ctx->st_in_a.p, 0, (in_tiles + 1) * sizeof(u32), ctx->stream));
     CK(cudaMemsetAsync(ctx->st_in_s.p, 0, (in_tiles + 1) * sizeof(u32), ctx->stream));
     ingest::Params ip;
-    ip.ev = ctx->events;
-    ip.n = n;
+    memset(&ip, 0, sizeof(ip));
+    ip.ev = src_ev;
+    ip.n = n_src;
     ip.g = g;
     ip.ks = ks;
+    ip.gidx = SH ? ctx->sh_sidx : nullptr;
     ip.tile_acc = P_<u32>(ctx->st_in_a);
     ip.tile_sync = P_<u32>(ctx->st_in_s);
     ip.hist_acc = P_<u32>(ctx->hist);
@@ -297,9 +322,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     ip.n_tiles = (u32)in_tiles;
     int occ = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ingest::k_ingest<0>, ingest::THREADS, 0);
-    const u64 grid = std::min<u64>((u64)sms * (occ > 0 ? occ : 1), in_tiles);
-    {
-        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n);  // pass 0 reads every event
+    const u64 grid = std::max<u64>(1, std::min<u64>((u64)sms * (occ > 0 ? occ : 1), in_tiles));
+    if (n_src > 0) {
+        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n_src);  // pass 0 reads every event
         ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
     }
     CK(cudaGetLastError());
@@ -309,34 +334,45 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 2 * 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaMemcpyAsync(&ctx->h_small[0], P_<u32>(ctx->st_in_a) + in_tiles, sizeof(u32), cudaMemcpyDeviceToHost,
                        ctx->stream));
-    CK(cudaMemcpyAsync(&ctx->h_small[1], P_<u32>(ctx->st_in_s) + in_tiles, sizeof(u32), cudaMemcpyDeviceToHost,
-                       ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     if (ctx->h_stats[2] != ~0ull) {
         ctx->bad_event = ctx->h_stats[2];
         ctx->err = "invalid event at index " + std::to_string(ctx->bad_event);
         return IGD_ETRACE;
     }
-    const u64 n_acc = ctx->h_small[0] & 0xFFFFFFFFull, n_sync = ctx->h_stats[4];
+    const u64 n_acc = SH ? ctx->sh_nrec : (ctx->h_small[0] & 0xFFFFFFFFull);
+    const u64 n_sync = ctx->h_stats[4];
     const u64 n_lock = ctx->h_stats[5];
+    const u64 wbase = SH ? ctx->sh_wbase : ctx->h_stats[0];
     if (n_sync + 64 > 0xFFFFFFFFull) return IGD_ETOOBIG;  // 32-bit record positions
+    if (!SH && n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32)) {
+        ctx->err = "accessed word range spans >= 2^32 words";
+        return IGD_ETOOBIG;
+    }
     if (ctx->sync_cap < n_sync) ctx->sync_cap = n_sync + n_sync / 8 + 4096;
     for (int b = 0; b < 2; b++) {
         // +64 entries: the check's 32-byte timestamp probes may read past the last list
         RET(ensure(ctx, ctx->syn_k[b], (ctx->sync_cap + 64) * sizeof(u32)));
         RET(ensure(ctx, ctx->syn_v[b], (ctx->sync_cap + 64) * sizeof(u32)));
     }
-    ip.acc_key = P_<u32>(ctx->acc_k[0]);
-    ip.acc_val = P_<u64>(ctx->acc_v[0]);
+    ip.acc_key = SH ? nullptr : P_<u32>(ctx->acc_k[0]);
+    ip.acc_val = SH ? nullptr : P_<u64>(ctx->acc_v[0]);
     ip.sync_key = P_<u32>(ctx->syn_k[0]);
     ip.sync_val = P_<u32>(ctx->syn_v[0]);
     ip.sync_cap = ctx->sync_cap;
-    {
+    if (n_src > 0) {
         // pass 1 re-reads the events and writes the (key, value) records
-        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
+        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n_src + (SH ? 0.0 : 12.0 * (double)n_acc) + 8.0 * (double)n_sync);
         ingest::k_ingest<1><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
     }
     CK(cudaGetLastError());
+    if (SH && n_acc > 0) {
+        // received records {key, index, tk, mask} -> sort keys + 16-byte payload
+        KTimer kt(ctx, KC_INGEST, 36.0 * (double)n_acc);
+        const unsigned sb = (unsigned)std::min<u64>((n_acc + 255) / 256, (u64)sms * 16);
+        shard::k_split_records<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
+                                                          P_<u32>(ctx->acc_k[0]), P_<uint4>(ctx->acc_v[0]));
+    }
     if (n_acc > 0) {
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digit histograms
         const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
@@ -346,11 +382,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     mark(ctx, 1);
-    if (n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32)) {
-        ctx->err = "accessed word range spans >= 2^32 words";
-        return IGD_ETOOBIG;
-    }
-    if (n_sync >= 0xFFFFFFFFull) return IGD_ETOOBIG;
     u32 h_hist_acc[1024], h_hist_sync[1024];
     memcpy(h_hist_acc, ctx->h_hist, sizeof(h_hist_acc));
     memcpy(h_hist_sync, ctx->h_hist + 1024, sizeof(h_hist_sync));
@@ -401,7 +432,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         CK(cudaMemsetAsync(ctx->wcnt.p, 0, ((u64)g.W + 1) * sizeof(u32), ctx->stream));
         CK(cudaMemsetAsync(ctx->tcnt.p, 0, ((u64)g.T + 1) * sizeof(u32), ctx->stream));
         syncx::LockParams lp;
-        lp.ev = ctx->events;
+        memset(&lp, 0, sizeof(lp));
+        lp.ev = src_ev;
+        lp.gidx = SH ? ctx->sh_sidx : nullptr;
+        lp.gn = (u32)n_src;
         lp.g = g;
         lp.ks = ks;
         lp.off = P_<u32>(ctx->off);
@@ -409,10 +443,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lp.switch_ts = P_<u32>(ctx->sw);
         lp.wcnt = P_<u32>(ctx->wcnt);
         lp.tcnt = P_<u32>(ctx->tcnt);
-        lp.woff = nullptr;
-        lp.toff = nullptr;
-        lp.wpts = nullptr;
-        lp.tpts = nullptr;
         const unsigned lblocks = (unsigned)(((u64)g.W * 32 + 255) / 256);
         {
             KTimer kt(ctx, KC_LOCK, 0);
@@ -448,9 +478,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     mark(ctx, 3);
     // ---------------- a5: accesses sorted by word, stable ----------------
     int acur = 0;
-    RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur, 8));
+    RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur,
+                   vbytes));
     ctx->last_acur = acur;
-    ctx->last_nacc = n_acc;
+    ctx->last_nacc = SH ? 0 : n_acc;
     mark(ctx, 4);
     // ---------------- a6: segmented shadow pass + check ----------------
     if (ctx->rep_cap == 0) ctx->rep_cap = 1 << 20;
@@ -459,14 +490,16 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         const u64 tiles = (n_acc + check::TILE - 1) / check::TILE;
         for (int attempt = 0;; attempt++) {
             RET(ensure(ctx, ctx->rep_raw, ctx->rep_cap * sizeof(igd_report)));
-            RET(ensure(ctx, ctx->rep_ctr, sizeof(u64)));
+            RET(ensure(ctx, ctx->rep_ctr, 2 * sizeof(u64)));
             RET(ensure(ctx, ctx->status, tiles * sizeof(u64)));
             CK(cudaMemsetAsync(ctx->status.p, 0, tiles * sizeof(u64), ctx->stream));
             CK(cudaMemsetAsync(ctx->ctr.p, 0, sizeof(u32), ctx->stream));
             CK(cudaMemsetAsync(ctx->rep_ctr.p, 0, sizeof(u64), ctx->stream));
             check::Params cp;
+            memset(&cp, 0, sizeof(cp));
             cp.key = P_<u32>(ctx->acc_k[acur]);
-            cp.val = P_<u64>(ctx->acc_v[acur]);
+            cp.val = ctx->acc_v[acur].p;
+            cp.wbase = wbase;
             cp.n = (u32)n_acc;
             cp.ev = ctx->events;
             cp.g = g;
@@ -486,9 +519,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.first_event = 0;
             cp.debug_stop = ctx->check_stop;
             {
-                // 4 B key + 4 B value streamed, one 16-B event gathered per access
-                KTimer kt(ctx, KC_CHECK, 12.0 * (double)n_acc);  // 4 B key + 8 B (index, tk) streamed
-                check::k_check<<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+                // key + payload streamed (12 or 20 bytes per access)
+                KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
+                if (SH) check::k_check<true><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+                else check::k_check<false><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
             }
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
@@ -546,6 +580,81 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     return IGD_OK;
 }
 
+// ---------------- sharded mode, stage 1: partition one rank's chunk ----------------
+static int shard_prepare_impl(igd_ctx* ctx, u32 P, u64* counts, u64* n_sync_stream, u64* bad, u64* minmax) {
+    const igd_trace_desc& D = ctx->desc;
+    const u64 n = D.n_events;
+    Geo g;
+    geo_init(g, D.n_blocks, D.block_dim);
+    KeySpace ks;
+    ks.init(g);
+    const int sms = sm_count(ctx);
+    const u64 tiles = (n + shard::TILE - 1) / shard::TILE;
+    const u64 row = tiles + 1;
+    RET(ensure(ctx, ctx->stats, 8 * sizeof(u64)));
+    RET(ensure(ctx, ctx->sh_cnt, (P + 1) * row * sizeof(u32)));
+    RET(ensure(ctx, ctx->sh_obase, (P + 1) * sizeof(u64)));
+    u64 init[8] = {~0ull, 0, ~0ull, 0, 0, 0, 0, 0};
+    memcpy(ctx->h_small, init, sizeof(init));
+    CK(cudaMemcpyAsync(ctx->stats.p, ctx->h_small, sizeof(init), cudaMemcpyHostToDevice, ctx->stream));
+    CK(cudaMemsetAsync(ctx->sh_cnt.p, 0, (P + 1) * row * sizeof(u32), ctx->stream));
+    shard::Params sp;
+    memset(&sp, 0, sizeof(sp));
+    sp.ev = ctx->events;
+    sp.n = n;
+    sp.first = D.first_event;
+    sp.g = g;
+    sp.ks = ks;
+    sp.P = P;
+    sp.n_tiles = (u32)tiles;
+    sp.cnt = P_<u32>(ctx->sh_cnt);
+    sp.stats = P_<u64>(ctx->stats);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, shard::k_shard<0>, shard::THREADS, 0);
+    const u64 grid = std::max<u64>(1, std::min<u64>((u64)sms * (occ > 0 ? occ : 1), tiles));
+    if (n > 0) {
+        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n);
+        shard::k_shard<0><<<(unsigned)grid, shard::THREADS, 0, ctx->stream>>>(sp);
+    }
+    CK(cudaGetLastError());
+    for (u32 o = 0; o <= P; o++) RET(scan_excl(ctx, P_<u32>(ctx->sh_cnt) + (u64)o * row, row));
+    std::vector<u32> tot(P + 1);
+    for (u32 o = 0; o <= P; o++)
+        CK(cudaMemcpyAsync(&tot[o], P_<u32>(ctx->sh_cnt) + (u64)o * row + tiles, sizeof(u32), cudaMemcpyDeviceToHost,
+                           ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_stats, ctx->stats.p, 8 * sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    bad[0] = ctx->h_stats[2];
+    minmax[0] = ctx->h_stats[0];
+    minmax[1] = ctx->h_stats[1];
+    std::vector<u64> ob(P + 1, 0);
+    u64 nrec = 0;
+    for (u32 o = 0; o < P; o++) {
+        counts[o] = tot[o];
+        ob[o] = nrec;
+        nrec += tot[o];
+    }
+    *n_sync_stream = tot[P];
+    ctx->sh_send_n = nrec;
+    ctx->sh_sync_n = tot[P];
+    RET(ensure(ctx, ctx->sh_send, (nrec + 1) * sizeof(uint4)));
+    RET(ensure(ctx, ctx->sh_sidx_buf, ((u64)tot[P] + 1) * sizeof(u32)));
+    RET(ensure(ctx, ctx->sh_sev_buf, ((u64)tot[P] + 1) * sizeof(uint4)));
+    if (bad[0] != ~0ull) return IGD_OK;  // the caller reduces the error across ranks
+    CK(cudaMemcpyAsync(ctx->sh_obase.p, ob.data(), (P + 1) * sizeof(u64), cudaMemcpyHostToDevice, ctx->stream));
+    sp.obase = P_<u64>(ctx->sh_obase);
+    sp.send = P_<uint4>(ctx->sh_send);
+    sp.sync_idx = P_<u32>(ctx->sh_sidx_buf);
+    sp.sync_ev = P_<uint4>(ctx->sh_sev_buf);
+    if (n > 0) {
+        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n + 16.0 * (double)nrec + 20.0 * (double)tot[P]);
+        shard::k_shard<1><<<(unsigned)grid, shard::THREADS, 0, ctx->stream>>>(sp);
+    }
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(ctx->stream));
+    return IGD_OK;
+}
+
 // ================================ C ABI =====================================================
 extern "C" {
 
@@ -574,6 +683,10 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
                          (int)rsort::onesweep_smem<u64>());
     cudaFuncSetAttribute(rsort::k_onesweep<1, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)rsort::onesweep_smem<u64>());
+    cudaFuncSetAttribute(rsort::k_onesweep<0, uint4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<uint4>());
+    cudaFuncSetAttribute(rsort::k_onesweep<1, uint4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<uint4>());
     cudaFuncSetAttribute(rsort::k_onesweep<0, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)rsort::onesweep_smem<u32>());
     cudaFuncSetAttribute(rsort::k_onesweep<1, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -602,10 +715,12 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
     if ((u64)desc->n_blocks * desc->block_dim > (1ull << 24)) return IGD_EINVAL;
     if (desc->n_events > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;
     if (desc->n_events > 0 && !events) return IGD_EINVAL;
-    if (desc->first_event != 0 || (desc->n_events_total != 0 && desc->n_events_total != desc->n_events)) {
-        ctx->err = "single-rank build: first_event must be 0 and n_events_total == n_events";
+    if (desc->n_events_total != 0 && desc->first_event + desc->n_events > desc->n_events_total) {
+        ctx->err = "first_event + n_events exceeds n_events_total";
         return IGD_EINVAL;
     }
+    if ((desc->n_events_total ? desc->n_events_total : desc->n_events) > 0xFFFFFFFFull - 2 * rsort::TILE)
+        return IGD_ETOOBIG;
     cudaSetDevice(ctx->device);
     ctx->desc = *desc;
     ctx->loaded = false;
@@ -622,13 +737,67 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
     return IGD_OK;
 }
 
+static void collect_timing(igd_ctx* ctx);
+
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     if (!ctx || !n_reports_global) return IGD_EINVAL;
     if (!ctx->loaded) return IGD_ESTATE;
+    if (ctx->desc.first_event != 0 ||
+        (ctx->desc.n_events_total != 0 && ctx->desc.n_events_total != ctx->desc.n_events)) {
+        ctx->err = "igd_detect checks a whole trace; a rank's chunk goes through igd_shard_*";
+        return IGD_EINVAL;
+    }
     cudaSetDevice(ctx->device);
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
+    ctx->shard = false;
     int rc = detect_impl(ctx, n_reports_global);
-    if (rc == IGD_OK && ctx->timing) {
+    if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
+    return rc;
+}
+
+int igd_shard_prepare(igd_ctx* ctx, uint32_t nranks, uint64_t* counts, uint64_t* n_sync_stream,
+                      uint64_t* bad_event, uint64_t* word_minmax) {
+    if (!ctx || !counts || !n_sync_stream || !bad_event || !word_minmax) return IGD_EINVAL;
+    if (nranks == 0 || nranks > (uint32_t)shard::MAXP) return IGD_EINVAL;
+    if (!ctx->loaded) return IGD_ESTATE;
+    cudaSetDevice(ctx->device);
+    ctx->launches = 0;
+    ctx->nk = 0;
+    return shard_prepare_impl(ctx, nranks, counts, n_sync_stream, bad_event, word_minmax);
+}
+
+int igd_shard_buffers(igd_ctx* ctx, void** d_records, void** d_sync_idx, void** d_sync_events) {
+    if (!ctx || !d_records || !d_sync_idx || !d_sync_events) return IGD_EINVAL;
+    *d_records = ctx->sh_send.p;
+    *d_sync_idx = ctx->sh_sidx_buf.p;
+    *d_sync_events = ctx->sh_sev_buf.p;
+    return IGD_OK;
+}
+
+int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, const uint32_t* d_sync_idx,
+                     const void* d_sync_events, uint64_t n_sync_stream, uint64_t min_word, uint32_t flags,
+                     uint64_t* n_reports) {
+    if (!ctx || !n_reports) return IGD_EINVAL;
+    if ((n_records && !d_records) || (n_sync_stream && (!d_sync_idx || !d_sync_events))) return IGD_EINVAL;
+    if (!ctx->loaded) return IGD_ESTATE;
+    cudaSetDevice(ctx->device);
+    ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
+    ctx->shard = true;
+    ctx->sh_rec = d_records;
+    ctx->sh_nrec = n_records;
+    ctx->sh_sidx = d_sync_idx;
+    ctx->sh_sev = d_sync_events;
+    ctx->sh_ns = n_sync_stream;
+    ctx->sh_wbase = min_word;
+    ctx->sh_ntotal = ctx->desc.n_events_total ? ctx->desc.n_events_total : ctx->desc.n_events;
+    int rc = detect_impl(ctx, n_reports);
+    ctx->shard = false;
+    if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
+    return rc;
+}
+
+static void collect_timing(igd_ctx* ctx) {
+    {
         cudaEventSynchronize(ctx->ev[8]);
         for (int s = 0; s < IGD_N_STAGES - 1; s++) cudaEventElapsedTime(&ctx->stage_ms[s], ctx->ev[s], ctx->ev[s + 1]);
         cudaEventElapsedTime(&ctx->stage_ms[IGD_N_STAGES - 1], ctx->ev[0], ctx->ev[7]);
@@ -645,7 +814,6 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
             ctx->cls_bytes[ctx->kcls[q]] += ctx->kbytes[q];
         }
     }
-    return rc;
 }
 
 int igd_reports(igd_ctx* ctx, igd_report* host_out, uint64_t cap, uint64_t* n_written) {
@@ -699,7 +867,8 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->sw,       &ctx->wcnt,
                   &ctx->tcnt,
                   &ctx->wpts,         &ctx->tpts,     &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
-                  &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist};
+                  &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
+                  &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf};
     for (Buf* b : all) buf_free(ctx, *b);
     cudaStreamSynchronize(ctx->stream);
     cudaFreeHost(ctx->h_stats);

@@ -32,6 +32,7 @@ struct Params {
     u32* sync_key;
     u32* sync_val;
     u64 sync_cap;  // records beyond capacity are counted, not written (host re-runs)
+    const u32* gidx;  // sharded mode: global timestamp of each input event (else its position)
     u32* tile_acc;   // [n_tiles + 1] pass 0: access records per tile; scanned to bases
     u32* tile_sync;  // [n_tiles + 1] pass 0: sync records per tile; scanned to bases
     u32* hist_acc;   // [4][256]
@@ -272,7 +273,7 @@ __global__ void __launch_bounds__(THREADS, 2) k_ingest(Params P) {
             const u32 f = dv[j].flags;
             const u32 wo = s_woff[j][warp];
             const u32 ex = excl[j];
-            if (f & 1u) {
+            if ((f & 1u) && P.acc_key) {
                 const u64 pos = ba + (wo & 0xFFFFu) + (ex & 0xFFFFu);
                 P.acc_key[pos] = dv[j].key;
                 P.acc_val[pos] = (base + (u64)j * THREADS + tid) | ((u64)dv[j].tk << 32);
@@ -280,7 +281,8 @@ __global__ void __launch_bounds__(THREADS, 2) k_ingest(Params P) {
             const u32 ns = (f >> 1) & 3u;
             if (ns) {
                 const u64 pos = bs + (wo >> 16) + (ex >> 16);
-                const u32 ts = (u32)(base + (u64)j * THREADS + tid);
+                const u64 i = base + (u64)j * THREADS + tid;
+                const u32 ts = P.gidx ? __ldg(P.gidx + i) : (u32)i;
                 if (pos + ns <= P.sync_cap) {
                     P.sync_key[pos] = dv[j].s0;
                     P.sync_val[pos] = ts;

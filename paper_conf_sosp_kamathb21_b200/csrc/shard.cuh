@@ -1,0 +1,167 @@
+// shard.cuh -- multi-GPU partitioning of one rank's trace chunk.
+//
+// Rank r holds the contiguous global range [first, first + n).  Words are hash-sharded:
+// owner(word) = fmix32(low 32 bits of the word) % P.  For the exchange each rank produces
+//   * its access records grouped by owner, each group in trace order:
+//       uint4 {key = low 32 bits of the word, global index, tk (+ mask summaries), active mask}
+//   * its synchronization stream (fences, barriers, grid syncs, CAS/EXCH), in trace order:
+//       global index + the raw 16-byte event,
+// with a stable count / scan / write structure like the ingest's.  After an all-to-all of the
+// records and an all-gather of the sync streams (torch.distributed over NCCL, issued by the
+// host binding) every rank rebuilds identical synchronization tables and checks the words it
+// owns: the union over ranks is exactly the single-GPU report set (address-shard invariance,
+// SURVEY 8(c) C.7 5(b)).
+#pragma once
+#include "common.cuh"
+#include "ingest.cuh"
+
+namespace shard {
+
+constexpr int THREADS = 256;
+constexpr int WARPS = THREADS / 32;
+constexpr int ITEMS = 8;
+constexpr int TILE = THREADS * ITEMS;
+constexpr int MAXP = 16;
+
+__device__ __forceinline__ u32 fmix32(u32 h) {
+    h ^= h >> 16;
+    h *= 0x85ebca6bu;
+    h ^= h >> 13;
+    h *= 0xc2b2ae35u;
+    h ^= h >> 16;
+    return h;
+}
+
+struct Params {
+    const igd_event* ev;
+    u64 n;          // events in this chunk
+    u64 first;      // global index of ev[0]
+    Geo g;
+    KeySpace ks;
+    u32 P;          // ranks (owners), <= MAXP
+    u32 n_tiles;
+    u32* cnt;       // [(P + 1) * (n_tiles + 1)]: row o < P = records for owner o per tile, row P =
+                    // sync-stream events per tile; scanned in place per row between the passes
+    const u64* obase;  // [P + 1] start of each owner's region in `send`; [P] unused
+    uint4* send;
+    u32* sync_idx;
+    uint4* sync_ev;
+    u64* stats;     // [0] min word, [1] max word, [2] first bad global index
+};
+
+template <int PASS>
+__global__ void __launch_bounds__(THREADS, 2) k_shard(Params P) {
+    __shared__ u32 s_wc[ITEMS][WARPS][MAXP + 1];  // per (item, warp, destination) counts, then offsets
+    const u32 tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const u32 lt = lanemask_lt();
+    const Geo g = P.g;
+    const KeySpace ks = P.ks;
+    const u32 NP = P.P;
+    u64 wmin = ~0ull, wmax = 0, bad = ~0ull;
+
+    for (u32 tile = blockIdx.x; tile < P.n_tiles; tile += gridDim.x) {
+        const u64 base = (u64)tile * TILE;
+        uint4 e[ITEMS];
+        u32 dst[ITEMS];  // owner for an access record; the sync stream uses bit 31 (both for CAS/EXCH)
+        u32 tk[ITEMS], rk[ITEMS], srk[ITEMS];
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const u64 i = base + (u64)j * THREADS + tid;
+            e[j] = (i < P.n) ? ld_event_stream(P.ev, i) : make_uint4(0, 0, 0, 0);
+            dst[j] = 0;
+            tk[j] = 0;
+            if (i < P.n) {
+                const ingest::Dec d = ingest::decode(e[j], g, ks);
+                if (d.flags & 16u) {
+                    bad = min(bad, P.first + i);
+                } else {
+                    const u32 kind = ev_kind(e[j]);
+                    if (d.flags & 1u) {
+                        dst[j] = 0x100u | (NP == 1 ? 0u : fmix32(d.key) % NP);
+                        tk[j] = d.tk;
+                        const u64 word = ev_addr(e[j]) >> 2;
+                        wmin = min(wmin, word);
+                        wmax = max(wmax, word);
+                    }
+                    if (kind >= IGD_FENCE || kind == IGD_CAS || kind == IGD_EXCH) dst[j] |= 0x80000000u;
+                }
+            }
+        }
+        // per item: warp counts and lane ranks per destination (owners, then the sync stream)
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            for (u32 o = 0; o <= NP; o++) {
+                const bool mine = (o < NP) ? ((dst[j] & 0x1FFu) == (0x100u | o)) : (dst[j] >> 31) != 0;
+                const u32 bal = __ballot_sync(IGD_FULL, mine);
+                if (mine) {
+                    if (o < NP) rk[j] = __popc(bal & lt);
+                    else srk[j] = __popc(bal & lt);
+                }
+                if (lane == 0) s_wc[j][warp][o] = __popc(bal);
+            }
+        }
+        __syncthreads();
+        if (PASS == 0) {
+            for (u32 o = tid; o <= NP; o += THREADS) {
+                u32 s = 0;
+                for (int j = 0; j < ITEMS; j++)
+                    for (int w = 0; w < WARPS; w++) s += s_wc[j][w][o];
+                P.cnt[(u64)o * (P.n_tiles + 1) + tile] = s;
+            }
+            __syncthreads();
+            continue;
+        }
+        // exclusive offsets in (item, warp) order per destination
+        for (u32 o = tid; o <= NP; o += THREADS) {
+            u32 s = 0;
+            for (int j = 0; j < ITEMS; j++)
+                for (int w = 0; w < WARPS; w++) {
+                    const u32 c = s_wc[j][w][o];
+                    s_wc[j][w][o] = s;
+                    s += c;
+                }
+        }
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const u64 i = base + (u64)j * THREADS + tid;
+            if (i >= P.n) continue;
+            const u32 gi = (u32)(P.first + i);
+            if (dst[j] & 0x100u) {
+                const u32 o = dst[j] & 0xFFu;
+                const u64 pos = P.obase[o] + P.cnt[(u64)o * (P.n_tiles + 1) + tile] + s_wc[j][warp][o] + rk[j];
+                const u32 key = (e[j].x >> 2) | (e[j].y << 30);
+                P.send[pos] = make_uint4(key, gi, tk[j], e[j].w);
+            }
+            if (dst[j] >> 31) {
+                const u64 pos = (u64)P.cnt[(u64)NP * (P.n_tiles + 1) + tile] + s_wc[j][warp][NP] + srk[j];
+                P.sync_idx[pos] = gi;
+                P.sync_ev[pos] = e[j];
+            }
+        }
+        __syncthreads();
+    }
+    if (PASS != 0) return;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        wmin = min(wmin, __shfl_xor_sync(IGD_FULL, wmin, o));
+        wmax = max(wmax, __shfl_xor_sync(IGD_FULL, wmax, o));
+        bad = min(bad, __shfl_xor_sync(IGD_FULL, bad, o));
+    }
+    if (lane == 0) {
+        if (wmin != ~0ull) atomicMin((unsigned long long*)&P.stats[0], (unsigned long long)wmin);
+        if (wmin != ~0ull) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
+        if (bad != ~0ull) atomicMin((unsigned long long*)&P.stats[2], (unsigned long long)bad);
+    }
+}
+
+// Received records (uint4 {key, idx, tk, mask}) -> sort keys + 16-byte payload.
+__global__ void k_split_records(const uint4* __restrict__ rec, u32 n, u32* __restrict__ keys, uint4* __restrict__ vals) {
+    for (u32 i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        const uint4 r = __ldcs(rec + i);
+        keys[i] = r.x;
+        vals[i] = make_uint4(r.y, r.z, r.w, 0u);
+    }
+}
+
+}  // namespace shard

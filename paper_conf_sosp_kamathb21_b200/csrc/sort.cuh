@@ -245,7 +245,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
             const u32 i = wbase + j * 32 + lane;
-            val[j] = i < P.n ? __ldcs(vin + i) : (VT)0;
+            val[j] = i < P.n ? __ldcs(vin + i) : VT{};
         }
     }
     __syncthreads();

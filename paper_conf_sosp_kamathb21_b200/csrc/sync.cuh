@@ -88,7 +88,22 @@ struct LockParams {
     const u32* toff;      // [T+1] (pass 1)
     u64* wpts;            // warp change points  (ts << 16 | bloom)
     u64* tpts;            // thread change points
+    const u32* gidx;      // sharded mode: global timestamps of the events in `ev` (sorted), else NULL
+    u32 gn;
 };
+
+// The event with timestamp ts: ev[ts] on one GPU; in sharded mode `ev` is the all-gathered
+// synchronization stream and its position is found by binary search on the timestamps.
+__device__ __forceinline__ uint4 event_at(const LockParams& P, u32 ts) {
+    if (!P.gidx) return ld_event(P.ev, ts);
+    u32 lo = 0, hi = P.gn;
+    while (lo < hi) {
+        const u32 mid = (lo + hi) >> 1;
+        if (__ldg(P.gidx + mid) < ts) lo = mid + 1;
+        else hi = mid;
+    }
+    return ld_event(P.ev, lo);
+}
 
 // One warp per traced warp.  WRITE = false: count change points; true: write them.
 template <bool WRITE>
@@ -147,7 +162,7 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
             g_lo++;
             g_next = (g_lo < g_hi) ? __ldg(P.sts + g_lo) : IGD_NONE32;
         } else if (ts == lk_next) {
-            const uint4 e = ld_event(P.ev, ts);
+            const uint4 e = event_at(P, ts);
             const u32 kind = ev_kind(e), s = norm_scope(ev_scope(e));
             const u32 h = lock_h18(ev_addr(e) >> 2);
             const u32 el = P.g.lane(ev_tid(e));
@@ -175,7 +190,7 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
             const u32 owner = __ffs(__ballot_sync(IGD_FULL, my_next == ts)) - 1;
             u32 s = 0;
             if (lane == owner) {
-                s = norm_scope(ev_scope(ld_event(P.ev, ts)));
+                s = norm_scope(ev_scope(event_at(P, ts)));
                 f_lo++;
                 my_next = (f_lo < f_hi) ? __ldg(P.sts + f_lo) : IGD_NONE32;
             }

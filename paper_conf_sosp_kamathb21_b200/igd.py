@@ -71,6 +71,13 @@ def load_library(build_if_missing: bool = True):
     lib.igd_kernel_stats.argtypes = [vp, i32, ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(u32),
                                      ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_double)]
     lib.igd_kernel_stats.restype = i32
+    lib.igd_shard_prepare.argtypes = [vp, u32, ctypes.POINTER(u64), ctypes.POINTER(u64), ctypes.POINTER(u64),
+                                      ctypes.POINTER(u64)]
+    lib.igd_shard_prepare.restype = i32
+    lib.igd_shard_buffers.argtypes = [vp, ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp)]
+    lib.igd_shard_buffers.restype = i32
+    lib.igd_shard_detect.argtypes = [vp, vp, u64, vp, vp, u64, u64, u32, ctypes.POINTER(u64)]
+    lib.igd_shard_detect.restype = i32
     lib.igd_ctx_destroy.argtypes = [vp]
     lib.igd_ctx_destroy.restype = None
     lib.igd_strerror.argtypes = [i32]
