@@ -146,6 +146,113 @@ def run_reference(args, fam, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def run_sharded(args, fam, rank, world, local):
+    """N GPUs (one process each): the trace is split into contiguous chunks, words are hash-sharded
+    and exchanged with NCCL all-to-all; sync streams all-gathered.  The same global
+    trace for every N (strong scaling); each rank generates only its chunk."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sosp_kamathb21_b200 as igd
+    import tracegen.families as F
+    from paper_conf_sosp_kamathb21_b200 import dist as D
+
+    torch.cuda.set_device(local % torch.cuda.device_count())
+    dev_index = torch.cuda.current_device()
+    if world == 1:  # --sharded on one GPU: a one-rank process group
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", str(29500 + os.getpid() % 1000))
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", "1")
+    if not dist.is_initialized():
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev_index))
+        else:
+            dist.init_process_group(args.backend)
+    comm = D.TorchComm()
+    t0 = time.time()
+    plan = F.Plan(fam, args.events or None)
+    n, nb, bd = plan.n_events, plan.n_blocks, plan.block_dim
+    lo, cnt = D.chunk_bounds(n, world, rank)
+    host = np.empty(cnt, igd.EVENT_DTYPE)
+    plan.fill(lo, cnt, out=host, threads=args.threads)
+    ledger_n = len(plan.ledger())
+    plan.close()
+    if rank == 0:
+        log(f"[bench] {F.FAMILY_NAMES[fam]}: {n} events over {world} ranks, chunk {cnt}, {time.time() - t0:.1f}s")
+    cudart = torch.cuda.cudart()
+    pinned = cudart.cudaHostRegister(host.ctypes.data, host.nbytes, 0) == 0
+    chunk = torch.from_numpy(host.view(np.uint8)).to(f"cuda:{dev_index}")
+    det = igd.Detector(dev_index)
+    stage = D.GpuStage(det)
+    for _ in range(args.warmup):
+        stage.load(chunk, lo, n, nb, bd)
+        rep = D.sharded_detect(stage, comm)
+    clocks = ClockSampler(dev_index)
+    clocks.start()
+    dist.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    kstats, launches = {}, 0
+    e0.record(det.stream)
+    for _ in range(args.steps):
+        stage.load(chunk, lo, n, nb, bd)
+        rep = D.sharded_detect(stage, comm, timing=True)
+        launches += det.launch_count()
+        for k, (c, ms_, b) in det.kernel_stats().items():
+            c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
+            kstats[k] = (c0 + c, m0 + ms_, b0 + b)
+    e1.record(det.stream)
+    torch.cuda.synchronize()
+    dist.barrier()
+    clk = clocks.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    ms = comm.allreduce_u64(int(ms * 1e6), "max", f"cuda:{dev_index}") / 1e6  # slowest rank
+    value = n / (ms / 1e3) / 1e9
+    # end to end: host chunk -> library H2D -> sharded check -> reports on the host
+    del chunk
+    torch.cuda.empty_cache()
+    e2e_times = []
+    for s in range(0 if args.no_e2e else args.e2e_steps + 1):
+        dist.barrier()
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        stage.load(host, lo, n, nb, bd)
+        out = D.sharded_detect(stage, comm)
+        torch.cuda.synchronize()
+        if s > 0:
+            e2e_times.append(time.perf_counter() - t)
+    e2e_s = sum(e2e_times) / len(e2e_times) if e2e_times else float("inf")
+    e2e_s = comm.allreduce_u64(int(e2e_s * 1e9) if e2e_times else 1 << 62, "max", f"cuda:{dev_index}") / 1e9
+    if pinned:
+        cudart.cudaHostUnregister(host.ctypes.data)
+    peak, peak_kind = peaks()
+    dom = max(kstats, key=lambda k: kstats[k][1])
+    c, kms, kbytes = kstats[dom]
+    achieved = kbytes / (kms / 1e3) / 1e9 if kms > 0 else 0.0
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
+                           "reports": int(len(rep)), "ledger_reports": ledger_n,
+                           "l2": "inputs larger than L2 (no flush)",
+                           "parallelism": f"{world} ranks: contiguous trace chunks, words hash-sharded "
+                                          f"(fmix32 % P), NCCL all-to-all + all-gather"},
+                "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                             "frac": achieved / peak, "peak_source": peak_kind, "traffic": None,
+                             "launches_per_step": c / args.steps, "rank": 0},
+                "cpu_baseline": None,
+                "e2e": {"value": n / e2e_s / 1e9 if e2e_times else None, "unit": "G events/s",
+                        "h2d_bytes_per_step": n * 16, "d2h_bytes_per_step": int(len(rep)) * 32 * world,
+                        "ms_per_step": e2e_s * 1e3},
+                "gpu_launches": launches, "clocks": clk}
+        print(json.dumps(line), flush=True)
+    det.close()
+    dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -159,6 +266,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer run (profiling)")
     ap.add_argument("--threads", type=int, default=0, help="generator threads (0 = all cores)")
+    ap.add_argument("--sharded", action="store_true", help="use the multi-GPU path even at N=1")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"], help="N>1 collectives")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     fam = CONFIGS[args.config]
@@ -168,6 +277,8 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
         return run_reference(args, fam, rank, world)
+    if world > 1 or args.sharded:
+        return run_sharded(args, fam, rank, world, local)
 
     import torch
     import torch.distributed as dist

@@ -273,8 +273,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const u64 n_src = SH ? ctx->sh_ns : D.n_events;                // events the ingest reads
     ctx->n_reports = 0;
     ctx->bad_event = 0;
-    ctx->launches = 0;
-    ctx->nk = 0;
+    if (!SH) {  // sharded: keep igd_shard_prepare's launches in the same accounting
+        ctx->launches = 0;
+        ctx->nk = 0;
+    }
     *n_out = 0;
     mark(ctx, 0);
     if (n == 0 || (n_src == 0 && (!SH || ctx->sh_nrec == 0))) {
@@ -592,6 +594,7 @@ static int shard_prepare_impl(igd_ctx* ctx, u32 P, u64* counts, u64* n_sync_stre
     const u64 tiles = (n + shard::TILE - 1) / shard::TILE;
     const u64 row = tiles + 1;
     RET(ensure(ctx, ctx->stats, 8 * sizeof(u64)));
+    RET(ensure(ctx, ctx->ctr, 64));
     RET(ensure(ctx, ctx->sh_cnt, (P + 1) * row * sizeof(u32)));
     RET(ensure(ctx, ctx->sh_obase, (P + 1) * sizeof(u64)));
     u64 init[8] = {~0ull, 0, ~0ull, 0, 0, 0, 0, 0};
@@ -763,6 +766,7 @@ int igd_shard_prepare(igd_ctx* ctx, uint32_t nranks, uint64_t* counts, uint64_t*
     cudaSetDevice(ctx->device);
     ctx->launches = 0;
     ctx->nk = 0;
+    ctx->timing = true;  // per-launch events are cheap; igd_shard_detect reports them with its own
     return shard_prepare_impl(ctx, nranks, counts, n_sync_stream, bad_event, word_minmax);
 }
 
@@ -790,6 +794,7 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     ctx->sh_ns = n_sync_stream;
     ctx->sh_wbase = min_word;
     ctx->sh_ntotal = ctx->desc.n_events_total ? ctx->desc.n_events_total : ctx->desc.n_events;
+    RET(buf_free(ctx, ctx->sh_send));  // the exchange is done: release the send buffer first
     int rc = detect_impl(ctx, n_reports);
     ctx->shard = false;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);

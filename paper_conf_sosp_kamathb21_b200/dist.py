@@ -56,6 +56,8 @@ def chunk_bounds(n_total: int, nranks: int, rank: int):
 
 def merge_reports(parts) -> np.ndarray:
     """Union of per-rank report arrays in canonical order (ascending cur; cur is unique)."""
+    parts = [p.cpu().numpy().reshape(-1).view(_igd.REPORT_DTYPE) if isinstance(p, torch.Tensor) else p
+             for p in parts]
     parts = [p for p in parts if len(p)]
     if not parts:
         return np.zeros(0, _igd.REPORT_DTYPE)
@@ -65,32 +67,35 @@ def merge_reports(parts) -> np.ndarray:
 
 # ---- communication ------------------------------------------------------------------------------
 class TorchComm:
-    """Collectives over a torch.distributed process group (NCCL on GPUs, gloo on CPU)."""
+    """Collectives over a torch.distributed process group: NCCL on GPUs (device tensors move over
+    NVLink / NVSwitch); with gloo, device tensors are staged through host memory."""
 
     def __init__(self, group=None):
         self.group = group
         self.rank = dist.get_rank(group)
         self.size = dist.get_world_size(group)
+        self.host_staged = dist.get_backend(group) == "gloo"
 
-    def _dev(self, like: torch.Tensor):
-        return like.device
+    def _in(self, t: torch.Tensor) -> torch.Tensor:
+        return t.cpu() if self.host_staged else t
 
     def allreduce_u64(self, value: int, op: str, device) -> int:
-        # values are < 2^63 except the NONE64 sentinel, which maps to -1 for MIN
-        v = -1 if value == NONE64 else int(value)
-        if op == "min_none":  # minimum of real values, NONE if all are NONE
+        """min / max of a non-negative int over ranks; "min_none" treats NONE64 as absent."""
+        if op == "min_none":
             v = (1 << 62) if value == NONE64 else int(value)
-            t = torch.tensor([v], dtype=torch.int64, device=device)
+            t = self._in(torch.tensor([v], dtype=torch.int64, device=device))
             dist.all_reduce(t, op=dist.ReduceOp.MIN, group=self.group)
             r = int(t.item())
             return NONE64 if r == (1 << 62) else r
-        t = torch.tensor([v], dtype=torch.int64, device=device)
+        t = self._in(torch.tensor([int(value)], dtype=torch.int64, device=device))
         dist.all_reduce(t, op=dist.ReduceOp.MIN if op == "min" else dist.ReduceOp.MAX, group=self.group)
         return int(t.item())
 
     def all_to_all_var(self, send: torch.Tensor, counts) -> torch.Tensor:
         """Rows of `send` grouped by destination rank (counts[d] rows for rank d) -> rows received
         from every rank, concatenated in source-rank order."""
+        dev = send.device
+        send = self._in(send)
         cnt = torch.tensor([int(c) for c in counts], dtype=torch.int64, device=send.device)
         rcnt = torch.empty_like(cnt)
         dist.all_to_all_single(rcnt, cnt, group=self.group)
@@ -98,10 +103,12 @@ class TorchComm:
         recv = torch.empty((sum(rc),) + tuple(send.shape[1:]), dtype=send.dtype, device=send.device)
         dist.all_to_all_single(recv, send, output_split_sizes=rc, input_split_sizes=[int(c) for c in counts],
                                group=self.group)
-        return recv
+        return recv.to(dev)
 
     def all_gather_var(self, t: torch.Tensor) -> torch.Tensor:
         """Concatenation over ranks (rank order) of variable-length tensors."""
+        dev = t.device
+        t = self._in(t)
         n = torch.tensor([t.shape[0]], dtype=torch.int64, device=t.device)
         ns = [torch.empty_like(n) for _ in range(self.size)]
         dist.all_gather(ns, n, group=self.group)
@@ -111,7 +118,7 @@ class TorchComm:
         pad[: t.shape[0]] = t
         outs = [torch.empty_like(pad) for _ in range(self.size)]
         dist.all_gather(outs, pad, group=self.group)
-        return torch.cat([o[:s] for o, s in zip(outs, sizes)])
+        return torch.cat([o[:s] for o, s in zip(outs, sizes)]).to(dev)
 
 
 # ---- device stage (libigd) ----------------------------------------------------------------------
@@ -178,8 +185,13 @@ class GpuStage:
                                   min_word, _igd.IGD_DETECT_TIMING if timing else 0, ctypes.byref(nrep))
         if rc != _igd.IGD_OK:
             raise _igd.IgdError(rc, lib.igd_last_error(self.det.ctx).decode())
-        self.det.n_reports = int(nrep.value)
-        return self.det.reports()
+        self.det.n_reports = n = int(nrep.value)
+        if n == 0:
+            return torch.zeros((0, 32), dtype=torch.uint8, device=self.device)
+        ptr, cnt = ctypes.c_void_p(), ctypes.c_uint64()
+        lib.igd_reports_device(self.det.ctx, ctypes.byref(ptr), ctypes.byref(cnt))
+        # device copy of the context-owned reports ([n, 32] bytes, ascending cur)
+        return torch.as_tensor(_CudaArray(ptr.value, (n, 32), "|u1"), device=self.device).clone()
 
 
 # ---- orchestration --------------------------------------------------------------------------------
@@ -204,9 +216,13 @@ def sharded_detect(stage, comm: TorchComm, timing: bool = False) -> np.ndarray:
     sidx = comm.all_gather_var(prep["sync_idx"].reshape(-1, 1)).reshape(-1)
     sev = comm.all_gather_var(prep["sync_ev"])
     local = stage.detect(recv, sidx, sev, lo if lo != (1 << 62) else 0, timing)
-    raw = torch.from_numpy(local.view(np.uint8).reshape(-1, 32).copy()).to(dev)
-    everything = comm.all_gather_var(raw).cpu().numpy()
-    return merge_reports([everything.reshape(-1).view(_igd.REPORT_DTYPE)])
+    if isinstance(local, np.ndarray):
+        local = torch.from_numpy(local.view(np.uint8).reshape(-1, 32).copy()).to(dev)
+    everything = comm.all_gather_var(local)           # [n, 32] bytes, rank order
+    if everything.shape[0] > 1:                       # merge by cur on the device (cur is unique)
+        cur = everything.view(torch.int64)[:, 1]
+        everything = everything[torch.argsort(cur)]
+    return everything.cpu().numpy().reshape(-1).view(_igd.REPORT_DTYPE)
 
 
 class LoopbackComm:
@@ -225,8 +241,8 @@ class LoopbackComm:
         offs = [np.concatenate([[0], np.cumsum(p["counts"])]) for p in preps]
         sidx = torch.cat([p["sync_idx"] for p in preps])
         sev = torch.cat([p["sync_ev"] for p in preps])
-        parts = []
-        for d, s in enumerate(stages):
-            recv = torch.cat([p["records"][int(o[d]):int(o[d + 1])] for p, o in zip(preps, offs)])
-            parts.append(s.detect(recv, sidx, sev, lo, timing))
+        # all exchanges first: a stage's detect releases its send buffer
+        recvs = [torch.cat([p["records"][int(o[d]):int(o[d + 1])] for p, o in zip(preps, offs)])
+                 for d in range(P)]
+        parts = [s.detect(recv, sidx, sev, lo, timing) for s, recv in zip(stages, recvs)]
         return merge_reports(parts)
