@@ -24,16 +24,19 @@ def needs_build() -> bool:
     return any(os.path.getmtime(s) > t for s in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, defines=None, out: str = None) -> str:
+    """Compile csrc/igd.cu into libigd.so (or `out`, e.g. a tuning variant with -D defines)."""
+    target = out or LIB
+    if out is None and not force and not needs_build():
         return LIB
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-    cmd = [nvcc, *NVCC_FLAGS, "-o", LIB + ".tmp", os.path.join(CSRC, "igd.cu")]
+    cmd = [nvcc, *NVCC_FLAGS, *[f"-D{d}" for d in (defines or [])], "-o", target + ".tmp",
+           os.path.join(CSRC, "igd.cu")]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

@@ -202,18 +202,23 @@ __device__ __forceinline__ Acc acc_at(const void* val, u32 k) {
 }
 
 template <bool MV>
-__global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
+#ifndef IGD_CHECK_MINB
+#define IGD_CHECK_MINB 6
+#endif
+__global__ void __launch_bounds__(THREADS, IGD_CHECK_MINB) k_check(Params P) {
     __shared__ u32 s_tile;
     __shared__ u64 s_wagg[WARPS];
     __shared__ u64 s_prefix;
     __shared__ u32 s_ready;
     __shared__ u32 s_qn;
     // queue of undecided accesses (SoA)
-    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_la[TILE], q_lt[TILE], q_k[TILE];
+    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_pos[TILE];  // q_pos: sorted position
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     if (t == 0) {
-        s_tile = atomicAdd(P.tile_ctr, 1u);
+        // tiles in launch order (the block scheduler dispatches CTAs in blockIdx order, as
+        // decoupled look-back scans rely on); no atomic round trip before the loads
+        s_tile = blockIdx.x;
         s_qn = 0;
         s_ready = 0;
     }
@@ -225,12 +230,16 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
     // K: word key, V: trace index, Z: the event's tk word (tid | kind | scope), carried by the sort
     u32 K[ITEMS], V[ITEMS], Z[ITEMS], M[ITEMS];
     if (!MV && first + ITEMS <= P.n) {
-        const uint4 k4 = __ldcs(reinterpret_cast<const uint4*>(P.key + first));
-        const uint4 v01 = __ldcs(reinterpret_cast<const uint4*>(P.val) + first / 2);
-        const uint4 v23 = __ldcs(reinterpret_cast<const uint4*>(P.val) + first / 2 + 1);
-        K[0] = k4.x; K[1] = k4.y; K[2] = k4.z; K[3] = k4.w;
-        V[0] = v01.x; Z[0] = v01.y; V[1] = v01.z; Z[1] = v01.w;
-        V[2] = v23.x; Z[2] = v23.y; V[3] = v23.z; Z[3] = v23.w;
+#pragma unroll
+        for (int q = 0; q < ITEMS / 4; q++) {
+            const uint4 k4 = __ldcs(reinterpret_cast<const uint4*>(P.key + first) + q);
+            K[4 * q] = k4.x; K[4 * q + 1] = k4.y; K[4 * q + 2] = k4.z; K[4 * q + 3] = k4.w;
+        }
+#pragma unroll
+        for (int q = 0; q < ITEMS / 2; q++) {
+            const uint4 v = __ldcs(reinterpret_cast<const uint4*>(P.val) + first / 2 + q);
+            V[2 * q] = v.x; Z[2 * q] = v.y; V[2 * q + 1] = v.z; Z[2 * q + 1] = v.w;
+        }
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) M[j] = 0;
     } else {
@@ -410,9 +419,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
                 q_md[q] = mdIdx;
                 q_c[q] = c | (flags << 24);
                 q_p[q] = p | (kind << 24) | (mdKind << 28);
-                q_la[q] = laIdx;
-                q_lt[q] = laTid;
-                q_k[q] = K[j];
+                q_pos[q] = first + j;
             }
         }
         laIdx = i;
@@ -445,7 +452,8 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
         }
         if (!type && P.lv.any) {  // R5: lock sets of the last accessor and of this access
             const u32 L = syncx::held_before(P.lv, g, c, i);
-            const u32 locks = syncx::held_before(P.lv, g, q_lt[q], q_la[q]);
+            const Acc la = acc_at<MV>(P.val, q_pos[q] - 1);  // the last accessor (rare path)
+            const u32 locks = syncx::held_before(P.lv, g, la.tk & 0xFFFFFFu, la.idx);
             if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
         }
         if (type) {
@@ -454,7 +462,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_check(Params P) {
             if (slot < P.rep_cap) {
                 igd_report r;
                 // full word from the 32-bit key: the accessed words span < 2^32 from wbase
-                r.addr = (P.wbase + (u32)(q_k[q] - (u32)P.wbase)) << 2;
+                r.addr = (P.wbase + (u32)(__ldg(P.key + q_pos[q]) - (u32)P.wbase)) << 2;
                 r.cur = P.first_event + i;
                 r.prev = P.first_event + mdIdx;
                 r.type = (uint8_t)type;

@@ -145,7 +145,10 @@ __device__ __forceinline__ void hist_add(u32* h, u32 digit, bool on, u32 lane) {
 // one, but every tile is independent: no look-back chain across 2M tiles (which bounded the
 // single-pass variant at ~40 G events/s on B200).
 template <int PASS>
-__global__ void __launch_bounds__(THREADS, 2) k_ingest(Params P) {
+#ifndef IGD_INGEST_MINB
+#define IGD_INGEST_MINB 3
+#endif
+__global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
     __shared__ u32 s_hacc[PASS == 0 ? 4 : 1][256];
     __shared__ u32 s_hsync[PASS == 0 ? 4 : 1][256];
     __shared__ u32 s_wtot[ITEMS][WARPS];  // packed (acc | nsync << 16) per (item, warp)

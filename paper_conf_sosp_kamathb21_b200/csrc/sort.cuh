@@ -95,7 +95,10 @@ constexpr size_t onesweep_smem() {
 }
 
 template <int MODE, typename VT>
-__global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
+#ifndef IGD_SORT_MINB
+#define IGD_SORT_MINB 3
+#endif
+__global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams P) {
     __shared__ u32 s_whist[WARPS][RADIX];
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
@@ -113,7 +116,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_onesweep(PassParams P) {
     if (t == 0) {
         // tile id, then TMA bulk copies of the tile's keys and values into shared memory: the
         // value copy lands while the keys are ranked
-        const u32 tile = atomicAdd(P.tile_ctr, 1u);
+        const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
         s_tile = tile;
         const u64 base = (u64)tile * TILE;
         if (base + TILE <= P.n) {

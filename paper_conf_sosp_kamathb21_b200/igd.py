@@ -44,11 +44,12 @@ def load_library(build_if_missing: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    if build_if_missing and _build.needs_build():
+    path = os.environ.get("IGD_LIB", _build.LIB)  # tuning variants (profiles/) only
+    if path == _build.LIB and build_if_missing and _build.needs_build():
         _build.build()
-    if not os.path.exists(_build.LIB):
-        raise ImportError(f"libigd.so not built at {_build.LIB}")
-    lib = ctypes.CDLL(_build.LIB)
+    if not os.path.exists(path):
+        raise ImportError(f"libigd.so not built at {path}")
+    lib = ctypes.CDLL(path)
     vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
     lib.igd_ctx_create.argtypes = [ctypes.POINTER(vp), i32, vp, i32, i32, vp, ALLOC_FN, FREE_FN, vp]
     lib.igd_ctx_create.restype = i32
