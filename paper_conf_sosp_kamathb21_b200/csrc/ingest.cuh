@@ -146,7 +146,7 @@ __device__ __forceinline__ void hist_add(u32* h, u32 digit, bool on, u32 lane) {
 // single-pass variant at ~40 G events/s on B200).
 template <int PASS>
 #ifndef IGD_INGEST_MINB
-#define IGD_INGEST_MINB 3
+#define IGD_INGEST_MINB 4
 #endif
 __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
     __shared__ u32 s_hacc[PASS == 0 ? 4 : 1][256];

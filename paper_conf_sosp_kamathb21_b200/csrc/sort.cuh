@@ -19,7 +19,13 @@ namespace rsort {
 
 constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
-constexpr int ITEMS = 16;
+#ifndef IGD_SORT_ITEMS
+#define IGD_SORT_ITEMS 16
+#endif
+#ifndef IGD_SORT_VDIRECT
+#define IGD_SORT_VDIRECT 0
+#endif
+constexpr int ITEMS = IGD_SORT_ITEMS;
 constexpr int TILE = THREADS * ITEMS;  // 4096
 constexpr int RADIX = 256;
 
@@ -251,6 +257,16 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             val[j] = i < P.n ? __ldcs(vin + i) : VT{};
         }
     }
+#if IGD_SORT_VDIRECT
+    // values straight to their output position (L2 merges the partial sectors)
+    __syncthreads();  // s_dig of every position written
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++)
+        if (full || wbase + j * 32 + lane < P.n) {
+            const u32 d = s_dig[rank[j]];
+            __stcs(vout + s_gbase[d] + (rank[j] - s_tile_excl[d]), val[j]);
+        }
+#else
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < ITEMS; j++)
@@ -264,6 +280,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             __stcs(vout + s_gbase[d] + (i - s_tile_excl[d]), s_v[i]);
         }
     }
+#endif
 }
 
 }  // namespace rsort
