@@ -175,3 +175,43 @@ def test_long_irregular_sync_lists(det, seed):
     drop = sync & ~burst & (rng.random(n) < 0.9)
     ev = ev[~drop]
     assert_same(det, ev, nb, bd, f"bursty {seed}")
+
+
+def test_c2_full_size_vs_oracle(det):
+    # BASELINE configs[1] at its full size (10^7 events), element by element against the oracle
+    import tracegen.families as F
+
+    ev, nb, bd, led = F.generate(2)
+    want = oracle.run(ev, nb, bd)
+    det.load(ev, nb, bd)
+    det.detect()
+    got = det.reports()
+    assert np.array_equal(got, want)
+    assert [(r["addr"], r["cur"], r["prev"], r["type"]) for r in got] == \
+           [(r["addr"], r["cur"], r["prev"], r["type"]) for r in led]
+
+
+def test_c3_full_size_sampled_words_vs_oracle(det):
+    # configs[2] at full size (10^8 events): the oracle checks a 1/16 address shard (replaying every
+    # synchronization event), the GPU result restricted to the same words must match exactly
+    import tracegen.families as F
+
+    ev, nb, bd, led = F.generate(3)
+    det.load(ev, nb, bd)
+    det.detect()
+    got = det.reports()
+    K = 16
+    want = oracle.run(ev, nb, bd, shard=(5, K))
+
+    def fmix(h):
+        h = h & 0xFFFFFFFF
+        h ^= h >> 16
+        h = (h * 0x85EBCA6B) & 0xFFFFFFFF
+        h ^= h >> 13
+        h = (h * 0xC2B2AE35) & 0xFFFFFFFF
+        return h ^ (h >> 16)
+
+    words = got["addr"] >> np.uint64(2)
+    mine = np.array([fmix(int(w) ^ (int(w) >> 32)) % K == 5 for w in words], bool)
+    assert np.array_equal(got[mine], want)
+    assert len(got) == len(led)
