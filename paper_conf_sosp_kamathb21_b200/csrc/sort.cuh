@@ -25,6 +25,12 @@ constexpr int WARPS = THREADS / 32;
 #ifndef IGD_SORT_VDIRECT
 #define IGD_SORT_VDIRECT 0
 #endif
+#ifndef IGD_SORT_SKIPBITS
+#define IGD_SORT_SKIPBITS 0
+#endif
+#ifndef IGD_SORT_NOLOOKBACK
+#define IGD_SORT_NOLOOKBACK 0
+#endif
 constexpr int ITEMS = IGD_SORT_ITEMS;
 constexpr int TILE = THREADS * ITEMS;  // 4096
 constexpr int RADIX = 256;
@@ -82,6 +88,19 @@ template <int MODE>
 __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     if (MODE == 0) {
         return __match_any_sync(IGD_FULL, d) & vmask;
+    } else if (IGD_SORT_SKIPBITS) {
+        // ballot only the digit bits that differ somewhere in the warp (high digits of
+        // clustered words are often warp-uniform)
+        u32 peers = vmask;
+        u32 diff = (__reduce_or_sync(IGD_FULL, d) ^ __reduce_and_sync(IGD_FULL, d)) & 0xFFu;
+        while (diff) {
+            const u32 b = __ffs(diff) - 1;
+            diff &= diff - 1;
+            const u32 bit = (d >> b) & 1u;
+            const u32 bal = __ballot_sync(IGD_FULL, bit);
+            peers &= bit ? bal : ~bal;
+        }
+        return peers;
     } else {
         u32 peers = vmask;
 #pragma unroll
@@ -209,7 +228,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     {
         const u32 d = t;
         u64 excl = 0;
-        if (tile > 0) {
+        if (tile > 0 && !IGD_SORT_NOLOOKBACK) {  // NOLOOKBACK: timing experiment only (wrong output)
             long tt = (long)tile - 1;
             while (tt >= 0) {
                 u64 s;
