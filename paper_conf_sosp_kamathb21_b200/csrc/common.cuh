@@ -84,6 +84,19 @@ __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
     return v;
 }
 
+// Wait until a look-back status word is published (non-zero state).  The back-off frees issue
+// slots for the other CTAs of the SM while a predecessor tile is still working.
+#ifndef IGD_SPIN_NS
+#define IGD_SPIN_NS 0
+#endif
+__device__ __forceinline__ u64 spin_status(const u64* p, u64 s) {
+    while ((s >> 62) == 0) {
+        if (IGD_SPIN_NS) __nanosleep(IGD_SPIN_NS);
+        s = ld_relaxed(p);
+    }
+    return s;
+}
+
 // Exclusive prefix of a u64 sum over tiles [0, tile): single thread walks back.
 __device__ __forceinline__ u64 lookback_sum(u64* status, u32 tile) {
     u64 excl = 0;

@@ -1,0 +1,249 @@
+// fused.cuh -- a1/a2/a4 write pass fused with the first a5 radix pass (single GPU).
+//
+// The unfused pipeline writes the compacted access records (12 B per access) in ingest pass 1
+// and the first radix pass reads them back and writes them again sorted by digit 0.  Here one
+// onesweep-style kernel reads each 4096-event tile of the trace once (one TMA bulk copy into
+// shared memory), decodes it, writes the tile's synchronization records at their trace-order
+// positions (bases from ingest pass 0), and ranks the tile's accesses by digit 0 of the word
+// key exactly like rsort::k_onesweep -- warp multisplit, per-tile digit counts, decoupled
+// look-back -- so the access records leave already sorted by digit 0 (stable: input order is
+// trace order).  Saves 24 B per access of HBM traffic and one launch over the accesses.
+//
+// Shared memory: the 64 KB event tile is dead once decoded, so the digit-sorted key / value
+// staging buffers alias it (3 CTAs per SM).
+#pragma once
+#include "common.cuh"
+#include "ingest.cuh"
+#include "sort.cuh"
+
+namespace fused {
+
+constexpr int THREADS = 256;
+constexpr int WARPS = THREADS / 32;
+constexpr int ITEMS = 16;
+constexpr int TILE = THREADS * ITEMS;  // events per tile == 2 ingest pass-0 tiles
+constexpr int RADIX = 256;
+#ifndef IGD_FUSED_EARLY
+#define IGD_FUSED_EARLY 1
+#endif
+static_assert(TILE == 2 * ingest::TILE, "sync-record bases come from ingest pass 0 tiles");
+static_assert(THREADS == RADIX, "one look-back digit per thread");
+
+struct Params {
+    const igd_event* ev;
+    u64 n;               // events
+    Geo g;
+    KeySpace ks;
+    const u32* tile_sync;  // exclusive sync-record base of every ingest pass-0 tile
+    u32* sync_key;
+    u32* sync_val;
+    u64 sync_cap;
+    const u32* digit_base;  // [256] exclusive global offsets of digit 0 of the access keys
+    u64* status;            // [n_tiles * 256], zeroed
+    u32* kout;              // access keys, sorted by digit 0
+    u64* vout;              // access payload (event index | tk << 32), same order
+};
+
+constexpr size_t smem_bytes() { return (size_t)TILE * sizeof(uint4); }  // 64 KB
+
+__global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
+    __shared__ u32 s_tile_excl[RADIX];
+    __shared__ u32 s_gbase[RADIX];
+    __shared__ u32 s_wsum[WARPS];
+    __shared__ u32 s_wsync[WARPS];
+    __shared__ u32 s_na;
+    __shared__ u32 s_cnt[RADIX];  // tile digit counts (early publication)
+    __shared__ __align__(8) u64 s_mbar;
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    // phase 1: the event tile (64 KB).  Phase 2 (events dead): digit-sorted keys [0, 16K),
+    // values [16K, 48K), digit per position [48K, 52K), per-warp digit counts [56K, 64K).
+    uint4* s_ev = reinterpret_cast<uint4*>(s_dyn);
+    u32* s_k = reinterpret_cast<u32*>(s_dyn);
+    u64* s_v = reinterpret_cast<u64*>(s_dyn + TILE * 4);
+    uint8_t* s_dig = s_dyn + TILE * 12;
+    u32(*s_whist)[RADIX] = reinterpret_cast<u32(*)[RADIX]>(s_dyn + TILE * 14);
+    static_assert(TILE * 14 + WARPS * RADIX * 4 <= TILE * 16, "phase-2 buffers fit the event tile");
+
+    const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
+    const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
+    const u64 base = (u64)tile * TILE;
+    const bool full = base + TILE <= P.n;
+    const u32 tile_e = full ? (u32)TILE : (u32)(P.n - base);
+    if (t == 0 && full) {
+        mbar_init(&s_mbar, 1);
+        mbar_expect_tx(&s_mbar, TILE * sizeof(uint4));
+        bulk_g2s(s_ev, P.ev + base, TILE * sizeof(uint4), &s_mbar);
+    }
+    s_cnt[t] = 0;
+    if (!full)
+        for (u32 i = t; i < TILE; i += THREADS)
+            s_ev[i] = i < tile_e ? ld_event_stream(P.ev, base + i) : make_uint4(0, 0, 0, 0);
+    __syncthreads();
+    if (full) mbar_wait(&s_mbar, 0);
+
+    // ---- decode: warp w owns events [w * 32 * ITEMS, (w + 1) * 32 * ITEMS) of the tile, item j
+    // of lane l being event w * 32 * ITEMS + j * 32 + l (warp-contiguous, item-major = trace order)
+    const Geo g = P.g;
+    const KeySpace ks = P.ks;
+    const u32 wofs = warp * 32 * ITEMS;
+    const u32 lt = lanemask_lt();
+    u32 key[ITEMS], tk[ITEMS];
+    u32 amask = 0;    // bit j: item j is an access
+    u32 nsync_w = 0;  // sync records of this warp (warp-uniform)
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++) {
+        const u32 p = wofs + j * 32 + lane;
+        const ingest::Dec d = ingest::decode(s_ev[p], g, ks);  // valid: ingest pass 0 checked every event
+        const bool in = p < tile_e;
+        key[j] = d.key;
+        tk[j] = d.tk;
+        amask |= ((in && (d.flags & 1u)) ? 1u : 0u) << j;
+        if (IGD_FUSED_EARLY && in && (d.flags & 1u)) atomicAdd(&s_cnt[d.key & 255u], 1u);
+        const u32 ns = in ? (d.flags >> 1) & 3u : 0u;
+        nsync_w += __popc(__ballot_sync(IGD_FULL, ns >= 1)) + __popc(__ballot_sync(IGD_FULL, ns == 2));
+    }
+    if (lane == 0) s_wsync[warp] = nsync_w;
+    __syncthreads();
+    // The tile's digit counts are known before any ranking: publish them now, so successors
+    // looking back rarely find this tile not ready (their spin was most of this kernel's issue
+    // slots when the aggregate was published after ranking, ncu r01 v5)
+    if (IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
+
+    // ---- synchronization records, in trace order: base of this tile (ingest pass 0) + earlier
+    // warps + earlier (item, lane) of this warp; decoded again from the staged tile
+    if (nsync_w) {
+        u32 wpre = 0;
+#pragma unroll
+        for (int w = 0; w < WARPS; w++)
+            if ((u32)w < warp) wpre += s_wsync[w];
+        u64 pos = (u64)P.tile_sync[2 * tile] + wpre;
+#pragma unroll 1
+        for (int j = 0; j < ITEMS; j++) {
+            const u32 p = wofs + j * 32 + lane;
+            const ingest::Dec d = ingest::decode(s_ev[p], g, ks);
+            const u32 ns = p < tile_e ? (d.flags >> 1) & 3u : 0u;
+            const u32 b1 = __ballot_sync(IGD_FULL, ns >= 1), b2 = __ballot_sync(IGD_FULL, ns == 2);
+            if (!(b1 | b2)) continue;
+            const u64 my = pos + __popc(b1 & lt) + __popc(b2 & lt);
+            if (ns && my + ns <= P.sync_cap) {
+                const u32 ts = (u32)(base + p);
+                P.sync_key[my] = d.s0;
+                P.sync_val[my] = ts;
+                if (ns == 2) {
+                    P.sync_key[my + 1] = d.s1;
+                    P.sync_val[my + 1] = ts;
+                }
+            }
+            pos += __popc(b1) + __popc(b2);
+        }
+    }
+    __syncthreads();  // the event tile is dead
+    for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_whist[0][0])[i] = 0;
+    __syncthreads();
+
+    // ---- rank the accesses by digit 0 (warp multisplit, as rsort::k_onesweep)
+    u32 rank2[ITEMS / 2];  // ranks (< TILE <= 2^16) packed in pairs: register budget of 3 CTAs/SM
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++) {
+        const bool valid = (amask >> j) & 1u;
+        const u32 vmask = __ballot_sync(IGD_FULL, valid);
+        const u32 d = key[j] & 255u;
+        const u32 peers = rsort::peers_of<1>(valid ? d : (0x100u | lane), vmask);
+        const u32 leader = __ffs(peers) - 1;
+        u32 old = 0;
+        if (lane == leader && valid) {
+            old = s_whist[warp][d];
+            s_whist[warp][d] = old + __popc(peers);
+        }
+        old = __shfl_sync(IGD_FULL, old, leader & 31u);
+        const u32 r = old + __popc(peers & lt);
+        if (j & 1) rank2[j / 2] |= r << 16;
+        else rank2[j / 2] = r;
+        __syncwarp();
+    }
+    __syncthreads();
+
+    // ---- per digit: exclusive over warps, tile count, publish the aggregate
+    u32 cnt;
+    {
+        const u32 d = t;
+        u32 sum = 0;
+#pragma unroll
+        for (int w = 0; w < WARPS; w++) {
+            const u32 c = s_whist[w][d];
+            s_whist[w][d] = sum;
+            sum += c;
+        }
+        cnt = sum;
+        if (!IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
+    }
+    {
+        u32 inc = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const u32 x = __shfl_up_sync(IGD_FULL, inc, o);
+            if (lane >= (u32)o) inc += x;
+        }
+        if (lane == 31) s_wsum[warp] = inc;
+        __syncthreads();
+        u32 wpre = 0;
+#pragma unroll
+        for (int w = 0; w < WARPS; w++)
+            if ((u32)w < warp) wpre += s_wsum[w];
+        s_tile_excl[t] = wpre + inc - cnt;
+        if (t == RADIX - 1) s_na = wpre + inc;  // accesses in this tile
+    }
+    // ---- look-back for digit t (LB statuses per round trip, as rsort::k_onesweep)
+    {
+        const u32 dg = t;
+        u64 excl = 0;
+        if (tile > 0) {
+            long tt = (long)tile - 1;
+            bool done = false;
+            while (!done) {
+                u64 s[IGD_SORT_LB];
+#pragma unroll
+                for (int q = 0; q < IGD_SORT_LB; q++)
+                    s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + dg) : ST_INC;
+#pragma unroll
+                for (int q = 0; q < IGD_SORT_LB; q++) {
+                    if (!done) {
+                        s[q] = spin_status(P.status + (u64)(tt - q) * RADIX + dg, s[q]);
+                        excl += s[q] & ST_VAL_MASK;
+                        done = (s[q] >> 62) == 2;
+                    }
+                }
+                tt -= IGD_SORT_LB;
+            }
+            st_relaxed(P.status + (u64)tile * RADIX + dg, ST_INC | (excl + cnt));
+        }
+        s_gbase[dg] = P.digit_base[dg] + (u32)excl;
+    }
+    __syncthreads();
+    // ---- records to their tile positions: key, payload (event index | tk << 32), digit
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++) {
+        if ((amask >> j) & 1u) {
+            const u32 d = key[j] & 255u;
+            const u32 r = ((rank2[j / 2] >> (16 * (j & 1))) & 0xFFFFu) + s_tile_excl[d] + s_whist[warp][d];
+            s_k[r] = key[j];
+            s_v[r] = (base + wofs + j * 32 + lane) | ((u64)tk[j] << 32);
+            s_dig[r] = (uint8_t)d;
+        }
+    }
+    __syncthreads();
+    // ---- out in digit runs
+    const u32 na = s_na;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const u32 i = t + k * THREADS;
+        if (i < na) {
+            const u32 d = s_dig[i];
+            const u32 o = s_gbase[d] + (i - s_tile_excl[d]);
+            __stcs(P.kout + o, s_k[i]);
+            __stcs(P.vout + o, s_v[i]);
+        }
+    }
+}
+
+}  // namespace fused

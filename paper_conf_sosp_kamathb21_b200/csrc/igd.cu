@@ -15,6 +15,7 @@
 
 #include "check.cuh"
 #include "common.cuh"
+#include "fused.cuh"
 #include "ingest.cuh"
 #include "sort.cuh"
 #include "shard.cuh"
@@ -58,8 +59,9 @@ struct igd_ctx {
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
-    int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any (IGD_SORT_MODE)
+    int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any, 2 = atomic-or (IGD_SORT_MODE)
     int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
+    int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
     bool shard = false;
     Buf sh_cnt, sh_obase, sh_send, sh_sidx_buf, sh_sev_buf;
@@ -190,13 +192,20 @@ static void mark(igd_ctx* ctx, int stage) {
     if (ctx->timing) cudaEventRecord(ctx->ev[stage], ctx->stream);
 }
 
+template <typename VT>
+static void launch_pass(int mode, unsigned gb, size_t smem, cudaStream_t st, const rsort::PassParams& pp) {
+    if (mode == 0) rsort::k_onesweep<0, VT><<<gb, rsort::THREADS, smem, st>>>(pp);
+    else if (mode == 2) rsort::k_onesweep<2, VT><<<gb, rsort::THREADS, smem, st>>>(pp);
+    else rsort::k_onesweep<1, VT><<<gb, rsort::THREADS, smem, st>>>(pp);
+}
+
 // Stable LSD radix sort of n (key, value) pairs in buffers k[cur], v[cur]; h_hist is the host
 // copy of the 4x256 digit histogram (device copy d_hist).  Digits above max_bits and digits
 // with one occupied bin are skipped.  Returns the buffer index holding the result.
 static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d_hist, const u32* h_hist,
-                      u32 max_bits, int* out_cur, int vbytes = 4) {
-    int cur = 0;
-    *out_cur = 0;
+                      u32 max_bits, int* out_cur, int vbytes = 4, u32 first_pass = 0, int first_cur = 0) {
+    int cur = first_cur;
+    *out_cur = cur;
     if (n <= 1) return IGD_OK;
     if (n > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;  // 32-bit tile indexing
     {
@@ -205,7 +214,7 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
     }
     const u64 tiles = (n + rsort::TILE - 1) / rsort::TILE;
     RET(ensure(ctx, ctx->status, tiles * rsort::RADIX * sizeof(u64)));
-    for (u32 p = 0; p < 4; p++) {
+    for (u32 p = first_pass; p < 4; p++) {
         if (p * 8 >= max_bits) break;
         bool trivial = false;
         for (int d = 0; d < 256; d++)
@@ -227,17 +236,9 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
             KTimer kt(ctx, cls, 2.0 * (4 + vbytes) * (double)n);  // read + write 4 B key and the value
             const unsigned gb = (unsigned)tiles;
             const size_t s8 = rsort::onesweep_smem<u64>(), s4 = rsort::onesweep_smem<u32>();
-            if (vbytes == 16) {
-                const size_t s16 = rsort::onesweep_smem<uint4>();
-                if (ctx->sort_mode == 0) rsort::k_onesweep<0, uint4><<<gb, rsort::THREADS, s16, ctx->stream>>>(pp);
-                else rsort::k_onesweep<1, uint4><<<gb, rsort::THREADS, s16, ctx->stream>>>(pp);
-            } else if (vbytes == 8) {
-                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u64><<<gb, rsort::THREADS, s8, ctx->stream>>>(pp);
-                else rsort::k_onesweep<1, u64><<<gb, rsort::THREADS, s8, ctx->stream>>>(pp);
-            } else {
-                if (ctx->sort_mode == 0) rsort::k_onesweep<0, u32><<<gb, rsort::THREADS, s4, ctx->stream>>>(pp);
-                else rsort::k_onesweep<1, u32><<<gb, rsort::THREADS, s4, ctx->stream>>>(pp);
-            }
+            if (vbytes == 16) launch_pass<uint4>(ctx->sort_mode, gb, rsort::onesweep_smem<uint4>(), ctx->stream, pp);
+            else if (vbytes == 8) launch_pass<u64>(ctx->sort_mode, gb, s8, ctx->stream, pp);
+            else launch_pass<u32>(ctx->sort_mode, gb, s4, ctx->stream, pp);
         }
         CK(cudaGetLastError());
         cur ^= 1;
@@ -322,6 +323,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     ip.hist_sync = P_<u32>(ctx->hist) + 1024;
     ip.stats = P_<u64>(ctx->stats);
     ip.n_tiles = (u32)in_tiles;
+    const bool FUSED = !SH && ctx->fused;
+    ip.hist0 = FUSED ? 1 : 0;
     int occ = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ingest::k_ingest<0>, ingest::THREADS, 0);
     const u64 grid = std::max<u64>(1, std::min<u64>((u64)sms * (occ > 0 ? occ : 1), in_tiles));
@@ -362,7 +365,36 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     ip.sync_key = P_<u32>(ctx->syn_k[0]);
     ip.sync_val = P_<u32>(ctx->syn_v[0]);
     ip.sync_cap = ctx->sync_cap;
-    if (n_src > 0) {
+    if (FUSED) {
+        // one pass: sync records + accesses sorted by digit 0 (fused.cuh) into acc_*[1]
+        const u64 ft = (n_src + fused::TILE - 1) / fused::TILE;
+        {
+            KTimer kt(ctx, KC_MISC, 0);
+            rsort::k_digit_base<<<1, rsort::RADIX, 0, ctx->stream>>>(P_<u32>(ctx->hist), P_<u32>(ctx->base));
+        }
+        RET(ensure(ctx, ctx->status, ft * fused::RADIX * sizeof(u64)));
+        CK(cudaMemsetAsync(ctx->status.p, 0, ft * fused::RADIX * sizeof(u64), ctx->stream));
+        fused::Params fp;
+        fp.ev = src_ev;
+        fp.n = n_src;
+        fp.g = g;
+        fp.ks = ks;
+        fp.tile_sync = P_<u32>(ctx->st_in_s);
+        fp.sync_key = P_<u32>(ctx->syn_k[0]);
+        fp.sync_val = P_<u32>(ctx->syn_v[0]);
+        fp.sync_cap = ctx->sync_cap;
+        fp.digit_base = P_<u32>(ctx->base);
+        fp.status = P_<u64>(ctx->status);
+        fp.kout = P_<u32>(ctx->acc_k[1]);
+        fp.vout = P_<u64>(ctx->acc_v[1]);
+        {
+            // reads every event once, writes the 12-byte access records and 8-byte sync records
+            KTimer kt(ctx, KC_SORT_ACC, 16.0 * (double)n_src + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
+            fused::k_ingest_sort0<<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
+        }
+        CK(cudaGetLastError());
+    }
+    if (n_src > 0 && !FUSED) {
         // pass 1 re-reads the events and writes the (key, value) records
         KTimer kt(ctx, KC_INGEST, 16.0 * (double)n_src + (SH ? 0.0 : 12.0 * (double)n_acc) + 8.0 * (double)n_sync);
         ingest::k_ingest<1><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
@@ -378,7 +410,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     if (n_acc > 0) {
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digit histograms
         const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
-        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[0]), (u32)n_acc, P_<u32>(ctx->hist));
+        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[FUSED ? 1 : 0]), (u32)n_acc,
+                                                         P_<u32>(ctx->hist), FUSED ? 1 : 0);
     }
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
@@ -481,7 +514,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     // ---------------- a5: accesses sorted by word, stable ----------------
     int acur = 0;
     RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur,
-                   vbytes));
+                   vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0));
     ctx->last_acur = acur;
     ctx->last_nacc = SH ? 0 : n_acc;
     mark(ctx, 4);
@@ -680,8 +713,11 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     ctx->afn = alloc_fn;
     ctx->ffn = free_fn;
     ctx->auser = alloc_user;
-    if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = atoi(m) == 0 ? 0 : 1;
+    if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = (atoi(m) >= 0 && atoi(m) <= 2) ? atoi(m) : 1;
     if (const char* m = getenv("IGD_CHECK_STOP")) ctx->check_stop = atoi(m);
+    if (const char* m = getenv("IGD_FUSED")) ctx->fused = atoi(m) != 0;
+    cudaFuncSetAttribute(fused::k_ingest_sort0, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)fused::smem_bytes());
     cudaFuncSetAttribute(rsort::k_onesweep<0, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)rsort::onesweep_smem<u64>());
     cudaFuncSetAttribute(rsort::k_onesweep<1, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -692,6 +728,12 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
                          (int)rsort::onesweep_smem<uint4>());
     cudaFuncSetAttribute(rsort::k_onesweep<0, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)rsort::onesweep_smem<u32>());
+    cudaFuncSetAttribute(rsort::k_onesweep<2, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<u32>());
+    cudaFuncSetAttribute(rsort::k_onesweep<2, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<u64>());
+    cudaFuncSetAttribute(rsort::k_onesweep<2, uint4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)rsort::onesweep_smem<uint4>());
     cudaFuncSetAttribute(rsort::k_onesweep<1, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)rsort::onesweep_smem<u32>());
     if (cudaMallocHost(&ctx->h_stats, 8 * sizeof(u64)) != cudaSuccess ||
@@ -936,7 +978,7 @@ int igd_debug_radix_sort(igd_ctx* ctx, uint32_t* d_keys, uint32_t* d_vals, uint6
                          float* ms) {
     if (!ctx || n >= 0xFFFFFFFFull || (n && (!d_keys || !d_vals))) return IGD_EINVAL;
     cudaSetDevice(ctx->device);
-    ctx->sort_mode = mode == 0 ? 0 : 1;
+    ctx->sort_mode = (mode >= 0 && mode <= 2) ? mode : 1;
     for (int b = 0; b < 2; b++) {
         RET(ensure(ctx, ctx->acc_k[b], n * sizeof(u32)));
         RET(ensure(ctx, ctx->acc_v[b], n * sizeof(u32)));

@@ -39,6 +39,7 @@ struct Params {
     u32* hist_sync;  // [4][256]
     u64* stats;      // [0] min word, [1] max word, [2] bad index, [3] n_acc, [4] n_sync, [5] n_lock
     u32 n_tiles;
+    int hist0;       // pass 0: digit-0 histogram of the access keys (for the fused first sort pass)
 };
 
 // Decoded event: flags bit 0 = access, bits 1..2 = number of sync records, bit 3 = CAS/EXCH,
@@ -202,7 +203,9 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
             const u32 v = (acc ? 1u : 0u) | (ns << 16);
             if (PASS == 0) {
                 if (f & 16u) bad = min(bad, base + (u64)j * THREADS + tid);
-                // (access-key digit histograms: k_hist_keys over the compacted keys)
+                // digit 0 of the access keys for the fused first radix pass (fused.cuh); the other
+                // digits: k_hist_keys over its output
+                if (P.hist0) hist_add(s_hacc[0], dv[j].key & 255u, (f & 1u) != 0, lane);
                 if (__any_sync(IGD_FULL, ns != 0)) {
 #pragma unroll
                     for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s0 >> (8 * p)) & 255u, ns != 0, lane);
@@ -326,7 +329,8 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
 
 // Digit histograms (4 x 8-bit) of the compacted access keys: a light, high-occupancy pass over
 // 4 bytes per access, with warp-uniform digits aggregated into one shared atomic.
-__global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys, u32 n, u32* __restrict__ hist) {
+__global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys, u32 n, u32* __restrict__ hist,
+                                                   int first_digit) {
     __shared__ u32 s[4][256];
     const u32 lane = threadIdx.x & 31u;
     for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&s[0][0])[i] = 0;
@@ -339,13 +343,15 @@ __global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys,
 #pragma unroll
         for (int e = 0; e < 4; e++)
 #pragma unroll
-            for (int p = 0; p < 4; p++) hist_add(s[p], (kk[e] >> (8 * p)) & 255u, in, lane);
+            for (int p = 0; p < 4; p++)
+                if (p >= first_digit) hist_add(s[p], (kk[e] >> (8 * p)) & 255u, in, lane);
     }
     if (blockIdx.x == 0)  // the n % 4 tail
         for (u32 i = n4 * 4 + threadIdx.x; i < n; i += blockDim.x) {
             const u32 k = keys[i];
 #pragma unroll
-            for (int p = 0; p < 4; p++) atomicAdd(&s[p][(k >> (8 * p)) & 255u], 1u);
+            for (int p = 0; p < 4; p++)
+                if (p >= first_digit) atomicAdd(&s[p][(k >> (8 * p)) & 255u], 1u);
         }
     __syncthreads();
     for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) {

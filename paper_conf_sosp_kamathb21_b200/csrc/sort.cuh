@@ -22,14 +22,17 @@ constexpr int WARPS = THREADS / 32;
 #ifndef IGD_SORT_ITEMS
 #define IGD_SORT_ITEMS 16
 #endif
-#ifndef IGD_SORT_VDIRECT
-#define IGD_SORT_VDIRECT 0
-#endif
 #ifndef IGD_SORT_SKIPBITS
 #define IGD_SORT_SKIPBITS 0
 #endif
 #ifndef IGD_SORT_NOLOOKBACK
 #define IGD_SORT_NOLOOKBACK 0
+#endif
+#ifndef IGD_SORT_EARLY
+#define IGD_SORT_EARLY 0
+#endif
+#ifndef IGD_SORT_LB
+#define IGD_SORT_LB 4
 #endif
 constexpr int ITEMS = IGD_SORT_ITEMS;
 constexpr int TILE = THREADS * ITEMS;  // 4096
@@ -129,6 +132,8 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     __shared__ u32 s_gbase[RADIX];
     __shared__ u32 s_tile;
     __shared__ u32 s_wsum[WARPS];
+    __shared__ u32 s_cnt[RADIX];  // tile digit counts (IGD_SORT_EARLY)
+    __shared__ u32 s_match[MODE == 2 ? WARPS : 1][RADIX];  // MODE 2: per-warp lane sets per digit
     __shared__ __align__(8) u64 s_mbar[2];
     extern __shared__ __align__(16) unsigned char s_dyn[];
     u32* s_k = reinterpret_cast<u32*>(s_dyn);                         // keys in, then keys out
@@ -154,6 +159,9 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         }
     }
     for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_whist[0][0])[i] = 0;
+    if (MODE == 2)
+        for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_match[0][0])[i] = 0;
+    if (IGD_SORT_EARLY) s_cnt[t] = 0;
     __syncthreads();
     const u32 tile = s_tile;
     const u32 base = tile * TILE;  // n <= 2^32 - 2^13 (checked by the host)
@@ -174,6 +182,14 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             key[j] = i < P.n ? __ldcs(P.kin + i) : 0u;
         }
     }
+    if (IGD_SORT_EARLY) {
+        // tile digit counts first, published before ranking (see fused.cuh)
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++)
+            if (full || wbase + j * 32 + lane < P.n) atomicAdd(&s_cnt[(key[j] >> shift) & 255u], 1u);
+        __syncthreads();
+        st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
+    }
     u32 rank[ITEMS];
     const u32 lt = lanemask_lt();
 #pragma unroll
@@ -181,13 +197,24 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         const bool valid = full || wbase + j * 32 + lane < P.n;
         const u32 vmask = full ? IGD_FULL : __ballot_sync(IGD_FULL, valid);
         const u32 d = (key[j] >> shift) & 255u;
-        // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set
-        const u32 peers = peers_of<MODE>(valid ? d : (0x100u | lane), vmask);
+        u32 peers;
+        if (MODE == 2) {
+            // lanes with digit d OR their bit into the warp's word for d; one shared atomic and
+            // one load per key instead of eight ballots (CUB's "match atomic-or" ranking)
+            if (valid) atomicOr(&s_match[MODE == 2 ? warp : 0][d], 1u << lane);
+            __syncwarp();
+            peers = valid ? s_match[MODE == 2 ? warp : 0][d] : (1u << lane);
+            __syncwarp();
+        } else {
+            // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set
+            peers = peers_of<MODE>(valid ? d : (0x100u | lane), vmask);
+        }
         const u32 leader = __ffs(peers) - 1;
         u32 old = 0;
         if (lane == leader && valid) {
             old = s_whist[warp][d];
             s_whist[warp][d] = old + __popc(peers);
+            if (MODE == 2) s_match[MODE == 2 ? warp : 0][d] = 0;
         }
         old = __shfl_sync(IGD_FULL, old, leader & 31u);
         rank[j] = old + __popc(peers & lt);
@@ -206,7 +233,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             sum += c;
         }
         cnt = sum;
-        st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
+        if (!IGD_SORT_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
     }
     // block exclusive scan of cnt over digits
     {
@@ -224,20 +251,30 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             if ((u32)w < warp) wpre += s_wsum[w];
         s_tile_excl[t] = wpre + inc - cnt;
     }
-    // decoupled look-back for this digit
+    // Decoupled look-back for this digit: LB predecessor statuses are requested at once, so a
+    // walk back over tiles that have published only their aggregate costs one L2 round trip per
+    // LB tiles instead of one per tile (C5: 127 -> 118 ms over 4 passes with LB = 4; issuing the
+    // first requests before the tile-local reorder to overlap them measured no further gain)
     {
         const u32 d = t;
         u64 excl = 0;
         if (tile > 0 && !IGD_SORT_NOLOOKBACK) {  // NOLOOKBACK: timing experiment only (wrong output)
             long tt = (long)tile - 1;
-            while (tt >= 0) {
-                u64 s;
-                do {
-                    s = ld_relaxed(P.status + (u64)tt * RADIX + d);
-                } while ((s >> 62) == 0);
-                excl += s & ST_VAL_MASK;
-                if ((s >> 62) == 2) break;
-                tt--;
+            bool done = false;
+            while (!done) {
+                u64 s[IGD_SORT_LB];
+#pragma unroll
+                for (int q = 0; q < IGD_SORT_LB; q++)
+                    s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + d) : ST_INC;
+#pragma unroll
+                for (int q = 0; q < IGD_SORT_LB; q++) {
+                    if (!done) {
+                        s[q] = spin_status(P.status + (u64)(tt - q) * RADIX + d, s[q]);
+                        excl += s[q] & ST_VAL_MASK;
+                        done = (s[q] >> 62) == 2;
+                    }
+                }
+                tt -= IGD_SORT_LB;
             }
             st_relaxed(P.status + (u64)tile * RADIX + d, ST_INC | (excl + cnt));
         }
@@ -276,16 +313,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             val[j] = i < P.n ? __ldcs(vin + i) : VT{};
         }
     }
-#if IGD_SORT_VDIRECT
-    // values straight to their output position (L2 merges the partial sectors)
-    __syncthreads();  // s_dig of every position written
-#pragma unroll
-    for (int j = 0; j < ITEMS; j++)
-        if (full || wbase + j * 32 + lane < P.n) {
-            const u32 d = s_dig[rank[j]];
-            __stcs(vout + s_gbase[d] + (rank[j] - s_tile_excl[d]), val[j]);
-        }
-#else
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < ITEMS; j++)
@@ -299,7 +326,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             __stcs(vout + s_gbase[d] + (i - s_tile_excl[d]), s_v[i]);
         }
     }
-#endif
 }
 
 }  // namespace rsort

@@ -215,3 +215,22 @@ def test_c3_full_size_sampled_words_vs_oracle(det):
     mine = np.array([fmix(int(w) ^ (int(w) >> 32)) % K == 5 for w in words], bool)
     assert np.array_equal(got[mine], want)
     assert len(got) == len(led)
+
+
+@pytest.mark.parametrize("env", [{"IGD_FUSED": "0"}, {"IGD_SORT_MODE": "2"}, {"IGD_SORT_MODE": "0"}],
+                         ids=["unfused_ingest", "atomic_or_multisplit", "match_any_multisplit"])
+def test_pipeline_variants_vs_oracle(monkeypatch, env):
+    """The alternate pipeline shapes (unfused ingest write pass + radix pass 0; the other warp
+    multisplit rankings) are selected per context from the environment: same report set."""
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    d = igd.Detector(0)
+    try:
+        w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+        for seed, n, words, nb, bd in [(21, 60_000, 40, 3, 96), (22, 200_000, 30_000, 16, 128)]:
+            ev, nb, bd = _fast_random(seed, n, words, nb, bd, w)
+            assert_same(d, ev, nb, bd, f"{env} seed {seed}")
+    finally:
+        d.close()
