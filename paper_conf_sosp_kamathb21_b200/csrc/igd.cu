@@ -407,14 +407,21 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         shard::k_split_records<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
                                                           P_<u32>(ctx->acc_k[0]), P_<uint4>(ctx->acc_v[0]));
     }
-    if (n_acc > 0) {
+    if (FUSED && n_sync > 0) {
+        // sync-key digit histograms over the records the fused pass wrote (trace order)
+        KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_sync);
+        const unsigned hb = (unsigned)std::min<u64>((n_sync / 4 + 255) / 256 + 1, (u64)sms * 8);
+        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->syn_k[0]), (u32)n_sync,
+                                                         P_<u32>(ctx->hist) + 1024, 0);
+    }
+    if (n_acc > 0 && !FUSED) {  // fused: ingest pass 0 built them
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digit histograms
         const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
-        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[FUSED ? 1 : 0]), (u32)n_acc,
-                                                         P_<u32>(ctx->hist), FUSED ? 1 : 0);
+        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[0]), (u32)n_acc, P_<u32>(ctx->hist), 0);
     }
     CK(cudaGetLastError());
-    CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_hist, ctx->hist.p, (FUSED ? 2048 : 1024) * sizeof(u32), cudaMemcpyDeviceToHost,
+                       ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     mark(ctx, 1);
     u32 h_hist_acc[1024], h_hist_sync[1024];

@@ -39,7 +39,9 @@ struct Params {
     u32* hist_sync;  // [4][256]
     u64* stats;      // [0] min word, [1] max word, [2] bad index, [3] n_acc, [4] n_sync, [5] n_lock
     u32 n_tiles;
-    int hist0;       // pass 0: digit-0 histogram of the access keys (for the fused first sort pass)
+    int hist0;       // pass 0, fused pipeline: the 4 digit histograms of the access keys (digit 0 for
+                     // fused.cuh, 1..3 for the later passes) and no sync-key histograms (k_hist_keys
+                     // over the written sync records instead)
 };
 
 // Decoded event: flags bit 0 = access, bits 1..2 = number of sync records, bit 3 = CAS/EXCH,
@@ -152,6 +154,7 @@ template <int PASS>
 __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
     __shared__ u32 s_hacc[PASS == 0 ? 4 : 1][256];
     __shared__ u32 s_hsync[PASS == 0 ? 4 : 1][256];
+    __shared__ u32 s_hup[PASS == 0 ? 3 : 1][256];  // fused pipeline: access-key digits 1..3
     __shared__ u32 s_wtot[ITEMS][WARPS];  // packed (acc | nsync << 16) per (item, warp)
     __shared__ u32 s_woff[ITEMS][WARPS];  // packed exclusive offsets (acc | sync << 16)
 
@@ -160,6 +163,7 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
         for (int i = tid; i < 4 * 256; i += THREADS) {
             (&s_hacc[0][0])[i] = 0;
             (&s_hsync[0][0])[i] = 0;
+            if (i < 3 * 256) (&s_hup[0][0])[i] = 0;
         }
     u64 wmin = ~0ull, wmax = 0, bad = ~0ull;
     u32 cnt_lock = 0;
@@ -205,8 +209,28 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
                 if (f & 16u) bad = min(bad, base + (u64)j * THREADS + tid);
                 // digit 0 of the access keys for the fused first radix pass (fused.cuh); the other
                 // digits: k_hist_keys over its output
-                if (P.hist0) hist_add(s_hacc[0], dv[j].key & 255u, (f & 1u) != 0, lane);
-                if (__any_sync(IGD_FULL, ns != 0)) {
+                // the low digit is nearly always distinct across lanes: plain shared atomics on
+                // four sub-histograms (warp & 3), no warp vote
+                if (P.hist0) {
+                    const bool acc = (f & 1u) != 0;
+                    if (acc) atomicAdd(&s_hacc[warp & 3u][dv[j].key & 255u], 1u);
+                    // digits 1..3: one set of atomics per warp when the lanes agree on the upper
+                    // 24 bits (lanes of one instruction touch neighbouring words), else per lane
+                    const u32 am = __ballot_sync(IGD_FULL, acc);
+                    if (am) {
+                        const u32 hi = dv[j].key >> 8;
+                        const u32 src = __ffs(am) - 1;
+                        const u32 h0 = __shfl_sync(IGD_FULL, hi, src);
+                        const bool uni = __all_sync(IGD_FULL, !acc || hi == h0);
+                        const u32 c = uni ? (lane == src ? __popc(am) : 0u) : (acc ? 1u : 0u);
+                        if (c) {
+                            atomicAdd(&s_hup[0][hi & 255u], c);
+                            atomicAdd(&s_hup[1][(hi >> 8) & 255u], c);
+                            atomicAdd(&s_hup[2][hi >> 16], c);
+                        }
+                    }
+                }
+                if (!P.hist0 && __any_sync(IGD_FULL, ns != 0)) {
 #pragma unroll
                     for (int p = 0; p < 4; p++) hist_add(s_hsync[p], (dv[j].s0 >> (8 * p)) & 255u, ns != 0, lane);
 #pragma unroll
@@ -305,8 +329,14 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
     // flush per-CTA results
     __syncthreads();
     for (int i = tid; i < 4 * 256; i += THREADS) {
-        const u32 a = (&s_hacc[0][0])[i];
-        if (a) atomicAdd(&P.hist_acc[i], a);
+        if (P.hist0) {
+            const u32 a = i < 256 ? s_hacc[0][i] + s_hacc[1][i] + s_hacc[2][i] + s_hacc[3][i]
+                                  : (&s_hup[0][0])[i - 256];
+            if (a) atomicAdd(&P.hist_acc[i], a);
+        } else {
+            const u32 a = (&s_hacc[0][0])[i];
+            if (a) atomicAdd(&P.hist_acc[i], a);
+        }
         const u32 s = (&s_hsync[0][0])[i];
         if (s) atomicAdd(&P.hist_sync[i], s);
     }
