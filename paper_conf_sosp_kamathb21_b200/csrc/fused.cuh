@@ -44,6 +44,42 @@ struct Params {
     u64* vout;              // access payload (event index | tk << 32), same order
 };
 
+// Decode of an event ingest pass 0 has already validated (the same fields as ingest::decode,
+// without the rule checks): access key and tk (+ mask summaries), or the sync record keys.
+struct FDec {
+    u32 key, tk, ns, s0, s1;
+    bool acc;
+};
+__device__ __forceinline__ FDec fdecode(const uint4& e, const Geo& g, const KeySpace& ks) {
+    FDec d;
+    const u32 tid = ev_tid(e), kind = ev_kind(e);
+    const u32 b = g.block(tid), off = tid - b * g.D, w = b * g.Wb + (off >> 5);
+    d.key = (e.x >> 2) | (e.y << 30);
+    d.tk = e.z;
+    d.ns = 1;
+    d.s1 = 0;
+    d.acc = kind <= IGD_EXCH;
+    if (d.acc) {
+        const u32 lanebit = 1u << (off & 31u);
+        d.tk |= (e.w == IGD_FULL ? (1u << 31) : 0u) | (e.w == lanebit ? (1u << 30) : 0u);
+        d.ns = kind >= IGD_CAS ? 1u : 0u;
+        d.s0 = ks.lock + w;
+    } else if (kind == IGD_FENCE) {
+        d.s0 = ks.any + tid;
+        if (norm_scope(ev_scope(e)) == IGD_SCOPE_DEVICE) {
+            d.s1 = ks.dev + tid;
+            d.ns = 2;
+        }
+    } else if (kind == IGD_SYNCWARP || kind == IGD_CG_TILE_SYNC) {
+        d.s0 = ks.wb + w;
+    } else if (kind == IGD_SYNCTHREADS || kind == IGD_CG_BLOCK_SYNC) {
+        d.s0 = ks.bb + b;
+    } else {
+        d.s0 = ks.grid;
+    }
+    return d;
+}
+
 constexpr size_t smem_bytes() { return (size_t)TILE * sizeof(uint4); }  // 64 KB
 
 __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
@@ -89,17 +125,21 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
     const u32 lt = lanemask_lt();
     u32 key[ITEMS], tk[ITEMS];
     u32 amask = 0;    // bit j: item j is an access
+    u32 nsbits = 0;   // bits 2j..2j+1: sync records of item j (0..2)
     u32 nsync_w = 0;  // sync records of this warp (warp-uniform)
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
         const u32 p = wofs + j * 32 + lane;
-        const ingest::Dec d = ingest::decode(s_ev[p], g, ks);  // valid: ingest pass 0 checked every event
+        const FDec d = fdecode(s_ev[p], g, ks);  // valid: ingest pass 0 checked every event
         const bool in = p < tile_e;
         key[j] = d.key;
         tk[j] = d.tk;
-        amask |= ((in && (d.flags & 1u)) ? 1u : 0u) << j;
-        if (IGD_FUSED_EARLY && in && (d.flags & 1u)) atomicAdd(&s_cnt[d.key & 255u], 1u);
-        const u32 ns = in ? (d.flags >> 1) & 3u : 0u;
+        amask |= ((in && d.acc) ? 1u : 0u) << j;
+        if (IGD_FUSED_EARLY && in && d.acc) atomicAdd(&s_cnt[d.key & 255u], 1u);
+        const u32 ns = in ? d.ns : 0u;
+        nsbits |= ns << (2 * j);
+        // the event's own slot now holds its sync record keys (read back by this thread only)
+        if (ns) *reinterpret_cast<uint2*>(&s_ev[p]) = make_uint2(d.s0, d.s1);
         nsync_w += __popc(__ballot_sync(IGD_FULL, ns >= 1)) + __popc(__ballot_sync(IGD_FULL, ns == 2));
     }
     if (lane == 0) s_wsync[warp] = nsync_w;
@@ -110,7 +150,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
     if (IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
 
     // ---- synchronization records, in trace order: base of this tile (ingest pass 0) + earlier
-    // warps + earlier (item, lane) of this warp; decoded again from the staged tile
+    // warps + earlier (item, lane) of this warp; keys from the event slots
     if (nsync_w) {
         u32 wpre = 0;
 #pragma unroll
@@ -120,17 +160,17 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
 #pragma unroll 1
         for (int j = 0; j < ITEMS; j++) {
             const u32 p = wofs + j * 32 + lane;
-            const ingest::Dec d = ingest::decode(s_ev[p], g, ks);
-            const u32 ns = p < tile_e ? (d.flags >> 1) & 3u : 0u;
+            const u32 ns = (nsbits >> (2 * j)) & 3u;
             const u32 b1 = __ballot_sync(IGD_FULL, ns >= 1), b2 = __ballot_sync(IGD_FULL, ns == 2);
             if (!(b1 | b2)) continue;
             const u64 my = pos + __popc(b1 & lt) + __popc(b2 & lt);
             if (ns && my + ns <= P.sync_cap) {
+                const uint2 sk = *reinterpret_cast<const uint2*>(&s_ev[p]);
                 const u32 ts = (u32)(base + p);
-                P.sync_key[my] = d.s0;
+                P.sync_key[my] = sk.x;
                 P.sync_val[my] = ts;
                 if (ns == 2) {
-                    P.sync_key[my + 1] = d.s1;
+                    P.sync_key[my + 1] = sk.y;
                     P.sync_val[my + 1] = ts;
                 }
             }
