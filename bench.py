@@ -253,6 +253,26 @@ def run_sharded(args, fam, rank, world, local):
     dist.destroy_process_group()
 
 
+# kernel class -> the kernel ncu names for it (classes made of one kernel)
+CLASS_KERNEL = {"sort_access": "rsort::k_onesweep<1, unsigned long>", "check": "check::k_check<0>",
+                "ingest_sort0": "fused::k_ingest_sort0"}
+TRAFFIC_JSON = os.path.join(ROOT, "profiles", "traffic_r01.json")
+
+
+def ncu_traffic(workload, n, kclass):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu launch list of this
+    workload at this size (profiles/traffic_r01.json, written by profiles/summarize_launches.py
+    from an `ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum` run of this bench)."""
+    k = CLASS_KERNEL.get(kclass)
+    try:
+        d = json.load(open(TRAFFIC_JSON)).get(f"{workload}@{n}", {})
+    except (OSError, ValueError):
+        return None, None
+    if k in d:
+        return d[k], f"ncu dram__bytes_read.sum + dram__bytes_write.sum, {os.path.basename(TRAFFIC_JSON)}"
+    return None, None
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -348,8 +368,9 @@ def main():
     total_alg = sum(v[2] for v in kstats.values()) / args.steps
     path_gbs = total_alg / (ms / 1e3) / 1e9
     f_acc = None
+    traffic, tsrc = ncu_traffic(F.FAMILY_NAMES[fam], n, dom)
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "peak_source": peak_kind, "traffic": None,
+                "frac": achieved / peak, "peak_source": peak_kind, "traffic": traffic, "traffic_source": tsrc,
                 "launches_per_step": cnt / args.steps, "ms_per_launch": kms / max(cnt, 1),
                 "alg_bytes_per_launch": kbytes / max(cnt, 1)}
     breakdown = {k: {"launches": v[0] // args.steps, "ms": v[1] / args.steps,

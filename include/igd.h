@@ -186,10 +186,10 @@ const char* igd_stage_name(int stage);
 uint64_t igd_last_launch_count(const igd_ctx* ctx);
 
 /* Per kernel class (0..IGD_N_KCLASS-1: ingest, sort_sync, csr_offsets, lock_infer, sort_access,
-   check, report, misc) of the last igd_detect run with IGD_DETECT_TIMING: launch count, summed
+   check, report, misc, ingest_sort0 = the ingest write pass fused with radix pass 0) of the last igd_detect run with IGD_DETECT_TIMING: launch count, summed
    device time (CUDA events on the context stream around each launch) and the algorithmic bytes
    those launches must move.  Any output pointer may be NULL. */
-#define IGD_N_KCLASS 8
+#define IGD_N_KCLASS 9
 int igd_kernel_stats(const igd_ctx* ctx, int kclass, const char** name, uint32_t* launches, float* ms,
                      double* alg_bytes);
 

@@ -24,7 +24,7 @@
 
 namespace {
 
-enum KClass { KC_INGEST = 0, KC_SORT_SYNC, KC_CSR, KC_LOCK, KC_SORT_ACC, KC_CHECK, KC_REPORT, KC_MISC };
+enum KClass { KC_INGEST = 0, KC_SORT_SYNC, KC_CSR, KC_LOCK, KC_SORT_ACC, KC_CHECK, KC_REPORT, KC_MISC, KC_FUSED };
 
 struct Buf {
     void* p = nullptr;
@@ -33,7 +33,7 @@ struct Buf {
 
 enum Stage { S_INGEST = 0, S_SYNC_SORT, S_TABLES, S_ACC_SORT, S_CHECK, S_REPORT, S_HOST, S_TOTAL };
 const char* kClassNames[IGD_N_KCLASS] = {"ingest", "sort_sync", "csr_offsets", "lock_infer",
-                                         "sort_access", "check", "report", "misc"};
+                                         "sort_access", "check", "report", "misc", "ingest_sort0"};
 constexpr int kMaxTimed = 128;
 const char* kStageNames[IGD_N_STAGES] = {"ingest", "sync_sort", "epoch_lock_tables", "access_sort",
                                          "check", "report_sort", "host_sync", "total"};
@@ -389,7 +389,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         fp.vout = P_<u64>(ctx->acc_v[1]);
         {
             // reads every event once, writes the 12-byte access records and 8-byte sync records
-            KTimer kt(ctx, KC_SORT_ACC, 16.0 * (double)n_src + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
+            KTimer kt(ctx, KC_FUSED, 16.0 * (double)n_src + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
             fused::k_ingest_sort0<<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
         }
         CK(cudaGetLastError());

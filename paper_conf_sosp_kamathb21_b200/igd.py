@@ -20,7 +20,7 @@ IGD_OK, IGD_EINVAL, IGD_ETRACE, IGD_ETOOBIG, IGD_ENOMEM, IGD_ECUDA, IGD_ENCCL, I
 IGD_TRACE_DEVICE_PTR = 1
 IGD_DETECT_TIMING = 1
 IGD_N_STAGES = 8
-IGD_N_KCLASS = 8
+IGD_N_KCLASS = 9
 
 
 class igd_trace_desc(ctypes.Structure):
