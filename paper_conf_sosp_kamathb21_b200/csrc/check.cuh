@@ -171,6 +171,10 @@ __device__ __forceinline__ bool q_grid(const PP& P, u32 a, u32 b) {
     return false;
 }
 
+#ifndef IGD_CHECK_WARPQ
+#define IGD_CHECK_WARPQ 1
+#endif
+
 // queue entry flags
 #define QF_SAME_W 1u
 #define QF_SAME_B 2u
@@ -212,7 +216,15 @@ __global__ void __launch_bounds__(THREADS, IGD_CHECK_MINB) k_check(Params P) {
     __shared__ u32 s_ready;
     __shared__ u32 s_qn;
     // queue of undecided accesses (SoA)
-    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_pos[TILE];  // q_pos: sorted position
+    // per-warp queues of undecided accesses (SoA; q_pos: sorted position): each warp answers
+    // its own queue right after its phase 1, with no CTA-wide barrier in between
+#if IGD_CHECK_WARPQ
+    constexpr int QCAP = 32 * ITEMS;
+    __shared__ u32 s_wqn[WARPS];
+#else
+    constexpr int QCAP = TILE;
+#endif
+    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_pos[TILE];
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     if (t == 0) {
@@ -220,6 +232,9 @@ __global__ void __launch_bounds__(THREADS, IGD_CHECK_MINB) k_check(Params P) {
         // decoupled look-back scans rely on); no atomic round trip before the loads
         s_tile = blockIdx.x;
         s_qn = 0;
+#if IGD_CHECK_WARPQ
+        for (int w = 0; w < WARPS; w++) s_wqn[w] = 0;
+#endif
         s_ready = 0;
     }
     __syncthreads();
@@ -411,7 +426,14 @@ __global__ void __launch_bounds__(THREADS, IGD_CHECK_MINB) k_check(Params P) {
         const u32 qmask = __ballot_sync(IGD_FULL, queue);
         if (qmask) {
             u32 qbase = 0;
+#if IGD_CHECK_WARPQ
+            if (lane == 0) {
+                qbase = warp * QCAP + s_wqn[warp];
+                s_wqn[warp] += __popc(qmask);
+            }
+#else
             if (lane == 0) qbase = atomicAdd(&s_qn, __popc(qmask));
+#endif
             qbase = __shfl_sync(IGD_FULL, qbase, 0);
             if (queue) {
                 const u32 q = qbase + __popc(qmask & lanemask_lt());
@@ -426,12 +448,21 @@ __global__ void __launch_bounds__(THREADS, IGD_CHECK_MINB) k_check(Params P) {
         laTid = c;
         laKind = kind;
     }
+#if IGD_CHECK_WARPQ
+    __syncwarp();
+    if (P.debug_stop == 2) return;
+    // ---- phase 2: the warp's queued accesses, densely over its lanes ----
+    const u32 qn = warp * QCAP + *(volatile u32*)&s_wqn[warp];
+    const KeySpace ks = P.ks;
+    for (u32 q = warp * QCAP + lane; q < qn; q += 32) {
+#else
     __syncthreads();
     if (P.debug_stop == 2) return;
     // ---- phase 2: the queued accesses, densely over the CTA ----
     const u32 qn = s_qn;
     const KeySpace ks = P.ks;
     for (u32 q = t; q < qn; q += THREADS) {
+#endif
         const u32 i = q_i[q], mdIdx = q_md[q];
         const u32 c = q_c[q] & 0xFFFFFFu, flags = q_c[q] >> 24;
         const u32 p = q_p[q] & 0xFFFFFFu;
