@@ -1,0 +1,464 @@
+// check4.cuh -- a6, ballot formulation: per-address segmented shadow-metadata pass + Table 2 check.
+//
+// Same contract as check::k_check (check.cuh) -- accesses sorted by (word, trace index); the
+// shadow state the paper keeps per 4-byte word (Fig. 4; updates P:1000-1058) before
+// access j is a pure function of its word-segment prefix -- but the segmented
+// scan is done with warp ballots instead of a shuffle scan of a packed 64-bit state:
+//
+//   A warp owns 32*ITEMS consecutive sorted accesses, striped: item j of lane l is position
+//   j*32 + l.  Six predicates per access are balloted (segment head, write, atomic, block-scoped
+//   atomic, DevShared pair, BlkShared pair: the adjacent-pair predicates of P:1001-1007, reading
+//   A5).  Every scan quantity the check needs is then "the highest set bit of a predicate mask
+//   at or below my position" compared with my segment's head position:
+//     lastW  = highest write  < j, if >= head      (segmented last-of: P:1013-1016, LW of Fig. 4)
+//     Atomic = highest atomic < j, if >= head, and its scope (reading A6)
+//     DevShared / BlkShared = a pair bit in (head, j]   (sticky OR, A5)
+//   Only accesses before the warp's first head need the state carried in from earlier warps
+//   (a CTA aggregate) and earlier tiles (decoupled look-back on the packed state of check.cuh).
+//
+// Phase 1 (history-free checks P1, P2, P3, P6, P4-lockstep) runs on every access; undecided
+// accesses go to a per-warp shared-memory queue that the warp drains densely (P4 syncwarp, P5,
+// R1..R5 via list queries), with the tile's payload staged in shared memory so md / last-accessor
+// lookups inside the tile are shared-memory reads.
+#pragma once
+#include "check.cuh"
+
+namespace check {
+
+#ifndef IGD_C4_ITEMS
+#define IGD_C4_ITEMS 4
+#endif
+#ifndef IGD_C4_MINB
+#define IGD_C4_MINB 6
+#endif
+#ifndef IGD_C4_STAGED
+#define IGD_C4_STAGED 0  // phase 2 with all list queries of an entry issued at once (measured slower)
+#endif
+constexpr int C4_ITEMS = IGD_C4_ITEMS;
+constexpr int C4_WT = 32 * C4_ITEMS;         // accesses per warp
+constexpr int C4_TILE = THREADS * C4_ITEMS;  // accesses per CTA
+
+__device__ __forceinline__ int hib(u32 m) { return 31 - (int)__clz(m); }  // m != 0
+
+#define QF_MASK 32u  // P4 lockstep clause pending: gather the event's active mask in phase 2
+
+// Staged interval query "is there x in list e with a < x < b" (check.cuh q_between, split so a
+// lane can have several in flight): bq_desc decides from the list descriptor {lo, hi, first,
+// last} or picks an interpolated 8-timestamp probe window; bq_probe decides from that window, or
+// finishes with a binary search (rare: a mis-guessed window).
+struct BQ {
+    u32 a, b, lo, hi, g0;
+    bool done, res;
+};
+__device__ __forceinline__ void bq_desc(BQ& q, const uint4 d) {
+    q.done = true;
+    q.res = false;
+    if (d.x == d.y || d.w <= q.a) return;  // empty, or every element <= a
+    if (d.z > q.a) {                        // the first element is the first one > a
+        q.res = d.z < q.b;
+        return;
+    }
+    q.lo = d.x + 1;
+    q.hi = d.y - 1;
+    u32 g = d.x + 1 + (u32)(__fdividef((float)(q.a - d.z), (float)(d.w - d.z)) * (float)(d.y - 1 - d.x));
+    g = min(max(g, q.lo), q.hi);
+    q.g0 = g & ~7u;
+    q.done = false;
+}
+__device__ __noinline__ bool bq_finish(const u32* __restrict__ ts, u32 lo, u32 hi, u32 a, u32 b) {
+    while (lo < hi) {
+        const u32 mid = (lo + hi) >> 1;
+        if (__ldg(ts + mid) <= a) lo = mid + 1;
+        else hi = mid;
+    }
+    return __ldg(ts + lo) < b;
+}
+__device__ __forceinline__ void bq_probe(BQ& q, const uint4 v0, const uint4 v1, const u32* __restrict__ ts) {
+    const u32 a = q.a, g0 = q.g0;
+    const u32 s0 = max(g0, q.lo), s1 = min(g0 + 8, q.hi + 1);  // probed positions inside [lo, hi]
+    const u32 lem = (u32)(v0.x <= a) | ((u32)(v0.y <= a) << 1) | ((u32)(v0.z <= a) << 2) | ((u32)(v0.w <= a) << 3) |
+                    ((u32)(v1.x <= a) << 4) | ((u32)(v1.y <= a) << 5) | ((u32)(v1.z <= a) << 6) |
+                    ((u32)(v1.w <= a) << 7);
+    const u32 rng = ((1u << (s1 - g0)) - 1u) & ~((1u << (s0 - g0)) - 1u);
+    const u32 le = __popc(lem & rng);
+    q.done = true;
+    if (le != 0 && le != s1 - s0) {  // the successor of a lies inside the window
+        const u32 k = s0 - g0 + le;
+        const uint4 h = k < 4 ? v0 : v1;
+        const u32 kk = k & 3u;
+        const u32 v = kk == 0 ? h.x : kk == 1 ? h.y : kk == 2 ? h.z : h.w;
+        q.res = v < q.b;
+        return;
+    }
+    q.res = le == 0 ? bq_finish(ts, q.lo, s0, a, q.b) : bq_finish(ts, s1, q.hi, a, q.b);
+}
+// grid query continued from list position x (the bucket's first entry was <= a)
+template <class PP>
+__device__ __noinline__ bool q_grid_from(const PP& P, u32 a, u32 b, u32 x) {
+#pragma unroll 1
+    for (int step = 0; x < P.ghi; step++, x++) {
+        const u32 v = __ldg(P.sts + x);
+        if (v > a) return v < b;
+        if (step == 8) return q_between(P.desc, P.sts, P.ks.grid, a, b);
+    }
+    return false;
+}
+
+template <bool MV>
+__global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
+    __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
+    __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
+    __shared__ uint8_t q_f[C4_TILE];              // queue flags
+    __shared__ u64 s_wagg[WARPS];
+    __shared__ u64 s_prefix;
+    __shared__ u32 s_ready;
+
+    const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
+    const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
+    const u32 tbase = tile * C4_TILE;
+    const u32 wloc = warp * C4_WT;
+    const u32 wbase = tbase + wloc;
+    const u32 n = P.n;
+    const Geo g = P.g;
+    if (t == 0) s_ready = 0;
+
+    u32 K[C4_ITEMS], V[C4_ITEMS], Z[C4_ITEMS], M[C4_ITEMS];
+#pragma unroll
+    for (int j = 0; j < C4_ITEMS; j++) {
+        const u32 x = wbase + j * 32 + lane;
+        const bool in = x < n;
+        K[j] = in ? __ldcs(P.key + x) : 0u;
+        if (MV) {
+            const uint4 v = in ? __ldcs(reinterpret_cast<const uint4*>(P.val) + x) : make_uint4(0, 0, 0, 0);
+            V[j] = v.x;
+            Z[j] = v.y;
+            M[j] = v.z;
+        } else {
+            const unsigned long long v = in ? __ldcs(reinterpret_cast<const unsigned long long*>(P.val) + x) : 0ull;
+            V[j] = (u32)v;
+            Z[j] = (u32)(v >> 32);
+            M[j] = 0;
+        }
+    }
+    // the access before the warp's first one
+    u32 cK = 0, cZ = 0;
+    if (lane == 0 && wbase > 0 && wbase <= n) {
+        cK = __ldg(P.key + wbase - 1);
+        cZ = acc_at<MV>(P.val, wbase - 1).tk;
+    }
+#pragma unroll
+    for (int j = 0; j < C4_ITEMS; j++) {
+        s_v[wloc + j * 32 + lane] = V[j];
+        s_z[wloc + j * 32 + lane] = Z[j];
+    }
+
+    // ---- predicates and ballots ----
+    u32 hm[C4_ITEMS], wm[C4_ITEMS], am[C4_ITEMS], bsm[C4_ITEMS], dm[C4_ITEMS], bm[C4_ITEMS];
+#pragma unroll
+    for (int j = 0; j < C4_ITEMS; j++) {
+        const u32 x = wbase + j * 32 + lane;
+        const u32 rK = __shfl_sync(IGD_FULL, K[j], (lane + 31u) & 31u);
+        const u32 rZ = __shfl_sync(IGD_FULL, Z[j], (lane + 31u) & 31u);
+        const u32 pK = lane ? rK : cK, pZ = lane ? rZ : cZ;
+        const bool pvalid = lane ? true : (j > 0 || wbase > 0);
+        cK = rK;  // lane 0: the last access of row j precedes row j+1's first
+        cZ = rZ;
+        const bool in = x < n;
+        const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
+        const bool head = !in || !pvalid || pK != K[j];
+        bool dev = false, blk = false;
+        if (!head) {
+            const u32 pt = pZ & 0xFFFFFFu;
+            const u32 bp = g.block(pt), bc = g.block(c);
+            dev = bp != bc;
+            blk = !dev && g.warp(pt) != g.warp(c);
+        }
+        const bool isA = in && kind >= IGD_ATOM && kind <= IGD_EXCH;
+        hm[j] = __ballot_sync(IGD_FULL, head);
+        wm[j] = __ballot_sync(IGD_FULL, in && kind != IGD_LD);
+        am[j] = __ballot_sync(IGD_FULL, isA);
+        bsm[j] = __ballot_sync(IGD_FULL, isA && norm_scope((Z[j] >> 28) & 3u) == IGD_SCOPE_BLOCK);
+        dm[j] = __ballot_sync(IGD_FULL, dev);
+        bm[j] = __ballot_sync(IGD_FULL, blk);
+    }
+
+    // ---- warp aggregate in the packed state of check.cuh (state after the warp's last access) ----
+    {
+        int H = -1, LW = -1, LA = -1, LD = -1, LB = -1;
+        u32 las = 0;
+#pragma unroll
+        for (int j = 0; j < C4_ITEMS; j++) {
+            if (hm[j]) H = j * 32 + hib(hm[j]);
+            if (wm[j]) LW = j * 32 + hib(wm[j]);
+            if (am[j]) {
+                LA = j * 32 + hib(am[j]);
+                las = (bsm[j] >> hib(am[j])) & 1u ? IGD_SCOPE_BLOCK : IGD_SCOPE_DEVICE;
+            }
+            if (dm[j]) LD = j * 32 + hib(dm[j]);
+            if (bm[j]) LB = j * 32 + hib(bm[j]);
+        }
+        const u64 agg = st_make((LW >= 0 && LW >= H) ? wbase + (u32)LW : IGD_NONE32,
+                                (LA >= 0 && LA >= H) ? las : 0u, LD > H ? 1u : 0u, LB > H ? 1u : 0u,
+                                H >= 0 ? 1u : 0u);
+        if (lane == 0) s_wagg[warp] = agg;
+    }
+    __syncthreads();
+    if (t == 0) {
+        u64 tagg = s_wagg[0];
+#pragma unroll
+        for (int w = 1; w < WARPS; w++) tagg = combine(tagg, s_wagg[w]);
+        u64 prefix = ST_IDENTITY;
+        st_relaxed(&P.status[tile], ((tile == 0 || st_head(tagg)) ? ST_INC : ST_AGG) | tagg);
+        if (tile > 0 && !(hm[0] & 1u) && P.debug_stop != 3) {  // a tile starting with a head needs no prefix
+            // combine predecessors back to an inclusive status or a head-containing aggregate;
+            // a tile with a head has published already (its successors never need more), its
+            // accesses before the first head still need the prefix
+            long tt = (long)tile - 1;
+            u64 acc = ST_IDENTITY;
+            bool have = false;
+            while (tt >= 0) {
+                u64 s;
+                do {
+                    s = ld_relaxed(&P.status[tt]);
+                } while ((s >> 62) == 0);
+                const u64 v = s & ST_VAL_MASK;
+                acc = have ? combine(v, acc) : v;
+                have = true;
+                if ((s >> 62) == 2 || st_head(v)) break;
+                tt--;
+            }
+            prefix = acc;
+            if (!st_head(tagg)) st_relaxed(&P.status[tile], ST_INC | combine(prefix, tagg));
+        }
+        s_prefix = prefix;
+        __threadfence_block();
+        *(volatile u32*)&s_ready = 1u;
+    }
+
+    // state carried into this warp's first segment (needed only before its first head)
+    u64 carry = ST_IDENTITY;
+    if (!(hm[0] & 1u)) {
+        for (u32 w = 0; w < warp; w++) carry = combine(carry, s_wagg[w]);
+        if (!st_head(carry) && tile > 0) {
+            if (P.debug_stop == 3) return;  // profiling: no look-back
+            while (*(volatile u32*)&s_ready == 0u) __nanosleep(32);
+            carry = combine(*(volatile u64*)&s_prefix, carry);
+        }
+    }
+    if (P.debug_stop == 1 || P.debug_stop == 3) {
+        if (carry == 0x123456789ull) P.rep_ctr[1] = carry;
+        return;
+    }
+
+    // ---- phase 1: scan quantities per access, history-free checks, queue the rest ----
+    const u32 lt = lanemask_lt(), le = lt | (1u << lane);
+    int cH = -1, cW = -1, cA = -1, cD = -1, cB = -1;  // highest bit in rows < j
+    u32 cAs = 0;
+    u32 qn = 0;  // warp-uniform queue length
+    const u32 qb = wloc;
+#pragma unroll
+    for (int j = 0; j < C4_ITEMS; j++) {
+        const u32 x = wbase + j * 32 + lane;
+        const bool isHead = (hm[j] >> lane) & 1u;
+        bool queue = false;
+        u32 mdp = 0, fl = 0;
+        if (!isHead) {
+            u32 m = hm[j] & le;
+            const int sH = m ? j * 32 + hib(m) : cH;
+            m = wm[j] & lt;
+            const int lw = m ? j * 32 + hib(m) : cW;
+            m = am[j] & lt;
+            const int la = m ? j * 32 + hib(m) : cA;
+            const u32 las = m ? (((bsm[j] >> hib(m)) & 1u) ? IGD_SCOPE_BLOCK : IGD_SCOPE_DEVICE) : cAs;
+            m = dm[j] & le;
+            const int ldv = m ? j * 32 + hib(m) : cD;
+            m = bm[j] & le;
+            const int lbv = m ? j * 32 + hib(m) : cB;
+            u32 lastW, as;
+            bool dev, blk;
+            if (sH >= 0) {
+                lastW = lw >= sH ? wbase + (u32)lw : IGD_NONE32;
+                as = la >= sH ? las : 0u;
+                dev = ldv > sH;
+                blk = lbv > sH;
+            } else {
+                lastW = lw >= 0 ? wbase + (u32)lw : st_lastW(carry);
+                as = la >= 0 ? las : st_as(carry);
+                dev = ldv >= 0 || st_dev(carry);
+                blk = lbv >= 0 || st_blk(carry);
+            }
+            const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
+            do {
+                if (kind == IGD_LD && lastW == IGD_NONE32) break;  // P2: never written
+                // md: the last writer for a load, the last accessor otherwise
+                mdp = kind == IGD_LD ? lastW : x - 1;
+                const u32 mdz = (mdp - tbase < (u32)C4_TILE) ? s_z[mdp - tbase] : acc_at<MV>(P.val, mdp).tk;
+                const u32 p = mdz & 0xFFFFFFu;
+                if (p == c) break;  // P3: program order
+                const bool isA = kind >= IGD_ATOM && kind <= IGD_EXCH;
+                const u32 bc = g.block(c);
+                const bool same_b = g.block(p) == bc;
+                if (as && isA && (same_b || as == IGD_SCOPE_DEVICE)) break;  // P6
+                const bool same_w = same_b && g.warp(p) == g.warp(c);
+                // P4 lockstep clause: md's lane in this instruction's active mask (tk bit 31: full
+                // warp; bit 30: own lane only; otherwise the mask itself -- in MV mode it travels
+                // with the payload, on one GPU the gather is deferred to phase 2's first round)
+                bool gather = false;
+                if (same_w && !(Z[j] >> 30)) {
+                    if (MV || !IGD_C4_STAGED) {
+                        if ((((MV ? M[j] : ld_event(P.ev, V[j]).w)) >> g.lane(p)) & 1u) break;
+                    } else {
+                        gather = true;
+                    }
+                }
+                if (same_w && (Z[j] >> 31)) break;
+                fl = (same_w ? QF_SAME_W : 0u) | (same_b ? QF_SAME_B : 0u) | (dev ? QF_DEV : 0u) |
+                     (blk ? QF_BLK : 0u) | (gather ? QF_MASK : 0u);
+                if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
+                    u32 lwTid = p;
+                    if (lastW != mdp)
+                        lwTid = ((lastW - tbase < (u32)C4_TILE) ? s_z[lastW - tbase] : acc_at<MV>(P.val, lastW).tk) &
+                                0xFFFFFFu;
+                    if (g.block(lwTid) != bc) fl |= QF_R1;
+                }
+                queue = true;
+            } while (0);
+        }
+        const u32 qmask = __ballot_sync(IGD_FULL, queue);
+        if (queue) {
+            const u32 q = qb + qn + __popc(qmask & lt);
+            q_x[q] = x;
+            q_md[q] = mdp;
+            q_f[q] = (uint8_t)fl;
+        }
+        qn += __popc(qmask);
+        if (hm[j]) cH = j * 32 + hib(hm[j]);
+        if (wm[j]) cW = j * 32 + hib(wm[j]);
+        if (am[j]) {
+            cA = j * 32 + hib(am[j]);
+            cAs = ((bsm[j] >> hib(am[j])) & 1u) ? IGD_SCOPE_BLOCK : IGD_SCOPE_DEVICE;
+        }
+        if (dm[j]) cD = j * 32 + hib(dm[j]);
+        if (bm[j]) cB = j * 32 + hib(bm[j]);
+    }
+    __syncwarp();
+    if (P.debug_stop == 2) return;
+
+    // ---- phase 2: the warp's queued accesses, densely over its lanes ----
+    // Every list query an entry may need is issued at once: round 1 loads the descriptors of
+    // md's warp / block / thread lists, the grid bucket and (deferred P4 lockstep) the event's
+    // active mask; round 2 the 32-byte timestamp probes.  Two dependent L2 round trips per entry
+    // instead of a chain of up to eight.
+    const KeySpace ks = P.ks;
+    for (u32 k = lane; k < qn; k += 32) {
+        const u32 x = q_x[qb + k], mdp = q_md[qb + k], flags = q_f[qb + k];
+        const u32 i = s_v[x - tbase], z = s_z[x - tbase];
+        const u32 c = z & 0xFFFFFFu, kind = (z >> 24) & 0xFu;
+        u32 mdIdx, mdz;
+        if (mdp - tbase < (u32)C4_TILE) {
+            mdIdx = s_v[mdp - tbase];
+            mdz = s_z[mdp - tbase];
+        } else {
+            const Acc a = acc_at<MV>(P.val, mdp);
+            mdIdx = a.idx;
+            mdz = a.tk;
+        }
+        const u32 p = mdz & 0xFFFFFFu;
+        const bool same_w = flags & QF_SAME_W, same_b = flags & QF_SAME_B;
+#if IGD_C4_STAGED
+        // round 1
+        const uint4 none4 = make_uint4(0, 0, 0, 0);
+        const uint4 dW = same_w ? __ldg(P.desc + ks.wb + g.warp(c)) : none4;
+        const uint4 dB = same_b ? __ldg(P.desc + ks.bb + g.block(c)) : none4;
+        const uint4 dF = __ldg(P.desc + (same_b ? ks.any : ks.dev) + p);
+        const bool hasG = P.glo != P.ghi;
+        const u32 gx = hasG ? __ldg(P.gtab + ((mdIdx + 1) >> P.gshift)) : 0u;
+        const u32 emask = (flags & QF_MASK) ? ld_event(P.ev, i).w : 0u;
+        if ((flags & QF_MASK) && ((emask >> g.lane(p)) & 1u)) continue;  // P4: lockstep
+        BQ qW, qB, qF;
+        qW.a = qB.a = qF.a = mdIdx;
+        qW.b = qB.b = qF.b = i;
+        bq_desc(qW, dW);
+        bq_desc(qB, dB);
+        bq_desc(qF, dF);
+        // round 2
+        uint4 w0 = none4, w1 = none4, b0 = none4, b1 = none4, f0 = none4, f1 = none4;
+        if (!qW.done) {
+            w0 = __ldg(reinterpret_cast<const uint4*>(P.sts + qW.g0));
+            w1 = __ldg(reinterpret_cast<const uint4*>(P.sts + qW.g0) + 1);
+        }
+        if (!qB.done) {
+            b0 = __ldg(reinterpret_cast<const uint4*>(P.sts + qB.g0));
+            b1 = __ldg(reinterpret_cast<const uint4*>(P.sts + qB.g0) + 1);
+        }
+        if (!qF.done) {
+            f0 = __ldg(reinterpret_cast<const uint4*>(P.sts + qF.g0));
+            f1 = __ldg(reinterpret_cast<const uint4*>(P.sts + qF.g0) + 1);
+        }
+        const u32 gv = (hasG && gx < P.ghi) ? __ldg(P.sts + gx) : 0xFFFFFFFFu;
+        if (!qW.done) bq_probe(qW, w0, w1, P.sts);
+        if (same_w && qW.res) continue;  // P4: syncwarp
+        bool grid = false;
+        if (hasG && gx < P.ghi) grid = gv > mdIdx ? gv < i : q_grid_from(P, mdIdx, i, gx + 1);
+        if (!qB.done) bq_probe(qB, b0, b1, P.sts);
+        if (same_b && (grid || qB.res)) continue;  // P5
+        if (!qF.done) bq_probe(qF, f0, f1, P.sts);
+        u32 type = (flags & QF_R1) ? IGD_R1 : 0u;
+        if (!type) {
+            if (same_b) {
+                // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread must
+                // not have fenced since md (A1, A30)
+                if (!(flags & QF_DEV) && !grid && !qF.res) type = (same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3;
+            } else if (!grid && !qF.res) {
+                type = IGD_R4;  // R4: other block, no device fence by md's thread
+            }
+        }
+#else
+        if (same_w && q_between(P.desc, P.sts, ks.wb + g.warp(c), mdIdx, i)) continue;  // P4: syncwarp
+        const bool grid = q_grid(P, mdIdx, i);
+        if (same_b && (grid || q_between(P.desc, P.sts, ks.bb + g.block(c), mdIdx, i))) continue;  // P5
+        u32 type = (flags & QF_R1) ? IGD_R1 : 0u;
+        if (!type) {
+            if (same_b) {
+                // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread must
+                // not have fenced since md (A1, A30)
+                if (!(flags & QF_DEV) && !grid && !q_between(P.desc, P.sts, ks.any + p, mdIdx, i))
+                    type = (same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3;
+            } else if (!grid && !q_between(P.desc, P.sts, ks.dev + p, mdIdx, i)) {
+                type = IGD_R4;  // R4: other block, no device fence by md's thread
+            }
+        }
+#endif
+        if (!type && P.lv.any) {  // R5: lock sets of the last accessor and of this access
+            const u32 L = syncx::held_before(P.lv, g, c, i);
+            u32 laIdx, laz;
+            if (x - 1 - tbase < (u32)C4_TILE) {
+                laIdx = s_v[x - 1 - tbase];
+                laz = s_z[x - 1 - tbase];
+            } else {
+                const Acc a = acc_at<MV>(P.val, x - 1);
+                laIdx = a.idx;
+                laz = a.tk;
+            }
+            const u32 locks = syncx::held_before(P.lv, g, laz & 0xFFFFFFu, laIdx);
+            if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
+        }
+        if (type) {
+            const unsigned long long slot = atomicAdd(P.rep_ctr, 1ull);
+            if (slot < P.rep_cap) {
+                igd_report r;
+                // full word from the 32-bit key: the accessed words span < 2^32 from wbase
+                r.addr = (P.wbase + (u32)(__ldg(P.key + x) - (u32)P.wbase)) << 2;
+                r.cur = P.first_event + i;
+                r.prev = P.first_event + mdIdx;
+                r.type = (uint8_t)type;
+                r.cur_kind = (uint8_t)kind;
+                r.prev_kind = (uint8_t)((mdz >> 24) & 0xFu);
+                for (int z2 = 0; z2 < 5; z2++) r.pad[z2] = 0;
+                P.rep[slot] = r;
+            }
+        }
+    }
+}
+
+}  // namespace check

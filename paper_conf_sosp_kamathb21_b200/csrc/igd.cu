@@ -14,6 +14,7 @@
 #include <string>
 
 #include "check.cuh"
+#include "check4.cuh"
 #include "common.cuh"
 #include "fused.cuh"
 #include "ingest.cuh"
@@ -61,6 +62,7 @@ struct igd_ctx {
     u64 rep_cap = 0;
     int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any, 2 = atomic-or (IGD_SORT_MODE)
     int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
+    int check_ver = 4;  // a6 kernel: 4 = ballot formulation (check4.cuh), 3 = shuffle scan (IGD_CHECK_VER)
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
     bool shard = false;
@@ -529,7 +531,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     if (ctx->rep_cap == 0) ctx->rep_cap = 1 << 20;
     u64 n_rep = 0;
     if (n_acc > 0) {
-        const u64 tiles = (n_acc + check::TILE - 1) / check::TILE;
+        const bool V4 = ctx->check_ver == 4;
+        const u64 ctile = V4 ? check::C4_TILE : check::TILE;
+        const u64 tiles = (n_acc + ctile - 1) / ctile;
         for (int attempt = 0;; attempt++) {
             RET(ensure(ctx, ctx->rep_raw, ctx->rep_cap * sizeof(igd_report)));
             RET(ensure(ctx, ctx->rep_ctr, 2 * sizeof(u64)));
@@ -563,8 +567,13 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
-                if (SH) check::k_check<true><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
-                else check::k_check<false><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+                if (V4) {
+                    if (SH) check::k_check4<true><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+                    else check::k_check4<false><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+                } else {
+                    if (SH) check::k_check<true><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+                    else check::k_check<false><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
+                }
             }
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
@@ -722,6 +731,7 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     ctx->auser = alloc_user;
     if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = (atoi(m) >= 0 && atoi(m) <= 2) ? atoi(m) : 1;
     if (const char* m = getenv("IGD_CHECK_STOP")) ctx->check_stop = atoi(m);
+    if (const char* m = getenv("IGD_CHECK_VER")) ctx->check_ver = atoi(m) == 3 ? 3 : 4;
     if (const char* m = getenv("IGD_FUSED")) ctx->fused = atoi(m) != 0;
     cudaFuncSetAttribute(fused::k_ingest_sort0, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes());

@@ -1,6 +1,6 @@
 """Event counters of the check kernel on a workload (what fraction of accesses reach which
 Table-2 stage, how many list queries and how they are answered).
-usage: python profiles/check_stats.py C4"""
+usage: python profiles/check_stats.py C4 [events]"""
 import ctypes
 import json
 import os
@@ -16,7 +16,7 @@ import tracegen.families as F  # noqa: E402
 NAMES = ["checked", "P2", "P3", "P6", "P4_lockstep", "mask_gather", "queued", "q_calls", "q_fast", "q_probe_hit",
          "q_bsearch", "reports", "prefix_waits", "md_lw_load"]
 fam = int(sys.argv[1][1:]) if len(sys.argv) > 1 else 4
-plan = F.Plan(fam)
+plan = F.Plan(fam, n=int(float(sys.argv[2])) if len(sys.argv) > 2 else None)
 ev = plan.fill()
 dev = torch.from_numpy(ev.view(np.uint8)).cuda()
 d = igd.Detector(0)

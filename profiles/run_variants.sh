@@ -4,6 +4,6 @@
 cfg=$1; shift
 for v in "$@"; do
   lib=variants/libigd_$v.so; [ "$v" = "default" ] && lib=paper_conf_sosp_kamathb21_b200/libigd.so
-  IGD_LIB=$lib timeout 600 python bench.py --config $cfg --steps 3 --no-e2e --no-cpu-baseline 2>/dev/null | \
+  IGD_LIB=$lib timeout 600 python bench.py --config $cfg --steps 3 ${EVARGS:-} --no-e2e --no-cpu-baseline 2>/dev/null | \
     python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$v', round(d['value'],3), round(d['ms_per_step'],1), d['config']['reports']==d['config']['ledger_reports'], json.dumps({k:round(v['ms'],1) for k,v in d['path']['kernels'].items()}))"
 done
