@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
     }
 
     // ---- predicates and ballots ----
-    u32 hm[C4_ITEMS], wm[C4_ITEMS], am[C4_ITEMS], bsm[C4_ITEMS], dm[C4_ITEMS], bm[C4_ITEMS];
+    u32 hm[C4_ITEMS], wm[C4_ITEMS], am[C4_ITEMS], bsm[C4_ITEMS], dm[C4_ITEMS], bm[C4_ITEMS], tm[C4_ITEMS];
 #pragma unroll
     for (int j = 0; j < C4_ITEMS; j++) {
         const u32 x = wbase + j * 32 + lane;
@@ -166,12 +166,13 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
         const bool in = x < n;
         const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
         const bool head = !in || !pvalid || pK != K[j];
-        bool dev = false, blk = false;
+        bool dev = false, blk = false, same_t = false;
         if (!head) {
             const u32 pt = pZ & 0xFFFFFFu;
             const u32 bp = g.block(pt), bc = g.block(c);
             dev = bp != bc;
             blk = !dev && g.warp(pt) != g.warp(c);
+            same_t = pt == c;
         }
         const bool isA = in && kind >= IGD_ATOM && kind <= IGD_EXCH;
         hm[j] = __ballot_sync(IGD_FULL, head);
@@ -180,6 +181,11 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
         bsm[j] = __ballot_sync(IGD_FULL, isA && norm_scope((Z[j] >> 28) & 3u) == IGD_SCOPE_BLOCK);
         dm[j] = __ballot_sync(IGD_FULL, dev);
         bm[j] = __ballot_sync(IGD_FULL, blk);
+        tm[j] = __ballot_sync(IGD_FULL, same_t);
+        // P4's lockstep clause will need this instruction's active mask when md is likely the
+        // previous access, from another lane of the same warp, and the mask is partial: gather
+        // it now so the trace read overlaps the scans (phase 1 re-checks the exact condition)
+        if (!MV && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) M[j] = ld_event(P.ev, V[j]).w;
     }
 
     // ---- warp aggregate in the packed state of check.cuh (state after the warp's last access) ----
@@ -251,6 +257,9 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
     }
 
     // ---- phase 1: scan quantities per access, history-free checks, queue the rest ----
+    auto tk_at = [&](u32 pos) -> u32 {  // tk of sorted position pos (tile: shared memory)
+        return (pos - tbase < (u32)C4_TILE) ? s_z[pos - tbase] : acc_at<MV>(P.val, pos).tk;
+    };
     const u32 lt = lanemask_lt(), le = lt | (1u << lane);
     int cH = -1, cW = -1, cA = -1, cD = -1, cB = -1;  // highest bit in rows < j
     u32 cAs = 0;
@@ -290,36 +299,48 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
             const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
             do {
                 if (kind == IGD_LD && lastW == IGD_NONE32) break;  // P2: never written
-                // md: the last writer for a load, the last accessor otherwise
-                mdp = kind == IGD_LD ? lastW : x - 1;
-                const u32 mdz = (mdp - tbase < (u32)C4_TILE) ? s_z[mdp - tbase] : acc_at<MV>(P.val, mdp).tk;
-                const u32 p = mdz & 0xFFFFFFu;
-                if (p == c) break;  // P3: program order
+                // md: the last writer for a load, the last accessor otherwise.  When
+                // md is the previous access of the segment (the common case) the thread / block /
+                // warp relations to it are the pair bits balloted above: no lookup, no division.
+                const bool prevMd = kind != IGD_LD || lastW == x - 1;
+                mdp = prevMd ? x - 1 : lastW;
                 const bool isA = kind >= IGD_ATOM && kind <= IGD_EXCH;
-                const u32 bc = g.block(c);
-                const bool same_b = g.block(p) == bc;
+                bool same_t, same_b, same_w;
+                u32 p = IGD_NONE32;  // md's thread, looked up only when needed
+                if (prevMd) {
+                    same_t = (tm[j] >> lane) & 1u;
+                    same_b = !((dm[j] >> lane) & 1u);
+                    same_w = same_b && !((bm[j] >> lane) & 1u);
+                } else {
+                    p = tk_at(mdp) & 0xFFFFFFu;
+                    same_t = p == c;
+                    same_b = g.block(p) == g.block(c);
+                    same_w = same_b && g.warp(p) == g.warp(c);
+                }
+                if (same_t) break;                                             // P3: program order
                 if (as && isA && (same_b || as == IGD_SCOPE_DEVICE)) break;  // P6
-                const bool same_w = same_b && g.warp(p) == g.warp(c);
                 // P4 lockstep clause: md's lane in this instruction's active mask (tk bit 31: full
-                // warp; bit 30: own lane only; otherwise the mask itself -- in MV mode it travels
-                // with the payload, on one GPU the gather is deferred to phase 2's first round)
+                // warp; bit 30: own lane only; otherwise the mask itself, from the payload in MV
+                // mode, else gathered from the trace)
+                if (same_w && (Z[j] >> 31)) break;
                 bool gather = false;
                 if (same_w && !(Z[j] >> 30)) {
+                    if (p == IGD_NONE32) p = tk_at(mdp) & 0xFFFFFFu;
                     if (MV || !IGD_C4_STAGED) {
-                        if ((((MV ? M[j] : ld_event(P.ev, V[j]).w)) >> g.lane(p)) & 1u) break;
+                        // prefetched unless md is an earlier writer (M[j] is the mask then only
+                        // if the previous access was also a same-warp candidate)
+                        const bool pre = MV || (prevMd && !(Z[j] >> 30));
+                        if ((((pre ? M[j] : ld_event(P.ev, V[j]).w)) >> g.lane(p)) & 1u) break;
                     } else {
                         gather = true;
                     }
                 }
-                if (same_w && (Z[j] >> 31)) break;
                 fl = (same_w ? QF_SAME_W : 0u) | (same_b ? QF_SAME_B : 0u) | (dev ? QF_DEV : 0u) |
                      (blk ? QF_BLK : 0u) | (gather ? QF_MASK : 0u);
                 if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
-                    u32 lwTid = p;
-                    if (lastW != mdp)
-                        lwTid = ((lastW - tbase < (u32)C4_TILE) ? s_z[lastW - tbase] : acc_at<MV>(P.val, lastW).tk) &
-                                0xFFFFFFu;
-                    if (g.block(lwTid) != bc) fl |= QF_R1;
+                    const bool other =
+                        lastW == mdp ? !same_b : g.block(tk_at(lastW) & 0xFFFFFFu) != g.block(c);
+                    if (other) fl |= QF_R1;
                 }
                 queue = true;
             } while (0);
@@ -429,8 +450,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
             }
         }
 #endif
-        if (!type && P.lv.any) {  // R5: lock sets of the last accessor and of this access
-            const u32 L = syncx::held_before(P.lv, g, c, i);
+        if (!type && P.lv.any && P.debug_stop != 4) {  // R5: lock sets of the last accessor and of this access
             u32 laIdx, laz;
             if (x - 1 - tbase < (u32)C4_TILE) {
                 laIdx = s_v[x - 1 - tbase];
@@ -440,7 +460,8 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
                 laIdx = a.idx;
                 laz = a.tk;
             }
-            const u32 locks = syncx::held_before(P.lv, g, laz & 0xFFFFFFu, laIdx);
+            u32 L, locks;
+            syncx::held_before2(P.lv, g, c, i, laz & 0xFFFFFFu, laIdx, L, locks);
             if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
         }
         if (type) {

@@ -38,12 +38,34 @@ struct Geo {
     u32 W;   // warps
     u32 B;   // blocks
     FastDiv fd;
-    __device__ __forceinline__ u32 block(u32 t) const { return fd.div(t); }
+    u32 dlog;  // log2(D) when D is a power of two, else 32
+    u32 a32;   // D % 32 == 0: warps never straddle blocks, so warp(t) = t / 32 and lane(t) = t % 32
+    __host__ void init(u32 nb, u32 bd) {
+        D = bd;
+        Wb = (bd + 31) / 32;
+        B = nb;
+        T = nb * bd;
+        W = nb * Wb;
+        fd.init(bd);
+        dlog = 32;
+        for (u32 l = 0; l < 32; l++)
+            if ((1u << l) == bd) dlog = l;
+        a32 = bd % 32 == 0 ? 1u : 0u;
+    }
+#ifndef IGD_GEO_FAST
+#define IGD_GEO_FAST 0
+#endif
+    __device__ __forceinline__ u32 block(u32 t) const {
+        if (IGD_GEO_FAST) return dlog < 32 ? t >> dlog : fd.div(t);
+        return fd.div(t);
+    }
     __device__ __forceinline__ u32 warp(u32 t) const {
+        if (IGD_GEO_FAST && a32) return t >> 5;
         u32 b = fd.div(t);
         return b * Wb + ((t - b * D) >> 5);
     }
     __device__ __forceinline__ u32 lane(u32 t) const {
+        if (IGD_GEO_FAST && a32) return t & 31u;
         u32 b = fd.div(t);
         return (t - b * D) & 31u;
     }

@@ -56,12 +56,13 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
-    Buf off, ldesc, gtab, sw, wcnt, tcnt, wpts, tpts;
+    Buf off, ldesc, gtab, sw, wcnt, tcnt, wpts, tpts, wdesc;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
     int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any, 2 = atomic-or (IGD_SORT_MODE)
     int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
+    int count_tma = 0;  // IGD_COUNT_TMA=1: ingest pass 0 through a TMA ring (ingest::k_count; measured slower: 8.6 vs 7.2 ms at C5 1e9, the pass is issue-bound)
     int check_ver = 4;  // a6 kernel: 4 = ballot formulation (check4.cuh), 3 = shuffle scan (IGD_CHECK_VER)
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
@@ -175,14 +176,7 @@ static u32 bits_needed(u64 maxval) {
     return b;
 }
 
-static void geo_init(Geo& g, u32 nb, u32 bd) {
-    g.D = bd;
-    g.Wb = (bd + 31) / 32;
-    g.B = nb;
-    g.T = nb * bd;
-    g.W = nb * g.Wb;
-    g.fd.init(bd);
-}
+static void geo_init(Geo& g, u32 nb, u32 bd) { g.init(nb, bd); }
 
 static int sm_count(igd_ctx* ctx) {
     int v = 148;
@@ -332,7 +326,16 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const u64 grid = std::max<u64>(1, std::min<u64>((u64)sms * (occ > 0 ? occ : 1), in_tiles));
     if (n_src > 0) {
         KTimer kt(ctx, KC_INGEST, 16.0 * (double)n_src);  // pass 0 reads every event
-        ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+        if (ctx->count_tma) {
+            // trace streamed through a TMA ring in shared memory (ingest::k_count)
+            const size_t smem = ingest::count_smem();
+            int occ2 = 0;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, ingest::k_count, ingest::THREADS, smem);
+            const u64 grid2 = std::max<u64>(1, std::min<u64>((u64)sms * (occ2 > 0 ? occ2 : 1), in_tiles));
+            ingest::k_count<<<(unsigned)grid2, ingest::THREADS, smem, ctx->stream>>>(ip);
+        } else {
+            ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+        }
     }
     CK(cudaGetLastError());
     RET(scan_excl(ctx, P_<u32>(ctx->st_in_a), in_tiles + 1));
@@ -510,6 +513,15 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             syncx::k_lock_infer<true><<<lblocks, 256, 0, ctx->stream>>>(lp);
         }
         CK(cudaGetLastError());
+        RET(ensure(ctx, ctx->wdesc, ((u64)g.W + 1) * sizeof(uint4)));
+        {
+            KTimer kt(ctx, KC_LOCK, 0);
+            const unsigned db = (unsigned)std::min<u64>(((u64)g.W + 255) / 256, (u64)sms * 8);
+            syncx::k_lock_desc<<<db, 256, 0, ctx->stream>>>(P_<u32>(ctx->off), ks.lock, P_<u32>(ctx->sw),
+                                                            P_<u32>(ctx->wcnt), g.W, P_<uint4>(ctx->wdesc));
+            CK(cudaGetLastError());
+        }
+        lv.wdesc = P_<uint4>(ctx->wdesc);
         lv.off = P_<u32>(ctx->off);
         lv.lock_key0 = ks.lock;
         lv.switch_ts = P_<u32>(ctx->sw);
@@ -731,8 +743,10 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     ctx->auser = alloc_user;
     if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = (atoi(m) >= 0 && atoi(m) <= 2) ? atoi(m) : 1;
     if (const char* m = getenv("IGD_CHECK_STOP")) ctx->check_stop = atoi(m);
+    if (const char* m = getenv("IGD_COUNT_TMA")) ctx->count_tma = atoi(m) != 0;
     if (const char* m = getenv("IGD_CHECK_VER")) ctx->check_ver = atoi(m) == 3 ? 3 : 4;
     if (const char* m = getenv("IGD_FUSED")) ctx->fused = atoi(m) != 0;
+    cudaFuncSetAttribute(ingest::k_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ingest::count_smem());
     cudaFuncSetAttribute(fused::k_ingest_sort0, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes());
     cudaFuncSetAttribute(rsort::k_onesweep<0, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -930,7 +944,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->sw,       &ctx->wcnt,
                   &ctx->tcnt,
-                  &ctx->wpts,         &ctx->tpts,     &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
+                  &ctx->wpts,         &ctx->tpts,     &ctx->wdesc,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf};
     for (Buf* b : all) buf_free(ctx, *b);

@@ -236,8 +236,59 @@ struct LockView {
     const u32* toff;
     const u64* wpts;
     const u64* tpts;
+    const uint4* wdesc;  // per warp {woff[w], woff[w+1], switch_ts[w], has CAS/EXCH} (k_lock_desc)
     u32 any;  // 0 when the trace has no CAS/EXCH at all
 };
+
+// One 16-byte descriptor per warp for the check's lock-set queries: one load decides "this warp
+// never takes a lock" and carries the bounds of its change-point list and its switch time.
+__global__ void k_lock_desc(const u32* __restrict__ off, u32 lock_key0, const u32* __restrict__ switch_ts,
+                            const u32* __restrict__ woff, u32 W, uint4* __restrict__ wdesc) {
+    for (u32 w = blockIdx.x * blockDim.x + threadIdx.x; w < W; w += gridDim.x * blockDim.x)
+        wdesc[w] = make_uint4(woff[w], woff[w + 1], switch_ts[w],
+                              off[lock_key0 + w] != off[lock_key0 + w + 1] ? 1u : 0u);
+}
+
+// Lock sets of two (thread, time) pairs at once -- the check's L(c, i) and L(la) of R5 -- with
+// the two descriptor loads and the two binary searches interleaved (independent L2 chains).
+__device__ __forceinline__ void held_before2(const LockView& V, const Geo& g, u32 c0, u32 i0, u32 c1, u32 i1,
+                                             u32& L0, u32& L1) {
+    L0 = L1 = 0;
+    const uint4 d0 = __ldg(V.wdesc + g.warp(c0)), d1 = __ldg(V.wdesc + g.warp(c1));
+    if (!d0.w && !d1.w) return;
+    // list bounds: the per-thread list after the warp's switch time, else the per-warp list
+    const bool t0 = d0.w && d0.z != IGD_NONE32 && i0 > d0.z, t1 = d1.w && d1.z != IGD_NONE32 && i1 > d1.z;
+    u32 lo0 = d0.x, hi0 = d0.w ? d0.y : d0.x, lo1 = d1.x, hi1 = d1.w ? d1.y : d1.x;
+    if (t0) {
+        lo0 = __ldg(V.toff + c0);
+        hi0 = __ldg(V.toff + c0 + 1);
+    }
+    if (t1) {
+        lo1 = __ldg(V.toff + c1);
+        hi1 = __ldg(V.toff + c1 + 1);
+    }
+    const u64* p0 = t0 ? V.tpts : V.wpts;
+    const u64* p1 = t1 ? V.tpts : V.wpts;
+    const u32 b0 = lo0, b1 = lo1;
+    // last entry with ts < i: first entry with ts >= i, minus one
+    while (lo0 < hi0 || lo1 < hi1) {
+        const u32 m0 = (lo0 + hi0) >> 1, m1 = (lo1 + hi1) >> 1;
+        const bool a0 = lo0 < hi0, a1 = lo1 < hi1;
+        const u64 v0 = a0 ? __ldg(p0 + m0) : 0ull, v1 = a1 ? __ldg(p1 + m1) : 0ull;
+        if (a0) {
+            if ((u32)(v0 >> 16) < i0) lo0 = m0 + 1;
+            else hi0 = m0;
+        }
+        if (a1) {
+            if ((u32)(v1 >> 16) < i1) lo1 = m1 + 1;
+            else hi1 = m1;
+        }
+    }
+    const u64 e0 = (d0.w && lo0 > b0) ? __ldg(p0 + lo0 - 1) : 0ull;
+    const u64 e1 = (d1.w && lo1 > b1) ? __ldg(p1 + lo1 - 1) : 0ull;
+    L0 = (u32)(e0 & 0xFFFFu);
+    L1 = (u32)(e1 & 0xFFFFu);
+}
 
 __device__ __forceinline__ u32 last_before(const u64* __restrict__ pts, u32 lo, u32 hi, u32 i) {
     // last entry with ts < i
