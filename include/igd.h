@@ -59,6 +59,12 @@ typedef struct {
 #define IGD_CG_TILE_SYNC 9 /* == SYNCWARP */
 #define IGD_CG_BLOCK_SYNC 10 /* == SYNCTHREADS */
 #define IGD_CG_GRID_SYNC 11  /* == GRID_SYNC */
+#define IGD_KERNEL_BOUNDARY 12 /* end of one kernel, start of the next (reading A31):
+                                  the implicit all-thread barrier at kernel end
+                                  orders everything before it before everything after it, so every
+                                  word's shadow state is discarded (its next access is P1), and the
+                                  locking protocol is inferred per kernel: every lock
+                                  table and isThread bit is reset.  One geometry for all kernels. */
 /* scope (tk bits 28..29) */
 #define IGD_SCOPE_NONE 0
 #define IGD_SCOPE_BLOCK 1
@@ -73,7 +79,8 @@ typedef struct {
  *   SYNCWARP, CG_TILE : addr 0, tid = any thread of the warp (< threads), scope NONE
  *   SYNCTHREADS, CG_BLOCK : addr 0, tid = any thread of the block (< threads), scope NONE
  *   GRID_SYNC, CG_GRID: addr 0, tid 0, scope NONE
- *   kind > 11 or tk bits 30..31 set: invalid.
+ *   KERNEL_BOUNDARY   : addr 0, tid 0, scope NONE
+ *   kind > 12 or tk bits 30..31 set: invalid.
  * Geometry: block(t) = t / block_dim, warps per block
  * Wb = ceil(block_dim/32), warp(t) = block(t)*Wb + (t % block_dim)/32,
  * lane(t) = (t % block_dim) % 32.

@@ -27,7 +27,8 @@
 
 /* ---- trace encoding, read with the oracle's own reader ---------------- */
 enum { O_LD = 0, O_ST = 1, O_ATOM = 2, O_CAS = 3, O_EXCH = 4, O_FENCE = 5, O_SYNCWARP = 6,
-       O_SYNCTHREADS = 7, O_GRID = 8, O_CG_TILE = 9, O_CG_BLOCK = 10, O_CG_GRID = 11 };
+       O_SYNCTHREADS = 7, O_GRID = 8, O_CG_TILE = 9, O_CG_BLOCK = 10, O_CG_GRID = 11,
+       O_KERNEL = 12 /* kernel boundary (reading A31) */ };
 enum { S_NONE = 0, S_BLOCK = 1, S_DEVICE = 2, S_SYSTEM = 3 };
 enum { R_NONE = 0, R1 = 1, R2 = 2, R3 = 3, R4 = 4, R5 = 5 };
 
@@ -93,6 +94,7 @@ typedef struct {
 
 typedef struct {
     uint64_t word;
+    uint64_t kernel;              /* kernel (boundaries before it) the entry was written in (A31) */
     uint8_t used;                 /* hash slot occupied */
     uint8_t valid, modified, atomic, ascope, devShared, blkShared;
     uint16_t locks;               /* Bloom of the last accessor's held locks (A7) */
@@ -152,7 +154,7 @@ static uint32_t o_fmix32(uint32_t h) {
 
 /* Field rules per kind. Returns 1 when the event is well-formed. */
 static int o_valid(const o_event* e, const o_geom* g) {
-    if (e->kind > O_CG_GRID) return 0;
+    if (e->kind > O_KERNEL) return 0;
     if (e->tid >= g->threads) return 0;
     uint32_t lanebit = 1u << g_lane(g, e->tid);
     switch (e->kind) {
@@ -164,7 +166,7 @@ static int o_valid(const o_event* e, const o_geom* g) {
         return e->addr == 0 && (e->mask & lanebit) && e->scope != S_NONE;
     case O_SYNCWARP: case O_CG_TILE: case O_SYNCTHREADS: case O_CG_BLOCK:
         return e->addr == 0 && e->scope == S_NONE;
-    case O_GRID: case O_CG_GRID:
+    case O_GRID: case O_CG_GRID: case O_KERNEL:
         return e->addr == 0 && e->scope == S_NONE && e->tid == 0;
     }
     return 0;
@@ -207,6 +209,7 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
     uint64_t* wbar = (uint64_t*)calloc(g.warps, sizeof(uint64_t));
     uint64_t* bbar = (uint64_t*)calloc(g.blocks, sizeof(uint64_t));
     uint64_t G = 0;
+    uint64_t kernel = 0; /* kernel boundaries so far (A31) */
     o_table* wt = (o_table*)calloc(g.warps, sizeof(o_table));
     o_table* tt = (o_table*)calloc(g.threads, sizeof(o_table));
     uint8_t* isThread = (uint8_t*)calloc(g.warps, 1);
@@ -262,6 +265,28 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
             continue;
         }
 
+        if (k == O_KERNEL) {
+            /* A31: the kernel ends.  Its implicit all-thread barrier orders
+               every access before it before every access after it: every word's shadow entry
+               is discarded (lazily, by kernel number), and the next kernel's locking protocol
+               is inferred afresh: lock tables and isThread bits reset. */
+            kernel++;
+            for (uint32_t q = 0; q < n_touched; q++) {
+                uint32_t w = touched_list[q];
+                memset(&wt[w], 0, sizeof(o_table));
+                isThread[w] = 0;
+                touched[w] = 0;
+                uint32_t b = w / g.Wb, wi = w % g.Wb;
+                for (uint32_t l = 0; l < 32; l++) {
+                    uint32_t off = wi * 32 + l;
+                    if (off >= g.D) break;
+                    memset(&tt[b * g.D + off], 0, sizeof(o_table));
+                }
+            }
+            n_touched = 0;
+            continue;
+        }
+
         /* ---- Step 3: an access (LD/ST/ATOM/CAS/EXCH) ---- */
         int isWrite = (k != O_LD);                                /* atomics are stores */
         int isAtomic = (k == O_ATOM || k == O_CAS || k == O_EXCH);
@@ -273,7 +298,13 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
         if (owned) {
             o_shadow* S = o_map_get(&map, word);
             if (!S) { rc = O_ENOMEM; goto done; }
-            if (!S->valid) goto writeback;                        /* P1: first access */
+            if (S->valid && S->kernel != kernel) {                /* A31: from an earlier kernel */
+                uint64_t wd = S->word;
+                memset(S, 0, sizeof(*S));
+                S->used = 1;
+                S->word = wd;
+            }
+            if (!S->valid) goto writeback;                        /* P1: first access (this kernel) */
 
             /* sharing flags vs the last accessor, sticky (A5) */
             {
@@ -323,6 +354,7 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
                 r.idx = i; r.tid = c; r.kind = e.kind;
                 r.sDEV = DEV(c); r.sANY = ANY(c); r.sWB = WB(w_c); r.sBB = BB(b_c);
                 S->valid = 1;
+                S->kernel = kernel;
                 S->LA = r;
                 S->locks = L;
                 if (isWrite) { S->modified = 1; S->LW = r; }
@@ -368,4 +400,4 @@ done:
 }
 
 /* Exported constants so the Python side can check it loaded this library. */
-int igdo_version(void) { return 1; }
+int igdo_version(void) { return 2; }

@@ -25,8 +25,9 @@ assert REPORT_DTYPE.itemsize == 32
 # kind codes
 LD, ST, ATOM, CAS, EXCH, FENCE, SYNCWARP, SYNCTHREADS, GRID_SYNC = range(9)
 CG_TILE_SYNC, CG_BLOCK_SYNC, CG_GRID_SYNC = 9, 10, 11
+KERNEL_BOUNDARY = 12  # multi-kernel traces
 KIND_NAMES = ["LD", "ST", "ATOM", "CAS", "EXCH", "FENCE", "SYNCWARP", "SYNCTHREADS", "GRID_SYNC",
-              "CG_TILE_SYNC", "CG_BLOCK_SYNC", "CG_GRID_SYNC"]
+              "CG_TILE_SYNC", "CG_BLOCK_SYNC", "CG_GRID_SYNC", "KERNEL_BOUNDARY"]
 # scope codes
 NONE, BLOCK, DEVICE, SYSTEM = 0, 1, 2, 3
 SCOPE_NAMES = ["NONE", "BLOCK", "DEVICE", "SYSTEM"]
@@ -114,6 +115,9 @@ class TraceBuilder:
     def grid_sync(self):
         return self.ev(GRID_SYNC, 0, 0, NONE, 0xFFFFFFFF)
 
+    def kernel_boundary(self):
+        return self.ev(KERNEL_BOUNDARY, 0, 0, NONE, 0xFFFFFFFF)
+
     def events(self):
         out = np.zeros(len(self.rows), EVENT_DTYPE)
         if self.rows:
@@ -141,9 +145,9 @@ def random_trace(seed: int, n: int, n_blocks: int = None, block_dim: int = None,
     if block_dim is None:
         block_dim = int(rng.choice([32, 64, 96]))
     g = Geometry(n_blocks, block_dim)
-    kinds = np.arange(12)
     if weights is None:
         weights = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    kinds = np.arange(len(weights))  # 13 weights: kernel boundaries too
     w = np.asarray(weights, float)
     w = w / w.sum()
     b = TraceBuilder(n_blocks, block_dim)
@@ -185,3 +189,23 @@ def random_trace(seed: int, n: int, n_blocks: int = None, block_dim: int = None,
         else:
             b.ev(k, 0, 0, NONE, 0xFFFFFFFF)
     return b.events(), n_blocks, block_dim
+
+
+def boundary_event() -> np.ndarray:
+    """One KERNEL_BOUNDARY event (addr 0, tid 0, scope NONE)."""
+    e = np.zeros(1, EVENT_DTYPE)
+    e["tk"] = pack_tk(0, KERNEL_BOUNDARY, NONE)
+    e["mask"] = 0xFFFFFFFF
+    return e
+
+
+def concat_kernels(traces) -> np.ndarray:
+    """Join per-kernel traces (same geometry) into one multi-kernel trace, a KERNEL_BOUNDARY
+    between consecutive kernels.  Returns the trace; kernel k's events start at
+    sum(len(t) + 1 for t in traces[:k])."""
+    parts = []
+    for k, t in enumerate(traces):
+        if k:
+            parts.append(boundary_event())
+        parts.append(np.asarray(t, EVENT_DTYPE))
+    return np.concatenate(parts) if parts else np.zeros(0, EVENT_DTYPE)
