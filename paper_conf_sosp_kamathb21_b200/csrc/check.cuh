@@ -1,26 +1,14 @@
-// check.cuh -- a6: per-address segmented shadow-metadata pass + Table 2 race check.
+// check.cuh -- a6 building blocks shared by the check kernel (check4.cuh) and the report stage:
 //
-// Input: accesses sorted by (word key, trace index).  Within one word's segment the shadow
-// state the paper keeps per 4-byte word (Fig. 4; updates P:1000-1058) before access
-// j is a pure function of the segment prefix ("equivalent formulation"):
-//   valid      = j is not the segment head                         (P1)
-//   LA         = access j-1                                          (last accessor)
-//   LW         = last write before j             -> segmented last-of scan
-//   Atomic/Scope = any atomic before j / scope of the last one       (reading A6)
-//   DevShared / BlkShared = OR of adjacent-pair predicates up to j   (A5)
-//   Locks      = held-lock Bloom of LA at LA's time                  (A7)
-//
-// Two phases per 1024-access tile (256 threads x 4 consecutive accesses):
-//  1. streaming: coalesced key/index loads, one 16-byte event gather per access, thread-local
-//     + warp-shuffle + block scans of the packed shadow state, decoupled look-back across tiles
-//     (a tile containing a segment head publishes its inclusive state at once, so only tiles
-//     inside one long hot-word segment wait), then the checks that need no synchronization
-//     history: P1, P2, P3, P6 and P4's lockstep clause.
-//  2. the accesses still undecided are queued in shared memory and processed densely by the
-//     whole CTA: P4 (syncwarp), P5, R1..R5.  The synchronization-counter comparisons of Table 2
-//     become interval queries on the a2 lists ("did md's thread fence in (md.idx, i)?", reading
-//     A1), answered by a per-list descriptor {lo, hi, first, last} and interpolation-guided
-//     32-byte probes (two dependent loads for the periodic lists of real kernels).
+// * the packed per-word shadow state carried across warps and tiles by the decoupled look-back
+//   (last-writer position, scope of the last atomic, DevShared, BlkShared, segment-head bit) and
+//   its segmented "last-of / OR" combine -- the state the paper keeps per 4-byte word (Fig. 4,
+//   P:763-829; updates P:1000-1058) as a function of the word's access prefix;
+// * interval queries on the a2 timestamp lists: "is there a sync of entity e in (a, b)?" -- the
+//   exact replacement of Table 2's counter comparisons (reading A16) -- answered from a per-list
+//   descriptor {lo, hi, first, last} and interpolation-guided 32-byte probes, and for grid syncs
+//   an L2-resident bucket table;
+// * report canonicalisation kernels (a7) and a gather micro-benchmark probe.
 #pragma once
 #include "common.cuh"
 #include "sync.cuh"
@@ -63,9 +51,12 @@ __global__ void k_list_desc(const u32* __restrict__ off, const u32* __restrict__
 // Optional event counters (igd_debug_check_stats): a debug aid, off unless enabled.
 __device__ int g_chk_stats_on;
 __device__ unsigned long long g_chk_stats[16];
-#define CSTAT(k)                                                \
-    do {                                                        \
-        if (g_chk_stats_on) atomicAdd(&g_chk_stats[k], 1ull);   \
+#ifndef IGD_CHECK_STATS
+#define IGD_CHECK_STATS 0  // build a variant with -DIGD_CHECK_STATS=1 for profiles/check_stats.py
+#endif
+#define CSTAT(k)                                                            \
+    do {                                                                    \
+        if (IGD_CHECK_STATS && g_chk_stats_on) atomicAdd(&g_chk_stats[k], 1ull); \
     } while (0)
 
 // Is there an element x of entity e's list with a < x < b ?
@@ -131,6 +122,7 @@ struct Params {
     const u32* gtab;    // grid-sync bucket table: first grid-list index at or after bucket start
     u32 gshift;         // bucket = t >> gshift
     u32 glo, ghi;       // the grid list inside sts
+    u32 has_kb;         // the trace has kernel boundaries (reading A31)
     const u32* sts;     // sync timestamps (sorted by entity, then time)
     syncx::LockView lv;
     u64* status;     // [n_tiles] zeroed
@@ -171,10 +163,6 @@ __device__ __forceinline__ bool q_grid(const PP& P, u32 a, u32 b) {
     return false;
 }
 
-#ifndef IGD_CHECK_WARPQ
-#define IGD_CHECK_WARPQ 1
-#endif
-
 // queue entry flags
 #define QF_SAME_W 1u
 #define QF_SAME_B 2u
@@ -203,307 +191,6 @@ __device__ __forceinline__ Acc acc_at(const void* val, u32 k) {
         a.mask = 0;
     }
     return a;
-}
-
-template <bool MV>
-#ifndef IGD_CHECK_MINB
-#define IGD_CHECK_MINB 6
-#endif
-__global__ void __launch_bounds__(THREADS, IGD_CHECK_MINB) k_check(Params P) {
-    __shared__ u32 s_tile;
-    __shared__ u64 s_wagg[WARPS];
-    __shared__ u64 s_prefix;
-    __shared__ u32 s_ready;
-    __shared__ u32 s_qn;
-    // queue of undecided accesses (SoA)
-    // per-warp queues of undecided accesses (SoA; q_pos: sorted position): each warp answers
-    // its own queue right after its phase 1, with no CTA-wide barrier in between
-#if IGD_CHECK_WARPQ
-    constexpr int QCAP = 32 * ITEMS;
-    __shared__ u32 s_wqn[WARPS];
-#else
-    constexpr int QCAP = TILE;
-#endif
-    __shared__ u32 q_i[TILE], q_md[TILE], q_c[TILE], q_p[TILE], q_pos[TILE];
-
-    const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
-    if (t == 0) {
-        // tiles in launch order (the block scheduler dispatches CTAs in blockIdx order, as
-        // decoupled look-back scans rely on); no atomic round trip before the loads
-        s_tile = blockIdx.x;
-        s_qn = 0;
-#if IGD_CHECK_WARPQ
-        for (int w = 0; w < WARPS; w++) s_wqn[w] = 0;
-#endif
-        s_ready = 0;
-    }
-    __syncthreads();
-    const u32 tile = s_tile;
-    const u32 first = tile * TILE + t * ITEMS;  // n <= 2^32 - 2^13
-    const Geo g = P.g;
-
-    // K: word key, V: trace index, Z: the event's tk word (tid | kind | scope), carried by the sort
-    u32 K[ITEMS], V[ITEMS], Z[ITEMS], M[ITEMS];
-    if (!MV && first + ITEMS <= P.n) {
-#pragma unroll
-        for (int q = 0; q < ITEMS / 4; q++) {
-            const uint4 k4 = __ldcs(reinterpret_cast<const uint4*>(P.key + first) + q);
-            K[4 * q] = k4.x; K[4 * q + 1] = k4.y; K[4 * q + 2] = k4.z; K[4 * q + 3] = k4.w;
-        }
-#pragma unroll
-        for (int q = 0; q < ITEMS / 2; q++) {
-            const uint4 v = __ldcs(reinterpret_cast<const uint4*>(P.val) + first / 2 + q);
-            V[2 * q] = v.x; Z[2 * q] = v.y; V[2 * q + 1] = v.z; Z[2 * q + 1] = v.w;
-        }
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) M[j] = 0;
-    } else {
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            const bool in = first + j < P.n;
-            const Acc a = in ? acc_at<MV>(P.val, first + j) : Acc{0, 0, 0};
-            K[j] = in ? P.key[first + j] : 0;
-            V[j] = a.idx;
-            Z[j] = a.tk;
-            M[j] = a.mask;
-        }
-    }
-
-    // previous element (first - 1): from the neighbour lane; lane 0 reads it
-    u32 pK = __shfl_up_sync(IGD_FULL, K[ITEMS - 1], 1);
-    u32 pV = __shfl_up_sync(IGD_FULL, V[ITEMS - 1], 1);
-    u32 pZ = __shfl_up_sync(IGD_FULL, Z[ITEMS - 1], 1);
-    if (lane == 0 && first > 0 && first - 1 < P.n) {
-        pK = __ldg(P.key + first - 1);
-        const Acc a = acc_at<MV>(P.val, first - 1);
-        pV = a.idx;
-        pZ = a.tk;
-    }
-
-    // per-access scan contributions
-    u64 contrib[ITEMS];
-    {
-        u32 prevTid = pZ & 0xFFFFFFu, prevKey = pK;
-        bool prevValid = first > 0;
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            const bool inr = first + j < P.n;
-            const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
-            const bool head = !prevValid || prevKey != K[j];
-            u32 dev = 0, blk = 0;
-            if (!head) {
-                const u32 bp = g.block(prevTid), bc = g.block(c);
-                if (bp != bc) dev = 1;
-                else if (g.warp(prevTid) != g.warp(c)) blk = 1;
-            }
-            const u32 lw = kind != IGD_LD ? first + j : IGD_NONE32;
-            const u32 as = (kind >= IGD_ATOM && kind <= IGD_EXCH) ? norm_scope((Z[j] >> 28) & 3u) : 0u;
-            contrib[j] = inr ? st_make(lw, as, dev, blk, head ? 1u : 0u) : ST_IDENTITY;
-            prevTid = c;
-            prevKey = K[j];
-            prevValid = true;
-        }
-    }
-    u64 agg = contrib[0];
-#pragma unroll
-    for (int j = 1; j < ITEMS; j++) agg = combine(agg, contrib[j]);
-    u64 inc = agg;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const u64 x = __shfl_up_sync(IGD_FULL, inc, o);
-        if (lane >= (u32)o) inc = combine(x, inc);
-    }
-    if (lane == 31) s_wagg[warp] = inc;
-    u64 wexcl = __shfl_up_sync(IGD_FULL, inc, 1);
-    if (lane == 0) wexcl = ST_IDENTITY;
-    __syncthreads();
-    // Tile-relative state.  Only accesses of the segment that continues from the previous tile
-    // (no head before them in this tile) need the look-back prefix; warp 0 lane 0 computes it
-    // while every other access proceeds.
-    if (t == 0) {
-        u64 tagg = s_wagg[0];
-#pragma unroll
-        for (int w = 1; w < WARPS; w++) tagg = combine(tagg, s_wagg[w]);
-        u64 prefix = ST_IDENTITY;
-        st_relaxed(&P.status[tile], ((tile == 0 || st_head(tagg)) ? ST_INC : ST_AGG) | tagg);
-        if (tile > 0) {
-            // combine predecessors back to an inclusive status or a head-containing aggregate
-            long tt = (long)tile - 1;
-            u64 acc = ST_IDENTITY;
-            bool have = false;
-            while (tt >= 0) {
-                u64 s;
-                do {
-                    s = ld_relaxed(&P.status[tt]);
-                } while ((s >> 62) == 0);
-                const u64 v = s & ST_VAL_MASK;
-                acc = have ? combine(v, acc) : v;
-                have = true;
-                if ((s >> 62) == 2 || st_head(v)) break;
-                tt--;
-            }
-            prefix = acc;
-            if (!st_head(tagg)) st_relaxed(&P.status[tile], ST_INC | combine(prefix, tagg));
-        }
-        s_prefix = prefix;
-        __threadfence_block();
-        *(volatile u32*)&s_ready = 1u;
-    }
-    u64 run = ST_IDENTITY;
-    for (u32 w = 0; w < warp; w++) run = combine(run, s_wagg[w]);
-    run = combine(run, wexcl);  // tile-relative shadow state before this thread's first access
-
-    if (P.debug_stop == 1) {
-        if (run == 0x123456789ull) P.rep_ctr[1] = run;  // keep the scans alive
-        return;
-    }
-    // ---- phase 1: history-free checks; queue the rest ----
-    u32 laIdx = pV, laTid = pZ & 0xFFFFFFu, laKind = (pZ >> 24) & 0xFu;
-#pragma unroll
-    for (int j = 0; j < ITEMS; j++) {
-        u64 before = run;
-        run = combine(run, contrib[j]);
-        if (!st_head(before) && first + j < P.n && !st_head(contrib[j])) {
-            // continues the previous tile's segment: wait for the look-back prefix
-            CSTAT(12);
-            while (*(volatile u32*)&s_ready == 0u) __nanosleep(64);
-            before = combine(*(volatile u64*)&s_prefix, before);
-        }
-        const u32 i = V[j];
-        const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
-        bool queue = false;
-        u32 mdIdx = laIdx, p = laTid, mdKind = laKind, flags = 0;
-        if (first + j < P.n && !st_head(contrib[j])) {
-            const u32 lastW = st_lastW(before), as = st_as(before);
-            CSTAT(0);
-            do {
-                if (kind == IGD_LD && lastW == IGD_NONE32) {  // P2: never written
-                    CSTAT(1);
-                    break;
-                }
-                if (kind == IGD_LD && lastW != first + j - 1) {  // md = last writer, further back
-                    CSTAT(13);
-                    const Acc mv = acc_at<MV>(P.val, lastW);
-                    mdIdx = mv.idx;
-                    p = mv.tk & 0xFFFFFFu;
-                    mdKind = (mv.tk >> 24) & 0xFu;
-                }
-                if (p == c) {  // P3: program order
-                    CSTAT(2);
-                    break;
-                }
-                const bool isA = kind >= IGD_ATOM && kind <= IGD_EXCH;
-                const u32 bc = g.block(c);
-                const bool same_b = g.block(p) == bc;
-                if (as && isA && (same_b || as == IGD_SCOPE_DEVICE)) {  // P6
-                    CSTAT(3);
-                    break;
-                }
-                const bool same_w = same_b && g.warp(p) == g.warp(c);
-                // P4, lockstep clause: md's lane is in this instruction's active mask.  The sort
-                // carries two mask summaries in tk bits 31 (full warp) and 30 (own lane only); the
-                // mask itself is gathered only for other partial masks
-                if (same_w && !(Z[j] >> 30)) CSTAT(5);
-                if (same_w && ((Z[j] >> 31) ||
-                               (!((Z[j] >> 30) & 1u) &&
-                                (((MV ? M[j] : ld_event(P.ev, i).w) >> g.lane(p)) & 1u)))) {
-                    CSTAT(4);
-                    break;
-                }
-                flags = (same_w ? QF_SAME_W : 0u) | (same_b ? QF_SAME_B : 0u) |
-                        ((st_dev(before) | st_dev(contrib[j])) ? QF_DEV : 0u) |
-                        ((st_blk(before) | st_blk(contrib[j])) ? QF_BLK : 0u);
-                if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
-                    u32 lwTid = p;
-                    if (kind != IGD_LD && lastW != first + j - 1)
-                        lwTid = acc_at<MV>(P.val, lastW).tk & 0xFFFFFFu;
-                    if (g.block(lwTid) != bc) flags |= QF_R1;
-                }
-                queue = true;
-                CSTAT(6);
-            } while (0);
-        }
-        const u32 qmask = __ballot_sync(IGD_FULL, queue);
-        if (qmask) {
-            u32 qbase = 0;
-#if IGD_CHECK_WARPQ
-            if (lane == 0) {
-                qbase = warp * QCAP + s_wqn[warp];
-                s_wqn[warp] += __popc(qmask);
-            }
-#else
-            if (lane == 0) qbase = atomicAdd(&s_qn, __popc(qmask));
-#endif
-            qbase = __shfl_sync(IGD_FULL, qbase, 0);
-            if (queue) {
-                const u32 q = qbase + __popc(qmask & lanemask_lt());
-                q_i[q] = i;
-                q_md[q] = mdIdx;
-                q_c[q] = c | (flags << 24);
-                q_p[q] = p | (kind << 24) | (mdKind << 28);
-                q_pos[q] = first + j;
-            }
-        }
-        laIdx = i;
-        laTid = c;
-        laKind = kind;
-    }
-#if IGD_CHECK_WARPQ
-    __syncwarp();
-    if (P.debug_stop == 2) return;
-    // ---- phase 2: the warp's queued accesses, densely over its lanes ----
-    const u32 qn = warp * QCAP + *(volatile u32*)&s_wqn[warp];
-    const KeySpace ks = P.ks;
-    for (u32 q = warp * QCAP + lane; q < qn; q += 32) {
-#else
-    __syncthreads();
-    if (P.debug_stop == 2) return;
-    // ---- phase 2: the queued accesses, densely over the CTA ----
-    const u32 qn = s_qn;
-    const KeySpace ks = P.ks;
-    for (u32 q = t; q < qn; q += THREADS) {
-#endif
-        const u32 i = q_i[q], mdIdx = q_md[q];
-        const u32 c = q_c[q] & 0xFFFFFFu, flags = q_c[q] >> 24;
-        const u32 p = q_p[q] & 0xFFFFFFu;
-        const bool same_w = flags & QF_SAME_W, same_b = flags & QF_SAME_B;
-        if (same_w && q_between(P.desc, P.sts, ks.wb + g.warp(c), mdIdx, i)) continue;  // P4: syncwarp
-        const bool grid = q_grid(P, mdIdx, i);
-        if (same_b && (grid || q_between(P.desc, P.sts, ks.bb + g.block(c), mdIdx, i))) continue;  // P5
-        u32 type = (flags & QF_R1) ? IGD_R1 : 0u;
-        if (!type) {
-            if (same_b) {
-                // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread must
-                // not have fenced since md (A1, A30)
-                if (!(flags & QF_DEV) && !grid && !q_between(P.desc, P.sts, ks.any + p, mdIdx, i))
-                    type = (same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3;
-            } else if (!grid && !q_between(P.desc, P.sts, ks.dev + p, mdIdx, i)) {
-                type = IGD_R4;  // R4: other block, no device fence by md's thread
-            }
-        }
-        if (!type && P.lv.any) {  // R5: lock sets of the last accessor and of this access
-            const u32 L = syncx::held_before(P.lv, g, c, i);
-            const Acc la = acc_at<MV>(P.val, q_pos[q] - 1);  // the last accessor (rare path)
-            const u32 locks = syncx::held_before(P.lv, g, la.tk & 0xFFFFFFu, la.idx);
-            if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
-        }
-        if (type) {
-            CSTAT(11);
-            const unsigned long long slot = atomicAdd(P.rep_ctr, 1ull);
-            if (slot < P.rep_cap) {
-                igd_report r;
-                // full word from the 32-bit key: the accessed words span < 2^32 from wbase
-                r.addr = (P.wbase + (u32)(__ldg(P.key + q_pos[q]) - (u32)P.wbase)) << 2;
-                r.cur = P.first_event + i;
-                r.prev = P.first_event + mdIdx;
-                r.type = (uint8_t)type;
-                r.cur_kind = (uint8_t)((q_p[q] >> 24) & 0xFu);
-                r.prev_kind = (uint8_t)(q_p[q] >> 28);
-                for (int z = 0; z < 5; z++) r.pad[z] = 0;
-                P.rep[slot] = r;
-            }
-        }
-    }
 }
 
 // Micro-benchmark probe: stream the sorted keys / indices and gather each access's event,

@@ -40,6 +40,22 @@ constexpr int C4_TILE = THREADS * C4_ITEMS;  // accesses per CTA
 
 __device__ __forceinline__ int hib(u32 m) { return 31 - (int)__clz(m); }  // m != 0
 
+// q_between without the call (no caller-saved spills in the scan loop): descriptor fast paths,
+// then a binary search -- for short lists such as the kernel boundaries
+__device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, const u32* __restrict__ ts, u32 e, u32 a,
+                                              u32 b) {
+    const uint4 d = __ldg(desc + e);
+    if (d.x == d.y || d.w <= a) return false;
+    if (d.z > a) return d.z < b;
+    u32 lo = d.x + 1, hi = d.y - 1;  // successor of a in [lo, hi]: ts[hi] = d.w > a
+    while (lo < hi) {
+        const u32 mid = (lo + hi) >> 1;
+        if (__ldg(ts + mid) <= a) lo = mid + 1;
+        else hi = mid;
+    }
+    return __ldg(ts + lo) < b;
+}
+
 #define QF_MASK 32u  // P4 lockstep clause pending: gather the event's active mask in phase 2
 
 // Staged interval query "is there x in list e with a < x < b" (check.cuh q_between, split so a
@@ -104,7 +120,9 @@ __device__ __noinline__ bool q_grid_from(const PP& P, u32 a, u32 b, u32 x) {
     return false;
 }
 
-template <bool MV>
+// KB: the trace has kernel boundaries (a separate instantiation: the boundary test costs
+// registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
+template <bool MV, bool KB>
 __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
     __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
     __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
@@ -141,10 +159,12 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
         }
     }
     // the access before the warp's first one
-    u32 cK = 0, cZ = 0;
+    u32 cK = 0, cZ = 0, cV = 0;
     if (lane == 0 && wbase > 0 && wbase <= n) {
         cK = __ldg(P.key + wbase - 1);
-        cZ = acc_at<MV>(P.val, wbase - 1).tk;
+        const Acc a = acc_at<MV>(P.val, wbase - 1);
+        cZ = a.tk;
+        cV = a.idx;
     }
 #pragma unroll
     for (int j = 0; j < C4_ITEMS; j++) {
@@ -165,7 +185,15 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
         cZ = rZ;
         const bool in = x < n;
         const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
-        const bool head = !in || !pvalid || pK != K[j];
+        bool head = !in || !pvalid || pK != K[j];
+        if (KB) {
+            // a kernel boundary between the previous access of this word and this one ends the
+            // word's history (reading A31): a new segment, as if the word were fresh
+            const u32 rV = __shfl_sync(IGD_FULL, V[j], (lane + 31u) & 31u);
+            const u32 pV = lane ? rV : cV;
+            cV = rV;
+            if (!head) head = q_between_inl(P.desc, P.sts, P.ks.kb, pV, V[j]);
+        }
         bool dev = false, blk = false, same_t = false;
         if (!head) {
             const u32 pt = pZ & 0xFFFFFFu;
@@ -298,7 +326,11 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
             }
             const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
             do {
-                if (kind == IGD_LD && lastW == IGD_NONE32) break;  // P2: never written
+                CSTAT(0);
+                if (kind == IGD_LD && lastW == IGD_NONE32) {  // P2: never written
+                    CSTAT(1);
+                    break;
+                }
                 // md: the last writer for a load, the last accessor otherwise.  When
                 // md is the previous access of the segment (the common case) the thread / block /
                 // warp relations to it are the pair bits balloted above: no lookup, no division.
@@ -317,8 +349,14 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
                     same_b = g.block(p) == g.block(c);
                     same_w = same_b && g.warp(p) == g.warp(c);
                 }
-                if (same_t) break;                                             // P3: program order
-                if (as && isA && (same_b || as == IGD_SCOPE_DEVICE)) break;  // P6
+                if (same_t) {  // P3: program order
+                    CSTAT(2);
+                    break;
+                }
+                if (as && isA && (same_b || as == IGD_SCOPE_DEVICE)) {  // P6
+                    CSTAT(3);
+                    break;
+                }
                 // P4 lockstep clause: md's lane in this instruction's active mask (tk bit 31: full
                 // warp; bit 30: own lane only; otherwise the mask itself, from the payload in MV
                 // mode, else gathered from the trace)
@@ -343,6 +381,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
                     if (other) fl |= QF_R1;
                 }
                 queue = true;
+                CSTAT(6);
             } while (0);
         }
         const u32 qmask = __ballot_sync(IGD_FULL, queue);
@@ -461,10 +500,11 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
                 laz = a.tk;
             }
             u32 L, locks;
-            syncx::held_before2(P.lv, g, c, i, laz & 0xFFFFFFu, laIdx, L, locks);
+            syncx::held_before2(P.lv, c, i, laz & 0xFFFFFFu, laIdx, L, locks);
             if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
         }
         if (type) {
+            CSTAT(11);
             const unsigned long long slot = atomicAdd(P.rep_ctr, 1ull);
             if (slot < P.rep_cap) {
                 igd_report r;

@@ -78,8 +78,9 @@ struct Geo {
 //   [2T+W,2T+W+B) syncthreads of block b          "BBar"
 //   2T+W+B  grid syncs                            "Grid"
 //   [2T+W+B+1, 2T+2W+B+1) CAS/EXCH of warp w      "Lock"
+//   2T+2W+B+1 kernel boundaries                   "Kb" (multi-kernel traces, reading A31)
 struct KeySpace {
-    u32 any, dev, wb, bb, grid, lock, E;
+    u32 any, dev, wb, bb, grid, lock, kb, E;
     __host__ void init(const Geo& g) {
         any = 0;
         dev = g.T;
@@ -87,7 +88,8 @@ struct KeySpace {
         bb = 2 * g.T + g.W;
         grid = bb + g.B;
         lock = grid + 1;
-        E = lock + g.W;
+        kb = lock + g.W;
+        E = kb + 1;
     }
 };
 

@@ -75,7 +75,7 @@ __device__ __forceinline__ FDec fdecode(const uint4& e, const Geo& g, const KeyS
     } else if (kind == IGD_SYNCTHREADS || kind == IGD_CG_BLOCK_SYNC) {
         d.s0 = ks.bb + b;
     } else {
-        d.s0 = ks.grid;
+        d.s0 = kind == IGD_KERNEL_BOUNDARY ? ks.kb : ks.grid;
     }
     return d;
 }

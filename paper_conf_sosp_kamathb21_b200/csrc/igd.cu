@@ -56,14 +56,13 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
-    Buf off, ldesc, gtab, sw, wcnt, tcnt, wpts, tpts, wdesc;
+    Buf off, ldesc, gtab, tcnt, tpts;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
     int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any, 2 = atomic-or (IGD_SORT_MODE)
     int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
     int count_tma = 0;  // IGD_COUNT_TMA=1: ingest pass 0 through a TMA ring (ingest::k_count; measured slower: 8.6 vs 7.2 ms at C5 1e9, the pass is issue-bound)
-    int check_ver = 4;  // a6 kernel: 4 = ballot formulation (check4.cuh), 3 = shuffle scan (IGD_CHECK_VER)
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
     bool shard = false;
@@ -456,8 +455,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         CK(cudaGetLastError());
     }
     // grid-sync bucket table (<= 2^22 buckets, L2-resident)
-    u32 glims[2] = {0, 0};
+    u32 glims[2] = {0, 0}, klims[2] = {0, 0};  // grid-sync list, kernel-boundary list
     CK(cudaMemcpyAsync(glims, P_<u32>(ctx->off) + ks.grid, 2 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(klims, P_<u32>(ctx->off) + ks.kb, 2 * sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     const u32 gshift = std::max<u32>(8, bits_needed(n) > 22 ? bits_needed(n) - 22 : 0);
     const u32 gnb = (u32)((n >> gshift) + 2);
@@ -473,10 +473,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     syncx::LockView lv;
     memset(&lv, 0, sizeof(lv));
     if (n_lock > 0) {
-        RET(ensure(ctx, ctx->sw, (u64)g.W * sizeof(u32)));
-        RET(ensure(ctx, ctx->wcnt, ((u64)g.W + 1) * sizeof(u32)));
         RET(ensure(ctx, ctx->tcnt, ((u64)g.T + 1) * sizeof(u32)));
-        CK(cudaMemsetAsync(ctx->wcnt.p, 0, ((u64)g.W + 1) * sizeof(u32), ctx->stream));
         CK(cudaMemsetAsync(ctx->tcnt.p, 0, ((u64)g.T + 1) * sizeof(u32), ctx->stream));
         syncx::LockParams lp;
         memset(&lp, 0, sizeof(lp));
@@ -487,8 +484,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lp.ks = ks;
         lp.off = P_<u32>(ctx->off);
         lp.sts = P_<u32>(ctx->syn_v[scur]);
-        lp.switch_ts = P_<u32>(ctx->sw);
-        lp.wcnt = P_<u32>(ctx->wcnt);
         lp.tcnt = P_<u32>(ctx->tcnt);
         const unsigned lblocks = (unsigned)(((u64)g.W * 32 + 255) / 256);
         {
@@ -496,38 +491,19 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             syncx::k_lock_infer<false><<<lblocks, 256, 0, ctx->stream>>>(lp);
         }
         CK(cudaGetLastError());
-        RET(scan_excl(ctx, P_<u32>(ctx->wcnt), (u64)g.W + 1));
         RET(scan_excl(ctx, P_<u32>(ctx->tcnt), (u64)g.T + 1));
-        u32 tot[2];
-        CK(cudaMemcpyAsync(&tot[0], P_<u32>(ctx->wcnt) + g.W, sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
-        CK(cudaMemcpyAsync(&tot[1], P_<u32>(ctx->tcnt) + g.T, sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+        u32 tot = 0;
+        CK(cudaMemcpyAsync(&tot, P_<u32>(ctx->tcnt) + g.T, sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
-        RET(ensure(ctx, ctx->wpts, ((u64)tot[0] + 1) * sizeof(u64)));
-        RET(ensure(ctx, ctx->tpts, ((u64)tot[1] + 1) * sizeof(u64)));
-        lp.woff = P_<u32>(ctx->wcnt);
+        RET(ensure(ctx, ctx->tpts, ((u64)tot + 1) * sizeof(u64)));
         lp.toff = P_<u32>(ctx->tcnt);
-        lp.wpts = P_<u64>(ctx->wpts);
         lp.tpts = P_<u64>(ctx->tpts);
         {
             KTimer kt(ctx, KC_LOCK, 0);
             syncx::k_lock_infer<true><<<lblocks, 256, 0, ctx->stream>>>(lp);
         }
         CK(cudaGetLastError());
-        RET(ensure(ctx, ctx->wdesc, ((u64)g.W + 1) * sizeof(uint4)));
-        {
-            KTimer kt(ctx, KC_LOCK, 0);
-            const unsigned db = (unsigned)std::min<u64>(((u64)g.W + 255) / 256, (u64)sms * 8);
-            syncx::k_lock_desc<<<db, 256, 0, ctx->stream>>>(P_<u32>(ctx->off), ks.lock, P_<u32>(ctx->sw),
-                                                            P_<u32>(ctx->wcnt), g.W, P_<uint4>(ctx->wdesc));
-            CK(cudaGetLastError());
-        }
-        lv.wdesc = P_<uint4>(ctx->wdesc);
-        lv.off = P_<u32>(ctx->off);
-        lv.lock_key0 = ks.lock;
-        lv.switch_ts = P_<u32>(ctx->sw);
-        lv.woff = P_<u32>(ctx->wcnt);
         lv.toff = P_<u32>(ctx->tcnt);
-        lv.wpts = P_<u64>(ctx->wpts);
         lv.tpts = P_<u64>(ctx->tpts);
         lv.any = 1;
     }
@@ -543,8 +519,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     if (ctx->rep_cap == 0) ctx->rep_cap = 1 << 20;
     u64 n_rep = 0;
     if (n_acc > 0) {
-        const bool V4 = ctx->check_ver == 4;
-        const u64 ctile = V4 ? check::C4_TILE : check::TILE;
+        const u64 ctile = check::C4_TILE;
         const u64 tiles = (n_acc + ctile - 1) / ctile;
         for (int attempt = 0;; attempt++) {
             RET(ensure(ctx, ctx->rep_raw, ctx->rep_cap * sizeof(igd_report)));
@@ -567,6 +542,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.gshift = gshift;
             cp.glo = glims[0];
             cp.ghi = glims[1];
+            cp.has_kb = klims[1] > klims[0] ? 1u : 0u;
             cp.sts = P_<u32>(ctx->syn_v[scur]);
             cp.lv = lv;
             cp.status = P_<u64>(ctx->status);
@@ -579,13 +555,11 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
-                if (V4) {
-                    if (SH) check::k_check4<true><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
-                    else check::k_check4<false><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
-                } else {
-                    if (SH) check::k_check<true><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
-                    else check::k_check<false><<<(unsigned)tiles, check::THREADS, 0, ctx->stream>>>(cp);
-                }
+                const unsigned tb = (unsigned)tiles;
+                if (SH && cp.has_kb) check::k_check4<true, true><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
+                else if (SH) check::k_check4<true, false><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
+                else if (cp.has_kb) check::k_check4<false, true><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
+                else check::k_check4<false, false><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
             }
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
@@ -744,7 +718,6 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = (atoi(m) >= 0 && atoi(m) <= 2) ? atoi(m) : 1;
     if (const char* m = getenv("IGD_CHECK_STOP")) ctx->check_stop = atoi(m);
     if (const char* m = getenv("IGD_COUNT_TMA")) ctx->count_tma = atoi(m) != 0;
-    if (const char* m = getenv("IGD_CHECK_VER")) ctx->check_ver = atoi(m) == 3 ? 3 : 4;
     if (const char* m = getenv("IGD_FUSED")) ctx->fused = atoi(m) != 0;
     cudaFuncSetAttribute(ingest::k_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ingest::count_smem());
     cudaFuncSetAttribute(fused::k_ingest_sort0, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -942,9 +915,8 @@ void igd_ctx_destroy(igd_ctx* ctx) {
     Buf* all[] = {&ctx->owned_events, &ctx->acc_k[0], &ctx->acc_k[1], &ctx->acc_v[0], &ctx->acc_v[1],
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
                   &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
-                  &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->sw,       &ctx->wcnt,
-                  &ctx->tcnt,
-                  &ctx->wpts,         &ctx->tpts,     &ctx->wdesc,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
+                  &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->tcnt,
+                  &ctx->tpts,         &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf};
     for (Buf* b : all) buf_free(ctx, *b);

@@ -67,7 +67,7 @@ __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpa
         lanebit = 1u << (off & 31u);
     }
     const bool inmask = (e.w & lanebit) != 0;
-    bool ok = (e.z >> 30) == 0 && tid_ok && kind <= IGD_CG_GRID_SYNC;
+    bool ok = (e.z >> 30) == 0 && tid_ok && kind <= IGD_KERNEL_BOUNDARY;
     if (ok) {
         switch (kind) {
             case IGD_LD:
@@ -88,7 +88,7 @@ __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpa
             case IGD_CG_BLOCK_SYNC:
                 ok = addr0 && scope == IGD_SCOPE_NONE;
                 break;
-            default:  // GRID_SYNC, CG_GRID_SYNC
+            default:  // GRID_SYNC, CG_GRID_SYNC, KERNEL_BOUNDARY
                 ok = addr0 && scope == IGD_SCOPE_NONE && tid == 0;
                 break;
         }
@@ -122,7 +122,7 @@ __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpa
         d.s0 = ks.bb + b;
         d.flags = 1u << 1;
     } else {
-        d.s0 = ks.grid;
+        d.s0 = kind == IGD_KERNEL_BOUNDARY ? ks.kb : ks.grid;
         d.flags = 1u << 1;
     }
     return d;

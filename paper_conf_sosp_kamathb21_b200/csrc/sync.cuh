@@ -8,10 +8,12 @@
 //     address hash (Valid, not Active), a fence of matching-or-wider scope activates entries,
 //     atomicExch invalidates the entry with the same hash and scope, a CAS executed by more
 //     than one lane switches the warp to per-thread tables for good, a grid sync
-//     is a device fence by every thread (reading A15).  One CUDA warp replays one traced warp,
-//     lane l owning thread l's per-thread table; it emits change points (ts, bloom) of the
-//     held-lock Bloom summary so the check can ask "locks of thread c just before
-//     event i" with one binary search.
+//     is a device fence by every thread (reading A15), a kernel boundary resets every table and
+//     the isThread bit (reading A31).  One CUDA warp replays one traced warp, lane l
+//     owning thread l's per-thread table; each lane emits change points (ts, bloom) of its
+//     thread's effective held-lock Bloom summary (the warp table's while isThread is
+//     unset, its own table after) so the check asks "locks of thread c just before event i" with
+//     one binary search on one list.
 #pragma once
 #include "common.cuh"
 
@@ -81,13 +83,9 @@ struct LockParams {
     KeySpace ks;
     const u32* off;       // CSR offsets of sync records
     const u32* sts;       // sorted sync timestamps
-    u32* switch_ts;       // [W] isThread switch time (NONE = never)
-    u32* wcnt;            // [W+1] warp change-point counts (pass 0) -> offsets after scan
-    u32* tcnt;            // [T+1] thread change-point counts
-    const u32* woff;      // [W+1] (pass 1)
+    u32* tcnt;            // [T+1] thread change-point counts (pass 0) -> offsets after the scan
     const u32* toff;      // [T+1] (pass 1)
-    u64* wpts;            // warp change points  (ts << 16 | bloom)
-    u64* tpts;            // thread change points
+    u64* tpts;            // thread change points (ts << 16 | bloom)
     const u32* gidx;      // sharded mode: global timestamps of the events in `ev` (sorted), else NULL
     u32 gn;
 };
@@ -112,50 +110,48 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     const u32 w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (w >= P.g.W) return;
     const KeySpace ks = P.ks;
-    u32 lk_lo = P.off[ks.lock + w];
-    const u32 lk_hi = P.off[ks.lock + w + 1];
-    if (lk_lo == lk_hi) {
-        if (!WRITE && lane == 0) {
-            P.wcnt[w] = 0;
-            P.switch_ts[w] = IGD_NONE32;
-        }
-        if (!WRITE) {
-            // thread counts of this warp's lanes
-            u32 b = w / P.g.Wb, wi = w - b * P.g.Wb;
-            u32 off = wi * 32 + lane;
-            if (off < P.g.D) P.tcnt[b * P.g.D + off] = 0;
-        }
-        return;
-    }
     const u32 b = w / P.g.Wb, wi = w - b * P.g.Wb;
     const u32 my_off = wi * 32 + lane;
     const bool has_thread = my_off < P.g.D;
     const u32 my_t = b * P.g.D + my_off;
+    u32 lk_lo = P.off[ks.lock + w];
+    const u32 lk_hi = P.off[ks.lock + w + 1];
+    if (lk_lo == lk_hi) {  // never a CAS / EXCH: no lock state
+        if (!WRITE && has_thread) P.tcnt[my_t] = 0;
+        return;
+    }
     u32 f_lo = 0, f_hi = 0;
     if (has_thread) {
         f_lo = P.off[ks.any + my_t];
         f_hi = P.off[ks.any + my_t + 1];
     }
     u32 g_lo = P.off[ks.grid], g_hi = P.off[ks.grid + 1];
+    u32 k_lo = P.off[ks.kb], k_hi = P.off[ks.kb + 1];
 
     Table wt, tt;
     wt.clear();
     tt.clear();
     bool isThread = false;
-    u32 sw = IGD_NONE32;
-    u32 held_w = 0, held_t = 0;
-    u32 nw = 0, nt = 0;
-    u32 wout = WRITE ? P.woff[w] : 0;
+    u32 held = 0;  // this lane's effective held-lock Bloom
+    u32 nt = 0;
     u32 tout = (WRITE && has_thread) ? P.toff[my_t] : 0;
 
     u32 my_next = (f_lo < f_hi) ? __ldg(P.sts + f_lo) : IGD_NONE32;
     u32 lk_next = __ldg(P.sts + lk_lo);
     u32 g_next = (g_lo < g_hi) ? __ldg(P.sts + g_lo) : IGD_NONE32;
+    u32 k_next = (k_lo < k_hi) ? __ldg(P.sts + k_lo) : IGD_NONE32;
     while (true) {
         const u32 f_min = __reduce_min_sync(IGD_FULL, my_next);
-        const u32 ts = min(f_min, min(lk_next, g_next));
+        const u32 ts = min(min(f_min, k_next), min(lk_next, g_next));
         if (ts == IGD_NONE32) break;
-        if (ts == g_next) {
+        if (ts == k_next) {
+            // kernel boundary: the next kernel's locking protocol is inferred afresh (A31)
+            wt.clear();
+            tt.clear();
+            isThread = false;
+            k_lo++;
+            k_next = (k_lo < k_hi) ? __ldg(P.sts + k_lo) : IGD_NONE32;
+        } else if (ts == g_next) {
             // grid sync: every thread fences at device scope (A15)
             wt.activate(IGD_SCOPE_DEVICE);
             tt.activate(IGD_SCOPE_DEVICE);
@@ -167,10 +163,7 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
             const u32 h = lock_h18(ev_addr(e) >> 2);
             const u32 el = P.g.lane(ev_tid(e));
             if (kind == IGD_CAS) {
-                if (!isThread && __popc(e.w) > 1) {
-                    isThread = true;
-                    sw = ts;
-                }
+                if (!isThread && __popc(e.w) > 1) isThread = true;
                 if (isThread) {
                     if (lane == el) tt.insert(h, s);
                 } else {
@@ -201,80 +194,35 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
                 wt.activate(s);
             }
         }
-        // change points
-        if (!isThread) {
-            const u32 hw = wt.held();
-            if (hw != held_w) {
-                if (WRITE && lane == 0) P.wpts[wout + nw] = ((u64)ts << 16) | hw;
-                nw++;
-                held_w = hw;
-            }
-        } else {
-            const u32 ht = tt.held();
-            if (ht != held_t) {
-                if (WRITE && has_thread) P.tpts[tout + nt] = ((u64)ts << 16) | ht;
-                nt++;
-                held_t = ht;
-            }
+        // change point of this lane's thread: effective table = per-warp until isThread is set
+        const u32 h = isThread ? tt.held() : wt.held();
+        if (h != held && has_thread) {
+            if (WRITE) P.tpts[tout + nt] = ((u64)ts << 16) | h;
+            nt++;
+            held = h;
         }
     }
-    if (!WRITE) {
-        if (lane == 0) {
-            P.wcnt[w] = nw;
-            P.switch_ts[w] = sw;
-        }
-        if (has_thread) P.tcnt[my_t] = nt;
-    }
+    if (!WRITE && has_thread) P.tcnt[my_t] = nt;
 }
 
-// held-lock Bloom of thread c just before event i (the check's L(c, i))
+// held-lock Bloom of thread c just before event i (the check's L(c, i)): the last change point
+// of c with ts < i
 struct LockView {
-    const u32* off;
-    u32 lock_key0;
-    const u32* switch_ts;
-    const u32* woff;
-    const u32* toff;
-    const u64* wpts;
-    const u64* tpts;
-    const uint4* wdesc;  // per warp {woff[w], woff[w+1], switch_ts[w], has CAS/EXCH} (k_lock_desc)
-    u32 any;  // 0 when the trace has no CAS/EXCH at all
+    const u32* toff;  // [T+1] per-thread change-point offsets
+    const u64* tpts;  // change points (ts << 16 | bloom)
+    u32 any;          // 0 when the trace has no CAS/EXCH at all
 };
 
-// One 16-byte descriptor per warp for the check's lock-set queries: one load decides "this warp
-// never takes a lock" and carries the bounds of its change-point list and its switch time.
-__global__ void k_lock_desc(const u32* __restrict__ off, u32 lock_key0, const u32* __restrict__ switch_ts,
-                            const u32* __restrict__ woff, u32 W, uint4* __restrict__ wdesc) {
-    for (u32 w = blockIdx.x * blockDim.x + threadIdx.x; w < W; w += gridDim.x * blockDim.x)
-        wdesc[w] = make_uint4(woff[w], woff[w + 1], switch_ts[w],
-                              off[lock_key0 + w] != off[lock_key0 + w + 1] ? 1u : 0u);
-}
-
-// Lock sets of two (thread, time) pairs at once -- the check's L(c, i) and L(la) of R5 -- with
-// the two descriptor loads and the two binary searches interleaved (independent L2 chains).
-__device__ __forceinline__ void held_before2(const LockView& V, const Geo& g, u32 c0, u32 i0, u32 c1, u32 i1,
-                                             u32& L0, u32& L1) {
-    L0 = L1 = 0;
-    const uint4 d0 = __ldg(V.wdesc + g.warp(c0)), d1 = __ldg(V.wdesc + g.warp(c1));
-    if (!d0.w && !d1.w) return;
-    // list bounds: the per-thread list after the warp's switch time, else the per-warp list
-    const bool t0 = d0.w && d0.z != IGD_NONE32 && i0 > d0.z, t1 = d1.w && d1.z != IGD_NONE32 && i1 > d1.z;
-    u32 lo0 = d0.x, hi0 = d0.w ? d0.y : d0.x, lo1 = d1.x, hi1 = d1.w ? d1.y : d1.x;
-    if (t0) {
-        lo0 = __ldg(V.toff + c0);
-        hi0 = __ldg(V.toff + c0 + 1);
-    }
-    if (t1) {
-        lo1 = __ldg(V.toff + c1);
-        hi1 = __ldg(V.toff + c1 + 1);
-    }
-    const u64* p0 = t0 ? V.tpts : V.wpts;
-    const u64* p1 = t1 ? V.tpts : V.wpts;
+// Lock sets of two (thread, time) pairs at once -- R5's L(c, i) and the last accessor's -- with
+// the two binary searches interleaved (independent L2 chains).
+__device__ __forceinline__ void held_before2(const LockView& V, u32 c0, u32 i0, u32 c1, u32 i1, u32& L0, u32& L1) {
+    u32 lo0 = __ldg(V.toff + c0), hi0 = __ldg(V.toff + c0 + 1);
+    u32 lo1 = __ldg(V.toff + c1), hi1 = __ldg(V.toff + c1 + 1);
     const u32 b0 = lo0, b1 = lo1;
-    // last entry with ts < i: first entry with ts >= i, minus one
     while (lo0 < hi0 || lo1 < hi1) {
         const u32 m0 = (lo0 + hi0) >> 1, m1 = (lo1 + hi1) >> 1;
         const bool a0 = lo0 < hi0, a1 = lo1 < hi1;
-        const u64 v0 = a0 ? __ldg(p0 + m0) : 0ull, v1 = a1 ? __ldg(p1 + m1) : 0ull;
+        const u64 v0 = a0 ? __ldg(V.tpts + m0) : 0ull, v1 = a1 ? __ldg(V.tpts + m1) : 0ull;
         if (a0) {
             if ((u32)(v0 >> 16) < i0) lo0 = m0 + 1;
             else hi0 = m0;
@@ -284,30 +232,8 @@ __device__ __forceinline__ void held_before2(const LockView& V, const Geo& g, u3
             else hi1 = m1;
         }
     }
-    const u64 e0 = (d0.w && lo0 > b0) ? __ldg(p0 + lo0 - 1) : 0ull;
-    const u64 e1 = (d1.w && lo1 > b1) ? __ldg(p1 + lo1 - 1) : 0ull;
-    L0 = (u32)(e0 & 0xFFFFu);
-    L1 = (u32)(e1 & 0xFFFFu);
-}
-
-__device__ __forceinline__ u32 last_before(const u64* __restrict__ pts, u32 lo, u32 hi, u32 i) {
-    // last entry with ts < i
-    u32 L = lo, H = hi;
-    while (L < H) {
-        u32 mid = (L + H) >> 1;
-        if ((u32)(__ldg(pts + mid) >> 16) < i) L = mid + 1;
-        else H = mid;
-    }
-    return (L > lo) ? (u32)(__ldg(pts + L - 1) & 0xFFFFu) : 0u;
-}
-
-__device__ __forceinline__ u32 held_before(const LockView& V, const Geo& g, u32 c, u32 i) {
-    if (!V.any) return 0;
-    const u32 w = g.warp(c);
-    if (__ldg(V.off + V.lock_key0 + w) == __ldg(V.off + V.lock_key0 + w + 1)) return 0;
-    const u32 sw = __ldg(V.switch_ts + w);
-    if (sw != IGD_NONE32 && i > sw) return last_before(V.tpts, __ldg(V.toff + c), __ldg(V.toff + c + 1), i);
-    return last_before(V.wpts, __ldg(V.woff + w), __ldg(V.woff + w + 1), i);
+    L0 = lo0 > b0 ? (u32)(__ldg(V.tpts + lo0 - 1) & 0xFFFFu) : 0u;
+    L1 = lo1 > b1 ? (u32)(__ldg(V.tpts + lo1 - 1) & 0xFFFFu) : 0u;
 }
 
 // ---------------------------------------------------------------------------------------------

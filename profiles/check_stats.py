@@ -1,6 +1,8 @@
 """Event counters of the check kernel on a workload (what fraction of accesses reach which
 Table-2 stage, how many list queries and how they are answered).
-usage: python profiles/check_stats.py C4 [events]"""
+usage: python profiles/build_variants.py stats:IGD_CHECK_STATS=1
+       IGD_LIB=variants/libigd_stats.so python profiles/check_stats.py C4 [events]
+(counters not instrumented in the current kernel read 0)"""
 import ctypes
 import json
 import os
