@@ -64,3 +64,16 @@ def test_invalid_event_reported_globally():
     with pytest.raises(igd.IgdError) as ei:
         sharded(ev, nb, bd, 4)
     assert ei.value.code == igd.igd.IGD_ETRACE and ei.value.bad_index == 31_337
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_multi_kernel_sharded(P):
+    # kernel boundaries (reading A31) travel with the synchronization stream to every rank
+    w = [12, 10, 6, 10, 8, 12, 2, 2, 1, 1, 1, 1]
+    for seed in range(30):
+        parts = [tg.random_trace(seed * 7 + k, 150, n_blocks=2, block_dim=64, weights=w, lock_words=3,
+                                 p_lock_data=0.3)[0] for k in range(3)]
+        ev = tg.concat_kernels(parts)
+        assert np.array_equal(sharded(ev, 2, 64, P), oracle.run(ev, 2, 64)), f"seed {seed} P {P}"
+    big = tg.concat_kernels([_fast_random(90 + k, 80_000, 500, 4, 64, w, lock_words=16)[0] for k in range(3)])
+    assert np.array_equal(sharded(big, 4, 64, P), oracle.run(big, 4, 64))
