@@ -29,7 +29,7 @@ constexpr int WARPS = THREADS / 32;
 #define IGD_SORT_NOLOOKBACK 0
 #endif
 #ifndef IGD_SORT_EARLY
-#define IGD_SORT_EARLY 0
+#define IGD_SORT_EARLY 1  // publish tile digit counts before ranking (C5@1e9: 21.6 -> 21.2 ms over 3 passes)
 #endif
 #ifndef IGD_SORT_LB
 #define IGD_SORT_LB 4
