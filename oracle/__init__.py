@@ -12,6 +12,9 @@ Parity status per function:
   * igdo_run                -- pinned: worked examples W1-W9 (tests/golden), from-scratch
                                brute force, pairwise evaluator, sync-free closed form,
                                zero-report families, injection ledgers.
+  * coalesced mode (A32)    -- pinned: equals the plain replay of the trace with the coalesced
+                               members deleted (group detection restated in numpy in the
+                               test), worked example (one report per warp instruction).
   * Bloom/hash constants    -- parity unpinned by the paper (reading A8): pinned only by
                                agreement with the brute force, which restates them.
 """
@@ -60,13 +63,19 @@ def _load():
         lib.igdo_run.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                  ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
                                  ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
+        lib.igdo_run_ex.restype = ctypes.c_int
+        lib.igdo_run_ex.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                    ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p,
+                                    ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
         _lib = lib
     return _lib
 
 
-def run(events: np.ndarray, n_blocks: int, block_dim: int, shard=(0, 1), cap: int = None):
+def run(events: np.ndarray, n_blocks: int, block_dim: int, shard=(0, 1), cap: int = None,
+        coalesce: bool = False):
     """Replay ``events`` (EVENT_DTYPE, 16 B each) and return the report array (REPORT_DTYPE),
-    ascending by ``cur``.  ``shard=(k, K)`` checks only words owned by shard k (C.7 5(b))."""
+    ascending by ``cur``.  ``shard=(k, K)`` checks only words owned by shard k (C.7 5(b)).
+    ``coalesce``: warp-coalesced check mode (§6.5, reading A32)."""
     lib = _load()
     ev = np.ascontiguousarray(events)
     assert ev.dtype.itemsize == 16
@@ -77,8 +86,8 @@ def run(events: np.ndarray, n_blocks: int, block_dim: int, shard=(0, 1), cap: in
         out = np.zeros(cap, REPORT_DTYPE)
         nrep = ctypes.c_uint64(0)
         bad = ctypes.c_uint64(0)
-        rc = lib.igdo_run(ev.ctypes.data if n else None, n, n_blocks, block_dim, shard[0], shard[1],
-                          out.ctypes.data, cap, ctypes.byref(nrep), ctypes.byref(bad))
+        rc = lib.igdo_run_ex(ev.ctypes.data if n else None, n, n_blocks, block_dim, shard[0], shard[1],
+                             1 if coalesce else 0, out.ctypes.data, cap, ctypes.byref(nrep), ctypes.byref(bad))
         if rc != O_OK:
             raise OracleError(rc, bad.value if rc == O_ETRACE else None)
         if nrep.value <= cap:

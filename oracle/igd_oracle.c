@@ -173,6 +173,37 @@ static int o_valid(const o_event* e, const o_geom* g) {
 }
 
 /*
+ * Warp-coalesced check mode (reading A32, §6.5): "if the active threads within a
+ * warp are accessing the same location using load or atomic instructions ... only a single
+ * thread checks for races ... on behalf of all active threads".  A coalesced group is a run of
+ * popcount(mask) >= 2 consecutive events of one warp instruction -- same warp, kind (LD or ATOM;
+ * CAS / EXCH are lock operations, and stay per lane), scope, mask and word, lanes
+ * strictly ascending -- starting at the mask's lowest lane.  Every member but the first is
+ * neither checked nor recorded in the word's shadow entry (Step 3).
+ */
+static void o_mark_coalesced(const uint8_t* events, uint64_t n, const o_geom* g, uint8_t* skip) {
+    for (uint64_t i = 0; i < n; i++) {
+        o_event e;
+        o_read_event(events + 16 * i, &e);
+        if (e.kind != O_LD && e.kind != O_ATOM) continue;
+        uint32_t cnt = (uint32_t)__builtin_popcount(e.mask);
+        if (cnt < 2 || g_lane(g, e.tid) != (uint32_t)__builtin_ctz(e.mask) || i + cnt > n) continue;
+        int ok = 1;
+        uint32_t prev_lane = g_lane(g, e.tid);
+        for (uint32_t q = 1; q < cnt && ok; q++) {
+            o_event f;
+            o_read_event(events + 16 * (i + q), &f);
+            ok = f.kind == e.kind && f.scope == e.scope && f.mask == e.mask &&
+                 g_warp(g, f.tid) == g_warp(g, e.tid) && (f.addr >> 2) == (e.addr >> 2) &&
+                 g_lane(g, f.tid) > prev_lane;
+            prev_lane = g_lane(g, f.tid);
+        }
+        if (ok)
+            for (uint32_t q = 1; q < cnt; q++) skip[i + q] = 1;
+    }
+}
+
+/*
  * igdo_run: replay events[0..n) (16-byte records) of one kernel with grid geometry
  * (n_blocks, block_dim).  Only words w with shard(w) == shard_k (of shard_K; K=1 means
  * all) are shadow-checked; all synchronization and lock events are replayed regardless
@@ -180,9 +211,9 @@ static int o_valid(const o_event* e, const o_geom* g) {
  * total is returned in *n_reports.  On an ill-formed event returns O_ETRACE and its index
  * in *bad_index.
  */
-int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,
-             uint32_t shard_k, uint32_t shard_K, o_report* out, uint64_t cap,
-             uint64_t* n_reports, uint64_t* bad_index) {
+int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,
+                uint32_t shard_k, uint32_t shard_K, uint32_t flags, o_report* out, uint64_t cap,
+                uint64_t* n_reports, uint64_t* bad_index) {
     *n_reports = 0;
     *bad_index = 0;
     if (n_blocks == 0 || block_dim == 0) return O_EINVAL;
@@ -217,11 +248,14 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
     uint32_t* touched_list = (uint32_t*)calloc(g.warps, sizeof(uint32_t));
     uint32_t n_touched = 0;
     o_map map = {0, 0, 0};
+    uint8_t* skip = (flags & 1u) ? (uint8_t*)calloc(n ? n : 1, 1) : NULL; /* A32 coalesced members */
     int rc = O_OK;
-    if (!devF || !anyF || !wbar || !bbar || !wt || !tt || !isThread || !touched || !touched_list) {
+    if (!devF || !anyF || !wbar || !bbar || !wt || !tt || !isThread || !touched || !touched_list ||
+        ((flags & 1u) && !skip)) {
         rc = O_ENOMEM;
         goto done;
     }
+    if (skip) o_mark_coalesced(events, n, &g, skip);
 
 #define DEV(t) (devF[t] + G)
 #define ANY(t) (anyF[t] + G)
@@ -295,6 +329,7 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
         uint16_t L = o_held_of(TABLE(c));                        /* 3.1: before own update (A11) */
 
         int owned = (shard_K == 1) || ((o_fmix32((uint32_t)word ^ (uint32_t)(word >> 32)) % shard_K) == shard_k);
+        if (skip && skip[i]) owned = 0; /* A32: checked by its group's first lane */
         if (owned) {
             o_shadow* S = o_map_get(&map, word);
             if (!S) { rc = O_ENOMEM; goto done; }
@@ -395,8 +430,14 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
 
 done:
     free(devF); free(anyF); free(wbar); free(bbar); free(wt); free(tt);
-    free(isThread); free(touched); free(touched_list); free(map.slot);
+    free(isThread); free(touched); free(touched_list); free(map.slot); free(skip);
     return rc;
+}
+
+int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,
+             uint32_t shard_k, uint32_t shard_K, o_report* out, uint64_t cap,
+             uint64_t* n_reports, uint64_t* bad_index) {
+    return igdo_run_ex(events, n, n_blocks, block_dim, shard_k, shard_K, 0, out, cap, n_reports, bad_index);
 }
 
 /* Exported constants so the Python side can check it loaded this library. */

@@ -209,3 +209,51 @@ def concat_kernels(traces) -> np.ndarray:
             parts.append(boundary_event())
         parts.append(np.asarray(t, EVENT_DTYPE))
     return np.concatenate(parts) if parts else np.zeros(0, EVENT_DTYPE)
+
+
+def warp_instr_trace(seed: int, n_instr: int, n_blocks: int = 2, block_dim: int = 64, n_words: int = 24,
+                     p_shared: float = 0.5, weights=None):
+    """Warp-instruction-shaped fuzz trace: each step picks a warp, an active mask and a kind and
+    emits one event per active lane in ascending lane order (the trace convention of
+    include/igd.h).  With probability ``p_shared`` an access instruction's lanes all touch one
+    word (the shape §6.5's coalescing targets), else each lane picks its own word.
+    Returns (events, n_blocks, block_dim)."""
+    rng = np.random.default_rng(seed)
+    g = Geometry(n_blocks, block_dim)
+    b = TraceBuilder(n_blocks, block_dim)
+    if weights is None:
+        weights = [30, 14, 16, 3, 2, 8, 4, 3, 1]   # LD ST ATOM CAS EXCH FENCE SYNCWARP SYNCTHREADS GRID
+    w = np.asarray(weights, float)
+    w = w / w.sum()
+    for _ in range(n_instr):
+        k = int(rng.choice(len(weights), p=w))
+        blk = int(rng.integers(0, n_blocks))
+        wi = int(rng.integers(0, (block_dim + 31) // 32))
+        lanes_here = min(32, block_dim - wi * 32)
+        full = (1 << lanes_here) - 1
+        r = rng.random()
+        mask = full if r < 0.4 else (int(rng.integers(1, 1 << lanes_here)) if r < 0.9 else 1 << int(rng.integers(0, lanes_here)))
+        lanes = [l for l in range(lanes_here) if (mask >> l) & 1]
+        tid0 = blk * block_dim + wi * 32
+        if k in (LD, ST, ATOM, CAS, EXCH):
+            scope = NONE if k in (LD, ST) else int(rng.integers(1, 4))
+            if k in (CAS, EXCH):
+                shared_word = 500 + int(rng.integers(0, 3))
+            else:
+                shared_word = int(rng.integers(0, n_words))
+            shared = rng.random() < p_shared or k in (CAS, EXCH)
+            for l in lanes:
+                word = shared_word if shared else int(rng.integers(0, n_words))
+                b.ev(k, tid0 + l, word, scope, mask)
+        elif k == FENCE:
+            s = int(rng.integers(1, 4))
+            for l in lanes:
+                b.ev(FENCE, tid0 + l, 0, s, mask)
+        elif k == SYNCWARP:
+            b.ev(SYNCWARP, tid0 + lanes[0], 0, NONE, mask)
+        elif k == SYNCTHREADS:
+            b.ev(SYNCTHREADS, blk * block_dim, 0, NONE, 0xFFFFFFFF)
+        else:
+            b.ev(GRID_SYNC, 0, 0, NONE, 0xFFFFFFFF)
+    _ = g
+    return b.events(), n_blocks, block_dim
