@@ -140,7 +140,13 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
 /* Run the race check over the attached trace.  On success *n_reports_global holds the number
    of reports; the reports stay in context-owned device memory until the next igd_detect or
    igd_ctx_destroy.  Returns IGD_ETRACE (igd_bad_event gives the index) on an ill-formed
-   event, IGD_ETOOBIG if the accessed words span >= 2^32 words.  flags: 0. */
+   event, IGD_ETOOBIG if the accessed words span >= 2^32 words.
+   flags: IGD_DETECT_TIMING (per-stage timings, below) | IGD_DETECT_COALESCE (warp-coalesced
+   check, §6.5, reading A32: of a warp instruction whose >= 2 active lanes all LD, or
+   all ATOM, one word -- consecutive events, same warp / kind / scope / mask / word, lanes
+   ascending from the mask's lowest -- only the first lane is checked and recorded; the
+   reports then differ from the per-lane default).  Single-context (not sharded) only. */
+#define IGD_DETECT_COALESCE 2u
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
 
 /* ---- multi-GPU sharding, driven by the host over torch.distributed / NCCL ----

@@ -42,6 +42,7 @@ struct Params {
     u64* status;            // [n_tiles * 256], zeroed
     u32* kout;              // access keys, sorted by digit 0
     u64* vout;              // access payload (event index | tk << 32), same order
+    const u32* skip_bits;   // coalesced mode (A32): bit i = event i is not an access record
 };
 
 // Decode of an event ingest pass 0 has already validated (the same fields as ingest::decode,
@@ -130,8 +131,10 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
         const u32 p = wofs + j * 32 + lane;
-        const FDec d = fdecode(s_ev[p], g, ks);  // valid: ingest pass 0 checked every event
+        FDec d = fdecode(s_ev[p], g, ks);  // valid: ingest pass 0 checked every event
         const bool in = p < tile_e;
+        if (P.skip_bits && d.acc && in && ((__ldg(P.skip_bits + ((base + p) >> 5)) >> (p & 31u)) & 1u))
+            d.acc = false;  // A32: checked by its coalesced group's first lane
         key[j] = d.key;
         tk[j] = d.tk;
         amask |= ((in && d.acc) ? 1u : 0u) << j;

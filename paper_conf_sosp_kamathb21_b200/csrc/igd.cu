@@ -15,6 +15,7 @@
 
 #include "check.cuh"
 #include "check4.cuh"
+#include "coalesce.cuh"
 #include "common.cuh"
 #include "fused.cuh"
 #include "ingest.cuh"
@@ -56,13 +57,14 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
-    Buf off, ldesc, gtab, tcnt, tpts;
+    Buf off, ldesc, gtab, tcnt, tpts, skipb;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
     int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any, 2 = atomic-or (IGD_SORT_MODE)
     int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
     int count_tma = 0;  // IGD_COUNT_TMA=1: ingest pass 0 through a TMA ring (ingest::k_count; measured slower: 8.6 vs 7.2 ms at C5 1e9, the pass is issue-bound)
+    bool coalesce = false;  // IGD_DETECT_COALESCE of the running igd_detect (reading A32)
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
     bool shard = false;
@@ -318,6 +320,18 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     ip.hist_sync = P_<u32>(ctx->hist) + 1024;
     ip.stats = P_<u64>(ctx->stats);
     ip.n_tiles = (u32)in_tiles;
+    ip.skip_bits = nullptr;
+    if (ctx->coalesce && !SH && n_src > 0) {
+        // warp-coalesced mode (A32): mark the events checked by their group's first lane
+        const u64 rows = (n_src + 31) / 32;
+        RET(ensure(ctx, ctx->skipb, rows * sizeof(u32)));
+        const u64 warps = (rows + coal::ROWS - 1) / coal::ROWS;
+        KTimer kt(ctx, KC_INGEST, 16.0 * (double)n_src);
+        coal::k_coalesce_marks<<<(unsigned)((warps * 32 + coal::THREADS - 1) / coal::THREADS), coal::THREADS, 0,
+                                 ctx->stream>>>(src_ev, n_src, g, P_<u32>(ctx->skipb));
+        CK(cudaGetLastError());
+        ip.skip_bits = P_<u32>(ctx->skipb);
+    }
     const bool FUSED = !SH && ctx->fused;
     ip.hist0 = FUSED ? 1 : 0;
     int occ = 0;
@@ -391,6 +405,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         fp.status = P_<u64>(ctx->status);
         fp.kout = P_<u32>(ctx->acc_k[1]);
         fp.vout = P_<u64>(ctx->acc_v[1]);
+        fp.skip_bits = ip.skip_bits;
         {
             // reads every event once, writes the 12-byte access records and 8-byte sync records
             KTimer kt(ctx, KC_FUSED, 16.0 * (double)n_src + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
@@ -798,8 +813,10 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     }
     cudaSetDevice(ctx->device);
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
+    ctx->coalesce = (flags & IGD_DETECT_COALESCE) != 0;
     ctx->shard = false;
     int rc = detect_impl(ctx, n_reports_global);
+    ctx->coalesce = false;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
     return rc;
 }
@@ -916,7 +933,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
                   &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->tcnt,
-                  &ctx->tpts,         &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
+                  &ctx->tpts,         &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf};
     for (Buf* b : all) buf_free(ctx, *b);

@@ -39,6 +39,7 @@ struct Params {
     u32* hist_sync;  // [4][256]
     u64* stats;      // [0] min word, [1] max word, [2] bad index, [3] n_acc, [4] n_sync, [5] n_lock
     u32 n_tiles;
+    const u32* skip_bits;  // coalesced mode (A32): bit i = event i is checked by its group's first lane
     int hist0;       // pass 0, fused pipeline: the 4 digit histograms of the access keys (digit 0 for
                      // fused.cuh, 1..3 for the later passes) and no sync-key histograms (k_hist_keys
                      // over the written sync records instead)
@@ -186,6 +187,8 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
                 const u64 i = base + (u64)j * THREADS + tid;
                 if (i < P.n) {
                     dv[j] = decode(e[j], g, ks);
+                    if (P.skip_bits && (dv[j].flags & 1u) && ((__ldg(P.skip_bits + (i >> 5)) >> (i & 31u)) & 1u))
+                        dv[j].flags &= ~1u;  // A32: not an access record
                     if (PASS == 0 && (dv[j].flags & 1u)) {
                         const u64 word = ev_addr(e[j]) >> 2;
                         wmin = min(wmin, word);
@@ -426,6 +429,8 @@ __global__ void __launch_bounds__(THREADS, IGD_COUNT_MINB) k_count(Params P) {
             Dec dv;
             if (in) {
                 dv = decode(e, g, ks);
+                if (P.skip_bits && (dv.flags & 1u) && ((__ldg(P.skip_bits + (i >> 5)) >> (i & 31u)) & 1u))
+                    dv.flags &= ~1u;  // A32: not an access record
                 if (dv.flags & 1u) {
                     const u64 word = ev_addr(e) >> 2;
                     wmin = min(wmin, word);

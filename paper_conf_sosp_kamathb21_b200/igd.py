@@ -19,6 +19,7 @@ REPORT_DTYPE = np.dtype([("addr", "<u8"), ("cur", "<u8"), ("prev", "<u8"), ("typ
 IGD_OK, IGD_EINVAL, IGD_ETRACE, IGD_ETOOBIG, IGD_ENOMEM, IGD_ECUDA, IGD_ENCCL, IGD_ESTATE = 0, -1, -2, -3, -4, -5, -6, -7
 IGD_TRACE_DEVICE_PTR = 1
 IGD_DETECT_TIMING = 1
+IGD_DETECT_COALESCE = 2
 IGD_N_STAGES = 8
 IGD_N_KCLASS = 9
 
@@ -194,8 +195,10 @@ class Detector:
             self._borrowed = None
             igd_trace_load(self.ctx, n_blocks, block_dim, ev.ctypes.data if len(ev) else 0, len(ev), False)
 
-    def detect(self, timing: bool = False) -> int:
-        self.n_reports = igd_detect(self.ctx, IGD_DETECT_TIMING if timing else 0)
+    def detect(self, timing: bool = False, coalesce: bool = False) -> int:
+        """igd_detect; ``coalesce``: warp-coalesced check mode (IGD_DETECT_COALESCE)."""
+        flags = (IGD_DETECT_TIMING if timing else 0) | (IGD_DETECT_COALESCE if coalesce else 0)
+        self.n_reports = igd_detect(self.ctx, flags)
         return self.n_reports
 
     def reports(self) -> np.ndarray:
