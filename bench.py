@@ -136,7 +136,7 @@ def run_reference(args, fam, rank, world):
     value = sample / t / 1e9
     sample_desc = f"first {sample} of {n_total} events of {F.FAMILY_NAMES[fam]} (single-threaded oracle)"
     line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic", "impl": "reference",
             "config": {"workload": F.FAMILY_NAMES[fam], "events": n_total, "sample_events": sample,
                        "n_blocks": nb, "block_dim": bd},
@@ -427,7 +427,7 @@ def main():
     b_alg = 16 + 32 * f_acc  # read the event + read/write a 16-B metadata entry per access
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
-                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": "u32", "data": "synthetic",
                 "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
                            "f_acc": f_acc, "reports": int(nrep),
