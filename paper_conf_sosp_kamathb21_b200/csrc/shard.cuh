@@ -19,7 +19,13 @@ namespace shard {
 
 constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
-constexpr int ITEMS = 8;
+#ifndef IGD_SHARD_ITEMS
+#define IGD_SHARD_ITEMS 4  // 4 items, 4 CTAs/SM: sharded C5@1e9 at N=1 108 -> 95 ms per step
+#endif
+#ifndef IGD_SHARD_MINB
+#define IGD_SHARD_MINB 4
+#endif
+constexpr int ITEMS = IGD_SHARD_ITEMS;
 constexpr int TILE = THREADS * ITEMS;
 constexpr int MAXP = 16;
 
@@ -50,7 +56,7 @@ struct Params {
 };
 
 template <int PASS>
-__global__ void __launch_bounds__(THREADS, 2) k_shard(Params P) {
+__global__ void __launch_bounds__(THREADS, IGD_SHARD_MINB) k_shard(Params P) {
     __shared__ u32 s_wc[ITEMS][WARPS][MAXP + 1];  // per (item, warp, destination) counts, then offsets
     const u32 tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const u32 lt = lanemask_lt();
