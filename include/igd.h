@@ -170,7 +170,8 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
    all ranks concatenated in source-rank order; d_sync_idx / d_sync_events = the global sync stream;
    min_word = global minimum accessed word.  Device pointers are borrowed for the call.  Reports (global
    indices) are read with igd_reports / igd_reports_device; the union over ranks is the single-GPU
-   report set (address-shard invariance).  flags: IGD_DETECT_TIMING or 0. */
+   report set (address-shard invariance).  flags: IGD_DETECT_TIMING or 0 (IGD_DETECT_COALESCE:
+   IGD_EINVAL, a coalesced group may straddle two ranks' chunks). */
 int igd_shard_prepare(igd_ctx* ctx, uint32_t nranks, uint64_t* counts, uint64_t* n_sync_stream,
                       uint64_t* bad_event, uint64_t* word_minmax);
 int igd_shard_buffers(igd_ctx* ctx, void** d_records, void** d_sync_idx, void** d_sync_events);

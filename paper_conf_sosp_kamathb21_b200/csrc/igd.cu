@@ -847,6 +847,10 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     if (!ctx || !n_reports) return IGD_EINVAL;
     if ((n_records && !d_records) || (n_sync_stream && (!d_sync_idx || !d_sync_events))) return IGD_EINVAL;
     if (!ctx->loaded) return IGD_ESTATE;
+    if (flags & IGD_DETECT_COALESCE) {  // reading A32: a group may straddle two ranks' chunks
+        ctx->err = "IGD_DETECT_COALESCE is a single-context mode";
+        return IGD_EINVAL;
+    }
     cudaSetDevice(ctx->device);
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
     ctx->shard = true;
