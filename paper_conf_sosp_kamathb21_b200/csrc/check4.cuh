@@ -31,6 +31,9 @@ namespace check {
 #ifndef IGD_C4_MINB
 #define IGD_C4_MINB 6
 #endif
+#ifndef IGD_C4_NOGATHER
+#define IGD_C4_NOGATHER 0  // timing experiment only (wrong results): no active-mask gathers (C5@1e9: the gathers cost ~1.5 ms of ~15)
+#endif
 #ifndef IGD_C4_WLB
 #define IGD_C4_WLB 0  // 1: warp-parallel look-back (measured slower: 14.9 -> 15.9 ms at C5@1e9; walks are short)
 #endif
@@ -219,7 +222,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
         // P4's lockstep clause will need this instruction's active mask when md is likely the
         // previous access, from another lane of the same warp, and the mask is partial: gather
         // it now so the trace read overlaps the scans (phase 1 re-checks the exact condition)
-        if (!MV && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) M[j] = ld_event(P.ev, V[j]).w;
+        if (!MV && !IGD_C4_NOGATHER && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) M[j] = ld_event(P.ev, V[j]).w;
     }
 
     // ---- warp aggregate in the packed state of check.cuh (state after the warp's last access) ----
@@ -418,7 +421,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
                         // prefetched unless md is an earlier writer (M[j] is the mask then only
                         // if the previous access was also a same-warp candidate)
                         const bool pre = MV || (prevMd && !(Z[j] >> 30));
-                        if ((((pre ? M[j] : ld_event(P.ev, V[j]).w)) >> g.lane(p)) & 1u) break;
+                        if ((((pre || IGD_C4_NOGATHER ? M[j] : ld_event(P.ev, V[j]).w)) >> g.lane(p)) & 1u) break;
                     } else {
                         gather = true;
                     }
