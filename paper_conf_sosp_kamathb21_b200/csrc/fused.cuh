@@ -260,7 +260,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
             }
             st_relaxed(P.status + (u64)tile * RADIX + dg, ST_INC | (excl + cnt));
         }
-        s_gbase[dg] = P.digit_base[dg] + (u32)excl;
+        s_gbase[dg] = P.digit_base[dg] + (u32)excl - s_tile_excl[dg];  // position = s_gbase[d] + i
     }
     __syncthreads();
     // ---- records to their tile positions: key, payload (event index | tk << 32), digit
@@ -282,7 +282,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
         const u32 i = t + k * THREADS;
         if (i < na) {
             const u32 d = s_dig[i];
-            const u32 o = s_gbase[d] + (i - s_tile_excl[d]);
+            const u32 o = s_gbase[d] + i;
             __stcs(P.kout + o, s_k[i]);
             __stcs(P.vout + o, s_v[i]);
         }

@@ -278,7 +278,9 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             }
             st_relaxed(P.status + (u64)tile * RADIX + d, ST_INC | (excl + cnt));
         }
-        s_gbase[d] = P.digit_base[d] + (u32)excl;
+        // output position of tile position i with digit d = s_gbase[d] + i (u32 arithmetic wraps
+        // back into range): one shared load per written element instead of two
+        s_gbase[d] = P.digit_base[d] + (u32)excl - s_tile_excl[d];
     }
     __syncthreads();
     // keys: reorder in shared memory (rank[] becomes the tile position), write digit runs
@@ -297,7 +299,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             const u32 kk = s_k[i];
             const u32 d = (kk >> shift) & 255u;
             s_dig[i] = (uint8_t)d;
-            __stcs(P.kout + s_gbase[d] + (i - s_tile_excl[d]), kk);
+            __stcs(P.kout + (s_gbase[d] + i), kk);
         }
     }
     // values: same permutation, in place through the staged buffer
@@ -323,7 +325,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         const u32 i = t + k * THREADS;
         if (i < tile_n) {
             const u32 d = s_dig[i];
-            __stcs(vout + s_gbase[d] + (i - s_tile_excl[d]), s_v[i]);
+            __stcs(vout + (s_gbase[d] + i), s_v[i]);
         }
     }
 }
