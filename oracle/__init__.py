@@ -15,6 +15,9 @@ Parity status per function:
   * coalesced mode (A32)    -- pinned: equals the plain replay of the trace with the coalesced
                                members deleted (group detection restated in numpy in the
                                test), worked example (one report per warp instruction).
+  * paper-width counters (A33) -- pinned: the from-scratch evaluator counting sync events
+                               modulo the widths (tests/pins.py), equality with the exact
+                               mode below the widths, a worked 64-fence example.
   * Bloom/hash constants    -- parity unpinned by the paper (reading A8): pinned only by
                                agreement with the brute force, which restates them.
 """
@@ -72,10 +75,11 @@ def _load():
 
 
 def run(events: np.ndarray, n_blocks: int, block_dim: int, shard=(0, 1), cap: int = None,
-        coalesce: bool = False):
+        coalesce: bool = False, paper_counters: bool = False):
     """Replay ``events`` (EVENT_DTYPE, 16 B each) and return the report array (REPORT_DTYPE),
     ascending by ``cur``.  ``shard=(k, K)`` checks only words owned by shard k (C.7 5(b)).
-    ``coalesce``: warp-coalesced check mode (§6.5, reading A32)."""
+    ``coalesce``: warp-coalesced check mode (§6.5, reading A32).  ``paper_counters``: the
+    synchronization IDs wrap at Fig. 4's widths (reading A33)."""
     lib = _load()
     ev = np.ascontiguousarray(events)
     assert ev.dtype.itemsize == 16
@@ -87,7 +91,7 @@ def run(events: np.ndarray, n_blocks: int, block_dim: int, shard=(0, 1), cap: in
         nrep = ctypes.c_uint64(0)
         bad = ctypes.c_uint64(0)
         rc = lib.igdo_run_ex(ev.ctypes.data if n else None, n, n_blocks, block_dim, shard[0], shard[1],
-                             1 if coalesce else 0, out.ctypes.data, cap, ctypes.byref(nrep), ctypes.byref(bad))
+                             (1 if coalesce else 0) | (2 if paper_counters else 0), out.ctypes.data, cap, ctypes.byref(nrep), ctypes.byref(bad))
         if rc != O_OK:
             raise OracleError(rc, bad.value if rc == O_ETRACE else None)
         if nrep.value <= cap:

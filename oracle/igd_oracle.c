@@ -249,6 +249,7 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
     uint32_t n_touched = 0;
     o_map map = {0, 0, 0};
     uint8_t* skip = (flags & 1u) ? (uint8_t*)calloc(n ? n : 1, 1) : NULL; /* A32 coalesced members */
+    const int wrap = (flags & 2u) != 0; /* A33: paper-width synchronization IDs */
     int rc = O_OK;
     if (!devF || !anyF || !wbar || !bbar || !wt || !tt || !isThread || !touched || !touched_list ||
         ((flags & 1u) && !skip)) {
@@ -355,14 +356,27 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
                 uint32_t w_p = g_warp(&g, p), b_p = g_block(&g, p);
                 /* preliminary checks (reading A4: md.* = relation between md and curr) */
                 int P3 = (p == c);
-                int P4 = (w_p == w_c) && (WB(w_c) != md->sWB || (e.mask >> g_lane(&g, p)) & 1u);
-                int P5 = (b_p == b_c) && (BB(b_c) != md->sBB);
+                int P4, P5, noAny, noDev;
+                if (!wrap) {
+                    P4 = (w_p == w_c) && (WB(w_c) != md->sWB || (e.mask >> g_lane(&g, p)) & 1u);
+                    P5 = (b_p == b_c) && (BB(b_c) != md->sBB);
+                    noAny = (ANY(p) == md->sANY); /* A1: md's thread has not fenced since */
+                    noDev = (DEV(p) == md->sDEV);
+                } else {
+                    /* A33: the IDs have Fig. 4's widths -- WarpBarID 6, BlkBarID 8, DevFenceID 6,
+                       BlkFenceID 6 bits -- so "unchanged" means a multiple of 2^width events */
+                    uint64_t dWB = WB(w_c) - md->sWB, dBB = BB(b_c) - md->sBB;
+                    uint64_t dDev = DEV(p) - md->sDEV;
+                    uint64_t dBlk = (ANY(p) - DEV(p)) - (md->sANY - md->sDEV); /* block-scope fences */
+                    P4 = (w_p == w_c) && ((dWB & 63u) != 0 || (e.mask >> g_lane(&g, p)) & 1u);
+                    P5 = (b_p == b_c) && ((dBB & 255u) != 0);
+                    noDev = (dDev & 63u) == 0;
+                    noAny = noDev && (dBlk & 63u) == 0;
+                }
                 int P6 = S->atomic && isAtomic && (b_p == b_c || S->ascope == S_DEVICE);
                 if (P3 || P4 || P5 || P6) goto writeback;
 
                 /* race checks in order; first true is reported */
-                int noAny = (ANY(p) == md->sANY);   /* A1: md's thread has not fenced since */
-                int noDev = (DEV(p) == md->sDEV);
                 int type = R_NONE;
                 if (S->atomic && S->ascope == S_BLOCK && g_block(&g, S->LW.tid) != b_c) type = R1;
                 else if (w_p == w_c && noAny && !S->devShared && !S->blkShared) type = R2;

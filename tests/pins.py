@@ -120,9 +120,31 @@ def _sync_between(kind, tid, scope, geo, lo, hi, what, ent):
     return False
 
 
-def bf_scratch(events, nb, bd):
+def _sync_count(kind, tid, scope, geo, lo, hi, what, ent):
+    """Number of events strictly inside (lo, hi) that advance the paper's ID ``what`` of
+    entity ``ent`` (Fig. 4 fields; grid syncs are a device fence by every thread and a barrier
+    for every block, A15)."""
+    n = 0
+    for x in range(lo + 1, hi):
+        k = kind[x]
+        if what == "WarpBarID":
+            n += k == SYNCWARP and geo.warp(tid[x]) == ent
+        elif what == "BlkBarID":
+            n += (k == SYNCTHREADS and geo.block(tid[x]) == ent) or k == GRID
+        elif what == "DevFenceID":
+            n += (k == FENCE and tid[x] == ent and scope[x] >= 2) or k == GRID
+        elif what == "BlkFenceID":
+            n += k == FENCE and tid[x] == ent and scope[x] == 1
+    return n
+
+
+WIDTH = {"WarpBarID": 6, "BlkBarID": 8, "DevFenceID": 6, "BlkFenceID": 6}  # Fig. 4 (P:763-829)
+
+
+def bf_scratch(events, nb, bd, paper_counters=False):
     """From-scratch evaluator (C.7 1).  Returns a list of (addr, cur, prev, type, cur_kind,
-    prev_kind) sorted by cur."""
+    prev_kind) sorted by cur.  ``paper_counters``: an ID counts as changed only when the number
+    of its events since md is not a multiple of 2^width (reading A33)."""
     geo = _Geo(nb, bd)
     addr, tid, kind, scope, mask, rawkind = _decode(events)
     L = lock_replay(events, nb, bd)
@@ -153,13 +175,23 @@ def bf_scratch(events, nb, bd):
                 same_w = geo.warp(p) == geo.warp(c)
                 same_b = geo.block(p) == geo.block(c)
                 P3 = p == c
-                P4 = same_w and (_sync_between(kind, tid, scope, geo, md, i, "warp_bar", geo.warp(c))
-                                 or (mask[i] >> geo.lane(p)) & 1 == 1)
-                P5 = same_b and _sync_between(kind, tid, scope, geo, md, i, "block_bar", geo.block(c))
+                if paper_counters:
+                    def moved(what, ent):
+                        return _sync_count(kind, tid, scope, geo, md, i, what, ent) % (1 << WIDTH[what]) != 0
+                    P4 = same_w and (moved("WarpBarID", geo.warp(c)) or (mask[i] >> geo.lane(p)) & 1 == 1)
+                    P5 = same_b and moved("BlkBarID", geo.block(c))
+                else:
+                    P4 = same_w and (_sync_between(kind, tid, scope, geo, md, i, "warp_bar", geo.warp(c))
+                                     or (mask[i] >> geo.lane(p)) & 1 == 1)
+                    P5 = same_b and _sync_between(kind, tid, scope, geo, md, i, "block_bar", geo.block(c))
                 P6 = atomic and k in ATOMICS and (same_b or ascope == 2)
                 if not (P3 or P4 or P5 or P6):
-                    noAny = not _sync_between(kind, tid, scope, geo, md, i, "any_fence", p)
-                    noDev = not _sync_between(kind, tid, scope, geo, md, i, "dev_fence", p)
+                    if paper_counters:
+                        noDev = not moved("DevFenceID", p)
+                        noAny = noDev and not moved("BlkFenceID", p)
+                    else:
+                        noAny = not _sync_between(kind, tid, scope, geo, md, i, "any_fence", p)
+                        noDev = not _sync_between(kind, tid, scope, geo, md, i, "dev_fence", p)
                     typ = 0
                     if atomic and ascope == 1 and geo.block(tid[LW]) != geo.block(c):
                         typ = 1

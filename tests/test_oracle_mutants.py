@@ -18,8 +18,11 @@ REPORT = np.dtype([("addr", "<u8"), ("cur", "<u8"), ("prev", "<u8"), ("type", "u
                    ("cur_kind", "u1"), ("prev_kind", "u1"), ("pad", "u1", (5,))])
 
 MUTANTS = {
-    "noAny_uses_current_thread": ("int noAny = (ANY(p) == md->sANY);", "int noAny = (ANY(c) == md->sANY);"),
-    "noDev_uses_any": ("int noDev = (DEV(p) == md->sDEV);", "int noDev = (ANY(p) == md->sDEV);"),
+    "noAny_uses_current_thread": ("noAny = (ANY(p) == md->sANY);", "noAny = (ANY(c) == md->sANY);"),
+    "noDev_uses_any": ("noDev = (DEV(p) == md->sDEV);", "noDev = (ANY(p) == md->sDEV);"),
+    "A33_devfence_width_7": ("noDev = (dDev & 63u) == 0;", "noDev = (dDev & 127u) == 0;"),
+    "A33_blkfence_ignored": ("noAny = noDev && (dBlk & 63u) == 0;", "noAny = noDev;"),
+    "A33_barrier_width_6": ("((dBB & 255u) != 0)", "((dBB & 63u) != 0)"),
     "md_always_last_accessor": ("(k == O_LD) ? &S->LW : &S->LA", "&S->LA"),
     "P4_drops_mask_clause": ("|| (e.mask >> g_lane(&g, p)) & 1u", "|| 0"),
     "P4_mask_uses_current_lane": ("(e.mask >> g_lane(&g, p))", "(e.mask >> g_lane(&g, c))"),
@@ -58,7 +61,21 @@ def _build(mutant_src, d):
     lib.igdo_run.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                              ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
                              ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
+    lib.igdo_run_ex.restype = ctypes.c_int
+    lib.igdo_run_ex.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
+                                ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
     return lib
+
+
+def _run_paper_counters(lib, ev, nb, bd):
+    cap = 4096
+    out = np.zeros(cap, REPORT)
+    nrep, bad = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    rc = lib.igdo_run_ex(ev.ctypes.data if len(ev) else None, len(ev), nb, bd, 0, 1, 2, out.ctypes.data, cap,
+                         ctypes.byref(nrep), ctypes.byref(bad))
+    assert rc == 0
+    return full_tuples(out[: nrep.value])
 
 
 def _run(lib, ev, nb, bd):
@@ -83,6 +100,11 @@ def _caught(lib):
         ev, nb, bd = tg.random_trace(seed, int(rng.integers(20, 160)), n_words=int(rng.integers(1, 10)), **kw)
         if _run(lib, ev, nb, bd) != bf_scratch(ev, nb, bd):
             return f"bruteforce seed {seed}"
+    from test_paper_counters import _burst_trace  # paper-width IDs (A33)
+    for seed in range(100):
+        ev, nb, bd = _burst_trace(seed, 40, threads=[0, 1, 33, 64] if seed % 2 else None)
+        if _run_paper_counters(lib, ev, nb, bd) != bf_scratch(ev, nb, bd, paper_counters=True):
+            return f"paper-counter bursts seed {seed}"
     return None
 
 
