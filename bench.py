@@ -94,19 +94,19 @@ def peaks():
         return 6650.0, "fallback"
 
 
-def oracle_baseline(ev, nb, bd, budget_s=15.0, coalesce=False):
+def oracle_baseline(ev, nb, bd, budget_s=15.0, coalesce=False, paper_counters=False):
     """Time the CPU oracle (as it stands, single-threaded) on a bounded prefix of the trace."""
     import oracle
 
     n = min(len(ev), 2_000_000)
     t0 = time.perf_counter()
-    oracle.run(ev[:n], nb, bd, coalesce=coalesce)
+    oracle.run(ev[:n], nb, bd, coalesce=coalesce, paper_counters=paper_counters)
     dt = time.perf_counter() - t0
     rate = n / dt
     n2 = int(min(len(ev), max(n, rate * budget_s)))
     if n2 > n:
         t0 = time.perf_counter()
-        oracle.run(ev[:n2], nb, bd, coalesce=coalesce)
+        oracle.run(ev[:n2], nb, bd, coalesce=coalesce, paper_counters=paper_counters)
         dt = time.perf_counter() - t0
         n = n2
     return n, dt
@@ -288,6 +288,8 @@ def main():
     ap.add_argument("--threads", type=int, default=0, help="generator threads (0 = all cores)")
     ap.add_argument("--sharded", action="store_true", help="use the multi-GPU path even at N=1")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"], help="N>1 collectives")
+    ap.add_argument("--paper-counters", action="store_true",
+                    help="Fig. 4-width synchronization IDs (IGD_DETECT_PAPER_COUNTERS, reading A33)")
     ap.add_argument("--coalesce", action="store_true",
                     help="warp-coalesced check mode (IGD_DETECT_COALESCE, reading A32; 1 GPU)")
     args = ap.parse_args()
@@ -332,8 +334,9 @@ def main():
     stream = det.stream
     det.load(dev, nb, bd)
     co = args.coalesce
+    pc = args.paper_counters
     for _ in range(args.warmup):
-        nrep = det.detect(coalesce=co)
+        nrep = det.detect(coalesce=co, paper_counters=pc)
     # ---------------- timed region (device-resident trace) ----------------
     clocks = ClockSampler(local)
     clocks.start()
@@ -346,7 +349,7 @@ def main():
     launches = 0
     e0.record(stream)
     for _ in range(args.steps):
-        nrep = det.detect(timing=True, coalesce=co)
+        nrep = det.detect(timing=True, coalesce=co, paper_counters=pc)
         launches += det.launch_count()
         for k, (cnt, ms, b) in det.kernel_stats().items():
             c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
@@ -396,7 +399,7 @@ def main():
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         det.load(host, nb, bd)           # H2D copy of the trace inside the library
-        nr = det.detect(coalesce=co)
+        nr = det.detect(coalesce=co, paper_counters=pc)
         out = det.reports()              # D2H of the reports
         torch.cuda.synchronize()
         dt = time.perf_counter() - t0
@@ -416,7 +419,7 @@ def main():
     # ---------------- CPU oracle baseline (rank 0, N=1) ----------------
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        sn, sdt = oracle_baseline(host, nb, bd, coalesce=co)
+        sn, sdt = oracle_baseline(host, nb, bd, coalesce=co, paper_counters=pc)
         cpu = {"value": sn / sdt / 1e9, "unit": "G events/s", "cores": 1, "kind": "oracle",
                "sample": f"first {sn} events of {F.FAMILY_NAMES[fam]} ({sdt:.1f}s, single-threaded C oracle)"}
     if pinned:
@@ -431,8 +434,9 @@ def main():
                 "vs_baseline": None, "dtype": "u32", "data": "synthetic",
                 "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
                            "f_acc": f_acc, "reports": int(nrep),
-                           "ledger_reports": None if co else ledger_n,  # the ledger counts per-lane reports
-                           "check_mode": "warp-coalesced (A32)" if co else "per-lane",
+                           "ledger_reports": None if (co or pc) else ledger_n,  # ledger: per-lane, exact IDs
+                           "check_mode": ("warp-coalesced (A32)" if co else "per-lane")
+                           + (", paper-width IDs (A33)" if pc else ""),
                            "l2": "inputs larger than L2 (no flush)",
                            "parallelism": f"{world} GPU(s), one process per GPU"},
                 "roofline": roofline,

@@ -147,6 +147,12 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
    ascending from the mask's lowest -- only the first lane is checked and recorded; the
    reports then differ from the per-lane default).  Single-context (not sharded) only. */
 #define IGD_DETECT_COALESCE 2u
+/* IGD_DETECT_PAPER_COUNTERS (reading A33): the synchronization IDs copied into a
+   word's metadata keep Fig. 4's widths -- WarpBarID 6, BlkBarID 8, DevFenceID 6,
+   BlkFenceID 6 bits -- so an ID whose events since md number a multiple of 2^width reads as
+   unchanged (the paper's bounded-counter false positives, §6.7).  Default: exact counters (A16).
+   Also accepted by igd_shard_detect. */
+#define IGD_DETECT_PAPER_COUNTERS 4u
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
 
 /* ---- multi-GPU sharding, driven by the host over torch.distributed / NCCL ----
@@ -170,7 +176,7 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
    all ranks concatenated in source-rank order; d_sync_idx / d_sync_events = the global sync stream;
    min_word = global minimum accessed word.  Device pointers are borrowed for the call.  Reports (global
    indices) are read with igd_reports / igd_reports_device; the union over ranks is the single-GPU
-   report set (address-shard invariance).  flags: IGD_DETECT_TIMING or 0 (IGD_DETECT_COALESCE:
+   report set (address-shard invariance).  flags: IGD_DETECT_TIMING | IGD_DETECT_PAPER_COUNTERS (IGD_DETECT_COALESCE:
    IGD_EINVAL, a coalesced group may straddle two ranks' chunks). */
 int igd_shard_prepare(igd_ctx* ctx, uint32_t nranks, uint64_t* counts, uint64_t* n_sync_stream,
                       uint64_t* bad_event, uint64_t* word_minmax);

@@ -49,6 +49,27 @@ constexpr int C4_TILE = THREADS * C4_ITEMS;  // accesses per CTA
 
 __device__ __forceinline__ int hib(u32 m) { return 31 - (int)__clz(m); }  // m != 0
 
+// Number of entries x of entity e's list with a < x < b (paper-width IDs, reading A33):
+// lower_bound(b) - upper_bound(a), with the descriptor's fast paths
+__device__ __noinline__ u32 q_count(const uint4* __restrict__ desc, const u32* __restrict__ ts, u32 e, u32 a, u32 b) {
+    const uint4 d = __ldg(desc + e);
+    if (d.x == d.y || d.w <= a || d.z >= b || b <= a + 1) return 0;
+    u32 lo = d.x, hi = d.y;  // upper_bound(a)
+    while (lo < hi) {
+        const u32 mid = (lo + hi) >> 1;
+        if (__ldg(ts + mid) <= a) lo = mid + 1;
+        else hi = mid;
+    }
+    const u32 ua = lo;
+    hi = d.y;  // lower_bound(b) in [ua, d.y)
+    while (lo < hi) {
+        const u32 mid = (lo + hi) >> 1;
+        if (__ldg(ts + mid) < b) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo - ua;
+}
+
 // q_between without the call (no caller-saved spills in the scan loop): descriptor fast paths,
 // then a binary search -- for short lists such as the kernel boundaries
 __device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, const u32* __restrict__ ts, u32 e, u32 a,
@@ -131,7 +152,7 @@ __device__ __noinline__ bool q_grid_from(const PP& P, u32 a, u32 b, u32 x) {
 
 // KB: the trace has kernel boundaries (a separate instantiation: the boundary test costs
 // registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
-template <bool MV, bool KB>
+template <bool MV, bool KB, bool WRAP>
 __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
     __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
     __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
@@ -527,10 +548,31 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
             }
         }
 #else
+        u32 type;
+        if (WRAP) {
+            // reading A33: an ID moved iff the number of its events since md is not a multiple of
+            // 2^width (Fig. 4: WarpBarID 6, BlkBarID 8, DevFenceID 6, BlkFenceID 6 bits)
+            const u32 gcnt = P.glo != P.ghi ? q_count(P.desc, P.sts, ks.grid, mdIdx, i) : 0u;
+            if (same_w && (q_count(P.desc, P.sts, ks.wb + g.warp(c), mdIdx, i) & 63u)) continue;  // P4
+            if (same_b && ((q_count(P.desc, P.sts, ks.bb + g.block(c), mdIdx, i) + gcnt) & 255u)) continue;  // P5
+            type = (flags & QF_R1) ? IGD_R1 : 0u;
+            if (!type) {
+                const u32 dfen = q_count(P.desc, P.sts, ks.dev + p, mdIdx, i);  // device fences of md's thread
+                const bool noDev = ((dfen + gcnt) & 63u) == 0;
+                if (same_b) {
+                    if (!(flags & QF_DEV)) {
+                        const u32 bfen = q_count(P.desc, P.sts, ks.any + p, mdIdx, i) - dfen;  // block-scope
+                        if (noDev && (bfen & 63u) == 0) type = (same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3;
+                    }
+                } else if (noDev) {
+                    type = IGD_R4;
+                }
+            }
+        } else {
         if (same_w && q_between(P.desc, P.sts, ks.wb + g.warp(c), mdIdx, i)) continue;  // P4: syncwarp
         const bool grid = q_grid(P, mdIdx, i);
         if (same_b && (grid || q_between(P.desc, P.sts, ks.bb + g.block(c), mdIdx, i))) continue;  // P5
-        u32 type = (flags & QF_R1) ? IGD_R1 : 0u;
+        type = (flags & QF_R1) ? IGD_R1 : 0u;
         if (!type) {
             if (same_b) {
                 // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread must
@@ -540,6 +582,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
             } else if (!grid && !q_between(P.desc, P.sts, ks.dev + p, mdIdx, i)) {
                 type = IGD_R4;  // R4: other block, no device fence by md's thread
             }
+        }
         }
 #endif
         if (!type && P.lv.any && P.debug_stop != 4) {  // R5: lock sets of the last accessor and of this access

@@ -65,6 +65,7 @@ struct igd_ctx {
     int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
     int count_tma = 0;  // IGD_COUNT_TMA=1: ingest pass 0 through a TMA ring (ingest::k_count; measured slower: 8.6 vs 7.2 ms at C5 1e9, the pass is issue-bound)
     bool coalesce = false;  // IGD_DETECT_COALESCE of the running igd_detect (reading A32)
+    bool paper_counters = false;  // IGD_DETECT_PAPER_COUNTERS (reading A33)
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
     bool shard = false;
@@ -242,6 +243,19 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
     }
     *out_cur = cur;
     return IGD_OK;
+}
+
+// a6 kernel instantiation: sharded payload (MV), kernel boundaries (KB), paper-width IDs (WRAP)
+template <bool MV, bool KB>
+static void launch_check_w(bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
+    if (wrap) check::k_check4<MV, KB, true><<<tb, check::THREADS, 0, st>>>(cp);
+    else check::k_check4<MV, KB, false><<<tb, check::THREADS, 0, st>>>(cp);
+}
+static void launch_check(bool mv, bool kb, bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
+    if (mv && kb) launch_check_w<true, true>(wrap, tb, st, cp);
+    else if (mv) launch_check_w<true, false>(wrap, tb, st, cp);
+    else if (kb) launch_check_w<false, true>(wrap, tb, st, cp);
+    else launch_check_w<false, false>(wrap, tb, st, cp);
 }
 
 static int scan_excl(igd_ctx* ctx, u32* data, u64 n) {
@@ -570,11 +584,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
-                const unsigned tb = (unsigned)tiles;
-                if (SH && cp.has_kb) check::k_check4<true, true><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
-                else if (SH) check::k_check4<true, false><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
-                else if (cp.has_kb) check::k_check4<false, true><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
-                else check::k_check4<false, false><<<tb, check::THREADS, 0, ctx->stream>>>(cp);
+                launch_check(SH, cp.has_kb != 0, ctx->paper_counters, (unsigned)tiles, ctx->stream, cp);
             }
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
@@ -814,9 +824,11 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     cudaSetDevice(ctx->device);
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
     ctx->coalesce = (flags & IGD_DETECT_COALESCE) != 0;
+    ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
     ctx->shard = false;
     int rc = detect_impl(ctx, n_reports_global);
     ctx->coalesce = false;
+    ctx->paper_counters = false;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
     return rc;
 }
@@ -853,6 +865,7 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     }
     cudaSetDevice(ctx->device);
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
+    ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
     ctx->shard = true;
     ctx->sh_rec = d_records;
     ctx->sh_nrec = n_records;
@@ -864,6 +877,7 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     RET(buf_free(ctx, ctx->sh_send));  // the exchange is done: release the send buffer first
     int rc = detect_impl(ctx, n_reports);
     ctx->shard = false;
+    ctx->paper_counters = false;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
     return rc;
 }

@@ -173,7 +173,8 @@ class GpuStage:
                 "sync_ev": _wrap(sev.value, nsync.value, EVENT_INTS, self.device),
                 "bad": int(bad.value), "min_word": int(mm[0]), "max_word": int(mm[1])}
 
-    def detect(self, recv, sync_idx, sync_ev, min_word: int, timing: bool = False) -> np.ndarray:
+    def detect(self, recv, sync_idx, sync_ev, min_word: int, timing: bool = False,
+               paper_counters: bool = False) -> np.ndarray:
         lib = _igd.load_library()
         recv = recv.contiguous()
         sync_idx = sync_idx.contiguous()
@@ -182,7 +183,8 @@ class GpuStage:
         rc = lib.igd_shard_detect(self.det.ctx, ctypes.c_void_p(recv.data_ptr() if recv.numel() else None),
                                   recv.shape[0], ctypes.c_void_p(sync_idx.data_ptr() if sync_idx.numel() else None),
                                   ctypes.c_void_p(sync_ev.data_ptr() if sync_ev.numel() else None), sync_idx.shape[0],
-                                  min_word, _igd.IGD_DETECT_TIMING if timing else 0, ctypes.byref(nrep))
+                                  min_word, (_igd.IGD_DETECT_TIMING if timing else 0)
+                                  | (_igd.IGD_DETECT_PAPER_COUNTERS if paper_counters else 0), ctypes.byref(nrep))
         if rc != _igd.IGD_OK:
             raise _igd.IgdError(rc, lib.igd_last_error(self.det.ctx).decode())
         self.det.n_reports = n = int(nrep.value)
@@ -202,7 +204,7 @@ def _check_prepared(bad: int, lo: int, hi: int, any_access: bool):
         raise _igd.IgdError(_igd.IGD_ETOOBIG, "accessed word range spans >= 2^32 words")
 
 
-def sharded_detect(stage, comm: TorchComm, timing: bool = False) -> np.ndarray:
+def sharded_detect(stage, comm: TorchComm, timing: bool = False, paper_counters: bool = False) -> np.ndarray:
     """One rank's part of the distributed check (the chunk is already loaded in `stage`).
     Returns the global report set (identical on every rank)."""
     prep = stage.prepare(comm.size)
@@ -215,7 +217,7 @@ def sharded_detect(stage, comm: TorchComm, timing: bool = False) -> np.ndarray:
     recv = comm.all_to_all_var(prep["records"], prep["counts"])
     sidx = comm.all_gather_var(prep["sync_idx"].reshape(-1, 1)).reshape(-1)
     sev = comm.all_gather_var(prep["sync_ev"])
-    local = stage.detect(recv, sidx, sev, lo if lo != (1 << 62) else 0, timing)
+    local = stage.detect(recv, sidx, sev, lo if lo != (1 << 62) else 0, timing, paper_counters)
     if isinstance(local, np.ndarray):
         local = torch.from_numpy(local.view(np.uint8).reshape(-1, 32).copy()).to(dev)
     everything = comm.all_gather_var(local)           # [n, 32] bytes, rank order
@@ -230,7 +232,7 @@ class LoopbackComm:
     ranks at once (single-GPU tests of the sharded path)."""
 
     @staticmethod
-    def run(stages, timing: bool = False) -> np.ndarray:
+    def run(stages, timing: bool = False, paper_counters: bool = False) -> np.ndarray:
         P = len(stages)
         preps = [s.prepare(P) for s in stages]
         bad = min((p["bad"] for p in preps), default=NONE64)
@@ -244,5 +246,5 @@ class LoopbackComm:
         # all exchanges first: a stage's detect releases its send buffer
         recvs = [torch.cat([p["records"][int(o[d]):int(o[d + 1])] for p, o in zip(preps, offs)])
                  for d in range(P)]
-        parts = [s.detect(recv, sidx, sev, lo, timing) for s, recv in zip(stages, recvs)]
+        parts = [s.detect(recv, sidx, sev, lo, timing, paper_counters) for s, recv in zip(stages, recvs)]
         return merge_reports(parts)

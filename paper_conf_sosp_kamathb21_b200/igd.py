@@ -20,6 +20,7 @@ IGD_OK, IGD_EINVAL, IGD_ETRACE, IGD_ETOOBIG, IGD_ENOMEM, IGD_ECUDA, IGD_ENCCL, I
 IGD_TRACE_DEVICE_PTR = 1
 IGD_DETECT_TIMING = 1
 IGD_DETECT_COALESCE = 2
+IGD_DETECT_PAPER_COUNTERS = 4
 IGD_N_STAGES = 8
 IGD_N_KCLASS = 9
 
@@ -195,9 +196,11 @@ class Detector:
             self._borrowed = None
             igd_trace_load(self.ctx, n_blocks, block_dim, ev.ctypes.data if len(ev) else 0, len(ev), False)
 
-    def detect(self, timing: bool = False, coalesce: bool = False) -> int:
-        """igd_detect; ``coalesce``: warp-coalesced check mode (IGD_DETECT_COALESCE)."""
-        flags = (IGD_DETECT_TIMING if timing else 0) | (IGD_DETECT_COALESCE if coalesce else 0)
+    def detect(self, timing: bool = False, coalesce: bool = False, paper_counters: bool = False) -> int:
+        """igd_detect; ``coalesce``: warp-coalesced check mode (IGD_DETECT_COALESCE, reading A32);
+        ``paper_counters``: Fig. 4-width synchronization IDs (IGD_DETECT_PAPER_COUNTERS, A33)."""
+        flags = ((IGD_DETECT_TIMING if timing else 0) | (IGD_DETECT_COALESCE if coalesce else 0)
+                 | (IGD_DETECT_PAPER_COUNTERS if paper_counters else 0))
         self.n_reports = igd_detect(self.ctx, flags)
         return self.n_reports
 

@@ -40,7 +40,7 @@ class CpuStage:
                 "sync_ev": torch.from_numpy(np.ascontiguousarray(sev)), "bad": NONE64, "min_word": wmin,
                 "max_word": wmax}
 
-    def detect(self, recv, sync_idx, sync_ev, min_word, timing=False):
+    def detect(self, recv, sync_idx, sync_ev, min_word, timing=False, paper_counters=False):
         me = getattr(self, "rank", None)
         recv = recv.numpy()
         sidx = sync_idx.numpy().astype(np.uint32).astype(np.int64)
@@ -57,7 +57,7 @@ class CpuStage:
         allev = np.concatenate([sev, racc])
         uniq, first = np.unique(allidx, return_index=True)
         trace = allev[first]
-        rep = oracle.run(trace, self.nb, self.bd)
+        rep = oracle.run(trace, self.nb, self.bd, paper_counters=paper_counters)
         mine = owner_of(rep["addr"] >> np.uint64(2), self.P) == self.rank
         rep = rep[mine].copy()
         rep["cur"] = uniq[rep["cur"].astype(np.int64)]

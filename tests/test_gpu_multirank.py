@@ -12,7 +12,7 @@ from test_gpu_parity import _fast_random
 pytestmark = pytest.mark.gpu
 
 
-def sharded(ev, nb, bd, P):
+def sharded_stages_run(ev, nb, bd, P, **kw):
     import paper_conf_sosp_kamathb21_b200 as igd
     from paper_conf_sosp_kamathb21_b200 import dist as D
 
@@ -23,10 +23,14 @@ def sharded(ev, nb, bd, P):
         s.load(ev[lo:lo + cnt], lo, len(ev), nb, bd)
         stages.append(s)
     try:
-        return D.LoopbackComm.run(stages)
+        return D.LoopbackComm.run(stages, **kw)
     finally:
         for s in stages:
             s.det.close()
+
+
+def sharded(ev, nb, bd, P):
+    return sharded_stages_run(ev, nb, bd, P)
 
 
 @pytest.mark.parametrize("P", [1, 2, 3, 8])

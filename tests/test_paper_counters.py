@@ -160,3 +160,14 @@ def test_gpu_families(det):
     for fam, n in ((2, 2_000_000), (3, 2_000_000), (4, 3_000_000)):
         ev, nb, bd, _ = F.generate(fam, n)
         _same(det, ev, nb, bd, f"C{fam}")
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("P", [2, 4])
+def test_gpu_sharded(P):
+    from test_gpu_multirank import sharded_stages_run
+
+    for seed in range(30):
+        ev, nb, bd = _burst_trace(seed, 40, threads=[0, 1, 33, 64] if seed % 2 else None)
+        got = sharded_stages_run(ev, nb, bd, P, paper_counters=True)
+        assert np.array_equal(got, oracle.run(ev, nb, bd, paper_counters=True)), f"seed {seed} P {P}"
