@@ -45,7 +45,12 @@ namespace check {
 #endif
 constexpr int C4_ITEMS = IGD_C4_ITEMS;
 constexpr int C4_WT = 32 * C4_ITEMS;         // accesses per warp
-constexpr int C4_TILE = THREADS * C4_ITEMS;  // accesses per CTA
+#ifndef IGD_C4_THREADS
+#define IGD_C4_THREADS 256
+#endif
+constexpr int C4_THREADS = IGD_C4_THREADS;
+constexpr int C4_WARPS = C4_THREADS / 32;
+constexpr int C4_TILE = C4_THREADS * C4_ITEMS;  // accesses per CTA
 
 __device__ __forceinline__ int hib(u32 m) { return 31 - (int)__clz(m); }  // m != 0
 
@@ -153,11 +158,11 @@ __device__ __noinline__ bool q_grid_from(const PP& P, u32 a, u32 b, u32 x) {
 // KB: the trace has kernel boundaries (a separate instantiation: the boundary test costs
 // registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
 template <bool MV, bool KB, bool WRAP>
-__global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
+__global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
     __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
     __shared__ uint8_t q_f[C4_TILE];              // queue flags
-    __shared__ u64 s_wagg[WARPS];
+    __shared__ u64 s_wagg[C4_WARPS];
     __shared__ u64 s_prefix;
     __shared__ u32 s_ready;
 
@@ -275,7 +280,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
         // associative; identity on the left is neutral)
         u64 tagg = s_wagg[0];
 #pragma unroll
-        for (int w = 1; w < WARPS; w++) tagg = combine(tagg, s_wagg[w]);
+        for (int w = 1; w < C4_WARPS; w++) tagg = combine(tagg, s_wagg[w]);
         u64 prefix = ST_IDENTITY;
         if (lane == 0) st_relaxed(&P.status[tile], ((tile == 0 || st_head(tagg)) ? ST_INC : ST_AGG) | tagg);
         if (tile > 0 && !(hm[0] & 1u) && P.debug_stop != 3) {  // a tile starting with a head needs no prefix
@@ -313,7 +318,7 @@ __global__ void __launch_bounds__(THREADS, IGD_C4_MINB) k_check4(Params P) {
     if (t == 0) {
         u64 tagg = s_wagg[0];
 #pragma unroll
-        for (int w = 1; w < WARPS; w++) tagg = combine(tagg, s_wagg[w]);
+        for (int w = 1; w < C4_WARPS; w++) tagg = combine(tagg, s_wagg[w]);
         u64 prefix = ST_IDENTITY;
         st_relaxed(&P.status[tile], ((tile == 0 || st_head(tagg)) ? ST_INC : ST_AGG) | tagg);
         if (tile > 0 && !(hm[0] & 1u) && P.debug_stop != 3) {  // a tile starting with a head needs no prefix

@@ -248,8 +248,8 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
 // a6 kernel instantiation: sharded payload (MV), kernel boundaries (KB), paper-width IDs (WRAP)
 template <bool MV, bool KB>
 static void launch_check_w(bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
-    if (wrap) check::k_check4<MV, KB, true><<<tb, check::THREADS, 0, st>>>(cp);
-    else check::k_check4<MV, KB, false><<<tb, check::THREADS, 0, st>>>(cp);
+    if (wrap) check::k_check4<MV, KB, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
+    else check::k_check4<MV, KB, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
 }
 static void launch_check(bool mv, bool kb, bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
     if (mv && kb) launch_check_w<true, true>(wrap, tb, st, cp);
