@@ -440,6 +440,11 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         shard::k_split_records<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
                                                           P_<u32>(ctx->acc_k[0]), P_<uint4>(ctx->acc_v[0]));
     }
+    if (FUSED && IGD_HIST_UP_LATE && n_acc > 0) {
+        KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digits 1..3
+        const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
+        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[1]), (u32)n_acc, P_<u32>(ctx->hist), 1);
+    }
     if (FUSED && n_sync > 0) {
         // sync-key digit histograms over the records the fused pass wrote (trace order)
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_sync);

@@ -21,6 +21,9 @@ constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
 constexpr int ITEMS = 8;
 constexpr int TILE = THREADS * ITEMS;
+#ifndef IGD_HIST_UP_LATE
+#define IGD_HIST_UP_LATE 0  // 1: access-key digits 1..3 histogrammed after the fused pass (k_hist_keys; measured +0.8 ms per 1e9 events)
+#endif
 
 struct Params {
     const igd_event* ev;
@@ -219,7 +222,7 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
                     if (acc) atomicAdd(&s_hacc[warp & 3u][dv[j].key & 255u], 1u);
                     // digits 1..3: one set of atomics per warp when the lanes agree on the upper
                     // 24 bits (lanes of one instruction touch neighbouring words), else per lane
-                    const u32 am = __ballot_sync(IGD_FULL, acc);
+                    const u32 am = IGD_HIST_UP_LATE ? 0u : __ballot_sync(IGD_FULL, acc);
                     if (am) {
                         const u32 hi = dv[j].key >> 8;
                         const u32 src = __ffs(am) - 1;
