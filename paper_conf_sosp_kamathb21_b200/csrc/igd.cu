@@ -191,10 +191,39 @@ static void mark(igd_ctx* ctx, int stage) {
 }
 
 template <typename VT>
-static void launch_pass(int mode, unsigned gb, size_t smem, cudaStream_t st, const rsort::PassParams& pp) {
-    if (mode == 0) rsort::k_onesweep<0, VT><<<gb, rsort::THREADS, smem, st>>>(pp);
-    else if (mode == 2) rsort::k_onesweep<2, VT><<<gb, rsort::THREADS, smem, st>>>(pp);
-    else rsort::k_onesweep<1, VT><<<gb, rsort::THREADS, smem, st>>>(pp);
+static void launch_mode(int mode, bool tail, unsigned gb, size_t smem, cudaStream_t st, const rsort::PassParams& pp) {
+    if (tail) {
+        if (mode == 0) rsort::k_onesweep<0, VT, true><<<gb, rsort::THREADS, smem, st>>>(pp);
+        else if (mode == 2) rsort::k_onesweep<2, VT, true><<<gb, rsort::THREADS, smem, st>>>(pp);
+        else rsort::k_onesweep<1, VT, true><<<gb, rsort::THREADS, smem, st>>>(pp);
+    } else {
+        if (mode == 0) rsort::k_onesweep<0, VT, false><<<gb, rsort::THREADS, smem, st>>>(pp);
+        else if (mode == 2) rsort::k_onesweep<2, VT, false><<<gb, rsort::THREADS, smem, st>>>(pp);
+        else rsort::k_onesweep<1, VT, false><<<gb, rsort::THREADS, smem, st>>>(pp);
+    }
+}
+// One radix pass over n keys: the full tiles, then (if any) the partial last tile.
+template <typename VT>
+static void launch_pass(int mode, u64 n, size_t smem, cudaStream_t st, rsort::PassParams pp) {
+    const u64 full = n / rsort::TILE;
+    if (full) {
+        pp.tile0 = 0;
+        launch_mode<VT>(mode, false, (unsigned)full, smem, st, pp);
+    }
+    if (n % rsort::TILE) {
+        pp.tile0 = (u32)full;
+        launch_mode<VT>(mode, true, 1u, smem, st, pp);
+    }
+}
+template <typename VT>
+static void set_pass_smem() {
+    const int b = (int)rsort::onesweep_smem<VT>();
+    cudaFuncSetAttribute(rsort::k_onesweep<0, VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<1, VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<2, VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<0, VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<1, VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<2, VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
 }
 
 // Stable LSD radix sort of n (key, value) pairs in buffers k[cur], v[cur]; h_hist is the host
@@ -232,12 +261,11 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         pp.tile_ctr = P_<u32>(ctx->ctr);
         {
             KTimer kt(ctx, cls, 2.0 * (4 + vbytes) * (double)n);  // read + write 4 B key and the value
-            const unsigned gb = (unsigned)tiles;
-            const size_t s8 = rsort::onesweep_smem<u64>(), s4 = rsort::onesweep_smem<u32>();
-            if (vbytes == 16) launch_pass<uint4>(ctx->sort_mode, gb, rsort::onesweep_smem<uint4>(), ctx->stream, pp);
-            else if (vbytes == 8) launch_pass<u64>(ctx->sort_mode, gb, s8, ctx->stream, pp);
-            else launch_pass<u32>(ctx->sort_mode, gb, s4, ctx->stream, pp);
+            if (vbytes == 16) launch_pass<uint4>(ctx->sort_mode, n, rsort::onesweep_smem<uint4>(), ctx->stream, pp);
+            else if (vbytes == 8) launch_pass<u64>(ctx->sort_mode, n, rsort::onesweep_smem<u64>(), ctx->stream, pp);
+            else launch_pass<u32>(ctx->sort_mode, n, rsort::onesweep_smem<u32>(), ctx->stream, pp);
         }
+        if (n > rsort::TILE && n % rsort::TILE) ctx->launches++;  // the partial-tile launch
         CK(cudaGetLastError());
         cur ^= 1;
     }
@@ -752,24 +780,9 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     cudaFuncSetAttribute(ingest::k_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ingest::count_smem());
     cudaFuncSetAttribute(fused::k_ingest_sort0, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes());
-    cudaFuncSetAttribute(rsort::k_onesweep<0, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<u64>());
-    cudaFuncSetAttribute(rsort::k_onesweep<1, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<u64>());
-    cudaFuncSetAttribute(rsort::k_onesweep<0, uint4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<uint4>());
-    cudaFuncSetAttribute(rsort::k_onesweep<1, uint4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<uint4>());
-    cudaFuncSetAttribute(rsort::k_onesweep<0, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<u32>());
-    cudaFuncSetAttribute(rsort::k_onesweep<2, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<u32>());
-    cudaFuncSetAttribute(rsort::k_onesweep<2, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<u64>());
-    cudaFuncSetAttribute(rsort::k_onesweep<2, uint4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<uint4>());
-    cudaFuncSetAttribute(rsort::k_onesweep<1, u32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)rsort::onesweep_smem<u32>());
+    set_pass_smem<u32>();
+    set_pass_smem<u64>();
+    set_pass_smem<uint4>();
     if (cudaMallocHost(&ctx->h_stats, 8 * sizeof(u64)) != cudaSuccess ||
         cudaMallocHost(&ctx->h_hist, 3 * 1024 * sizeof(u32)) != cudaSuccess ||
         cudaMallocHost(&ctx->h_small, 8 * sizeof(u64)) != cudaSuccess) {

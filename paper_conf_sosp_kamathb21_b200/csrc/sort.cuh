@@ -84,6 +84,7 @@ struct PassParams {
     const u32* digit_base;  // [256] exclusive global offsets of this pass's digits
     u64* status;            // [n_tiles * 256], zeroed
     u32* tile_ctr;          // zeroed
+    u32 tile0;              // tile index of blockIdx.x 0 (the TAIL launch holds the last, partial tile)
 };
 
 // Mask of the lanes (within vmask) whose 8-bit digit equals this lane's.
@@ -122,7 +123,9 @@ constexpr size_t onesweep_smem() {
     return (size_t)TILE * sizeof(u32) + (size_t)TILE * sizeof(VT) + TILE;
 }
 
-template <int MODE, typename VT>
+// TAIL = false: every tile of the launch is full (no bounds tests on the hot path); TAIL = true:
+// the one partial last tile, launched after the full ones (its look-back finds them published).
+template <int MODE, typename VT, bool TAIL>
 #ifndef IGD_SORT_MINB
 #define IGD_SORT_MINB 3
 #endif
@@ -146,10 +149,10 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     if (t == 0) {
         // tile id, then TMA bulk copies of the tile's keys and values into shared memory: the
         // value copy lands while the keys are ranked
-        const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
+        const u32 tile = P.tile0 + blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
         s_tile = tile;
         const u64 base = (u64)tile * TILE;
-        if (base + TILE <= P.n) {
+        if (!TAIL) {
             mbar_init(&s_mbar[0], 1);
             mbar_init(&s_mbar[1], 1);
             mbar_expect_tx(&s_mbar[0], TILE * sizeof(u32));
@@ -168,7 +171,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     const u32 wofs = warp * 32 * ITEMS;
     const u32 wbase = base + wofs;
     const u32 shift = P.shift;
-    const bool full = (u64)base + TILE <= P.n;
+    constexpr bool full = !TAIL;
 
     u32 key[ITEMS];
     if (full) {
