@@ -112,7 +112,7 @@ __device__ __noinline__ bool q_between(const uint4* __restrict__ desc, const u32
 
 struct Params {
     const u32* key;  // sorted word keys
-    const void* val; // sorted payload: u64 (index | tk << 32), or uint4 {index, tk, mask, 0} (MV)
+    const void* val; // sorted payload: u64 (index | tk << 32), or uint4 {key, index, tk, mask} (MV)
     u64 wbase;       // smallest accessed word (reports rebuild the 64-bit word from the key)
     u32 n;           // number of accesses
     const igd_event* ev;
@@ -171,7 +171,7 @@ __device__ __forceinline__ bool q_grid(const PP& P, u32 a, u32 b) {
 #define QF_R1 16u
 
 // Sorted payload of one access: single GPU = u64 (trace index | tk << 32), the active mask is
-// gathered from the trace when needed; sharded = uint4 {index, tk, mask, 0} (the events of
+// gathered from the trace when needed; sharded = the record uint4 {key, index, tk, mask} (the events of
 // other ranks are not resident).
 struct Acc {
     u32 idx, tk, mask;
@@ -179,11 +179,11 @@ struct Acc {
 template <bool MV>
 __device__ __forceinline__ Acc acc_at(const void* val, u32 k) {
     Acc a;
-    if (MV) {
+    if (MV) {  // the received record {key, idx, tk, mask}
         const uint4 v = __ldg(reinterpret_cast<const uint4*>(val) + k);
-        a.idx = v.x;
-        a.tk = v.y;
-        a.mask = v.z;
+        a.idx = v.y;
+        a.tk = v.z;
+        a.mask = v.w;
     } else {
         const unsigned long long v = __ldg(reinterpret_cast<const unsigned long long*>(val) + k);
         a.idx = (u32)v;

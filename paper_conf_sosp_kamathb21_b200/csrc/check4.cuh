@@ -181,11 +181,11 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         const u32 x = wbase + j * 32 + lane;
         const bool in = x < n;
         K[j] = in ? __ldcs(P.key + x) : 0u;
-        if (MV) {
+        if (MV) {  // the received record {key, idx, tk, mask}
             const uint4 v = in ? __ldcs(reinterpret_cast<const uint4*>(P.val) + x) : make_uint4(0, 0, 0, 0);
-            V[j] = v.x;
-            Z[j] = v.y;
-            M[j] = v.z;
+            V[j] = v.y;
+            Z[j] = v.z;
+            M[j] = v.w;
         } else {
             const unsigned long long v = in ? __ldcs(reinterpret_cast<const unsigned long long*>(P.val) + x) : 0ull;
             V[j] = (u32)v;

@@ -229,11 +229,18 @@ static void set_pass_smem() {
 // Stable LSD radix sort of n (key, value) pairs in buffers k[cur], v[cur]; h_hist is the host
 // copy of the 4x256 digit histogram (device copy d_hist).  Digits above max_bits and digits
 // with one occupied bin are skipped.  Returns the buffer index holding the result.
+// vin_first: values of the input (instead of v[first_cur]) for the first pass that runs -- the
+// sharded path sorts the received records in place of a split copy.
 static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d_hist, const u32* h_hist,
-                      u32 max_bits, int* out_cur, int vbytes = 4, u32 first_pass = 0, int first_cur = 0) {
+                      u32 max_bits, int* out_cur, int vbytes = 4, u32 first_pass = 0, int first_cur = 0,
+                      const void* vin_first = nullptr) {
     int cur = first_cur;
     *out_cur = cur;
-    if (n <= 1) return IGD_OK;
+    bool ran = false;
+    if (n <= 1) {
+        if (n == 1 && vin_first) CK(cudaMemcpyAsync(v[cur].p, vin_first, vbytes, cudaMemcpyDeviceToDevice, ctx->stream));
+        return IGD_OK;
+    }
     if (n > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;  // 32-bit tile indexing
     {
         KTimer kt(ctx, KC_MISC, 0);
@@ -251,7 +258,8 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
         rsort::PassParams pp;
         pp.kin = P_<u32>(k[cur]);
-        pp.vin = v[cur].p;
+        pp.vin = (!ran && vin_first) ? vin_first : v[cur].p;
+        ran = true;
         pp.kout = P_<u32>(k[cur ^ 1]);
         pp.vout = v[cur ^ 1].p;
         pp.n = (u32)n;
@@ -269,6 +277,8 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         CK(cudaGetLastError());
         cur ^= 1;
     }
+    if (!ran && vin_first)  // every digit trivial: the values still have to land in v[cur]
+        CK(cudaMemcpyAsync(v[cur].p, vin_first, n * vbytes, cudaMemcpyDeviceToDevice, ctx->stream));
     *out_cur = cur;
     return IGD_OK;
 }
@@ -462,11 +472,12 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     }
     CK(cudaGetLastError());
     if (SH && n_acc > 0) {
-        // received records {key, index, tk, mask} -> sort keys + 16-byte payload
-        KTimer kt(ctx, KC_INGEST, 36.0 * (double)n_acc);
-        const unsigned sb = (unsigned)std::min<u64>((n_acc + 255) / 256, (u64)sms * 16);
-        shard::k_split_records<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
-                                                          P_<u32>(ctx->acc_k[0]), P_<uint4>(ctx->acc_v[0]));
+        // received records {key, index, tk, mask}: the sort keys and their digit histograms; the
+        // records themselves are the payload of the first radix pass
+        KTimer kt(ctx, KC_INGEST, 20.0 * (double)n_acc);
+        const unsigned sb = (unsigned)std::min<u64>((n_acc + 255) / 256, (u64)sms * 8);
+        shard::k_record_keys<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
+                                                         P_<u32>(ctx->acc_k[0]), P_<u32>(ctx->hist));
     }
     if (FUSED && IGD_HIST_UP_LATE && n_acc > 0) {
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digits 1..3
@@ -480,7 +491,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->syn_k[0]), (u32)n_sync,
                                                          P_<u32>(ctx->hist) + 1024, 0);
     }
-    if (n_acc > 0 && !FUSED) {  // fused: ingest pass 0 built them
+    if (n_acc > 0 && !FUSED && !SH) {  // fused: ingest pass 0 built them; sharded: k_record_keys
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digit histograms
         const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
         ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[0]), (u32)n_acc, P_<u32>(ctx->hist), 0);
@@ -573,7 +584,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     // ---------------- a5: accesses sorted by word, stable ----------------
     int acur = 0;
     RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur,
-                   vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0));
+                   vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0, SH ? ctx->sh_rec : nullptr));
     ctx->last_acur = acur;
     ctx->last_nacc = SH ? 0 : n_acc;
     mark(ctx, 4);

@@ -161,12 +161,26 @@ __global__ void __launch_bounds__(THREADS, IGD_SHARD_MINB) k_shard(Params P) {
     }
 }
 
-// Received records (uint4 {key, idx, tk, mask}) -> sort keys + 16-byte payload.
-__global__ void k_split_records(const uint4* __restrict__ rec, u32 n, u32* __restrict__ keys, uint4* __restrict__ vals) {
+// Received records (uint4 {key, idx, tk, mask}) -> the sort keys and their 4 x 8-bit digit
+// histograms.  The records themselves are the sort payload (the check reads idx, tk, mask from
+// .y .z .w), so no split copy of them is written.
+__global__ void __launch_bounds__(256) k_record_keys(const uint4* __restrict__ rec, u32 n, u32* __restrict__ keys,
+                                                     u32* __restrict__ hist) {
+    __shared__ u32 s[4][256];
+    for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&s[0][0])[i] = 0;
+    __syncthreads();
     for (u32 i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-        const uint4 r = __ldcs(rec + i);
-        keys[i] = r.x;
-        vals[i] = make_uint4(r.y, r.z, r.w, 0u);
+        const u32 k = __ldcs(rec + i).x;
+        keys[i] = k;
+        atomicAdd(&s[0][k & 255u], 1u);
+        atomicAdd(&s[1][(k >> 8) & 255u], 1u);
+        atomicAdd(&s[2][(k >> 16) & 255u], 1u);
+        atomicAdd(&s[3][k >> 24], 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) {
+        const u32 v = (&s[0][0])[i];
+        if (v) atomicAdd(&hist[i], v);
     }
 }
 
