@@ -234,7 +234,8 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             const u32 pt = pZ & 0xFFFFFFu;
             const u32 bp = g.block(pt), bc = g.block(c);
             dev = bp != bc;
-            blk = !dev && g.warp(pt) != g.warp(c);
+            // same block: different warps iff the in-block offsets differ in their warp index
+            blk = !dev && ((pt - bp * g.D) >> 5) != ((c - bc * g.D) >> 5);
             same_t = pt == c;
         }
         const bool isA = in && kind >= IGD_ATOM && kind <= IGD_EXCH;
@@ -425,8 +426,9 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 } else {
                     p = tk_at(mdp) & 0xFFFFFFu;
                     same_t = p == c;
-                    same_b = g.block(p) == g.block(c);
-                    same_w = same_b && g.warp(p) == g.warp(c);
+                    const u32 bp = g.block(p), bc = g.block(c);
+                    same_b = bp == bc;
+                    same_w = same_b && ((p - bp * g.D) >> 5) == ((c - bc * g.D) >> 5);
                 }
                 if (same_t) {  // P3: program order
                     CSTAT(2);
