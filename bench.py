@@ -254,8 +254,8 @@ def run_sharded(args, fam, rank, world, local):
 
 
 # kernel class -> the kernel ncu names for it (classes made of one kernel)
-CLASS_KERNEL = {"sort_access": "rsort::k_onesweep<1, unsigned long>", "check": "check::k_check<0>",
-                "ingest_sort0": "fused::k_ingest_sort0"}
+CLASS_KERNEL = {"sort_access": "rsort::k_onesweep<1, unsigned long, 0>", "check": "check::k_check4<0, 0, 0>",
+                "ingest_sort0": "fused::k_ingest_sort0", "ingest": "ingest::k_ingest<0>"}
 TRAFFIC_JSON = os.path.join(ROOT, "profiles", "traffic_r01.json")
 
 
