@@ -119,7 +119,7 @@ struct Params {
     Geo g;
     KeySpace ks;
     const uint4* desc;  // per-entity list descriptors
-    const u32* gtab;    // grid-sync bucket table: first grid-list index at or after bucket start
+    const u64* gtab;    // grid-sync bucket table: {first grid-list index at or after the bucket start, its timestamp}
     u32 gshift;         // bucket = t >> gshift
     u32 glo, ghi;       // the grid list inside sts
     u32 has_kb;         // the trace has kernel boundaries (reading A31)
@@ -134,10 +134,11 @@ struct Params {
     int debug_stop;  // profiling only (IGD_CHECK_STOP): 1 = stop after the scans, 2 = after phase 1
 };
 
-// Grid-sync bucket table: gtab[b] = index of the first grid sync with timestamp >= b << shift.
-// The grid list is global and short, so "a grid sync in (a, b)?" -- the most frequent query of
-// P5 / R2..R4 -- becomes one L2-resident table load plus a step or two along the list.
-__global__ void k_grid_table(const u32* __restrict__ ts, u32 glo, u32 ghi, u32 shift, u32 nb, u32* __restrict__ gtab) {
+// Grid-sync bucket table: gtab[b] = {index, timestamp} of the first grid sync with timestamp >=
+// b << shift (timestamp NONE past the last).  The grid list is global and short, so "a grid sync
+// in (a, b)?" -- the most frequent query of P5 / R2..R4 -- is one L2-resident 8-byte load in the
+// common case (no grid sync between the bucket start and a), else a step or two along the list.
+__global__ void k_grid_table(const u32* __restrict__ ts, u32 glo, u32 ghi, u32 shift, u32 nb, u64* __restrict__ gtab) {
     for (u64 b = (u64)blockIdx.x * blockDim.x + threadIdx.x; b < nb; b += (u64)gridDim.x * blockDim.x) {
         const u64 start = b << shift;
         u32 lo = glo, hi = ghi;
@@ -146,14 +147,19 @@ __global__ void k_grid_table(const u32* __restrict__ ts, u32 glo, u32 ghi, u32 s
             if ((u64)ts[mid] < start) lo = mid + 1;
             else hi = mid;
         }
-        gtab[b] = lo;
+        gtab[b] = (u64)lo | ((u64)(lo < ghi ? ts[lo] : IGD_NONE32) << 32);
     }
 }
 
 template <class PP>
 __device__ __forceinline__ bool q_grid(const PP& P, u32 a, u32 b) {
     if (P.glo == P.ghi) return false;
-    u32 x = __ldg(P.gtab + ((a + 1) >> P.gshift));  // first grid sync at or after a's bucket
+    const u64 e = __ldg(P.gtab + ((a + 1) >> P.gshift));  // first grid sync at or after a's bucket
+    u32 x = (u32)e;
+    const u32 v0 = (u32)(e >> 32);
+    if (x >= P.ghi) return false;
+    if (v0 > a) return v0 < b;
+    x++;
 #pragma unroll 1
     for (int step = 0; x < P.ghi; step++, x++) {
         const u32 v = __ldg(P.sts + x);

@@ -513,7 +513,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         const uint4 dB = same_b ? __ldg(P.desc + ks.bb + g.block(c)) : none4;
         const uint4 dF = __ldg(P.desc + (same_b ? ks.any : ks.dev) + p);
         const bool hasG = P.glo != P.ghi;
-        const u32 gx = hasG ? __ldg(P.gtab + ((mdIdx + 1) >> P.gshift)) : 0u;
+        const u32 gx = hasG ? (u32)__ldg(P.gtab + ((mdIdx + 1) >> P.gshift)) : 0u;
         const u32 emask = (flags & QF_MASK) ? ld_event(P.ev, i).w : 0u;
         if ((flags & QF_MASK) && ((emask >> g.lane(p)) & 1u)) continue;  // P4: lockstep
         BQ qW, qB, qF;

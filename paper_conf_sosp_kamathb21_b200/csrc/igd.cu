@@ -534,12 +534,12 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     CK(cudaStreamSynchronize(ctx->stream));
     const u32 gshift = std::max<u32>(8, bits_needed(n) > 22 ? bits_needed(n) - 22 : 0);
     const u32 gnb = (u32)((n >> gshift) + 2);
-    RET(ensure(ctx, ctx->gtab, (u64)gnb * sizeof(u32)));
+    RET(ensure(ctx, ctx->gtab, (u64)gnb * sizeof(u64)));
     if (glims[1] > glims[0]) {
         unsigned blocks = (unsigned)std::min<u64>((gnb + 255) / 256, (u64)sms * 16);
-        KTimer kt(ctx, KC_CSR, 4.0 * (double)gnb);
+        KTimer kt(ctx, KC_CSR, 8.0 * (double)gnb);
         check::k_grid_table<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->syn_v[scur]), glims[0], glims[1], gshift,
-                                                            gnb, P_<u32>(ctx->gtab));
+                                                            gnb, P_<u64>(ctx->gtab));
         CK(cudaGetLastError());
     }
     // ---------------- a3: lock inference ----------------
@@ -611,7 +611,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.g = g;
             cp.ks = ks;
             cp.desc = P_<uint4>(ctx->ldesc);
-            cp.gtab = P_<u32>(ctx->gtab);
+            cp.gtab = P_<u64>(ctx->gtab);
             cp.gshift = gshift;
             cp.glo = glims[0];
             cp.ghi = glims[1];
