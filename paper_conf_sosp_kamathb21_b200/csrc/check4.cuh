@@ -486,10 +486,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     if (P.debug_stop == 2) return;
 
     // ---- phase 2: the warp's queued accesses, densely over its lanes ----
-    // Every list query an entry may need is issued at once: round 1 loads the descriptors of
-    // md's warp / block / thread lists, the grid bucket and (deferred P4 lockstep) the event's
-    // active mask; round 2 the 32-byte timestamp probes.  Two dependent L2 round trips per entry
-    // instead of a chain of up to eight.
+    // One entry per lane, its list queries in Table 2's order with early exits.  Issuing all of an
+    // entry's queries at once (IGD_C4_STAGED) and interleaving two entries per lane were both
+    // measured slower (20.9 and 22.2 vs 14.8 ms at C5@1e9): this phase is bound by the queries'
+    // total L2 / issue work, not by the latency of one chain.
     const KeySpace ks = P.ks;
     for (u32 k = lane; k < qn; k += 32) {
         const u32 x = q_x[qb + k], mdp = q_md[qb + k], flags = q_f[qb + k];
@@ -507,6 +507,8 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         const u32 p = mdz & 0xFFFFFFu;
         const bool same_w = flags & QF_SAME_W, same_b = flags & QF_SAME_B;
 #if IGD_C4_STAGED
+        // all queries of the entry at once: round 1 descriptors + grid bucket + active mask,
+        // round 2 the 32-byte timestamp probes
         // round 1
         const uint4 none4 = make_uint4(0, 0, 0, 0);
         const uint4 dW = same_w ? __ldg(P.desc + ks.wb + g.warp(c)) : none4;
