@@ -191,6 +191,49 @@ def test_c2_full_size_vs_oracle(det):
            [(r["addr"], r["cur"], r["prev"], r["type"]) for r in led]
 
 
+def _shard_of(words, K):
+    h = (words ^ (words >> np.uint64(32))).astype(np.uint64) & np.uint64(0xFFFFFFFF)
+    h ^= h >> np.uint64(16)
+    h = (h * np.uint64(0x85EBCA6B)) & np.uint64(0xFFFFFFFF)
+    h ^= h >> np.uint64(13)
+    h = (h * np.uint64(0xC2B2AE35)) & np.uint64(0xFFFFFFFF)
+    return (h ^ (h >> np.uint64(16))) % np.uint64(K)
+
+
+def test_c4_full_size_sampled_words_vs_oracle(det):
+    # configs[3] at its full size (5*10^8 events): the oracle replays every event but checks a 1/64
+    # address shard; the GPU reports restricted to those words must be identical, and the whole GPU
+    # report set must equal the generator's injection ledger
+    import tracegen.families as F
+
+    ev, nb, bd, led = F.generate(4)
+    det.load(ev, nb, bd)
+    det.detect()
+    got = det.reports()
+    want = oracle.run(ev, nb, bd, shard=(5, 64))
+    mine = _shard_of(got["addr"] >> np.uint64(2), 64) == 5
+    assert len(want) > 0 and np.array_equal(got[mine], want)
+    assert [(r["addr"], r["cur"], r["prev"], r["type"]) for r in got] == \
+           [(r["addr"], r["cur"], r["prev"], r["type"]) for r in led]
+
+
+def test_c5_prefix_sampled_words_vs_oracle(det):
+    # configs[4]'s workload (the 4*10^9-event mix over 2^30 words): its first 4*10^8 events are a
+    # valid trace (the check of access i depends only on events <= i); oracle on a 1/64 shard
+    import tracegen.families as F
+
+    plan = F.Plan(5)
+    ev = plan.fill(0, 400_000_000)
+    nb, bd = plan.n_blocks, plan.block_dim
+    plan.close()
+    det.load(ev, nb, bd)
+    det.detect()
+    got = det.reports()
+    want = oracle.run(ev, nb, bd, shard=(9, 64))
+    mine = _shard_of(got["addr"] >> np.uint64(2), 64) == 9
+    assert len(want) > 0 and np.array_equal(got[mine], want)
+
+
 def test_c3_full_size_sampled_words_vs_oracle(det):
     # configs[2] at full size (10^8 events): the oracle checks a 1/16 address shard (replaying every
     # synchronization event), the GPU result restricted to the same words must match exactly
