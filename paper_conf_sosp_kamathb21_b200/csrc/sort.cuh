@@ -31,6 +31,9 @@ constexpr int WARPS = THREADS / 32;
 #ifndef IGD_SORT_EARLY
 #define IGD_SORT_EARLY 1  // publish tile digit counts before ranking (C5@1e9: 21.6 -> 21.2 ms over 3 passes)
 #endif
+#ifndef IGD_SORT_MIX
+#define IGD_SORT_MIX 2  // every other row ranked with match.any: C5@1e9 sort 20.4 -> 19.8 ms
+#endif
 #ifndef IGD_SORT_LB
 #define IGD_SORT_LB 4
 #endif
@@ -210,7 +213,14 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             __syncwarp();
         } else {
             // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set
-            peers = peers_of<MODE>(valid ? d : (0x100u | lane), vmask);
+            // IGD_SORT_MIX: alternate rows between match.any (MIO pipe) and the 8 ballots (ALU /
+            // issue), which bottleneck on different units
+            // IGD_SORT_MIX = N: one row in N uses match.any; negative -N: all rows but one in N
+            if (IGD_SORT_MIX && MODE == 1 &&
+                (IGD_SORT_MIX > 0 ? (j % IGD_SORT_MIX) == IGD_SORT_MIX - 1 : (j % -IGD_SORT_MIX) != 0))
+                peers = peers_of<0>(valid ? d : (0x100u | lane), vmask);
+            else
+                peers = peers_of<MODE>(valid ? d : (0x100u | lane), vmask);
         }
         const u32 leader = __ffs(peers) - 1;
         u32 old = 0;
