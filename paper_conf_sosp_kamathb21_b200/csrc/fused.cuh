@@ -24,7 +24,7 @@ constexpr int ITEMS = 16;
 constexpr int TILE = THREADS * ITEMS;  // events per tile == 2 ingest pass-0 tiles
 constexpr int RADIX = 256;
 #ifndef IGD_FUSED_MIX
-#define IGD_FUSED_MIX 0  // 1: every other row ranked with match.any (measured slightly slower here)
+#define IGD_FUSED_MIX 4  // N: one row in N ranked with match.any (N = 2 measured slower, 4 neutral-to-better)
 #endif
 #ifndef IGD_FUSED_EARLY
 #define IGD_FUSED_EARLY 1
@@ -194,7 +194,8 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
         const bool valid = (amask >> j) & 1u;
         const u32 vmask = __ballot_sync(IGD_FULL, valid);
         const u32 d = key[j] & 255u;
-        const u32 peers = (IGD_FUSED_MIX && (j & 1)) ? rsort::peers_of<0>(valid ? d : (0x100u | lane), vmask)
+        const u32 peers = (IGD_FUSED_MIX && (j % IGD_FUSED_MIX) == IGD_FUSED_MIX - 1)
+                              ? rsort::peers_of<0>(valid ? d : (0x100u | lane), vmask)
                                                     : rsort::peers_of<1>(valid ? d : (0x100u | lane), vmask);
         const u32 leader = __ffs(peers) - 1;
         u32 old = 0;
