@@ -34,6 +34,9 @@ namespace check {
 #ifndef IGD_C4_NOGATHER
 #define IGD_C4_NOGATHER 0  // timing experiment only (wrong results): no active-mask gathers (C5@1e9: the gathers cost ~1.5 ms of ~15)
 #endif
+#ifndef IGD_C4_MBAR
+#define IGD_C4_MBAR 1  // warps wait for the tile prefix on an mbarrier (0: poll a shared flag)
+#endif
 #ifndef IGD_C4_WLB
 #define IGD_C4_WLB 0  // 1: warp-parallel look-back (measured slower: 14.9 -> 15.9 ms at C5@1e9; walks are short)
 #endif
@@ -165,6 +168,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     __shared__ u64 s_wagg[C4_WARPS];
     __shared__ u64 s_prefix;
     __shared__ u32 s_ready;
+    __shared__ __align__(8) u64 s_rbar;  // IGD_C4_MBAR: the tile prefix is ready (one arrival)
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
@@ -173,7 +177,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     const u32 wbase = tbase + wloc;
     const u32 n = P.n;
     const Geo g = P.g;
-    if (t == 0) s_ready = 0;
+    if (t == 0) {
+        s_ready = 0;
+        if (IGD_C4_MBAR) mbar_init(&s_rbar, 1);  // visible to every thread after the __syncthreads below
+    }
 
     u32 K[C4_ITEMS], V[C4_ITEMS], Z[C4_ITEMS], M[C4_ITEMS];
 #pragma unroll
@@ -346,6 +353,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         s_prefix = prefix;
         __threadfence_block();
         *(volatile u32*)&s_ready = 1u;
+        if (IGD_C4_MBAR) mbar_arrive(&s_rbar);  // release: s_prefix before the phase flips
     }
 
 #endif
@@ -355,7 +363,11 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         for (u32 w = 0; w < warp; w++) carry = combine(carry, s_wagg[w]);
         if (!st_head(carry) && tile > 0) {
             if (P.debug_stop == 3) return;  // profiling: no look-back
-            while (*(volatile u32*)&s_ready == 0u) __nanosleep(IGD_C4_SLEEP);
+            if (IGD_C4_MBAR && !IGD_C4_WLB) {
+                mbar_wait(&s_rbar, 0);  // suspended in hardware, not polling issue slots
+            } else {
+                while (*(volatile u32*)&s_ready == 0u) __nanosleep(IGD_C4_SLEEP);
+            }
             carry = combine(*(volatile u64*)&s_prefix, carry);
         }
     }

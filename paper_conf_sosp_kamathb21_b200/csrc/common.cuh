@@ -181,6 +181,9 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, 
         "l"(src), "r"(bytes), "r"(smem_u32(mbar))
         : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(u64* mbar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(mbar)) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(u64* mbar, u32 phase) {
     asm volatile(
         "{\n"
