@@ -20,8 +20,15 @@ namespace fused {
 
 constexpr int THREADS = 256;
 constexpr int WARPS = THREADS / 32;
-constexpr int ITEMS = 16;
-constexpr int TILE = THREADS * ITEMS;  // events per tile == 2 ingest pass-0 tiles
+#ifndef IGD_FUSED_ITEMS
+#define IGD_FUSED_ITEMS 16  // 8 items x 4-5 CTAs/SM measured slower (10.6 -> 10.9 ms at C5@1e9)
+#endif
+#ifndef IGD_FUSED_MINB
+#define IGD_FUSED_MINB 3
+#endif
+constexpr int ITEMS = IGD_FUSED_ITEMS;
+constexpr int TILE = THREADS * ITEMS;  // events per tile: a whole number of ingest pass-0 tiles
+constexpr int TPI = TILE / ingest::TILE;  // ingest pass-0 tiles per fused tile
 constexpr int RADIX = 256;
 #ifndef IGD_FUSED_MIX
 #define IGD_FUSED_MIX 4  // N: one row in N ranked with match.any (N = 2 measured slower, 4 neutral-to-better)
@@ -29,7 +36,7 @@ constexpr int RADIX = 256;
 #ifndef IGD_FUSED_EARLY
 #define IGD_FUSED_EARLY 1
 #endif
-static_assert(TILE == 2 * ingest::TILE, "sync-record bases come from ingest pass 0 tiles");
+static_assert(TILE % ingest::TILE == 0, "sync-record bases come from ingest pass 0 tiles");
 static_assert(THREADS == RADIX, "one look-back digit per thread");
 
 struct Params {
@@ -84,9 +91,13 @@ __device__ __forceinline__ FDec fdecode(const uint4& e, const Geo& g, const KeyS
     return d;
 }
 
-constexpr size_t smem_bytes() { return (size_t)TILE * sizeof(uint4); }  // 64 KB
+// the event tile (16 B per event), or the phase-2 buffers aliasing it if those are larger
+constexpr size_t smem_bytes() {
+    return (size_t)TILE * 16 > (size_t)TILE * 14 + WARPS * RADIX * 4 ? (size_t)TILE * 16
+                                                                     : (size_t)TILE * 14 + WARPS * RADIX * 4;
+}
 
-__global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
+__global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params P) {
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
     __shared__ u32 s_wsum[WARPS];
@@ -102,7 +113,6 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
     u64* s_v = reinterpret_cast<u64*>(s_dyn + TILE * 4);
     uint8_t* s_dig = s_dyn + TILE * 12;
     u32(*s_whist)[RADIX] = reinterpret_cast<u32(*)[RADIX]>(s_dyn + TILE * 14);
-    static_assert(TILE * 14 + WARPS * RADIX * 4 <= TILE * 16, "phase-2 buffers fit the event tile");
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
@@ -162,7 +172,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_ingest_sort0(Params P) {
 #pragma unroll
         for (int w = 0; w < WARPS; w++)
             if ((u32)w < warp) wpre += s_wsync[w];
-        u64 pos = (u64)P.tile_sync[2 * tile] + wpre;
+        u64 pos = (u64)P.tile_sync[TPI * tile] + wpre;
 #pragma unroll 1
         for (int j = 0; j < ITEMS; j++) {
             const u32 p = wofs + j * 32 + lane;
