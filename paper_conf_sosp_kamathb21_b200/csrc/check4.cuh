@@ -160,7 +160,7 @@ __device__ __noinline__ bool q_grid_from(const PP& P, u32 a, u32 b, u32 x) {
 
 // KB: the trace has kernel boundaries (a separate instantiation: the boundary test costs
 // registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
-template <bool MV, bool KB, bool WRAP>
+template <bool MV, bool KB, bool WRAP, bool GEO2>
 __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
     __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
@@ -177,6 +177,11 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     const u32 wbase = tbase + wloc;
     const u32 n = P.n;
     const Geo g = P.g;
+    // GEO2: block_dim is a power of two >= 32, so block / warp / lane are shifts and masks
+    const u32 dlog = g.dlog;
+    auto blk_of = [&](u32 t) -> u32 { return GEO2 ? t >> dlog : g.block(t); };
+    auto warp_of = [&](u32 t) -> u32 { return GEO2 ? t >> 5 : g.warp(t); };
+    auto lane_of = [&](u32 t) -> u32 { return GEO2 ? t & 31u : g.lane(t); };
     if (t == 0) {
         s_ready = 0;
         if (IGD_C4_MBAR) mbar_init(&s_rbar, 1);  // visible to every thread after the __syncthreads below
@@ -239,10 +244,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         bool dev = false, blk = false, same_t = false;
         if (!head) {
             const u32 pt = pZ & 0xFFFFFFu;
-            const u32 bp = g.block(pt), bc = g.block(c);
+            const u32 bp = blk_of(pt), bc = blk_of(c);
             dev = bp != bc;
             // same block: different warps iff the in-block offsets differ in their warp index
-            blk = !dev && ((pt - bp * g.D) >> 5) != ((c - bc * g.D) >> 5);
+            blk = !dev && (GEO2 ? (pt >> 5) != (c >> 5) : ((pt - bp * g.D) >> 5) != ((c - bc * g.D) >> 5));
             same_t = pt == c;
         }
         const bool isA = in && kind >= IGD_ATOM && kind <= IGD_EXCH;
@@ -438,9 +443,9 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 } else {
                     p = tk_at(mdp) & 0xFFFFFFu;
                     same_t = p == c;
-                    const u32 bp = g.block(p), bc = g.block(c);
+                    const u32 bp = blk_of(p), bc = blk_of(c);
                     same_b = bp == bc;
-                    same_w = same_b && ((p - bp * g.D) >> 5) == ((c - bc * g.D) >> 5);
+                    same_w = same_b && (GEO2 ? (p >> 5) == (c >> 5) : ((p - bp * g.D) >> 5) == ((c - bc * g.D) >> 5));
                 }
                 if (same_t) {  // P3: program order
                     CSTAT(2);
@@ -461,7 +466,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                         // prefetched unless md is an earlier writer (M[j] is the mask then only
                         // if the previous access was also a same-warp candidate)
                         const bool pre = MV || (prevMd && !(Z[j] >> 30));
-                        if ((((pre || IGD_C4_NOGATHER ? M[j] : ld_event(P.ev, V[j]).w)) >> g.lane(p)) & 1u) break;
+                        if ((((pre || IGD_C4_NOGATHER ? M[j] : ld_event(P.ev, V[j]).w)) >> lane_of(p)) & 1u) break;
                     } else {
                         gather = true;
                     }
@@ -470,7 +475,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                      (blk ? QF_BLK : 0u) | (gather ? QF_MASK : 0u);
                 if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
                     const bool other =
-                        lastW == mdp ? !same_b : g.block(tk_at(lastW) & 0xFFFFFFu) != g.block(c);
+                        lastW == mdp ? !same_b : blk_of(tk_at(lastW) & 0xFFFFFFu) != blk_of(c);
                     if (other) fl |= QF_R1;
                 }
                 queue = true;
@@ -574,8 +579,8 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             // reading A33: an ID moved iff the number of its events since md is not a multiple of
             // 2^width (Fig. 4: WarpBarID 6, BlkBarID 8, DevFenceID 6, BlkFenceID 6 bits)
             const u32 gcnt = P.glo != P.ghi ? q_count(P.desc, P.sts, ks.grid, mdIdx, i) : 0u;
-            if (same_w && (q_count(P.desc, P.sts, ks.wb + g.warp(c), mdIdx, i) & 63u)) continue;  // P4
-            if (same_b && ((q_count(P.desc, P.sts, ks.bb + g.block(c), mdIdx, i) + gcnt) & 255u)) continue;  // P5
+            if (same_w && (q_count(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i) & 63u)) continue;  // P4
+            if (same_b && ((q_count(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i) + gcnt) & 255u)) continue;  // P5
             type = (flags & QF_R1) ? IGD_R1 : 0u;
             if (!type) {
                 const u32 dfen = q_count(P.desc, P.sts, ks.dev + p, mdIdx, i);  // device fences of md's thread
@@ -590,9 +595,9 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 }
             }
         } else {
-        if (same_w && q_between(P.desc, P.sts, ks.wb + g.warp(c), mdIdx, i)) continue;  // P4: syncwarp
+        if (same_w && q_between(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i)) continue;  // P4: syncwarp
         const bool grid = q_grid(P, mdIdx, i);
-        if (same_b && (grid || q_between(P.desc, P.sts, ks.bb + g.block(c), mdIdx, i))) continue;  // P5
+        if (same_b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) continue;  // P5
         type = (flags & QF_R1) ? IGD_R1 : 0u;
         if (!type) {
             if (same_b) {

@@ -286,8 +286,15 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
 // a6 kernel instantiation: sharded payload (MV), kernel boundaries (KB), paper-width IDs (WRAP)
 template <bool MV, bool KB>
 static void launch_check_w(bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
-    if (wrap) check::k_check4<MV, KB, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
-    else check::k_check4<MV, KB, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+    // power-of-two geometry (block_dim >= 32): shift / mask instead of divisions (common case)
+    const bool geo2 = cp.g.dlog < 32 && cp.g.D >= 32;
+    if (wrap) {
+        if (geo2) check::k_check4<MV, KB, true, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
+        else check::k_check4<MV, KB, true, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+    } else {
+        if (geo2) check::k_check4<MV, KB, false, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
+        else check::k_check4<MV, KB, false, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+    }
 }
 static void launch_check(bool mv, bool kb, bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
     if (mv && kb) launch_check_w<true, true>(wrap, tb, st, cp);
