@@ -239,7 +239,7 @@ def run_sharded(args, fam, rank, world, local):
                            "reports": int(len(rep)), "ledger_reports": ledger_n,
                            "l2": "inputs larger than L2 (no flush)",
                            "parallelism": f"{world} ranks: contiguous trace chunks, words hash-sharded "
-                                          f"(fmix32 % P), NCCL all-to-all + all-gather"},
+                                          f"(fmix32 % P), {args.backend.upper()} all-to-all + all-gather"},
                 "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                              "frac": achieved / peak, "peak_source": peak_kind, "traffic": None,
                              "launches_per_step": c / args.steps, "rank": 0},
