@@ -64,6 +64,9 @@ def test_random_small(det, batch):
     (3, 300_000, 1, 4, 64),        # one hot word: a single segment across ~300 tiles
     (4, 200_000, 70_000, 16, 128),
     (5, 150_000, 3, 1, 32),
+    (6, 100_000, 500, 5, 48),      # block_dim not a power of two: the division geometry path
+    (7, 80_000, 200, 9, 16),       # block_dim < 32: partial warps, one per block
+    (8, 120_000, 2_000, 3, 1024),  # largest block: 32 warps per block on the shift path
 ])
 def test_random_multi_tile(det, seed, n, words, nb, bd):
     w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
