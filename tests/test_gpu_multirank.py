@@ -52,6 +52,13 @@ def test_multi_tile_trace(P):
     assert np.array_equal(sharded(ev, nb, bd, P), oracle.run(ev, nb, bd))
 
 
+@pytest.mark.parametrize("P,bd", [(3, 96), (2, 16)])
+def test_multi_tile_trace_odd_geometry(P, bd):
+    # block_dim not a power of two / below a warp: the sharded check on the division geometry path
+    ev, nb, bd = _fast_random(78, 200_000, 2_000, 5, bd, [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1], lock_words=20)
+    assert np.array_equal(sharded(ev, nb, bd, P), oracle.run(ev, nb, bd))
+
+
 @pytest.mark.parametrize("fam,n,rate", [(1, None, 1.0), (2, 2_000_000, 3.0), (4, 3_000_000, 8.0)])
 def test_families_sharded_equal_ledger(fam, n, rate):
     ev, nb, bd, led = F.generate(fam, n, rate=rate)
