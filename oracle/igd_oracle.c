@@ -419,17 +419,18 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
                 if (!isThread[w_c] && __builtin_popcount(e.mask) > 1) isThread[w_c] = 1;
                 if (!touched[w_c]) { touched[w_c] = 1; touched_list[n_touched++] = w_c; }
                 o_table* T = TABLE(c);
+                /* "up to 3 separate locks": a CAS on a lock already in the table
+                   (same hash and scope, e.g. the retries of a spin loop) adds nothing (A9) */
                 int present = 0;
                 for (int q = 0; q < 3; q++)
                     if (T->e[q].valid && T->e[q].h18 == h && T->e[q].scope == s) present = 1;
+                int slot = -1; /* the lowest free slot */
+                for (int q = 2; q >= 0; q--)
+                    if (!T->e[q].valid) slot = q;
+                if (slot < 0) present = 1; /* full table: the insert is dropped (A9) */
                 if (!present) {
-                    for (int q = 0; q < 3; q++) {
-                        if (!T->e[q].valid) {
-                            T->e[q].valid = 1; T->e[q].active = 0;
-                            T->e[q].scope = (uint8_t)s; T->e[q].h18 = h;
-                            break;
-                        }
-                    } /* full table: the insert is dropped (A9) */
+                    T->e[slot].valid = 1; T->e[slot].active = 0;
+                    T->e[slot].scope = (uint8_t)s; T->e[slot].h18 = h;
                 }
             } else {
                 /* atomicExch unsets Valid of entries matching hash and scope */
@@ -452,6 +453,14 @@ int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t bloc
              uint32_t shard_k, uint32_t shard_K, o_report* out, uint64_t cap,
              uint64_t* n_reports, uint64_t* bad_index) {
     return igdo_run_ex(events, n, n_blocks, block_dim, shard_k, shard_K, 0, out, cap, n_reports, bad_index);
+}
+
+/* Test hook (reading A8): the 18-bit lock hash of a word and its 16-bit Bloom summary, so
+   tests can pin what the paper fixes -- an 18-bit hash and a 16-bit summary with two
+   hash functions, "2-way bloom filter". */
+void igdo_lock_hash(uint64_t word, uint32_t* h18, uint32_t* bloom) {
+    *h18 = o_h18(word);
+    *bloom = o_bloom(*h18);
 }
 
 /* Exported constants so the Python side can check it loaded this library. */

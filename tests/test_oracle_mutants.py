@@ -47,6 +47,12 @@ MUTANTS = {
                             "if (isAtomic) { if (!S->atomic) S->ascope = (uint8_t)s; S->atomic = 1; }"),
     "check_after_lock_update": ("uint16_t L = o_held_of(TABLE(c));", "uint16_t L = o_held_of(TABLE(c)) | (k == O_CAS ? o_bloom(o_h18(e.addr >> 2)) : 0);"),
     "bloom_single_bit": ("| (1u << ((h >> 4) & 15u))", ""),
+    # reading A9 (lock-table capacity, duplicates, overflow): W10 / W11 discriminate
+    "A9_no_dedup": ("T->e[q].scope == s) present = 1;", "T->e[q].scope == s) present = 0;"),
+    "A9_evict_oldest": ("if (slot < 0) present = 1;",
+                        "if (slot < 0) { T->e[0] = T->e[1]; T->e[1] = T->e[2]; T->e[2].valid = 0; slot = 2; }"),
+    "A9_replace_last": ("if (slot < 0) present = 1;", "if (slot < 0) slot = 2;"),
+    "A9_four_entries": ("if (slot < 0) present = 1;", "if (slot < 0) { memset(T, 0, sizeof(*T)); slot = 0; }"),
 }
 
 
