@@ -133,7 +133,8 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
    memory owned by the context, asynchronously on the context stream from the caller's
    buffer; the call synchronizes the stream before returning, so the caller may free the
    buffer afterwards.  Device `events` are BORROWED: they must stay valid and unmodified until
-   igd_detect returns.  Returns IGD_EINVAL on bad geometry / desc, IGD_ETOOBIG when
+   igd_detect returns, and be 16-byte aligned.  Returns IGD_EINVAL on bad geometry / desc or a
+   misaligned device pointer, IGD_ETOOBIG when
    n_events >= 2^32 - 1.  Field validation happens in igd_detect. */
 int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* events);
 
@@ -166,7 +167,9 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
    ranks and must not continue if any rank has one); word_minmax = min / max accessed word of the chunk
    (the caller reduces them; the global span must be < 2^32 words).  Returns IGD_OK even when
    *bad_event is set.
-   igd_shard_buffers: device pointers (context-owned, valid until the next prepare) to the records
+   igd_shard_buffers: device pointers (context-owned, valid until the next prepare or until
+   igd_shard_detect returns, which releases the record buffer -- after the check when the
+   caller passes it back as d_records) to the records
    (uint4 {low 32 bits of the word, global index, tk, active mask}, grouped by owner in rank order,
    trace order inside a group), the sync-stream global indices (u32) and events (16 B).
    Exchange (caller): all-to-all of the record groups; all-gather of the sync streams concatenated

@@ -10,8 +10,8 @@ extern "C" {
 #endif
 
 /* Stable LSD radix sort (the a5 kernel) of n (key, value) u32 pairs held in DEVICE memory,
-   in place, over the low max_bits key bits.  mode: 1 = ballot multisplit, 0 = match.any,
-   2 = shared-memory atomic-or multisplit.
+   in place, over the low max_bits key bits.  mode: ignored (one multisplit policy, rows ranked
+   alternately by ballots and match.any; kept for ABI stability).
    *ms = device time of the sort passes (CUDA events on the context stream). */
 int igd_debug_radix_sort(igd_ctx* ctx, uint32_t* d_keys, uint32_t* d_vals, uint64_t n, uint32_t max_bits, int mode,
                          float* ms);

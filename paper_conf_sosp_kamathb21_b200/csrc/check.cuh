@@ -126,12 +126,11 @@ struct Params {
     const u32* sts;     // sync timestamps (sorted by entity, then time)
     syncx::LockView lv;
     u64* status;     // [n_tiles] zeroed
-    u32* tile_ctr;   // zeroed
+    u32* tile_ctr;   // zeroed: tile tickets
     igd_report* rep;
     u64 rep_cap;
     unsigned long long* rep_ctr;
     u64 first_event; // global index offset (multi-rank)
-    int debug_stop;  // profiling only (IGD_CHECK_STOP): 1 = stop after the scans, 2 = after phase 1
 };
 
 // Grid-sync bucket table: gtab[b] = {index, timestamp} of the first grid sync with timestamp >=

@@ -31,20 +31,11 @@ namespace check {
 #ifndef IGD_C4_MINB
 #define IGD_C4_MINB 6
 #endif
-#ifndef IGD_C4_NOGATHER
-#define IGD_C4_NOGATHER 0  // timing experiment only (wrong results): no active-mask gathers (C5@1e9: the gathers cost ~1.5 ms of ~15)
-#endif
 #ifndef IGD_C4_MBAR
 #define IGD_C4_MBAR 1  // warps wait for the tile prefix on an mbarrier (0: poll a shared flag)
 #endif
-#ifndef IGD_C4_WLB
-#define IGD_C4_WLB 0  // 1: warp-parallel look-back (measured slower: 14.9 -> 15.9 ms at C5@1e9; walks are short)
-#endif
 #ifndef IGD_C4_SLEEP
 #define IGD_C4_SLEEP 32  // ns between polls of the tile prefix
-#endif
-#ifndef IGD_C4_STAGED
-#define IGD_C4_STAGED 0  // phase 2 with all list queries of an entry issued at once (measured slower)
 #endif
 constexpr int C4_ITEMS = IGD_C4_ITEMS;
 constexpr int C4_WT = 32 * C4_ITEMS;         // accesses per warp
@@ -94,70 +85,6 @@ __device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, co
     return __ldg(ts + lo) < b;
 }
 
-#define QF_MASK 32u  // P4 lockstep clause pending: gather the event's active mask in phase 2
-
-// Staged interval query "is there x in list e with a < x < b" (check.cuh q_between, split so a
-// lane can have several in flight): bq_desc decides from the list descriptor {lo, hi, first,
-// last} or picks an interpolated 8-timestamp probe window; bq_probe decides from that window, or
-// finishes with a binary search (rare: a mis-guessed window).
-struct BQ {
-    u32 a, b, lo, hi, g0;
-    bool done, res;
-};
-__device__ __forceinline__ void bq_desc(BQ& q, const uint4 d) {
-    q.done = true;
-    q.res = false;
-    if (d.x == d.y || d.w <= q.a) return;  // empty, or every element <= a
-    if (d.z > q.a) {                        // the first element is the first one > a
-        q.res = d.z < q.b;
-        return;
-    }
-    q.lo = d.x + 1;
-    q.hi = d.y - 1;
-    u32 g = d.x + 1 + (u32)(__fdividef((float)(q.a - d.z), (float)(d.w - d.z)) * (float)(d.y - 1 - d.x));
-    g = min(max(g, q.lo), q.hi);
-    q.g0 = g & ~7u;
-    q.done = false;
-}
-__device__ __noinline__ bool bq_finish(const u32* __restrict__ ts, u32 lo, u32 hi, u32 a, u32 b) {
-    while (lo < hi) {
-        const u32 mid = (lo + hi) >> 1;
-        if (__ldg(ts + mid) <= a) lo = mid + 1;
-        else hi = mid;
-    }
-    return __ldg(ts + lo) < b;
-}
-__device__ __forceinline__ void bq_probe(BQ& q, const uint4 v0, const uint4 v1, const u32* __restrict__ ts) {
-    const u32 a = q.a, g0 = q.g0;
-    const u32 s0 = max(g0, q.lo), s1 = min(g0 + 8, q.hi + 1);  // probed positions inside [lo, hi]
-    const u32 lem = (u32)(v0.x <= a) | ((u32)(v0.y <= a) << 1) | ((u32)(v0.z <= a) << 2) | ((u32)(v0.w <= a) << 3) |
-                    ((u32)(v1.x <= a) << 4) | ((u32)(v1.y <= a) << 5) | ((u32)(v1.z <= a) << 6) |
-                    ((u32)(v1.w <= a) << 7);
-    const u32 rng = ((1u << (s1 - g0)) - 1u) & ~((1u << (s0 - g0)) - 1u);
-    const u32 le = __popc(lem & rng);
-    q.done = true;
-    if (le != 0 && le != s1 - s0) {  // the successor of a lies inside the window
-        const u32 k = s0 - g0 + le;
-        const uint4 h = k < 4 ? v0 : v1;
-        const u32 kk = k & 3u;
-        const u32 v = kk == 0 ? h.x : kk == 1 ? h.y : kk == 2 ? h.z : h.w;
-        q.res = v < q.b;
-        return;
-    }
-    q.res = le == 0 ? bq_finish(ts, q.lo, s0, a, q.b) : bq_finish(ts, s1, q.hi, a, q.b);
-}
-// grid query continued from list position x (the bucket's first entry was <= a)
-template <class PP>
-__device__ __noinline__ bool q_grid_from(const PP& P, u32 a, u32 b, u32 x) {
-#pragma unroll 1
-    for (int step = 0; x < P.ghi; step++, x++) {
-        const u32 v = __ldg(P.sts + x);
-        if (v > a) return v < b;
-        if (step == 8) return q_between(P.desc, P.sts, P.ks.grid, a, b);
-    }
-    return false;
-}
-
 // KB: the trace has kernel boundaries (a separate instantiation: the boundary test costs
 // registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
 template <bool MV, bool KB, bool WRAP, bool GEO2>
@@ -169,9 +96,19 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     __shared__ u64 s_prefix;
     __shared__ u32 s_ready;
     __shared__ __align__(8) u64 s_rbar;  // IGD_C4_MBAR: the tile prefix is ready (one arrival)
+    __shared__ u32 s_tile;
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
-    const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
+    // Tile ids in the order CTAs start (a ticket, not blockIdx.x): a tile only waits on tiles
+    // that are already running, so the decoupled look-back cannot deadlock whatever order the
+    // hardware dispatches CTAs in (MPS, SM partitions).
+    if (t == 0) {
+        s_tile = atomicAdd(P.tile_ctr, 1u);
+        s_ready = 0;
+        if (IGD_C4_MBAR) mbar_init(&s_rbar, 1);
+    }
+    __syncthreads();
+    const u32 tile = s_tile;
     const u32 tbase = tile * C4_TILE;
     const u32 wloc = warp * C4_WT;
     const u32 wbase = tbase + wloc;
@@ -182,11 +119,6 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     auto blk_of = [&](u32 t) -> u32 { return GEO2 ? t >> dlog : g.block(t); };
     auto warp_of = [&](u32 t) -> u32 { return GEO2 ? t >> 5 : g.warp(t); };
     auto lane_of = [&](u32 t) -> u32 { return GEO2 ? t & 31u : g.lane(t); };
-    if (t == 0) {
-        s_ready = 0;
-        if (IGD_C4_MBAR) mbar_init(&s_rbar, 1);  // visible to every thread after the __syncthreads below
-    }
-
     u32 K[C4_ITEMS], V[C4_ITEMS], Z[C4_ITEMS], M[C4_ITEMS];
 #pragma unroll
     for (int j = 0; j < C4_ITEMS; j++) {
@@ -261,7 +193,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         // P4's lockstep clause will need this instruction's active mask when md is likely the
         // previous access, from another lane of the same warp, and the mask is partial: gather
         // it now so the trace read overlaps the scans (phase 1 re-checks the exact condition)
-        if (!MV && !IGD_C4_NOGATHER && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) M[j] = ld_event(P.ev, V[j]).w;
+        if (!MV && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) M[j] = ld_event(P.ev, V[j]).w;
     }
 
     // ---- warp aggregate in the packed state of check.cuh (state after the warp's last access) ----
@@ -285,56 +217,13 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         if (lane == 0) s_wagg[warp] = agg;
     }
     __syncthreads();
-#if IGD_C4_WLB
-    if (warp == 0) {
-        // Warp 0 publishes the tile's aggregate and looks back 32 predecessors per round: lane l
-        // reads tile - 1 - l - 32r; the closest inclusive-or-head status ends the walk; the
-        // statuses in between are combined in time order by a shuffle reduction (combine is
-        // associative; identity on the left is neutral)
-        u64 tagg = s_wagg[0];
-#pragma unroll
-        for (int w = 1; w < C4_WARPS; w++) tagg = combine(tagg, s_wagg[w]);
-        u64 prefix = ST_IDENTITY;
-        if (lane == 0) st_relaxed(&P.status[tile], ((tile == 0 || st_head(tagg)) ? ST_INC : ST_AGG) | tagg);
-        if (tile > 0 && !(hm[0] & 1u) && P.debug_stop != 3) {  // a tile starting with a head needs no prefix
-            u64 acc = ST_IDENTITY;
-            for (long top = (long)tile - 1;; top -= 32) {
-                const long tt = top - (long)lane;
-                u64 s = ST_INC | ST_IDENTITY;  // before tile 0: an inclusive identity
-                if (tt >= 0) {
-                    do {
-                        s = ld_relaxed(&P.status[tt]);
-                    } while ((s >> 62) == 0);
-                }
-                u64 v = s & ST_VAL_MASK;
-                const u32 stop = __ballot_sync(IGD_FULL, (s >> 62) == 2 || st_head(v));
-                const u32 k = stop ? (u32)(__ffs(stop) - 1) : 31u;
-                if (lane > k) v = ST_IDENTITY;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {  // lane l <- x_{l+o} (earlier) combined before x_l
-                    const u64 y = __shfl_down_sync(IGD_FULL, v, o);
-                    if (lane + o < 32) v = combine(y, v);
-                }
-                acc = combine(__shfl_sync(IGD_FULL, v, 0), acc);
-                if (stop) break;
-            }
-            prefix = acc;
-            if (lane == 0 && !st_head(tagg)) st_relaxed(&P.status[tile], ST_INC | combine(prefix, tagg));
-        }
-        if (lane == 0) {
-            s_prefix = prefix;
-            __threadfence_block();
-            *(volatile u32*)&s_ready = 1u;
-        }
-    }
-#else
     if (t == 0) {
         u64 tagg = s_wagg[0];
 #pragma unroll
         for (int w = 1; w < C4_WARPS; w++) tagg = combine(tagg, s_wagg[w]);
         u64 prefix = ST_IDENTITY;
         st_relaxed(&P.status[tile], ((tile == 0 || st_head(tagg)) ? ST_INC : ST_AGG) | tagg);
-        if (tile > 0 && !(hm[0] & 1u) && P.debug_stop != 3) {  // a tile starting with a head needs no prefix
+        if (tile > 0 && !(hm[0] & 1u)) {  // a tile starting with a head needs no prefix
             // combine predecessors back to an inclusive status or a head-containing aggregate;
             // a tile with a head has published already (its successors never need more), its
             // accesses before the first head still need the prefix
@@ -361,24 +250,18 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         if (IGD_C4_MBAR) mbar_arrive(&s_rbar);  // release: s_prefix before the phase flips
     }
 
-#endif
     // state carried into this warp's first segment (needed only before its first head)
     u64 carry = ST_IDENTITY;
     if (!(hm[0] & 1u)) {
         for (u32 w = 0; w < warp; w++) carry = combine(carry, s_wagg[w]);
         if (!st_head(carry) && tile > 0) {
-            if (P.debug_stop == 3) return;  // profiling: no look-back
-            if (IGD_C4_MBAR && !IGD_C4_WLB) {
+            if (IGD_C4_MBAR) {
                 mbar_wait(&s_rbar, 0);  // suspended in hardware, not polling issue slots
             } else {
                 while (*(volatile u32*)&s_ready == 0u) __nanosleep(IGD_C4_SLEEP);
             }
             carry = combine(*(volatile u64*)&s_prefix, carry);
         }
-    }
-    if (P.debug_stop == 1 || P.debug_stop == 3) {
-        if (carry == 0x123456789ull) P.rep_ctr[1] = carry;
-        return;
     }
 
     // ---- phase 1: scan quantities per access, history-free checks, queue the rest ----
@@ -459,20 +342,15 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 // warp; bit 30: own lane only; otherwise the mask itself, from the payload in MV
                 // mode, else gathered from the trace)
                 if (same_w && (Z[j] >> 31)) break;
-                bool gather = false;
                 if (same_w && !(Z[j] >> 30)) {
                     if (p == IGD_NONE32) p = tk_at(mdp) & 0xFFFFFFu;
-                    if (MV || !IGD_C4_STAGED) {
-                        // prefetched unless md is an earlier writer (M[j] is the mask then only
-                        // if the previous access was also a same-warp candidate)
-                        const bool pre = MV || (prevMd && !(Z[j] >> 30));
-                        if ((((pre || IGD_C4_NOGATHER ? M[j] : ld_event(P.ev, V[j]).w)) >> lane_of(p)) & 1u) break;
-                    } else {
-                        gather = true;
-                    }
+                    // prefetched unless md is an earlier writer (M[j] is the mask then only
+                    // if the previous access was also a same-warp candidate)
+                    const bool pre = MV || (prevMd && !(Z[j] >> 30));
+                    if (((pre ? M[j] : ld_event(P.ev, V[j]).w) >> lane_of(p)) & 1u) break;
                 }
                 fl = (same_w ? QF_SAME_W : 0u) | (same_b ? QF_SAME_B : 0u) | (dev ? QF_DEV : 0u) |
-                     (blk ? QF_BLK : 0u) | (gather ? QF_MASK : 0u);
+                     (blk ? QF_BLK : 0u);
                 if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
                     const bool other =
                         lastW == mdp ? !same_b : blk_of(tk_at(lastW) & 0xFFFFFFu) != blk_of(c);
@@ -500,13 +378,12 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         if (bm[j]) cB = j * 32 + hib(bm[j]);
     }
     __syncwarp();
-    if (P.debug_stop == 2) return;
 
     // ---- phase 2: the warp's queued accesses, densely over its lanes ----
     // One entry per lane, its list queries in Table 2's order with early exits.  Issuing all of an
-    // entry's queries at once (IGD_C4_STAGED) and interleaving two entries per lane were both
-    // measured slower (20.9 and 22.2 vs 14.8 ms at C5@1e9): this phase is bound by the queries'
-    // total L2 / issue work, not by the latency of one chain.
+    // entry's queries at once and interleaving two entries per lane were both measured slower
+    // (20.9 and 22.2 vs 14.8 ms at C5@1e9, round 1): this phase is bound by the queries' total
+    // L2 / issue work, not by the latency of one chain.
     const KeySpace ks = P.ks;
     for (u32 k = lane; k < qn; k += 32) {
         const u32 x = q_x[qb + k], mdp = q_md[qb + k], flags = q_f[qb + k];
@@ -523,57 +400,6 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         }
         const u32 p = mdz & 0xFFFFFFu;
         const bool same_w = flags & QF_SAME_W, same_b = flags & QF_SAME_B;
-#if IGD_C4_STAGED
-        // all queries of the entry at once: round 1 descriptors + grid bucket + active mask,
-        // round 2 the 32-byte timestamp probes
-        // round 1
-        const uint4 none4 = make_uint4(0, 0, 0, 0);
-        const uint4 dW = same_w ? __ldg(P.desc + ks.wb + g.warp(c)) : none4;
-        const uint4 dB = same_b ? __ldg(P.desc + ks.bb + g.block(c)) : none4;
-        const uint4 dF = __ldg(P.desc + (same_b ? ks.any : ks.dev) + p);
-        const bool hasG = P.glo != P.ghi;
-        const u32 gx = hasG ? (u32)__ldg(P.gtab + ((mdIdx + 1) >> P.gshift)) : 0u;
-        const u32 emask = (flags & QF_MASK) ? ld_event(P.ev, i).w : 0u;
-        if ((flags & QF_MASK) && ((emask >> g.lane(p)) & 1u)) continue;  // P4: lockstep
-        BQ qW, qB, qF;
-        qW.a = qB.a = qF.a = mdIdx;
-        qW.b = qB.b = qF.b = i;
-        bq_desc(qW, dW);
-        bq_desc(qB, dB);
-        bq_desc(qF, dF);
-        // round 2
-        uint4 w0 = none4, w1 = none4, b0 = none4, b1 = none4, f0 = none4, f1 = none4;
-        if (!qW.done) {
-            w0 = __ldg(reinterpret_cast<const uint4*>(P.sts + qW.g0));
-            w1 = __ldg(reinterpret_cast<const uint4*>(P.sts + qW.g0) + 1);
-        }
-        if (!qB.done) {
-            b0 = __ldg(reinterpret_cast<const uint4*>(P.sts + qB.g0));
-            b1 = __ldg(reinterpret_cast<const uint4*>(P.sts + qB.g0) + 1);
-        }
-        if (!qF.done) {
-            f0 = __ldg(reinterpret_cast<const uint4*>(P.sts + qF.g0));
-            f1 = __ldg(reinterpret_cast<const uint4*>(P.sts + qF.g0) + 1);
-        }
-        const u32 gv = (hasG && gx < P.ghi) ? __ldg(P.sts + gx) : 0xFFFFFFFFu;
-        if (!qW.done) bq_probe(qW, w0, w1, P.sts);
-        if (same_w && qW.res) continue;  // P4: syncwarp
-        bool grid = false;
-        if (hasG && gx < P.ghi) grid = gv > mdIdx ? gv < i : q_grid_from(P, mdIdx, i, gx + 1);
-        if (!qB.done) bq_probe(qB, b0, b1, P.sts);
-        if (same_b && (grid || qB.res)) continue;  // P5
-        if (!qF.done) bq_probe(qF, f0, f1, P.sts);
-        u32 type = (flags & QF_R1) ? IGD_R1 : 0u;
-        if (!type) {
-            if (same_b) {
-                // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread must
-                // not have fenced since md (A1, A30)
-                if (!(flags & QF_DEV) && !grid && !qF.res) type = (same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3;
-            } else if (!grid && !qF.res) {
-                type = IGD_R4;  // R4: other block, no device fence by md's thread
-            }
-        }
-#else
         u32 type;
         if (WRAP) {
             // reading A33: an ID moved iff the number of its events since md is not a multiple of
@@ -610,8 +436,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             }
         }
         }
-#endif
-        if (!type && P.lv.any && P.debug_stop != 4) {  // R5: lock sets of the last accessor and of this access
+        if (!type && P.lv.any) {  // R5: lock sets of the last accessor and of this access
             u32 laIdx, laz;
             if (x - 1 - tbase < (u32)C4_TILE) {
                 laIdx = s_v[x - 1 - tbase];

@@ -50,6 +50,7 @@ struct Params {
     u64 sync_cap;
     const u32* digit_base;  // [256] exclusive global offsets of digit 0 of the access keys
     u64* status;            // [n_tiles * 256], zeroed
+    u32* tile_ctr;          // zeroed: tile tickets (CTA start order, see rsort::k_onesweep)
     u32* kout;              // access keys, sorted by digit 0
     u64* vout;              // access payload (event index | tk << 32), same order
     const u32* skip_bits;   // coalesced mode (A32): bit i = event i is not an access record
@@ -105,6 +106,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     __shared__ u32 s_na;
     __shared__ u32 s_cnt[RADIX];  // tile digit counts (early publication)
     __shared__ __align__(8) u64 s_mbar;
+    __shared__ u32 s_tile;
     extern __shared__ __align__(16) unsigned char s_dyn[];
     // phase 1: the event tile (64 KB).  Phase 2 (events dead): digit-sorted keys [0, 16K),
     // values [16K, 48K), digit per position [48K, 52K), per-warp digit counts [56K, 64K).
@@ -115,16 +117,24 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     u32(*s_whist)[RADIX] = reinterpret_cast<u32(*)[RADIX]>(s_dyn + TILE * 14);
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
-    const u32 tile = blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
+    if (t == 0) {
+        // tile ticket in CTA start order (decoupled look-back never waits on an unstarted tile),
+        // then one TMA bulk copy of the tile's events
+        const u32 tl = atomicAdd(P.tile_ctr, 1u);
+        s_tile = tl;
+        const u64 b0 = (u64)tl * TILE;
+        if (b0 + TILE <= P.n) {
+            mbar_init(&s_mbar, 1);
+            mbar_expect_tx(&s_mbar, TILE * sizeof(uint4));
+            bulk_g2s(s_ev, P.ev + b0, TILE * sizeof(uint4), &s_mbar);
+        }
+    }
+    s_cnt[t] = 0;
+    __syncthreads();
+    const u32 tile = s_tile;
     const u64 base = (u64)tile * TILE;
     const bool full = base + TILE <= P.n;
     const u32 tile_e = full ? (u32)TILE : (u32)(P.n - base);
-    if (t == 0 && full) {
-        mbar_init(&s_mbar, 1);
-        mbar_expect_tx(&s_mbar, TILE * sizeof(uint4));
-        bulk_g2s(s_ev, P.ev + base, TILE * sizeof(uint4), &s_mbar);
-    }
-    s_cnt[t] = 0;
     if (!full)
         for (u32 i = t; i < TILE; i += THREADS)
             s_ev[i] = i < tile_e ? ld_event_stream(P.ev, base + i) : make_uint4(0, 0, 0, 0);

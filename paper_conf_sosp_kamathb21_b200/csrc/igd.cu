@@ -61,9 +61,6 @@ struct igd_ctx {
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
-    int sort_mode = 1;  // warp multisplit: 1 = ballots (default), 0 = match.any, 2 = atomic-or (IGD_SORT_MODE)
-    int check_stop = 0; // profiling knob IGD_CHECK_STOP (results invalid when set)
-    int count_tma = 0;  // IGD_COUNT_TMA=1: ingest pass 0 through a TMA ring (ingest::k_count; measured slower: 8.6 vs 7.2 ms at C5 1e9, the pass is issue-bound)
     bool coalesce = false;  // IGD_DETECT_COALESCE of the running igd_detect (reading A32)
     bool paper_counters = false;  // IGD_DETECT_PAPER_COUNTERS (reading A33)
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
@@ -190,40 +187,19 @@ static void mark(igd_ctx* ctx, int stage) {
     if (ctx->timing) cudaEventRecord(ctx->ev[stage], ctx->stream);
 }
 
+// One radix pass over n keys: the full tiles, then (if any) the partial last tile (same tile
+// counter: the tail's ticket is the last tile).
 template <typename VT>
-static void launch_mode(int mode, bool tail, unsigned gb, size_t smem, cudaStream_t st, const rsort::PassParams& pp) {
-    if (tail) {
-        if (mode == 0) rsort::k_onesweep<0, VT, true><<<gb, rsort::THREADS, smem, st>>>(pp);
-        else if (mode == 2) rsort::k_onesweep<2, VT, true><<<gb, rsort::THREADS, smem, st>>>(pp);
-        else rsort::k_onesweep<1, VT, true><<<gb, rsort::THREADS, smem, st>>>(pp);
-    } else {
-        if (mode == 0) rsort::k_onesweep<0, VT, false><<<gb, rsort::THREADS, smem, st>>>(pp);
-        else if (mode == 2) rsort::k_onesweep<2, VT, false><<<gb, rsort::THREADS, smem, st>>>(pp);
-        else rsort::k_onesweep<1, VT, false><<<gb, rsort::THREADS, smem, st>>>(pp);
-    }
-}
-// One radix pass over n keys: the full tiles, then (if any) the partial last tile.
-template <typename VT>
-static void launch_pass(int mode, u64 n, size_t smem, cudaStream_t st, rsort::PassParams pp) {
+static void launch_pass(u64 n, size_t smem, cudaStream_t st, const rsort::PassParams& pp) {
     const u64 full = n / rsort::TILE;
-    if (full) {
-        pp.tile0 = 0;
-        launch_mode<VT>(mode, false, (unsigned)full, smem, st, pp);
-    }
-    if (n % rsort::TILE) {
-        pp.tile0 = (u32)full;
-        launch_mode<VT>(mode, true, 1u, smem, st, pp);
-    }
+    if (full) rsort::k_onesweep<VT, false><<<(unsigned)full, rsort::THREADS, smem, st>>>(pp);
+    if (n % rsort::TILE) rsort::k_onesweep<VT, true><<<1u, rsort::THREADS, smem, st>>>(pp);
 }
 template <typename VT>
 static void set_pass_smem() {
     const int b = (int)rsort::onesweep_smem<VT>();
-    cudaFuncSetAttribute(rsort::k_onesweep<0, VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
-    cudaFuncSetAttribute(rsort::k_onesweep<1, VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
-    cudaFuncSetAttribute(rsort::k_onesweep<2, VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
-    cudaFuncSetAttribute(rsort::k_onesweep<0, VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
-    cudaFuncSetAttribute(rsort::k_onesweep<1, VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
-    cudaFuncSetAttribute(rsort::k_onesweep<2, VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
 }
 
 // Stable LSD radix sort of n (key, value) pairs in buffers k[cur], v[cur]; h_hist is the host
@@ -269,9 +245,9 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         pp.tile_ctr = P_<u32>(ctx->ctr);
         {
             KTimer kt(ctx, cls, 2.0 * (4 + vbytes) * (double)n);  // read + write 4 B key and the value
-            if (vbytes == 16) launch_pass<uint4>(ctx->sort_mode, n, rsort::onesweep_smem<uint4>(), ctx->stream, pp);
-            else if (vbytes == 8) launch_pass<u64>(ctx->sort_mode, n, rsort::onesweep_smem<u64>(), ctx->stream, pp);
-            else launch_pass<u32>(ctx->sort_mode, n, rsort::onesweep_smem<u32>(), ctx->stream, pp);
+            if (vbytes == 16) launch_pass<uint4>(n, rsort::onesweep_smem<uint4>(), ctx->stream, pp);
+            else if (vbytes == 8) launch_pass<u64>(n, rsort::onesweep_smem<u64>(), ctx->stream, pp);
+            else launch_pass<u32>(n, rsort::onesweep_smem<u32>(), ctx->stream, pp);
         }
         if (n > rsort::TILE && n % rsort::TILE) ctx->launches++;  // the partial-tile launch
         CK(cudaGetLastError());
@@ -398,16 +374,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const u64 grid = std::max<u64>(1, std::min<u64>((u64)sms * (occ > 0 ? occ : 1), in_tiles));
     if (n_src > 0) {
         KTimer kt(ctx, KC_INGEST, 16.0 * (double)n_src);  // pass 0 reads every event
-        if (ctx->count_tma) {
-            // trace streamed through a TMA ring in shared memory (ingest::k_count)
-            const size_t smem = ingest::count_smem();
-            int occ2 = 0;
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, ingest::k_count, ingest::THREADS, smem);
-            const u64 grid2 = std::max<u64>(1, std::min<u64>((u64)sms * (occ2 > 0 ? occ2 : 1), in_tiles));
-            ingest::k_count<<<(unsigned)grid2, ingest::THREADS, smem, ctx->stream>>>(ip);
-        } else {
-            ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
-        }
+        ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
     }
     CK(cudaGetLastError());
     RET(scan_excl(ctx, P_<u32>(ctx->st_in_a), in_tiles + 1));
@@ -451,6 +418,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         }
         RET(ensure(ctx, ctx->status, ft * fused::RADIX * sizeof(u64)));
         CK(cudaMemsetAsync(ctx->status.p, 0, ft * fused::RADIX * sizeof(u64), ctx->stream));
+        CK(cudaMemsetAsync(ctx->ctr.p, 0, sizeof(u32), ctx->stream));
         fused::Params fp;
         fp.ev = src_ev;
         fp.n = n_src;
@@ -462,6 +430,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         fp.sync_cap = ctx->sync_cap;
         fp.digit_base = P_<u32>(ctx->base);
         fp.status = P_<u64>(ctx->status);
+        fp.tile_ctr = P_<u32>(ctx->ctr);
         fp.kout = P_<u32>(ctx->acc_k[1]);
         fp.vout = P_<u64>(ctx->acc_v[1]);
         fp.skip_bits = ip.skip_bits;
@@ -631,7 +600,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.rep_cap = ctx->rep_cap;
             cp.rep_ctr = P_<unsigned long long>(ctx->rep_ctr);
             cp.first_event = 0;
-            cp.debug_stop = ctx->check_stop;
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
@@ -791,11 +759,7 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     ctx->afn = alloc_fn;
     ctx->ffn = free_fn;
     ctx->auser = alloc_user;
-    if (const char* m = getenv("IGD_SORT_MODE")) ctx->sort_mode = (atoi(m) >= 0 && atoi(m) <= 2) ? atoi(m) : 1;
-    if (const char* m = getenv("IGD_CHECK_STOP")) ctx->check_stop = atoi(m);
-    if (const char* m = getenv("IGD_COUNT_TMA")) ctx->count_tma = atoi(m) != 0;
     if (const char* m = getenv("IGD_FUSED")) ctx->fused = atoi(m) != 0;
-    cudaFuncSetAttribute(ingest::k_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ingest::count_smem());
     cudaFuncSetAttribute(fused::k_ingest_sort0, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes());
     set_pass_smem<u32>();
@@ -835,6 +799,11 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
     ctx->desc = *desc;
     ctx->loaded = false;
     if (desc->flags & IGD_TRACE_DEVICE_PTR) {
+        // the kernels read events with 16-byte vector loads and TMA bulk copies
+        if (((uintptr_t)events & 15u) != 0) {
+            ctx->err = "device events must be 16-byte aligned";
+            return IGD_EINVAL;
+        }
         ctx->events = events;
     } else {
         const size_t bytes = desc->n_events * sizeof(igd_event);
@@ -894,6 +863,10 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
                      uint64_t* n_reports) {
     if (!ctx || !n_reports) return IGD_EINVAL;
     if ((n_records && !d_records) || (n_sync_stream && (!d_sync_idx || !d_sync_events))) return IGD_EINVAL;
+    if ((((uintptr_t)d_records | (uintptr_t)d_sync_events) & 15u) != 0) {
+        ctx->err = "records and sync events must be 16-byte aligned";
+        return IGD_EINVAL;
+    }
     if (!ctx->loaded) return IGD_ESTATE;
     if (flags & IGD_DETECT_COALESCE) {  // reading A32: a group may straddle two ranks' chunks
         ctx->err = "IGD_DETECT_COALESCE is a single-context mode";
@@ -910,8 +883,14 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     ctx->sh_ns = n_sync_stream;
     ctx->sh_wbase = min_word;
     ctx->sh_ntotal = ctx->desc.n_events_total ? ctx->desc.n_events_total : ctx->desc.n_events;
-    RET(buf_free(ctx, ctx->sh_send));  // the exchange is done: release the send buffer first
+    // the exchange is done: release the send buffer first, unless the caller passes (part of) it
+    // back as the received records (one rank, or an in-place exchange) -- then after the check
+    const char* sb = (const char*)ctx->sh_send.p;
+    const char* rb = (const char*)d_records;
+    const bool aliased = sb && rb && rb < sb + ctx->sh_send.cap && rb + n_records * 16 > sb;
+    if (!aliased) RET(buf_free(ctx, ctx->sh_send));
     int rc = detect_impl(ctx, n_reports);
+    if (aliased) buf_free(ctx, ctx->sh_send);
     ctx->shard = false;
     ctx->paper_counters = false;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
@@ -1052,7 +1031,7 @@ int igd_debug_radix_sort(igd_ctx* ctx, uint32_t* d_keys, uint32_t* d_vals, uint6
                          float* ms) {
     if (!ctx || n >= 0xFFFFFFFFull || (n && (!d_keys || !d_vals))) return IGD_EINVAL;
     cudaSetDevice(ctx->device);
-    ctx->sort_mode = (mode >= 0 && mode <= 2) ? mode : 1;
+    (void)mode;  // one multisplit policy (IGD_SORT_MIX); kept in the signature for the hook's callers
     for (int b = 0; b < 2; b++) {
         RET(ensure(ctx, ctx->acc_k[b], n * sizeof(u32)));
         RET(ensure(ctx, ctx->acc_v[b], n * sizeof(u32)));

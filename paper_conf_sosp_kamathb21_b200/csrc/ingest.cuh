@@ -374,153 +374,6 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
     if (tid == 0 && cta_sync) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cta_sync);
 }
 
-// Pass 0 with the trace streamed through shared memory: persistent CTAs, a ring of STAGES tiles
-// filled by TMA bulk copies (cp.async.bulk + mbarrier) that thread 0 issues STAGES - 1 tiles ahead,
-// so the HBM reads of later tiles overlap the decode / histogram work of the current one (the
-// register-staged k_ingest<0> left the loads idle during that work: 2.2 TB/s on C5, ncu r01 v5).
-// Same outputs as k_ingest<0>.
-#ifndef IGD_COUNT_STAGES
-#define IGD_COUNT_STAGES 3
-#endif
-#ifndef IGD_COUNT_MINB
-#define IGD_COUNT_MINB 2
-#endif
-constexpr int CSTAGES = IGD_COUNT_STAGES;
-constexpr size_t count_smem() { return (size_t)CSTAGES * TILE * sizeof(uint4); }
-
-__global__ void __launch_bounds__(THREADS, IGD_COUNT_MINB) k_count(Params P) {
-    __shared__ u32 s_hacc[4][256];
-    __shared__ u32 s_hsync[4][256];
-    __shared__ u32 s_hup[3][256];
-    __shared__ u32 s_wtot[WARPS];
-    __shared__ __align__(8) u64 s_mbar[CSTAGES];
-    extern __shared__ __align__(16) unsigned char s_dyn[];
-    uint4* s_ev = reinterpret_cast<uint4*>(s_dyn);
-
-    const u32 tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
-    for (int i = tid; i < 4 * 256; i += THREADS) {
-        (&s_hacc[0][0])[i] = 0;
-        (&s_hsync[0][0])[i] = 0;
-        if (i < 3 * 256) (&s_hup[0][0])[i] = 0;
-    }
-    auto issue = [&](u32 tile, int stage) {
-        const u64 base = (u64)tile * TILE;
-        const u32 cnt = (u32)(P.n - base < (u64)TILE ? P.n - base : (u64)TILE);
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        mbar_expect_tx(&s_mbar[stage], cnt * (u32)sizeof(uint4));
-        bulk_g2s(s_ev + (size_t)stage * TILE, P.ev + base, cnt * (u32)sizeof(uint4), &s_mbar[stage]);
-    };
-    if (tid == 0) {
-        for (int s = 0; s < CSTAGES; s++) mbar_init(&s_mbar[s], 1);
-        for (int s = 0; s < CSTAGES - 1; s++) {
-            const u32 tl = blockIdx.x + s * gridDim.x;
-            if (tl < P.n_tiles) issue(tl, s);
-        }
-    }
-    __syncthreads();
-    u64 wmin = ~0ull, wmax = 0, bad = ~0ull;
-    u32 cnt_lock = 0;
-    u64 cta_sync = 0;
-    const Geo g = P.g;
-    const KeySpace ks = P.ks;
-    u32 it = 0;
-    for (u32 tile = blockIdx.x; tile < P.n_tiles; tile += gridDim.x, it++) {
-        const int stage = (int)(it % CSTAGES);
-        if (tid == 0) {  // refill the stage freed at the end of the previous iteration
-            const u32 ahead = tile + (CSTAGES - 1) * gridDim.x;
-            if (ahead < P.n_tiles) issue(ahead, (int)((it + CSTAGES - 1) % CSTAGES));
-        }
-        mbar_wait(&s_mbar[stage], (it / CSTAGES) & 1u);
-        const uint4* ev = s_ev + (size_t)stage * TILE;
-        const u64 base = (u64)tile * TILE;
-        u32 wsum = 0;
-#pragma unroll 4
-        for (int j = 0; j < ITEMS; j++) {
-            const u32 p = (u32)j * THREADS + tid;
-            const u64 i = base + p;
-            const bool in = i < P.n;
-            const uint4 e = ev[p];
-            Dec dv;
-            if (in) {
-                dv = decode(e, g, ks);
-                if (P.skip_bits && (dv.flags & 1u) && ((__ldg(P.skip_bits + (i >> 5)) >> (i & 31u)) & 1u))
-                    dv.flags &= ~1u;  // A32: not an access record
-                if (dv.flags & 1u) {
-                    const u64 word = ev_addr(e) >> 2;
-                    wmin = min(wmin, word);
-                    wmax = max(wmax, word);
-                }
-            } else {
-                dv.flags = 0;
-                dv.key = dv.s0 = dv.s1 = dv.tk = 0;
-            }
-            const u32 f = dv.flags;
-            const bool acc = (f & 1u) != 0;
-            const u32 ns = (f >> 1) & 3u;
-            if (f & 16u) bad = min(bad, i);
-            if (P.hist0) {
-                if (acc) atomicAdd(&s_hacc[warp & 3u][dv.key & 255u], 1u);
-                const u32 am = __ballot_sync(IGD_FULL, acc);
-                if (am) {
-                    const u32 hi = dv.key >> 8;
-                    const u32 src = __ffs(am) - 1;
-                    const u32 h0 = __shfl_sync(IGD_FULL, hi, src);
-                    const bool uni = __all_sync(IGD_FULL, !acc || hi == h0);
-                    const u32 c = uni ? (lane == src ? __popc(am) : 0u) : (acc ? 1u : 0u);
-                    if (c) {
-                        atomicAdd(&s_hup[0][hi & 255u], c);
-                        atomicAdd(&s_hup[1][(hi >> 8) & 255u], c);
-                        atomicAdd(&s_hup[2][hi >> 16], c);
-                    }
-                }
-            } else {  // unfused pipeline: access-key histograms by k_hist_keys over the written keys
-                if (__any_sync(IGD_FULL, ns != 0)) {
-#pragma unroll
-                    for (int q = 0; q < 4; q++) hist_add(s_hsync[q], (dv.s0 >> (8 * q)) & 255u, ns != 0, lane);
-#pragma unroll
-                    for (int q = 0; q < 4; q++) hist_add(s_hsync[q], (dv.s1 >> (8 * q)) & 255u, ns == 2, lane);
-                }
-            }
-            cnt_lock += (f >> 3) & 1u;
-            wsum += __reduce_add_sync(IGD_FULL, (acc ? 1u : 0u) | (ns << 16));
-        }
-        if (lane == 0) s_wtot[warp] = wsum;
-        __syncthreads();  // also: every thread is done with this stage's events
-        if (warp == 0) {
-            const u32 x = lane < WARPS ? s_wtot[lane] : 0u;
-            const u32 ta = __reduce_add_sync(IGD_FULL, x & 0xFFFFu);
-            const u32 ts = __reduce_add_sync(IGD_FULL, x >> 16);
-            if (lane == 0) {
-                P.tile_acc[tile] = ta;
-                P.tile_sync[tile] = ts;
-                cta_sync += ts;
-            }
-        }
-    }
-    __syncthreads();
-    for (int i = tid; i < 4 * 256; i += THREADS) {
-        const u32 a = i < 256 ? s_hacc[0][i] + s_hacc[1][i] + s_hacc[2][i] + s_hacc[3][i] : (&s_hup[0][0])[i - 256];
-        if (a) atomicAdd(&P.hist_acc[i], a);
-        const u32 s = (&s_hsync[0][0])[i];
-        if (s) atomicAdd(&P.hist_sync[i], s);
-    }
-    u64 cl = cnt_lock;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        wmin = min(wmin, __shfl_xor_sync(IGD_FULL, wmin, o));
-        wmax = max(wmax, __shfl_xor_sync(IGD_FULL, wmax, o));
-        bad = min(bad, __shfl_xor_sync(IGD_FULL, bad, o));
-        cl += __shfl_xor_sync(IGD_FULL, cl, o);
-    }
-    if (lane == 0) {
-        if (wmin != ~0ull) atomicMin((unsigned long long*)&P.stats[0], (unsigned long long)wmin);
-        if (wmin != ~0ull) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
-        if (bad != ~0ull) atomicMin((unsigned long long*)&P.stats[2], (unsigned long long)bad);
-        if (cl) atomicAdd((unsigned long long*)&P.stats[5], (unsigned long long)cl);
-    }
-    if (tid == 0 && cta_sync) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cta_sync);
-}
-
 // Digit histograms (4 x 8-bit) of the compacted access keys: a light, high-occupancy pass over
 // 4 bytes per access, with warp-uniform digits aggregated into one shared atomic.
 __global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys, u32 n, u32* __restrict__ hist,

@@ -22,12 +22,6 @@ constexpr int WARPS = THREADS / 32;
 #ifndef IGD_SORT_ITEMS
 #define IGD_SORT_ITEMS 16
 #endif
-#ifndef IGD_SORT_SKIPBITS
-#define IGD_SORT_SKIPBITS 0
-#endif
-#ifndef IGD_SORT_NOLOOKBACK
-#define IGD_SORT_NOLOOKBACK 0
-#endif
 #ifndef IGD_SORT_EARLY
 #define IGD_SORT_EARLY 1  // publish tile digit counts before ranking (C5@1e9: 21.6 -> 21.2 ms over 3 passes)
 #endif
@@ -86,8 +80,7 @@ struct PassParams {
     u32 shift;
     const u32* digit_base;  // [256] exclusive global offsets of this pass's digits
     u64* status;            // [n_tiles * 256], zeroed
-    u32* tile_ctr;          // zeroed
-    u32 tile0;              // tile index of blockIdx.x 0 (the TAIL launch holds the last, partial tile)
+    u32* tile_ctr;          // zeroed before the pass: tile tickets (the TAIL launch follows the full one)
 };
 
 // Mask of the lanes (within vmask) whose 8-bit digit equals this lane's.
@@ -95,19 +88,6 @@ template <int MODE>
 __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     if (MODE == 0) {
         return __match_any_sync(IGD_FULL, d) & vmask;
-    } else if (IGD_SORT_SKIPBITS) {
-        // ballot only the digit bits that differ somewhere in the warp (high digits of
-        // clustered words are often warp-uniform)
-        u32 peers = vmask;
-        u32 diff = (__reduce_or_sync(IGD_FULL, d) ^ __reduce_and_sync(IGD_FULL, d)) & 0xFFu;
-        while (diff) {
-            const u32 b = __ffs(diff) - 1;
-            diff &= diff - 1;
-            const u32 bit = (d >> b) & 1u;
-            const u32 bal = __ballot_sync(IGD_FULL, bit);
-            peers &= bit ? bal : ~bal;
-        }
-        return peers;
     } else {
         u32 peers = vmask;
 #pragma unroll
@@ -120,7 +100,7 @@ __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     }
 }
 
-// Dynamic shared memory of k_onesweep<MODE, VT>: staged keys, staged values, digit per position.
+// Dynamic shared memory of k_onesweep<VT>: staged keys, staged values, digit per position.
 template <typename VT>
 constexpr size_t onesweep_smem() {
     return (size_t)TILE * sizeof(u32) + (size_t)TILE * sizeof(VT) + TILE;
@@ -128,7 +108,7 @@ constexpr size_t onesweep_smem() {
 
 // TAIL = false: every tile of the launch is full (no bounds tests on the hot path); TAIL = true:
 // the one partial last tile, launched after the full ones (its look-back finds them published).
-template <int MODE, typename VT, bool TAIL>
+template <typename VT, bool TAIL>
 #ifndef IGD_SORT_MINB
 #define IGD_SORT_MINB 3
 #endif
@@ -139,7 +119,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     __shared__ u32 s_tile;
     __shared__ u32 s_wsum[WARPS];
     __shared__ u32 s_cnt[RADIX];  // tile digit counts (IGD_SORT_EARLY)
-    __shared__ u32 s_match[MODE == 2 ? WARPS : 1][RADIX];  // MODE 2: per-warp lane sets per digit
     __shared__ __align__(8) u64 s_mbar[2];
     extern __shared__ __align__(16) unsigned char s_dyn[];
     u32* s_k = reinterpret_cast<u32*>(s_dyn);                         // keys in, then keys out
@@ -151,8 +130,10 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     if (t == 0) {
         // tile id, then TMA bulk copies of the tile's keys and values into shared memory: the
-        // value copy lands while the keys are ranked
-        const u32 tile = P.tile0 + blockIdx.x;  // CTAs dispatch in blockIdx order (decoupled look-back)
+        // value copy lands while the keys are ranked.  The id is a ticket in CTA start order (the
+        // full-tile launch takes 0..full-1, the tail launch after it the last one), so a tile's
+        // look-back only waits on running tiles, whatever the dispatch order.
+        const u32 tile = atomicAdd(P.tile_ctr, 1u);
         s_tile = tile;
         const u64 base = (u64)tile * TILE;
         if (!TAIL) {
@@ -165,8 +146,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         }
     }
     for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_whist[0][0])[i] = 0;
-    if (MODE == 2)
-        for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_match[0][0])[i] = 0;
     if (IGD_SORT_EARLY) s_cnt[t] = 0;
     __syncthreads();
     const u32 tile = s_tile;
@@ -203,31 +182,17 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         const bool valid = full || wbase + j * 32 + lane < P.n;
         const u32 vmask = full ? IGD_FULL : __ballot_sync(IGD_FULL, valid);
         const u32 d = (key[j] >> shift) & 255u;
-        u32 peers;
-        if (MODE == 2) {
-            // lanes with digit d OR their bit into the warp's word for d; one shared atomic and
-            // one load per key instead of eight ballots (CUB's "match atomic-or" ranking)
-            if (valid) atomicOr(&s_match[MODE == 2 ? warp : 0][d], 1u << lane);
-            __syncwarp();
-            peers = valid ? s_match[MODE == 2 ? warp : 0][d] : (1u << lane);
-            __syncwarp();
-        } else {
-            // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set
-            // IGD_SORT_MIX: alternate rows between match.any (MIO pipe) and the 8 ballots (ALU /
-            // issue), which bottleneck on different units
-            // IGD_SORT_MIX = N: one row in N uses match.any; negative -N: all rows but one in N
-            if (IGD_SORT_MIX && MODE == 1 &&
-                (IGD_SORT_MIX > 0 ? (j % IGD_SORT_MIX) == IGD_SORT_MIX - 1 : (j % -IGD_SORT_MIX) != 0))
-                peers = peers_of<0>(valid ? d : (0x100u | lane), vmask);
-            else
-                peers = peers_of<MODE>(valid ? d : (0x100u | lane), vmask);
-        }
+        // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set.
+        // IGD_SORT_MIX = N: one row in N is ranked with match.any (MIO pipe), the others with the
+        // 8 ballots (ALU / issue): the two bottleneck on different units
+        const u32 peers = (IGD_SORT_MIX && (j % IGD_SORT_MIX) == IGD_SORT_MIX - 1)
+                              ? peers_of<0>(valid ? d : (0x100u | lane), vmask)
+                              : peers_of<1>(valid ? d : (0x100u | lane), vmask);
         const u32 leader = __ffs(peers) - 1;
         u32 old = 0;
         if (lane == leader && valid) {
             old = s_whist[warp][d];
             s_whist[warp][d] = old + __popc(peers);
-            if (MODE == 2) s_match[MODE == 2 ? warp : 0][d] = 0;
         }
         old = __shfl_sync(IGD_FULL, old, leader & 31u);
         rank[j] = old + __popc(peers & lt);
@@ -271,7 +236,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     {
         const u32 d = t;
         u64 excl = 0;
-        if (tile > 0 && !IGD_SORT_NOLOOKBACK) {  // NOLOOKBACK: timing experiment only (wrong output)
+        if (tile > 0) {
             long tt = (long)tile - 1;
             bool done = false;
             while (!done) {

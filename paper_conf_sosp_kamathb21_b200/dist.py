@@ -141,8 +141,15 @@ class GpuStage:
         self.det = det
         self.device = torch.device("cuda", det.device)
 
+    def _order(self):
+        """libigd runs on the Detector's stream: make it wait for the work the caller queued on
+        the current torch stream (e.g. the NCCL exchange that fills recv / sync buffers)."""
+        if self.device.type == "cuda":
+            self.det.stream.wait_stream(torch.cuda.current_stream(self.device))
+
     def load(self, chunk, first_event: int, n_total: int, n_blocks: int, block_dim: int):
         lib = _igd.load_library()
+        self._order()
         if isinstance(chunk, torch.Tensor):
             n = chunk.numel() * chunk.element_size() // 16
             ptr, flags = (chunk.data_ptr() if n else 0), _igd.IGD_TRACE_DEVICE_PTR
@@ -159,6 +166,7 @@ class GpuStage:
 
     def prepare(self, nranks: int):
         lib = _igd.load_library()
+        self._order()
         counts = (ctypes.c_uint64 * nranks)()
         nsync, bad = ctypes.c_uint64(), ctypes.c_uint64()
         mm = (ctypes.c_uint64 * 2)()
@@ -177,6 +185,7 @@ class GpuStage:
                paper_counters: bool = False) -> np.ndarray:
         lib = _igd.load_library()
         recv = recv.contiguous()
+        self._order()
         sync_idx = sync_idx.contiguous()
         sync_ev = sync_ev.contiguous()
         nrep = ctypes.c_uint64()

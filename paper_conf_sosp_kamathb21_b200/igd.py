@@ -187,6 +187,7 @@ class Detector:
         torch = self._torch
         if isinstance(events, torch.Tensor):
             assert events.is_cuda and events.is_contiguous() and events.numel() * events.element_size() % 16 == 0
+            assert events.data_ptr() % 16 == 0, "device events must be 16-byte aligned"
             n = events.numel() * events.element_size() // 16
             self._borrowed = events
             igd_trace_load(self.ctx, n_blocks, block_dim, events.data_ptr() if n else 0, n, True)

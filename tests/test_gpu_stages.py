@@ -1,5 +1,5 @@
 """Stage-level GPU tests: each kernel against a host reference of THAT stage.
-a5 radix sort: stable by key == numpy stable argsort (all three multisplit variants)."""
+a5 radix sort: stable by key == numpy stable argsort."""
 import ctypes
 
 import numpy as np
@@ -33,7 +33,7 @@ def gpu_sort(det, keys, vals, bits, mode):
     return k.cpu().numpy().view(np.uint32), v.cpu().numpy().view(np.uint32), ms.value
 
 
-@pytest.mark.parametrize("mode", [0, 1, 2])
+@pytest.mark.parametrize("mode", [1])
 @pytest.mark.parametrize("n,dist", [(1, "u"), (2, "u"), (4095, "u"), (4097, "u"), (1_000_003, "u"),
                                     (777_777, "skew"), (300_000, "const"), (2_000_001, "hi")])
 def test_radix_sort_stable(det, mode, n, dist):
