@@ -321,7 +321,8 @@ def main():
     n, nb, bd = plan.n_events, plan.n_blocks, plan.block_dim
     host = np.empty(n, igd.EVENT_DTYPE)
     plan.fill(out=host, threads=args.threads)
-    ledger_n = len(plan.ledger())
+    lg = plan.ledger()
+    ledger_n = len(lg)
     plan.close()
     log(f"[bench] {F.FAMILY_NAMES[fam]}: {n} events, {nb}x{bd} threads, generated in {time.time() - t0:.1f}s")
     cudart = torch.cuda.cudart()
@@ -425,6 +426,14 @@ def main():
     if pinned:
         cudart.cudaHostUnregister(host.ctypes.data)
 
+    # full-size parity against the generator's injection ledger, element by element on
+    # (addr, cur, prev, type): the whole report array, not just its length
+    ledger_match = None
+    if not (co or pc):
+        ledger_match = bool(len(lg) == len(reports)
+                            and np.array_equal(lg["addr"], reports["addr"]) and np.array_equal(lg["cur"], reports["cur"])
+                            and np.array_equal(lg["prev"], reports["prev"])
+                            and np.array_equal(lg["type"].astype(np.uint8), reports["type"]))
     kinds = np.bincount(((host["tk"] >> 24) & 0xF).astype(np.int64), minlength=12)
     f_acc = float(kinds[:5].sum()) / max(n, 1)
     b_alg = 16 + 32 * f_acc  # read the event + read/write a 16-B metadata entry per access
@@ -435,6 +444,7 @@ def main():
                 "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
                            "f_acc": f_acc, "reports": int(nrep),
                            "ledger_reports": None if (co or pc) else ledger_n,  # ledger: per-lane, exact IDs
+                           "ledger_match": ledger_match,
                            "check_mode": ("warp-coalesced (A32)" if co else "per-lane")
                            + (", paper-width IDs (A33)" if pc else ""),
                            "l2": "inputs larger than L2 (no flush)",
