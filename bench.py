@@ -147,15 +147,17 @@ def run_reference(args, fam, rank, world):
 
 
 def run_sharded(args, fam, rank, world, local):
-    """N GPUs (one process each): the trace is split into contiguous chunks, words are hash-sharded
-    and exchanged with NCCL all-to-all; sync streams all-gathered.  The same global
-    trace for every N (strong scaling); each rank generates only its chunk."""
+    """N GPUs (one process each) through the collective C ABI: every rank
+    creates an igd context with the same NCCL unique id (torch.distributed only broadcasts the
+    128-byte id and brackets the timed region), loads its contiguous chunk of the trace, and
+    igd_detect runs the partition, the NCCL all-to-all / all-gathers, the sharded check and the
+    report merge inside libigd.  The same global trace for every N (strong scaling); each rank
+    generates only its chunk.  --sharded at N=1: the one-rank collective path."""
     import torch
     import torch.distributed as dist
 
     import paper_conf_sosp_kamathb21_b200 as igd
     import tracegen.families as F
-    from paper_conf_sosp_kamathb21_b200 import dist as D
 
     torch.cuda.set_device(local % torch.cuda.device_count())
     dev_index = torch.cuda.current_device()
@@ -169,25 +171,31 @@ def run_sharded(args, fam, rank, world, local):
             dist.init_process_group("nccl", device_id=torch.device("cuda", dev_index))
         else:
             dist.init_process_group(args.backend)
-    comm = D.TorchComm()
+    tdev = f"cuda:{dev_index}" if args.backend == "nccl" else "cpu"
+    idt = torch.zeros(128, dtype=torch.uint8, device=tdev)
+    if rank == 0:
+        idt.copy_(torch.frombuffer(bytearray(igd.igd_nccl_unique_id()), dtype=torch.uint8))
+    dist.broadcast(idt, 0)
+    nccl_id = bytes(idt.cpu().numpy().tobytes())
+
     t0 = time.time()
     plan = F.Plan(fam, args.events or None)
     n, nb, bd = plan.n_events, plan.n_blocks, plan.block_dim
-    lo, cnt = D.chunk_bounds(n, world, rank)
+    lo = n * rank // world
+    cnt = n * (rank + 1) // world - lo
     host = np.empty(cnt, igd.EVENT_DTYPE)
     plan.fill(lo, cnt, out=host, threads=args.threads)
-    ledger_n = len(plan.ledger())
+    lg = plan.ledger()
     plan.close()
     if rank == 0:
         log(f"[bench] {F.FAMILY_NAMES[fam]}: {n} events over {world} ranks, chunk {cnt}, {time.time() - t0:.1f}s")
     cudart = torch.cuda.cudart()
     pinned = cudart.cudaHostRegister(host.ctypes.data, host.nbytes, 0) == 0
     chunk = torch.from_numpy(host.view(np.uint8)).to(f"cuda:{dev_index}")
-    det = igd.Detector(dev_index)
-    stage = D.GpuStage(det)
+    det = igd.Detector(dev_index, nranks=world, rank=rank, nccl_id=nccl_id)
+    det.load(chunk, nb, bd, first_event=lo, n_events_total=n)
     for _ in range(args.warmup):
-        stage.load(chunk, lo, n, nb, bd)
-        rep = D.sharded_detect(stage, comm)
+        nrep = det.detect()
     clocks = ClockSampler(dev_index)
     clocks.start()
     dist.barrier()
@@ -197,8 +205,7 @@ def run_sharded(args, fam, rank, world, local):
     kstats, launches = {}, 0
     e0.record(det.stream)
     for _ in range(args.steps):
-        stage.load(chunk, lo, n, nb, bd)
-        rep = D.sharded_detect(stage, comm, timing=True)
+        nrep = det.detect(timing=True)
         launches += det.launch_count()
         for k, (c, ms_, b) in det.kernel_stats().items():
             c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
@@ -208,23 +215,33 @@ def run_sharded(args, fam, rank, world, local):
     dist.barrier()
     clk = clocks.stop()
     ms = e0.elapsed_time(e1) / args.steps
-    ms = comm.allreduce_u64(int(ms * 1e6), "max", f"cuda:{dev_index}") / 1e6  # slowest rank
+    t = torch.tensor([ms], dtype=torch.float64, device=tdev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)  # slowest rank
+    ms = float(t.item())
     value = n / (ms / 1e3) / 1e9
-    # end to end: host chunk -> library H2D -> sharded check -> reports on the host
+    rep = det.reports()
+    ledger_match = bool(len(lg) == len(rep) and np.array_equal(lg["addr"], rep["addr"])
+                        and np.array_equal(lg["cur"], rep["cur"]) and np.array_equal(lg["prev"], rep["prev"])
+                        and np.array_equal(lg["type"].astype(np.uint8), rep["type"]))
+    # end to end: host chunk -> library H2D -> collective check -> global reports on the host
     del chunk
+    det.load(np.zeros(0, igd.EVENT_DTYPE), nb, bd, first_event=lo, n_events_total=n)
     torch.cuda.empty_cache()
     e2e_times = []
     for s in range(0 if args.no_e2e else args.e2e_steps + 1):
         dist.barrier()
         torch.cuda.synchronize()
-        t = time.perf_counter()
-        stage.load(host, lo, n, nb, bd)
-        out = D.sharded_detect(stage, comm)
+        t1 = time.perf_counter()
+        det.load(host, nb, bd, first_event=lo, n_events_total=n)
+        det.detect()
+        out = det.reports()
         torch.cuda.synchronize()
         if s > 0:
-            e2e_times.append(time.perf_counter() - t)
-    e2e_s = sum(e2e_times) / len(e2e_times) if e2e_times else float("inf")
-    e2e_s = comm.allreduce_u64(int(e2e_s * 1e9) if e2e_times else 1 << 62, "max", f"cuda:{dev_index}") / 1e9
+            e2e_times.append(time.perf_counter() - t1)
+    e2e_s = sum(e2e_times) / len(e2e_times) if e2e_times else 0.0
+    t = torch.tensor([e2e_s], dtype=torch.float64, device=tdev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    e2e_s = float(t.item())
     if pinned:
         cudart.cudaHostUnregister(host.ctypes.data)
     peak, peak_kind = peaks()
@@ -236,16 +253,17 @@ def run_sharded(args, fam, rank, world, local):
                 "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": "u32", "data": "synthetic",
                 "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
-                           "reports": int(len(rep)), "ledger_reports": ledger_n,
+                           "reports": int(nrep), "ledger_reports": int(len(lg)), "ledger_match": ledger_match,
                            "l2": "inputs larger than L2 (no flush)",
                            "parallelism": f"{world} ranks: contiguous trace chunks, words hash-sharded "
-                                          f"(fmix32 % P), {args.backend.upper()} all-to-all + all-gather"},
+                                          "(fmix32 % P); NCCL all-to-all + all-gathers inside libigd "
+                                          "(collective igd_detect)"},
                 "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                              "frac": achieved / peak, "peak_source": peak_kind, "traffic": None,
                              "launches_per_step": c / args.steps, "rank": 0},
                 "cpu_baseline": None,
                 "e2e": {"value": n / e2e_s / 1e9 if e2e_times else None, "unit": "G events/s",
-                        "h2d_bytes_per_step": n * 16, "d2h_bytes_per_step": int(len(rep)) * 32 * world,
+                        "h2d_bytes_per_step": n * 16, "d2h_bytes_per_step": int(len(out)) * 32 * world,
                         "ms_per_step": e2e_s * 1e3},
                 "gpu_launches": launches, "clocks": clk}
         print(json.dumps(line), flush=True)

@@ -33,7 +33,7 @@ extern "C" {
 #define IGD_ETOOBIG (-3) /* n_events >= 2^32-1, or the accessed word range spans >= 2^32 words */
 #define IGD_ENOMEM (-4)  /* device allocation failed */
 #define IGD_ECUDA (-5)   /* a CUDA runtime call failed; see igd_last_error() */
-#define IGD_ENCCL (-6)   /* reserved for the multi-GPU exchange */
+#define IGD_ENCCL (-6)   /* an NCCL call failed, or libnccl.so.2 could not be loaded (multi-GPU) */
 #define IGD_ESTATE (-7)  /* call out of order (e.g. igd_detect before igd_trace_load) */
 
 /* ---- trace event: 16 bytes, little-endian, arrays 16-byte aligned ---------------- */
@@ -122,9 +122,15 @@ typedef void (*igd_free_fn)(void* p, void* stream, void* user);
 typedef struct igd_ctx igd_ctx; /* opaque; owns every device buffer it allocates */
 
 /* Create a context on `cuda_device`, issuing all work on `cuda_stream` (a cudaStream_t;
-   NULL = the legacy default stream).  nranks must be 1 in this build (multi-GPU sharding
-   is driven from the host binding; IGD_EINVAL otherwise).  nccl_unique_id is ignored when
-   nranks == 1 and may be NULL. */
+   NULL = the legacy default stream).
+   Multi-GPU: nranks > 1 processes (one per GPU) each create a context with their
+   rank in [0, nranks) and the SAME 128-byte NCCL unique id (igd_nccl_unique_id on one rank,
+   shared by the caller, e.g. a torch.distributed broadcast).  The call initialises an NCCL
+   communicator (ncclCommInitRank: blocks until every rank joins) and makes igd_detect collective.
+   nranks == 1 with a non-NULL id gives a one-rank communicator (the collective path on one GPU);
+   nranks == 1 with NULL is the single-GPU pipeline.  IGD_EINVAL: rank out of range, nranks > 1
+   without an id, one of alloc_fn / free_fn NULL; IGD_ENCCL: libnccl unavailable or the
+   communicator could not be created. */
 int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks, int rank,
                    const uint8_t* nccl_unique_id, igd_alloc_fn alloc_fn, igd_free_fn free_fn,
                    void* alloc_user);
@@ -155,6 +161,19 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
    Also accepted by igd_shard_detect. */
 #define IGD_DETECT_PAPER_COUNTERS 4u
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
+/* Collective contexts (created with an NCCL id): every rank calls igd_detect after loading its
+   contiguous chunk [desc.first_event, desc.first_event + desc.n_events) of one global trace of
+   desc.n_events_total events (chunks in rank order, covering the trace).  Words are
+   hash-sharded (owner = fmix32(low 32 bits of the word) % nranks); the access records move to
+   their owner by an NCCL all-to-all, the synchronization streams are all-gathered, each rank
+   checks the words it owns, and the reports are all-gathered and merged: every rank returns the
+   identical global report set (igd_reports), equal to the single-GPU result.  Errors are agreed
+   across ranks (the first invalid GLOBAL index for IGD_ETRACE), so every rank returns the same
+   code.  IGD_DETECT_COALESCE is rejected (IGD_EINVAL). */
+
+/* A fresh 128-byte NCCL unique id for igd_ctx_create (call on one rank, share with the others).
+   IGD_ENCCL when libnccl cannot be loaded. */
+int igd_nccl_unique_id(uint8_t* out128);
 
 /* ---- multi-GPU sharding, driven by the host over torch.distributed / NCCL ----
    Each rank loads its contiguous chunk with igd_trace_load (desc.first_event = global index of

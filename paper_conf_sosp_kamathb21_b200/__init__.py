@@ -6,4 +6,5 @@ every step of the check runs in the CUDA kernels, and loading fails loudly when 
 library or a GPU is missing.
 """
 from .igd import (EVENT_DTYPE, REPORT_DTYPE, Detector, IgdError, igd_ctx_create, igd_ctx_destroy,  # noqa: F401
-                  igd_detect, igd_reports, igd_strerror, igd_trace_load, lib_path, load_library)
+                  igd_detect, igd_nccl_unique_id, igd_reports, igd_strerror, igd_trace_load, lib_path,
+                  load_library)

@@ -98,6 +98,9 @@ constexpr size_t smem_bytes() {
                                                                      : (size_t)TILE * 14 + WARPS * RADIX * 4;
 }
 
+// COAL: warp-coalesced mode (A32) -- a separate instantiation so the default path carries no
+// skip-bit test (ncu r02b: 6% of the kernel's instructions)
+template <bool COAL>
 __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params P) {
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
@@ -156,7 +159,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
         const u32 p = wofs + j * 32 + lane;
         FDec d = fdecode(s_ev[p], g, ks);  // valid: ingest pass 0 checked every event
         const bool in = p < tile_e;
-        if (P.skip_bits && d.acc && in && ((__ldg(P.skip_bits + ((base + p) >> 5)) >> (p & 31u)) & 1u))
+        if (COAL && d.acc && in && ((__ldg(P.skip_bits + ((base + p) >> 5)) >> (p & 31u)) & 1u))
             d.acc = false;  // A32: checked by its coalesced group's first lane
         key[j] = d.key;
         tk[j] = d.tk;

@@ -22,6 +22,8 @@
 #include "sort.cuh"
 #include "shard.cuh"
 #include "sync.cuh"
+#include <dlfcn.h>
+#include <nccl.h>  // types and prototypes only: the library is resolved at run time (NcclApi)
 #include <vector>
 
 namespace {
@@ -40,11 +42,70 @@ constexpr int kMaxTimed = 128;
 const char* kStageNames[IGD_N_STAGES] = {"ingest", "sync_sort", "epoch_lock_tables", "access_sort",
                                          "check", "report_sort", "host_sync", "total"};
 
+// ---- NCCL, resolved at run time -------------------------------------------------------------
+// A process that uses torch.distributed already has torch's libnccl loaded: RTLD_NOLOAD finds that
+// copy, so libigd's communicator and torch's come from one library.  Otherwise the system
+// libnccl.so.2 is loaded.  Only multi-rank contexts need it (igd_ctx_create with an NCCL id).
+struct NcclApi {
+    bool ok = false;
+    std::string why;
+    decltype(&ncclGetUniqueId) GetUniqueId = nullptr;
+    decltype(&ncclCommInitRank) CommInitRank = nullptr;
+    decltype(&ncclCommDestroy) CommDestroy = nullptr;
+    decltype(&ncclAllReduce) AllReduce = nullptr;
+    decltype(&ncclAllGather) AllGather = nullptr;
+    decltype(&ncclBroadcast) Broadcast = nullptr;
+    decltype(&ncclSend) Send = nullptr;
+    decltype(&ncclRecv) Recv = nullptr;
+    decltype(&ncclGroupStart) GroupStart = nullptr;
+    decltype(&ncclGroupEnd) GroupEnd = nullptr;
+    decltype(&ncclGetErrorString) GetErrorString = nullptr;
+};
+NcclApi load_nccl() {
+    NcclApi a;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) {
+        const char* e = dlerror();
+        a.why = std::string("cannot load libnccl.so.2: ") + (e ? e : "?");
+        return a;
+    }
+#define IGD_NCCL_SYM(F)                                                  \
+    a.F = reinterpret_cast<decltype(a.F)>(dlsym(h, "nccl" #F));          \
+    if (!a.F) {                                                          \
+        a.why = "libnccl lacks nccl" #F;                                 \
+        return a;                                                        \
+    }
+    IGD_NCCL_SYM(GetUniqueId)
+    IGD_NCCL_SYM(CommInitRank)
+    IGD_NCCL_SYM(CommDestroy)
+    IGD_NCCL_SYM(AllReduce)
+    IGD_NCCL_SYM(AllGather)
+    IGD_NCCL_SYM(Broadcast)
+    IGD_NCCL_SYM(Send)
+    IGD_NCCL_SYM(Recv)
+    IGD_NCCL_SYM(GroupStart)
+    IGD_NCCL_SYM(GroupEnd)
+    IGD_NCCL_SYM(GetErrorString)
+#undef IGD_NCCL_SYM
+    a.ok = true;
+    return a;
+}
+NcclApi& nccl() {
+    static NcclApi api = load_nccl();
+    return api;
+}
+
 }  // namespace
 
 struct igd_ctx {
     int device = 0;
     cudaStream_t stream = nullptr;
+    // multi-GPU: an NCCL communicator makes igd_detect collective
+    int nranks = 1, rank = 0;
+    ncclComm_t comm = nullptr;
+    Buf cl_small, cl_mat, cl_recv, cl_sidx, cl_sev, cl_nrep, cl_rep;
     igd_alloc_fn afn = nullptr;
     igd_free_fn ffn = nullptr;
     void* auser = nullptr;
@@ -127,6 +188,14 @@ struct KTimer {
     do {                         \
         int r_ = (x);            \
         if (r_ != IGD_OK) return r_; \
+    } while (0)
+#define NK(call)                                                                               \
+    do {                                                                                       \
+        ncclResult_t e_ = (call);                                                              \
+        if (e_ != ncclSuccess) {                                                               \
+            ctx->err = std::string(#call) + ": " + nccl().GetErrorString(e_);                  \
+            return IGD_ENCCL;                                                                  \
+        }                                                                                      \
     } while (0)
 
 static int buf_free(igd_ctx* ctx, Buf& b) {
@@ -295,6 +364,48 @@ static int scan_excl(igd_ctx* ctx, u32* data, u64 n) {
     return IGD_OK;
 }
 
+// a7: reports `in[0..n)` (one per access, unique `cur` < n_time) in ascending `cur` order into
+// ctx->rep_out: a radix sort of the u32 keys cur, then a gather.
+static int canon_reports(igd_ctx* ctx, const igd_report* in, u64 n, u64 n_time) {
+    RET(ensure(ctx, ctx->rep_out, (n ? n : 1) * sizeof(igd_report)));
+    if (n == 1 && in != P_<igd_report>(ctx->rep_out)) {
+        CK(cudaMemcpyAsync(ctx->rep_out.p, in, sizeof(igd_report), cudaMemcpyDeviceToDevice, ctx->stream));
+    } else if (n > 1) {
+        const int sms = sm_count(ctx);
+        for (int b = 0; b < 2; b++) {
+            RET(ensure(ctx, ctx->rep_k[b], n * sizeof(u32)));
+            RET(ensure(ctx, ctx->rep_v[b], n * sizeof(u32)));
+        }
+        RET(ensure(ctx, ctx->rep_hist, 1024 * sizeof(u32)));
+        unsigned blocks = (unsigned)std::min<u64>((n + 255) / 256, (u64)sms * 8);
+        {
+            KTimer kt(ctx, KC_REPORT, 40.0 * (double)n);
+            check::k_report_keys<<<blocks, 256, 0, ctx->stream>>>(in, (u32)n, 0, P_<u32>(ctx->rep_k[0]),
+                                                                P_<u32>(ctx->rep_v[0]));
+        }
+        CK(cudaMemsetAsync(ctx->rep_hist.p, 0, 1024 * sizeof(u32), ctx->stream));
+        {
+            KTimer kt(ctx, KC_REPORT, 4.0 * (double)n);
+            rsort::k_hist4<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->rep_k[0]), n, P_<u32>(ctx->rep_hist));
+        }
+        CK(cudaMemcpyAsync(ctx->h_hist + 2048, ctx->rep_hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost,
+                           ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        u32 hh[1024];
+        memcpy(hh, ctx->h_hist + 2048, sizeof(hh));
+        int rcur = 0;
+        RET(radix_sort(ctx, KC_REPORT, ctx->rep_k, ctx->rep_v, n, P_<u32>(ctx->rep_hist), hh,
+                       bits_needed(n_time ? n_time - 1 : 0), &rcur));
+        {
+            KTimer kt(ctx, KC_REPORT, 68.0 * (double)n);
+            check::k_report_gather<<<blocks, 256, 0, ctx->stream>>>(in, P_<u32>(ctx->rep_v[rcur]), (u32)n,
+                                                                   P_<igd_report>(ctx->rep_out));
+        }
+        CK(cudaGetLastError());
+    }
+    return IGD_OK;
+}
+
 // The pipeline.  Single GPU: the trace is `ctx->events`.  Sharded (ctx->shard): the
 // synchronization side runs over the all-gathered sync stream (global timestamps in sh_sidx),
 // the access side over the records this rank received in the all-to-all.
@@ -437,7 +548,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         {
             // reads every event once, writes the 12-byte access records and 8-byte sync records
             KTimer kt(ctx, KC_FUSED, 16.0 * (double)n_src + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
-            fused::k_ingest_sort0<<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
+            if (fp.skip_bits)
+                fused::k_ingest_sort0<true><<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
+            else
+                fused::k_ingest_sort0<false><<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
         }
         CK(cudaGetLastError());
     }
@@ -616,42 +730,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     }
     mark(ctx, 5);
     // ---------------- a7: canonical order (ascending cur) ----------------
-    RET(ensure(ctx, ctx->rep_out, (n_rep ? n_rep : 1) * sizeof(igd_report)));
-    if (n_rep == 1) {
-        CK(cudaMemcpyAsync(ctx->rep_out.p, ctx->rep_raw.p, sizeof(igd_report), cudaMemcpyDeviceToDevice, ctx->stream));
-    } else if (n_rep > 1) {
-        for (int b = 0; b < 2; b++) {
-            RET(ensure(ctx, ctx->rep_k[b], n_rep * sizeof(u32)));
-            RET(ensure(ctx, ctx->rep_v[b], n_rep * sizeof(u32)));
-        }
-        RET(ensure(ctx, ctx->rep_hist, 1024 * sizeof(u32)));
-        unsigned blocks = (unsigned)std::min<u64>((n_rep + 255) / 256, (u64)sms * 8);
-        {
-            KTimer kt(ctx, KC_REPORT, 40.0 * (double)n_rep);
-            check::k_report_keys<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw), (u32)n_rep, 0,
-                                                                P_<u32>(ctx->rep_k[0]), P_<u32>(ctx->rep_v[0]));
-        }
-        CK(cudaMemsetAsync(ctx->rep_hist.p, 0, 1024 * sizeof(u32), ctx->stream));
-        {
-            KTimer kt(ctx, KC_REPORT, 4.0 * (double)n_rep);
-            rsort::k_hist4<<<blocks, 256, 0, ctx->stream>>>(P_<u32>(ctx->rep_k[0]), n_rep, P_<u32>(ctx->rep_hist));
-        }
-        CK(cudaMemcpyAsync(ctx->h_hist + 2048, ctx->rep_hist.p, 1024 * sizeof(u32), cudaMemcpyDeviceToHost,
-                           ctx->stream));
-        CK(cudaStreamSynchronize(ctx->stream));
-        u32 hh[1024];
-        memcpy(hh, ctx->h_hist + 2048, sizeof(hh));
-        int rcur = 0;
-        RET(radix_sort(ctx, KC_REPORT, ctx->rep_k, ctx->rep_v, n_rep, P_<u32>(ctx->rep_hist), hh, bits_needed(n - 1),
-                       &rcur));
-        {
-            KTimer kt(ctx, KC_REPORT, 68.0 * (double)n_rep);
-            check::k_report_gather<<<blocks, 256, 0, ctx->stream>>>(P_<igd_report>(ctx->rep_raw),
-                                                                   P_<u32>(ctx->rep_v[rcur]), (u32)n_rep,
-                                                                   P_<igd_report>(ctx->rep_out));
-        }
-        CK(cudaGetLastError());
-    }
+    RET(canon_reports(ctx, P_<igd_report>(ctx->rep_raw), n_rep, n));
     mark(ctx, 6);
     CK(cudaStreamSynchronize(ctx->stream));
     mark(ctx, 7);
@@ -737,15 +816,151 @@ static int shard_prepare_impl(igd_ctx* ctx, u32 P, u64* counts, u64* n_sync_stre
     return IGD_OK;
 }
 
+// ---------------- multi-GPU collective check ----------------
+// Every rank holds the contiguous global range [first_event, first_event + n_events) of one trace.
+// 1. partition the chunk: access records grouped by owner rank fmix32(word) % P, and the
+//    synchronization stream (shard_prepare_impl);
+// 2. NCCL: one all-reduce of {first bad index, min word, ~max word, local error} (min), an
+//    all-gather of every rank's per-owner record counts and sync-stream length;
+// 3. NCCL: all-to-all of the record groups (grouped send / recv: received groups land in
+//    source-rank order = trace order, so the stable radix sort keeps (word, time) order) and the
+//    sync streams of all ranks broadcast into one global stream (rank order = trace order);
+// 4. the words this rank owns are checked against the rebuilt global sync / lock tables
+//    (detect_impl, sharded mode);
+// 5. NCCL: every rank's reports are broadcast to all, then merged by `cur` (a7).
+// Every rank returns the same global report set.  Errors found by any rank (bad event, word span,
+// a local allocation failure) are agreed through step 2, so no rank is left inside a collective.
+static int collective_detect(igd_ctx* ctx, u64* n_out) {
+    NcclApi& N = nccl();
+    const u32 P = (u32)ctx->nranks, me = (u32)ctx->rank;
+    const ncclComm_t comm = ctx->comm;
+    cudaStream_t st = ctx->stream;
+    *n_out = 0;
+    ctx->n_reports = 0;
+    ctx->launches = 0;
+    ctx->nk = 0;
+    std::vector<u64> counts(P + 1, 0);
+    u64 nsync = 0, bad = ~0ull, mm[2] = {~0ull, 0};
+    RET(ensure(ctx, ctx->cl_small, 8 * sizeof(u64)));
+    int lrc = shard_prepare_impl(ctx, P, counts.data(), &nsync, &bad, mm);
+    u64 small[4] = {bad, mm[0], mm[0] == ~0ull ? ~0ull : ~mm[1], lrc == IGD_OK ? ~0ull : (u64)(-lrc)};
+    CK(cudaMemcpyAsync(ctx->cl_small.p, small, sizeof(small), cudaMemcpyHostToDevice, st));
+    NK(N.AllReduce(ctx->cl_small.p, ctx->cl_small.p, 4, ncclUint64, ncclMin, comm, st));
+    CK(cudaMemcpyAsync(small, ctx->cl_small.p, sizeof(small), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (small[3] != ~0ull) {
+        if (lrc == IGD_OK) ctx->err = "another rank failed in the partition stage (" + std::to_string(-(int64_t)small[3]) + ")";
+        return -(int)small[3];
+    }
+    if (small[0] != ~0ull) {
+        ctx->bad_event = small[0];
+        ctx->err = "invalid event at global index " + std::to_string(small[0]);
+        return IGD_ETRACE;
+    }
+    const bool any_acc = small[1] != ~0ull;
+    const u64 wmin = any_acc ? small[1] : 0, wmax = any_acc ? ~small[2] : 0;
+    if (any_acc && wmax - wmin >= (1ull << 32)) {
+        ctx->err = "accessed word range spans >= 2^32 words";
+        return IGD_ETOOBIG;
+    }
+    // count matrix: row r = rank r's records per owner, then its sync-stream length
+    const u64 W = P + 1;
+    RET(ensure(ctx, ctx->cl_mat, (W * P + W) * sizeof(u64)));
+    counts[P] = nsync;
+    CK(cudaMemcpyAsync(P_<u64>(ctx->cl_mat) + W * P, counts.data(), W * sizeof(u64), cudaMemcpyHostToDevice, st));
+    NK(N.AllGather(P_<u64>(ctx->cl_mat) + W * P, ctx->cl_mat.p, W, ncclUint64, comm, st));
+    std::vector<u64> M(W * P);
+    CK(cudaMemcpyAsync(M.data(), ctx->cl_mat.p, W * P * sizeof(u64), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    std::vector<u64> soff(P + 1, 0), roff(P + 1, 0), yoff(P + 1, 0);
+    for (u32 r = 0; r < P; r++) {
+        soff[r + 1] = soff[r] + M[me * W + r];  // my records for owner r
+        roff[r + 1] = roff[r] + M[r * W + me];  // records rank r sends me
+        yoff[r + 1] = yoff[r] + M[r * W + P];   // rank r's sync stream
+    }
+    const u64 nrecv = roff[P], nsy = yoff[P];
+    if (nsy + 64 > 0xFFFFFFFFull || nrecv > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;
+    RET(ensure(ctx, ctx->cl_recv, (nrecv + 1) * 16));
+    RET(ensure(ctx, ctx->cl_sidx, (nsy + 1) * sizeof(u32)));
+    RET(ensure(ctx, ctx->cl_sev, (nsy + 1) * 16));
+    {
+        // all-to-all of the access records (one grouped send / receive per peer, self included)
+        NK(N.GroupStart());
+        for (u32 r = 0; r < P; r++) {
+            const u64 ns = M[me * W + r], nr = M[r * W + me];
+            if (ns) NK(N.Send((const char*)ctx->sh_send.p + soff[r] * 16, ns * 16, ncclUint8, (int)r, comm, st));
+            if (nr) NK(N.Recv((char*)ctx->cl_recv.p + roff[r] * 16, nr * 16, ncclUint8, (int)r, comm, st));
+        }
+        NK(N.GroupEnd());
+        // the synchronization streams, concatenated in rank order (a variable all-gather)
+        NK(N.GroupStart());
+        for (u32 r = 0; r < P; r++) {
+            const u64 c = M[r * W + P];
+            if (!c) continue;
+            u32* di = P_<u32>(ctx->cl_sidx) + yoff[r];
+            char* de = (char*)ctx->cl_sev.p + yoff[r] * 16;
+            NK(N.Broadcast(r == me ? ctx->sh_sidx_buf.p : di, di, c, ncclUint32, (int)r, comm, st));
+            NK(N.Broadcast(r == me ? ctx->sh_sev_buf.p : de, de, c * 16, ncclUint8, (int)r, comm, st));
+        }
+        NK(N.GroupEnd());
+    }
+    RET(buf_free(ctx, ctx->sh_send));  // stream-ordered: after the sends
+    // the words this rank owns
+    ctx->shard = true;
+    ctx->sh_rec = ctx->cl_recv.p;
+    ctx->sh_nrec = nrecv;
+    ctx->sh_sidx = P_<u32>(ctx->cl_sidx);
+    ctx->sh_sev = ctx->cl_sev.p;
+    ctx->sh_ns = nsy;
+    ctx->sh_wbase = wmin;
+    ctx->sh_ntotal = ctx->desc.n_events_total ? ctx->desc.n_events_total : ctx->desc.n_events;
+    u64 nloc = 0;
+    lrc = detect_impl(ctx, &nloc);
+    ctx->shard = false;
+    // agree on success, then every rank's reports to every rank
+    RET(ensure(ctx, ctx->cl_nrep, 2 * P * sizeof(u64)));
+    u64 mine[2] = {lrc == IGD_OK ? nloc : 0, lrc == IGD_OK ? 0 : (u64)(-lrc)};
+    CK(cudaMemcpyAsync(P_<u64>(ctx->cl_nrep) + 2 * me, mine, sizeof(mine), cudaMemcpyHostToDevice, st));
+    NK(N.AllGather(P_<u64>(ctx->cl_nrep) + 2 * me, ctx->cl_nrep.p, 2, ncclUint64, comm, st));
+    std::vector<u64> NR(2 * P);
+    CK(cudaMemcpyAsync(NR.data(), ctx->cl_nrep.p, 2 * P * sizeof(u64), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    for (u32 r = 0; r < P; r++)
+        if (NR[2 * r + 1]) {
+            if (lrc == IGD_OK) ctx->err = "rank " + std::to_string(r) + " failed in the check stage";
+            return -(int)NR[2 * r + 1];
+        }
+    u64 total = 0;
+    std::vector<u64> off(P + 1, 0);
+    for (u32 r = 0; r < P; r++) off[r + 1] = off[r] + NR[2 * r];
+    total = off[P];
+    if (P > 1) {
+        RET(ensure(ctx, ctx->cl_rep, (total ? total : 1) * sizeof(igd_report)));
+        NK(N.GroupStart());
+        for (u32 r = 0; r < P; r++) {
+            const u64 c = NR[2 * r];
+            if (!c) continue;
+            char* d = (char*)ctx->cl_rep.p + off[r] * sizeof(igd_report);
+            NK(N.Broadcast(r == me ? ctx->rep_out.p : d, d, c * sizeof(igd_report), ncclUint8, (int)r, comm, st));
+        }
+        NK(N.GroupEnd());
+        RET(canon_reports(ctx, P_<igd_report>(ctx->cl_rep), total, ctx->sh_ntotal));
+    }
+    CK(cudaStreamSynchronize(st));
+    ctx->n_reports = total;
+    *n_out = total;
+    return IGD_OK;
+}
+
 // ================================ C ABI =====================================================
 extern "C" {
 
 int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks, int rank,
                    const uint8_t* nccl_unique_id, igd_alloc_fn alloc_fn, igd_free_fn free_fn, void* alloc_user) {
-    (void)nccl_unique_id;
     if (!out) return IGD_EINVAL;
     *out = nullptr;
-    if (nranks != 1 || rank != 0) return IGD_EINVAL;
+    if (nranks < 1 || rank < 0 || rank >= nranks) return IGD_EINVAL;
+    if (nranks > 1 && !nccl_unique_id) return IGD_EINVAL;
     if ((alloc_fn == nullptr) != (free_fn == nullptr)) return IGD_EINVAL;
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
@@ -760,7 +975,9 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     ctx->ffn = free_fn;
     ctx->auser = alloc_user;
     if (const char* m = getenv("IGD_FUSED")) ctx->fused = atoi(m) != 0;
-    cudaFuncSetAttribute(fused::k_ingest_sort0, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(fused::k_ingest_sort0<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)fused::smem_bytes());
+    cudaFuncSetAttribute(fused::k_ingest_sort0<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes());
     set_pass_smem<u32>();
     set_pass_smem<u64>();
@@ -778,6 +995,24 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
         ctx->cls_ms[i] = 0.f;
         ctx->cls_n[i] = 0;
         ctx->cls_bytes[i] = 0;
+    }
+    ctx->nranks = nranks;
+    ctx->rank = rank;
+    if (nccl_unique_id) {
+        // a communicator (also for nranks == 1: the collective path on one GPU); blocks until
+        // every rank has joined
+        NcclApi& N = nccl();
+        if (!N.ok) {
+            igd_ctx_destroy(ctx);
+            return IGD_ENCCL;
+        }
+        ncclUniqueId id;
+        memcpy(&id, nccl_unique_id, sizeof(id));
+        if (N.CommInitRank(&ctx->comm, nranks, id, rank) != ncclSuccess) {
+            ctx->comm = nullptr;
+            igd_ctx_destroy(ctx);
+            return IGD_ENCCL;
+        }
     }
     *out = ctx;
     return IGD_OK;
@@ -821,6 +1056,19 @@ static void collect_timing(igd_ctx* ctx);
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     if (!ctx || !n_reports_global) return IGD_EINVAL;
     if (!ctx->loaded) return IGD_ESTATE;
+    if (ctx->comm) {  // collective over the communicator's ranks
+        if (flags & IGD_DETECT_COALESCE) {  // reading A32: a group may straddle two ranks' chunks
+            ctx->err = "IGD_DETECT_COALESCE is a single-context mode";
+            return IGD_EINVAL;
+        }
+        cudaSetDevice(ctx->device);
+        ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
+        ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
+        int rc = collective_detect(ctx, n_reports_global);
+        ctx->paper_counters = false;
+        if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
+        return rc;
+    }
     if (ctx->desc.first_event != 0 ||
         (ctx->desc.n_events_total != 0 && ctx->desc.n_events_total != ctx->desc.n_events)) {
         ctx->err = "igd_detect checks a whole trace; a rank's chunk goes through igd_shard_*";
@@ -959,16 +1207,32 @@ int igd_kernel_stats(const igd_ctx* ctx, int kclass, const char** name, uint32_t
     return IGD_OK;
 }
 
+int igd_nccl_unique_id(uint8_t* out128) {
+    if (!out128) return IGD_EINVAL;
+    NcclApi& N = nccl();
+    if (!N.ok) return IGD_ENCCL;
+    ncclUniqueId id;
+    if (N.GetUniqueId(&id) != ncclSuccess) return IGD_ENCCL;
+    memcpy(out128, &id, sizeof(id));
+    return IGD_OK;
+}
+
 void igd_ctx_destroy(igd_ctx* ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->device);
+    if (ctx->comm) {
+        nccl().CommDestroy(ctx->comm);
+        ctx->comm = nullptr;
+    }
     Buf* all[] = {&ctx->owned_events, &ctx->acc_k[0], &ctx->acc_k[1], &ctx->acc_v[0], &ctx->acc_v[1],
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
                   &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->tcnt,
                   &ctx->tpts,         &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
-                  &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf};
+                  &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf,
+                  &ctx->cl_small,     &ctx->cl_mat,   &ctx->cl_recv,  &ctx->cl_sidx,  &ctx->cl_sev,
+                  &ctx->cl_nrep,      &ctx->cl_rep};
     for (Buf* b : all) buf_free(ctx, *b);
     cudaStreamSynchronize(ctx->stream);
     cudaFreeHost(ctx->h_stats);
@@ -987,7 +1251,7 @@ const char* igd_strerror(int code) {
         case IGD_ETOOBIG: return "trace too large for the 32-bit index path";
         case IGD_ENOMEM: return "device out of memory";
         case IGD_ECUDA: return "CUDA error";
-        case IGD_ENCCL: return "NCCL error";
+        case IGD_ENCCL: return "NCCL error (or libnccl unavailable)";
         case IGD_ESTATE: return "call out of order";
         default: return "unknown error";
     }

@@ -81,6 +81,8 @@ def load_library(build_if_missing: bool = True):
     lib.igd_shard_buffers.restype = i32
     lib.igd_shard_detect.argtypes = [vp, vp, u64, vp, vp, u64, u64, u32, ctypes.POINTER(u64)]
     lib.igd_shard_detect.restype = i32
+    lib.igd_nccl_unique_id.argtypes = [vp]
+    lib.igd_nccl_unique_id.restype = i32
     lib.igd_ctx_destroy.argtypes = [vp]
     lib.igd_ctx_destroy.restype = None
     lib.igd_strerror.argtypes = [i32]
@@ -103,20 +105,36 @@ def igd_strerror(code: int) -> str:
     return load_library().igd_strerror(code).decode()
 
 
+def igd_nccl_unique_id() -> bytes:
+    """A fresh 128-byte NCCL unique id (rank 0 creates it, the caller shares it with the others)."""
+    buf = (ctypes.c_uint8 * 128)()
+    rc = load_library().igd_nccl_unique_id(buf)
+    if rc != IGD_OK:
+        raise IgdError(rc, "igd_nccl_unique_id")
+    return bytes(buf)
+
+
 def igd_ctx_create(cuda_device: int, cuda_stream: int, alloc_fn=None, free_fn=None, nranks: int = 1,
-                   rank: int = 0):
+                   rank: int = 0, nccl_id: bytes = None):
     lib = load_library()
     ctx = ctypes.c_void_p()
-    rc = lib.igd_ctx_create(ctypes.byref(ctx), cuda_device, ctypes.c_void_p(cuda_stream), nranks, rank, None,
+    idbuf = None
+    if nccl_id is not None:
+        assert len(nccl_id) == 128
+        idbuf = (ctypes.c_uint8 * 128).from_buffer_copy(nccl_id)
+    rc = lib.igd_ctx_create(ctypes.byref(ctx), cuda_device, ctypes.c_void_p(cuda_stream), nranks, rank,
+                            ctypes.cast(idbuf, ctypes.c_void_p) if idbuf is not None else None,
                             alloc_fn or ALLOC_FN(), free_fn or FREE_FN(), None)
     if rc != IGD_OK:
         raise IgdError(rc, "igd_ctx_create")
     return ctx
 
 
-def igd_trace_load(ctx, n_blocks: int, block_dim: int, events_ptr: int, n_events: int, device_ptr: bool):
+def igd_trace_load(ctx, n_blocks: int, block_dim: int, events_ptr: int, n_events: int, device_ptr: bool,
+                   first_event: int = 0, n_events_total: int = None):
     lib = load_library()
-    d = igd_trace_desc(n_blocks, block_dim, n_events, 0, n_events, IGD_TRACE_DEVICE_PTR if device_ptr else 0)
+    d = igd_trace_desc(n_blocks, block_dim, n_events if n_events_total is None else n_events_total, first_event,
+                       n_events, IGD_TRACE_DEVICE_PTR if device_ptr else 0)
     rc = lib.igd_trace_load(ctx, ctypes.byref(d), ctypes.c_void_p(events_ptr or None))
     if rc != IGD_OK:
         raise IgdError(rc, lib.igd_last_error(ctx).decode())
@@ -153,7 +171,11 @@ class Detector:
     ``load`` accepts a host numpy EVENT_DTYPE array (copied by the library) or a CUDA
     tensor of the same bytes (borrowed: kept alive here until the next load)."""
 
-    def __init__(self, device: int = 0, stream=None):
+    def __init__(self, device: int = 0, stream=None, nranks: int = 1, rank: int = 0, nccl_id: bytes = None):
+        """``nranks`` / ``rank`` / ``nccl_id``: a collective context (one process per GPU, the same
+        id on every rank; igd_nccl_unique_id on one of them) -- detect() is then collective and
+        returns the global report set on every rank.  nranks == 1 with an id: the collective path
+        on one GPU."""
         import torch
 
         if not torch.cuda.is_available():
@@ -179,23 +201,28 @@ class Detector:
 
         self._afn = ALLOC_FN(_alloc)
         self._ffn = FREE_FN(_free)
-        self.ctx = igd_ctx_create(device, self.stream.cuda_stream, self._afn, self._ffn)
+        self.nranks, self.rank = nranks, rank
+        self.ctx = igd_ctx_create(device, self.stream.cuda_stream, self._afn, self._ffn, nranks, rank, nccl_id)
         self._borrowed = None
         self.n_reports = 0
 
-    def load(self, events, n_blocks: int, block_dim: int):
+    def load(self, events, n_blocks: int, block_dim: int, first_event: int = 0, n_events_total: int = None):
+        """Attach a trace (or, on a collective context, this rank's chunk starting at global index
+        ``first_event`` of an ``n_events_total``-event trace)."""
         torch = self._torch
         if isinstance(events, torch.Tensor):
             assert events.is_cuda and events.is_contiguous() and events.numel() * events.element_size() % 16 == 0
             assert events.data_ptr() % 16 == 0, "device events must be 16-byte aligned"
             n = events.numel() * events.element_size() // 16
             self._borrowed = events
-            igd_trace_load(self.ctx, n_blocks, block_dim, events.data_ptr() if n else 0, n, True)
+            igd_trace_load(self.ctx, n_blocks, block_dim, events.data_ptr() if n else 0, n, True, first_event,
+                           n_events_total)
         else:
             ev = np.ascontiguousarray(events)
             assert ev.dtype.itemsize == 16
             self._borrowed = None
-            igd_trace_load(self.ctx, n_blocks, block_dim, ev.ctypes.data if len(ev) else 0, len(ev), False)
+            igd_trace_load(self.ctx, n_blocks, block_dim, ev.ctypes.data if len(ev) else 0, len(ev), False,
+                           first_event, n_events_total)
 
     def detect(self, timing: bool = False, coalesce: bool = False, paper_counters: bool = False) -> int:
         """igd_detect; ``coalesce``: warp-coalesced check mode (IGD_DETECT_COALESCE, reading A32);

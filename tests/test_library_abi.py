@@ -75,3 +75,22 @@ def test_product_does_not_import_oracle():
                 txt = open(path).read()
                 assert not re.search(r"#include\s+[\"<].*oracle", txt), f
                 assert "igdo_" not in txt, f
+
+
+def test_nccl_unique_id_without_gpu():
+    # the multi-GPU boundary: libnccl is resolved at run time and an id is 128 bytes
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    a, b = igd.igd_nccl_unique_id(), igd.igd_nccl_unique_id()
+    assert len(a) == 128 and len(b) == 128 and a != b
+
+
+def test_collective_create_argument_errors_without_gpu():
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    lib = igd.load_library()
+    ctx = ctypes.c_void_p()
+    A, F = igd.igd.ALLOC_FN(), igd.igd.FREE_FN()
+    assert lib.igd_ctx_create(ctypes.byref(ctx), 0, None, 2, 0, None, A, F, None) == -1  # nranks > 1, no id
+    assert lib.igd_ctx_create(ctypes.byref(ctx), 0, None, 2, 2, None, A, F, None) == -1  # rank out of range
+    assert lib.igd_ctx_create(ctypes.byref(ctx), 0, None, 0, 0, None, A, F, None) == -1  # no ranks
