@@ -228,6 +228,7 @@ def run_sharded(args, fam, rank, world, local):
     det.load(np.zeros(0, igd.EVENT_DTYPE), nb, bd, first_event=lo, n_events_total=n)
     torch.cuda.empty_cache()
     e2e_times = []
+    out = rep
     for s in range(0 if args.no_e2e else args.e2e_steps + 1):
         dist.barrier()
         torch.cuda.synchronize()

@@ -30,7 +30,8 @@ extern "C" {
 #define IGD_OK 0
 #define IGD_EINVAL (-1)  /* bad argument or geometry (threads must be 1..2^24) */
 #define IGD_ETRACE (-2)  /* an event violates the field rules below; see igd_bad_event() */
-#define IGD_ETOOBIG (-3) /* n_events >= 2^32-1, or the accessed word range spans >= 2^32 words */
+#define IGD_ETOOBIG (-3) /* n_events >= 2^32 - 8192 (32-bit trace indices), or -- sharded / collective
+                            contexts only -- the accessed word range spans >= 2^32 words */
 #define IGD_ENOMEM (-4)  /* device allocation failed */
 #define IGD_ECUDA (-5)   /* a CUDA runtime call failed; see igd_last_error() */
 #define IGD_ENCCL (-6)   /* an NCCL call failed, or libnccl.so.2 could not be loaded (multi-GPU) */
@@ -147,7 +148,9 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
 /* Run the race check over the attached trace.  On success *n_reports_global holds the number
    of reports; the reports stay in context-owned device memory until the next igd_detect or
    igd_ctx_destroy.  Returns IGD_ETRACE (igd_bad_event gives the index) on an ill-formed
-   event, IGD_ETOOBIG if the accessed words span >= 2^32 words.
+   event.  Word keys (a4): the low 32 bits of the word when the accessed words span < 2^32
+   words, else u64 keys word - (min word rounded down to 256) sorted over ceil(bits(span)/8)
+   radix passes -- any 62-bit word range (e.g. sparse 48-bit virtual addresses) is exact.
    flags: IGD_DETECT_TIMING (per-stage timings, below) | IGD_DETECT_COALESCE (warp-coalesced
    check, §6.5, reading A32: of a warp instruction whose >= 2 active lanes all LD, or
    all ATOM, one word -- consecutive events, same warp / kind / scope / mask / word, lanes

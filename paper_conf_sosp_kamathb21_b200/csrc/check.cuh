@@ -111,9 +111,10 @@ __device__ __noinline__ bool q_between(const uint4* __restrict__ desc, const u32
 }
 
 struct Params {
-    const u32* key;  // sorted word keys
+    const void* key; // sorted word keys: u32 low 32 bits of the word, or u64 word - wbase (wide path)
     const void* val; // sorted payload: u64 (index | tk << 32), or uint4 {key, index, tk, mask} (MV)
-    u64 wbase;       // smallest accessed word (reports rebuild the 64-bit word from the key)
+    u64 wbase;       // u32 keys: smallest accessed word (reports rebuild the 64-bit word from the
+                     // key); u64 keys: the key base
     u32 n;           // number of accesses
     const igd_event* ev;
     Geo g;

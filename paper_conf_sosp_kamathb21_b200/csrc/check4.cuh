@@ -87,7 +87,8 @@ __device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, co
 
 // KB: the trace has kernel boundaries (a separate instantiation: the boundary test costs
 // registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
-template <bool MV, bool KB, bool WRAP, bool GEO2>
+// KT: u32 word keys (low 32 bits; spans < 2^32 words) or u64 keys (word - wbase, a4's wide path)
+template <bool MV, bool KB, bool WRAP, bool GEO2, typename KT = u32>
 __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
     __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
@@ -119,12 +120,14 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     auto blk_of = [&](u32 t) -> u32 { return GEO2 ? t >> dlog : g.block(t); };
     auto warp_of = [&](u32 t) -> u32 { return GEO2 ? t >> 5 : g.warp(t); };
     auto lane_of = [&](u32 t) -> u32 { return GEO2 ? t & 31u : g.lane(t); };
-    u32 K[C4_ITEMS], V[C4_ITEMS], Z[C4_ITEMS], M[C4_ITEMS];
+    const KT* keys = reinterpret_cast<const KT*>(P.key);
+    KT K[C4_ITEMS];
+    u32 V[C4_ITEMS], Z[C4_ITEMS], M[C4_ITEMS];
 #pragma unroll
     for (int j = 0; j < C4_ITEMS; j++) {
         const u32 x = wbase + j * 32 + lane;
         const bool in = x < n;
-        K[j] = in ? __ldcs(P.key + x) : 0u;
+        K[j] = in ? __ldcs(keys + x) : KT(0);
         if (MV) {  // the received record {key, idx, tk, mask}
             const uint4 v = in ? __ldcs(reinterpret_cast<const uint4*>(P.val) + x) : make_uint4(0, 0, 0, 0);
             V[j] = v.y;
@@ -138,9 +141,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         }
     }
     // the access before the warp's first one
-    u32 cK = 0, cZ = 0, cV = 0;
+    KT cK = 0;
+    u32 cZ = 0, cV = 0;
     if (lane == 0 && wbase > 0 && wbase <= n) {
-        cK = __ldg(P.key + wbase - 1);
+        cK = __ldg(keys + wbase - 1);
         const Acc a = acc_at<MV>(P.val, wbase - 1);
         cZ = a.tk;
         cV = a.idx;
@@ -156,9 +160,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
 #pragma unroll
     for (int j = 0; j < C4_ITEMS; j++) {
         const u32 x = wbase + j * 32 + lane;
-        const u32 rK = __shfl_sync(IGD_FULL, K[j], (lane + 31u) & 31u);
+        const KT rK = __shfl_sync(IGD_FULL, K[j], (lane + 31u) & 31u);
         const u32 rZ = __shfl_sync(IGD_FULL, Z[j], (lane + 31u) & 31u);
-        const u32 pK = lane ? rK : cK, pZ = lane ? rZ : cZ;
+        const KT pK = lane ? rK : cK;
+        const u32 pZ = lane ? rZ : cZ;
         const bool pvalid = lane ? true : (j > 0 || wbase > 0);
         cK = rK;  // lane 0: the last access of row j precedes row j+1's first
         cZ = rZ;
@@ -456,7 +461,8 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             if (slot < P.rep_cap) {
                 igd_report r;
                 // full word from the 32-bit key: the accessed words span < 2^32 from wbase
-                r.addr = (P.wbase + (u32)(__ldg(P.key + x) - (u32)P.wbase)) << 2;
+                if (sizeof(KT) == 8) r.addr = (P.wbase + (u64)__ldg(keys + x)) << 2;  // key = word - wbase
+                else r.addr = (P.wbase + (u32)((u32)__ldg(keys + x) - (u32)P.wbase)) << 2;
                 r.cur = P.first_event + i;
                 r.prev = P.first_event + mdIdx;
                 r.type = (uint8_t)type;

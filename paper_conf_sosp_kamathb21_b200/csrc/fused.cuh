@@ -51,7 +51,8 @@ struct Params {
     const u32* digit_base;  // [256] exclusive global offsets of digit 0 of the access keys
     u64* status;            // [n_tiles * 256], zeroed
     u32* tile_ctr;          // zeroed: tile tickets (CTA start order, see rsort::k_onesweep)
-    u32* kout;              // access keys, sorted by digit 0
+    void* kout;             // access keys (u32 or u64, template KT), sorted by digit 0
+    u64 kbase;              // KT = u64: key = word - kbase (kbase's low 8 bits are 0)
     u64* vout;              // access payload (event index | tk << 32), same order
     const u32* skip_bits;   // coalesced mode (A32): bit i = event i is not an access record
 };
@@ -92,15 +93,20 @@ __device__ __forceinline__ FDec fdecode(const uint4& e, const Geo& g, const KeyS
     return d;
 }
 
-// the event tile (16 B per event), or the phase-2 buffers aliasing it if those are larger
+// the event tile (16 B per event), or the phase-2 buffers aliasing it if those are larger:
+// keys (KT), values (8 B), digits (1 B), per-warp digit counts
+template <typename KT = u32>
 constexpr size_t smem_bytes() {
-    return (size_t)TILE * 16 > (size_t)TILE * 14 + WARPS * RADIX * 4 ? (size_t)TILE * 16
-                                                                     : (size_t)TILE * 14 + WARPS * RADIX * 4;
+    return (size_t)TILE * 16 > (size_t)TILE * (sizeof(KT) + 9) + WARPS * RADIX * 4
+               ? (size_t)TILE * 16
+               : (size_t)TILE * (sizeof(KT) + 9) + WARPS * RADIX * 4;
 }
 
 // COAL: warp-coalesced mode (A32) -- a separate instantiation so the default path carries no
 // skip-bit test (ncu r02b: 6% of the kernel's instructions)
-template <bool COAL>
+// KT: u32 keys (low 32 bits of the word; spans < 2^32 words) or u64 keys (word - kbase, the wide
+// path of a4)
+template <bool COAL, typename KT = u32>
 __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params P) {
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
@@ -111,13 +117,14 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     __shared__ __align__(8) u64 s_mbar;
     __shared__ u32 s_tile;
     extern __shared__ __align__(16) unsigned char s_dyn[];
-    // phase 1: the event tile (64 KB).  Phase 2 (events dead): digit-sorted keys [0, 16K),
-    // values [16K, 48K), digit per position [48K, 52K), per-warp digit counts [56K, 64K).
+    // phase 1: the event tile (64 KB).  Phase 2 (events dead), u32 keys: digit-sorted keys
+    // [0, 16K), values [16K, 48K), digit per position [48K, 52K), per-warp digit counts [52K, 60K).
     uint4* s_ev = reinterpret_cast<uint4*>(s_dyn);
-    u32* s_k = reinterpret_cast<u32*>(s_dyn);
-    u64* s_v = reinterpret_cast<u64*>(s_dyn + TILE * 4);
-    uint8_t* s_dig = s_dyn + TILE * 12;
-    u32(*s_whist)[RADIX] = reinterpret_cast<u32(*)[RADIX]>(s_dyn + TILE * 14);
+    KT* s_k = reinterpret_cast<KT*>(s_dyn);
+    u64* s_v = reinterpret_cast<u64*>(s_dyn + TILE * sizeof(KT));
+    uint8_t* s_dig = s_dyn + TILE * (sizeof(KT) + 8);
+    u32(*s_whist)[RADIX] = reinterpret_cast<u32(*)[RADIX]>(s_dyn + TILE * (sizeof(KT) + 9));
+    KT* kout = reinterpret_cast<KT*>(P.kout);
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     if (t == 0) {
@@ -150,21 +157,24 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     const KeySpace ks = P.ks;
     const u32 wofs = warp * 32 * ITEMS;
     const u32 lt = lanemask_lt();
-    u32 key[ITEMS], tk[ITEMS];
+    KT key[ITEMS];
+    u32 tk[ITEMS];
     u32 amask = 0;    // bit j: item j is an access
     u32 nsbits = 0;   // bits 2j..2j+1: sync records of item j (0..2)
     u32 nsync_w = 0;  // sync records of this warp (warp-uniform)
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
         const u32 p = wofs + j * 32 + lane;
-        FDec d = fdecode(s_ev[p], g, ks);  // valid: ingest pass 0 checked every event
+        const uint4 ev = s_ev[p];
+        FDec d = fdecode(ev, g, ks);  // valid: ingest pass 0 checked every event
         const bool in = p < tile_e;
         if (COAL && d.acc && in && ((__ldg(P.skip_bits + ((base + p) >> 5)) >> (p & 31u)) & 1u))
             d.acc = false;  // A32: checked by its coalesced group's first lane
-        key[j] = d.key;
+        if (sizeof(KT) == 8) key[j] = (KT)((((u64)ev.y << 32) | ev.x) >> 2) - (KT)P.kbase;
+        else key[j] = (KT)d.key;
         tk[j] = d.tk;
         amask |= ((in && d.acc) ? 1u : 0u) << j;
-        if (IGD_FUSED_EARLY && in && d.acc) atomicAdd(&s_cnt[d.key & 255u], 1u);
+        if (IGD_FUSED_EARLY && in && d.acc) atomicAdd(&s_cnt[(u32)key[j] & 255u], 1u);
         const u32 ns = in ? d.ns : 0u;
         nsbits |= ns << (2 * j);
         // the event's own slot now holds its sync record keys (read back by this thread only)
@@ -216,7 +226,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     for (int j = 0; j < ITEMS; j++) {
         const bool valid = (amask >> j) & 1u;
         const u32 vmask = __ballot_sync(IGD_FULL, valid);
-        const u32 d = key[j] & 255u;
+        const u32 d = (u32)key[j] & 255u;
         const u32 peers = (IGD_FUSED_MIX && (j % IGD_FUSED_MIX) == IGD_FUSED_MIX - 1)
                               ? rsort::peers_of<0>(valid ? d : (0x100u | lane), vmask)
                                                     : rsort::peers_of<1>(valid ? d : (0x100u | lane), vmask);
@@ -295,7 +305,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
         if ((amask >> j) & 1u) {
-            const u32 d = key[j] & 255u;
+            const u32 d = (u32)key[j] & 255u;
             const u32 r = ((rank2[j / 2] >> (16 * (j & 1))) & 0xFFFFu) + s_tile_excl[d] + s_whist[warp][d];
             s_k[r] = key[j];
             s_v[r] = (base + wofs + j * 32 + lane) | ((u64)tk[j] << 32);
@@ -311,7 +321,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
         if (i < na) {
             const u32 d = s_dig[i];
             const u32 o = s_gbase[d] + i;
-            __stcs(P.kout + o, s_k[i]);
+            __stcs(kout + o, s_k[i]);
             __stcs(P.vout + o, s_v[i]);
         }
     }

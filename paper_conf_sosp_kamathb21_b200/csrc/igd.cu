@@ -63,9 +63,11 @@ struct NcclApi {
 };
 NcclApi load_nccl() {
     NcclApi a;
+    // RTLD_LOCAL: a copy loaded here must not satisfy another library's later symbol lookups
+    // (torch resolves its own, newer NCCL symbols against the global namespace)
     void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
-    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
-    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_LOCAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_LOCAL);
     if (!h) {
         const char* e = dlerror();
         a.why = std::string("cannot load libnccl.so.2: ") + (e ? e : "?");
@@ -142,7 +144,7 @@ struct igd_ctx {
 
     // pinned host mirrors
     u64* h_stats = nullptr;  // 8
-    u32* h_hist = nullptr;   // 2 x 1024 (+ report hist 1024)
+    u32* h_hist = nullptr;   // 2 x 1024 (+ report hist 1024, + wide-key digits 4..7)
     u64* h_small = nullptr;  // 8
 
     bool timing = false;
@@ -258,27 +260,30 @@ static void mark(igd_ctx* ctx, int stage) {
 
 // One radix pass over n keys: the full tiles, then (if any) the partial last tile (same tile
 // counter: the tail's ticket is the last tile).
-template <typename VT>
-static void launch_pass(u64 n, size_t smem, cudaStream_t st, const rsort::PassParams& pp) {
+template <typename VT, typename KT = u32>
+static void launch_pass(u64 n, cudaStream_t st, const rsort::PassParams& pp) {
+    const size_t smem = rsort::onesweep_smem<VT, KT>();
     const u64 full = n / rsort::TILE;
-    if (full) rsort::k_onesweep<VT, false><<<(unsigned)full, rsort::THREADS, smem, st>>>(pp);
-    if (n % rsort::TILE) rsort::k_onesweep<VT, true><<<1u, rsort::THREADS, smem, st>>>(pp);
+    if (full) rsort::k_onesweep<VT, false, KT><<<(unsigned)full, rsort::THREADS, smem, st>>>(pp);
+    if (n % rsort::TILE) rsort::k_onesweep<VT, true, KT><<<1u, rsort::THREADS, smem, st>>>(pp);
 }
-template <typename VT>
+template <typename VT, typename KT = u32>
 static void set_pass_smem() {
-    const int b = (int)rsort::onesweep_smem<VT>();
-    cudaFuncSetAttribute(rsort::k_onesweep<VT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
-    cudaFuncSetAttribute(rsort::k_onesweep<VT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    const int b = (int)rsort::onesweep_smem<VT, KT>();
+    cudaFuncSetAttribute(rsort::k_onesweep<VT, false, KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+    cudaFuncSetAttribute(rsort::k_onesweep<VT, true, KT>, cudaFuncAttributeMaxDynamicSharedMemorySize, b);
 }
 
 // Stable LSD radix sort of n (key, value) pairs in buffers k[cur], v[cur]; h_hist is the host
-// copy of the 4x256 digit histogram (device copy d_hist).  Digits above max_bits and digits
-// with one occupied bin are skipped.  Returns the buffer index holding the result.
+// copy of the 4x256 (u32 keys) or 8x256 (kbytes = 8: u64 keys) digit histogram (device copy
+// d_hist).  Digits above max_bits and digits with one occupied bin are skipped.  Returns the
+// buffer index holding the result.
 // vin_first: values of the input (instead of v[first_cur]) for the first pass that runs -- the
 // sharded path sorts the received records in place of a split copy.
 static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d_hist, const u32* h_hist,
                       u32 max_bits, int* out_cur, int vbytes = 4, u32 first_pass = 0, int first_cur = 0,
-                      const void* vin_first = nullptr) {
+                      const void* vin_first = nullptr, int kbytes = 4) {
+    const u32 ndig = kbytes == 8 ? 8u : 4u;
     int cur = first_cur;
     *out_cur = cur;
     bool ran = false;
@@ -289,11 +294,11 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
     if (n > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;  // 32-bit tile indexing
     {
         KTimer kt(ctx, KC_MISC, 0);
-        rsort::k_digit_base<<<4, rsort::RADIX, 0, ctx->stream>>>(d_hist, P_<u32>(ctx->base));
+        rsort::k_digit_base<<<ndig, rsort::RADIX, 0, ctx->stream>>>(d_hist, P_<u32>(ctx->base));
     }
     const u64 tiles = (n + rsort::TILE - 1) / rsort::TILE;
     RET(ensure(ctx, ctx->status, tiles * rsort::RADIX * sizeof(u64)));
-    for (u32 p = first_pass; p < 4; p++) {
+    for (u32 p = first_pass; p < ndig; p++) {
         if (p * 8 >= max_bits) break;
         bool trivial = false;
         for (int d = 0; d < 256; d++)
@@ -302,10 +307,10 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         CK(cudaMemsetAsync(ctx->status.p, 0, tiles * rsort::RADIX * sizeof(u64), ctx->stream));
         CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
         rsort::PassParams pp;
-        pp.kin = P_<u32>(k[cur]);
+        pp.kin = k[cur].p;
         pp.vin = (!ran && vin_first) ? vin_first : v[cur].p;
         ran = true;
-        pp.kout = P_<u32>(k[cur ^ 1]);
+        pp.kout = k[cur ^ 1].p;
         pp.vout = v[cur ^ 1].p;
         pp.n = (u32)n;
         pp.shift = p * 8;
@@ -313,10 +318,11 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         pp.status = P_<u64>(ctx->status);
         pp.tile_ctr = P_<u32>(ctx->ctr);
         {
-            KTimer kt(ctx, cls, 2.0 * (4 + vbytes) * (double)n);  // read + write 4 B key and the value
-            if (vbytes == 16) launch_pass<uint4>(n, rsort::onesweep_smem<uint4>(), ctx->stream, pp);
-            else if (vbytes == 8) launch_pass<u64>(n, rsort::onesweep_smem<u64>(), ctx->stream, pp);
-            else launch_pass<u32>(n, rsort::onesweep_smem<u32>(), ctx->stream, pp);
+            KTimer kt(ctx, cls, 2.0 * (kbytes + vbytes) * (double)n);  // read + write the key and the value
+            if (kbytes == 8) launch_pass<u64, u64>(n, ctx->stream, pp);
+            else if (vbytes == 16) launch_pass<uint4>(n, ctx->stream, pp);
+            else if (vbytes == 8) launch_pass<u64>(n, ctx->stream, pp);
+            else launch_pass<u32>(n, ctx->stream, pp);
         }
         if (n > rsort::TILE && n % rsort::TILE) ctx->launches++;  // the partial-tile launch
         CK(cudaGetLastError());
@@ -341,7 +347,18 @@ static void launch_check_w(bool wrap, unsigned tb, cudaStream_t st, const check:
         else check::k_check4<MV, KB, false, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
     }
 }
-static void launch_check(bool mv, bool kb, bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
+static void launch_check(bool mv, bool kb, bool wrap, bool key64, unsigned tb, cudaStream_t st,
+                         const check::Params& cp) {
+    if (key64) {  // a4's wide path (single GPU): general geometry instantiation
+        if (kb) {
+            if (wrap) check::k_check4<false, true, true, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
+            else check::k_check4<false, true, false, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
+        } else {
+            if (wrap) check::k_check4<false, false, true, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
+            else check::k_check4<false, false, false, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
+        }
+        return;
+    }
     if (mv && kb) launch_check_w<true, true>(wrap, tb, st, cp);
     else if (mv) launch_check_w<true, false>(wrap, tb, st, cp);
     else if (kb) launch_check_w<false, true>(wrap, tb, st, cp);
@@ -436,8 +453,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     // ---------------- a1 + a2 + a4: ingest ----------------
     const u64 in_tiles = (n_src + ingest::TILE - 1) / ingest::TILE;
     RET(ensure(ctx, ctx->stats, 8 * sizeof(u64)));
-    RET(ensure(ctx, ctx->hist, 3 * 1024 * sizeof(u32)));
-    RET(ensure(ctx, ctx->base, 4 * 256 * sizeof(u32)));
+    // hist: [0, 1024) access-key digits 0..3, [1024, 2048) sync-key digits, [2048, 4096) the
+    // 8 digits of wide (u64) access keys
+    RET(ensure(ctx, ctx->hist, 4 * 1024 * sizeof(u32)));
+    RET(ensure(ctx, ctx->base, 8 * 256 * sizeof(u32)));
     RET(ensure(ctx, ctx->ctr, 64));
     RET(ensure(ctx, ctx->st_in_a, (in_tiles + 1) * sizeof(u32)));
     RET(ensure(ctx, ctx->st_in_s, (in_tiles + 1) * sizeof(u32)));
@@ -505,9 +524,16 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const u64 n_lock = ctx->h_stats[5];
     const u64 wbase = SH ? ctx->sh_wbase : ctx->h_stats[0];
     if (n_sync + 64 > 0xFFFFFFFFull) return IGD_ETOOBIG;  // 32-bit record positions
-    if (!SH && n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32)) {
-        ctx->err = "accessed word range spans >= 2^32 words";
-        return IGD_ETOOBIG;
+    // a4: accessed words spanning >= 2^32 words (sparse virtual addresses) take the wide path:
+    // u64 keys word - kbase, sorted over ceil(bits(span) / 8) digit passes
+    const bool key64 = !SH && n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32);
+    const u64 kbase = key64 ? (ctx->h_stats[0] & ~255ull) : 0;  // low digit unchanged: pass 0's histogram holds
+    if (key64) {
+        if (!FUSED) {
+            ctx->err = "word spans >= 2^32 words need the fused ingest pipeline (IGD_FUSED=1)";
+            return IGD_ETOOBIG;
+        }
+        for (int b = 0; b < 2; b++) RET(ensure(ctx, ctx->acc_k[b], acc_cap * sizeof(u64)));
     }
     if (ctx->sync_cap < n_sync) ctx->sync_cap = n_sync + n_sync / 8 + 4096;
     for (int b = 0; b < 2; b++) {
@@ -542,16 +568,22 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         fp.digit_base = P_<u32>(ctx->base);
         fp.status = P_<u64>(ctx->status);
         fp.tile_ctr = P_<u32>(ctx->ctr);
-        fp.kout = P_<u32>(ctx->acc_k[1]);
+        fp.kout = ctx->acc_k[1].p;
+        fp.kbase = kbase;
         fp.vout = P_<u64>(ctx->acc_v[1]);
         fp.skip_bits = ip.skip_bits;
         {
             // reads every event once, writes the 12-byte access records and 8-byte sync records
             KTimer kt(ctx, KC_FUSED, 16.0 * (double)n_src + 12.0 * (double)n_acc + 8.0 * (double)n_sync);
-            if (fp.skip_bits)
+            if (key64) {
+                const size_t sm64 = fused::smem_bytes<u64>();
+                if (fp.skip_bits) fused::k_ingest_sort0<true, u64><<<(unsigned)ft, fused::THREADS, sm64, ctx->stream>>>(fp);
+                else fused::k_ingest_sort0<false, u64><<<(unsigned)ft, fused::THREADS, sm64, ctx->stream>>>(fp);
+            } else if (fp.skip_bits) {
                 fused::k_ingest_sort0<true><<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
-            else
+            } else {
                 fused::k_ingest_sort0<false><<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
+            }
         }
         CK(cudaGetLastError());
     }
@@ -574,6 +606,16 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
         ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[1]), (u32)n_acc, P_<u32>(ctx->hist), 1);
     }
+    if (key64) {
+        // wide keys: digit 0 is pass 0's (kbase has a zero low digit); digits 1..7 over the keys
+        // the fused pass wrote
+        CK(cudaMemsetAsync(P_<u32>(ctx->hist) + 2048, 0, 2048 * sizeof(u32), ctx->stream));
+        CK(cudaMemcpyAsync(P_<u32>(ctx->hist) + 2048, ctx->hist.p, 256 * sizeof(u32), cudaMemcpyDeviceToDevice,
+                           ctx->stream));
+        KTimer kt(ctx, KC_INGEST, 8.0 * (double)n_acc);
+        const unsigned hb = (unsigned)std::min<u64>((n_acc + 255) / 256, (u64)sms * 8);
+        rsort::k_hist8<<<hb, 256, 0, ctx->stream>>>(P_<u64>(ctx->acc_k[1]), n_acc, P_<u32>(ctx->hist) + 2048, 1);
+    }
     if (FUSED && n_sync > 0) {
         // sync-key digit histograms over the records the fused pass wrote (trace order)
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_sync);
@@ -594,6 +636,14 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     u32 h_hist_acc[1024], h_hist_sync[1024];
     memcpy(h_hist_acc, ctx->h_hist, sizeof(h_hist_acc));
     memcpy(h_hist_sync, ctx->h_hist + 1024, sizeof(h_hist_sync));
+    std::vector<u32> h_hist64;
+    if (key64) {
+        h_hist64.resize(2048);
+        CK(cudaMemcpyAsync(ctx->h_hist + 2048, P_<u32>(ctx->hist) + 2048, 2048 * sizeof(u32), cudaMemcpyDeviceToHost,
+                           ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        memcpy(h_hist64.data(), ctx->h_hist + 2048, 2048 * sizeof(u32));
+    }
 
     // ---------------- a2: sync records sorted by entity, CSR offsets ----------------
     int scur = 0;
@@ -673,8 +723,12 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     mark(ctx, 3);
     // ---------------- a5: accesses sorted by word, stable ----------------
     int acur = 0;
-    RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur,
-                   vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0, SH ? ctx->sh_rec : nullptr));
+    if (key64)
+        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist) + 2048, h_hist64.data(),
+                       bits_needed(ctx->h_stats[1] - kbase), &acur, vbytes, 1, 1, nullptr, 8));
+    else
+        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur,
+                       vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0, SH ? ctx->sh_rec : nullptr));
     ctx->last_acur = acur;
     ctx->last_nacc = SH ? 0 : n_acc;
     mark(ctx, 4);
@@ -693,9 +747,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             CK(cudaMemsetAsync(ctx->rep_ctr.p, 0, sizeof(u64), ctx->stream));
             check::Params cp;
             memset(&cp, 0, sizeof(cp));
-            cp.key = P_<u32>(ctx->acc_k[acur]);
+            cp.key = ctx->acc_k[acur].p;
             cp.val = ctx->acc_v[acur].p;
-            cp.wbase = wbase;
+            cp.wbase = key64 ? kbase : wbase;
             cp.n = (u32)n_acc;
             cp.ev = ctx->events;
             cp.g = g;
@@ -717,7 +771,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
-                launch_check(SH, cp.has_kb != 0, ctx->paper_counters, (unsigned)tiles, ctx->stream, cp);
+                launch_check(SH, cp.has_kb != 0, ctx->paper_counters, key64, (unsigned)tiles, ctx->stream, cp);
             }
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
@@ -979,11 +1033,16 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
                          (int)fused::smem_bytes());
     cudaFuncSetAttribute(fused::k_ingest_sort0<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes());
+    cudaFuncSetAttribute(fused::k_ingest_sort0<false, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)fused::smem_bytes<u64>());
+    cudaFuncSetAttribute(fused::k_ingest_sort0<true, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)fused::smem_bytes<u64>());
     set_pass_smem<u32>();
     set_pass_smem<u64>();
     set_pass_smem<uint4>();
+    set_pass_smem<u64, u64>();
     if (cudaMallocHost(&ctx->h_stats, 8 * sizeof(u64)) != cudaSuccess ||
-        cudaMallocHost(&ctx->h_hist, 3 * 1024 * sizeof(u32)) != cudaSuccess ||
+        cudaMallocHost(&ctx->h_hist, 4 * 1024 * sizeof(u32)) != cudaSuccess ||
         cudaMallocHost(&ctx->h_small, 8 * sizeof(u64)) != cudaSuccess) {
         delete ctx;
         return IGD_ENOMEM;

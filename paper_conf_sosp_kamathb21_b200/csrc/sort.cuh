@@ -71,10 +71,26 @@ __global__ void k_hist4(const u32* __restrict__ keys, u64 n, u32* __restrict__ h
     }
 }
 
+// 8-digit histogram of u64 keys (the wide-key path of a4); digits >= first_digit.
+__global__ void k_hist8(const u64* __restrict__ keys, u64 n, u32* __restrict__ hist, int first_digit) {
+    __shared__ u32 s[8][RADIX];
+    for (int i = threadIdx.x; i < 8 * RADIX; i += blockDim.x) (&s[0][0])[i] = 0;
+    __syncthreads();
+    for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) {
+        const u64 k = keys[i];
+        for (int p = first_digit; p < 8; p++) atomicAdd(&s[p][(u32)(k >> (8 * p)) & 255u], 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < 8 * RADIX; i += blockDim.x) {
+        const u32 v = (&s[0][0])[i];
+        if (v) atomicAdd(&hist[i], v);
+    }
+}
+
 struct PassParams {
-    const u32* kin;
-    const void* vin;  // u32 or u64 values (template VT)
-    u32* kout;
+    const void* kin;  // u32 or u64 keys (template KT)
+    const void* vin;  // u32, u64 or uint4 values (template VT)
+    void* kout;
     void* vout;
     u32 n;
     u32 shift;
@@ -100,15 +116,16 @@ __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     }
 }
 
-// Dynamic shared memory of k_onesweep<VT>: staged keys, staged values, digit per position.
-template <typename VT>
+// Dynamic shared memory of k_onesweep<VT, TAIL, KT>: staged keys, staged values, digit per position.
+template <typename VT, typename KT = u32>
 constexpr size_t onesweep_smem() {
-    return (size_t)TILE * sizeof(u32) + (size_t)TILE * sizeof(VT) + TILE;
+    return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT) + TILE;
 }
 
 // TAIL = false: every tile of the launch is full (no bounds tests on the hot path); TAIL = true:
 // the one partial last tile, launched after the full ones (its look-back finds them published).
-template <typename VT, bool TAIL>
+// KT = u32 (word spans < 2^32 words) or u64 keys (reading a4's wide path: up to 8 digit passes)
+template <typename VT, bool TAIL, typename KT = u32>
 #ifndef IGD_SORT_MINB
 #define IGD_SORT_MINB 3
 #endif
@@ -121,11 +138,13 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     __shared__ u32 s_cnt[RADIX];  // tile digit counts (IGD_SORT_EARLY)
     __shared__ __align__(8) u64 s_mbar[2];
     extern __shared__ __align__(16) unsigned char s_dyn[];
-    u32* s_k = reinterpret_cast<u32*>(s_dyn);                         // keys in, then keys out
-    VT* s_v = reinterpret_cast<VT*>(s_dyn + TILE * sizeof(u32));      // values in, then values out
-    uint8_t* s_dig = s_dyn + TILE * sizeof(u32) + TILE * sizeof(VT);  // digit of each output position
+    KT* s_k = reinterpret_cast<KT*>(s_dyn);                           // keys in, then keys out
+    VT* s_v = reinterpret_cast<VT*>(s_dyn + TILE * sizeof(KT));       // values in, then values out
+    uint8_t* s_dig = s_dyn + TILE * sizeof(KT) + TILE * sizeof(VT);   // digit of each output position
     const VT* vin = reinterpret_cast<const VT*>(P.vin);
     VT* vout = reinterpret_cast<VT*>(P.vout);
+    const KT* kin = reinterpret_cast<const KT*>(P.kin);
+    KT* kout = reinterpret_cast<KT*>(P.kout);
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
     if (t == 0) {
@@ -139,8 +158,8 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         if (!TAIL) {
             mbar_init(&s_mbar[0], 1);
             mbar_init(&s_mbar[1], 1);
-            mbar_expect_tx(&s_mbar[0], TILE * sizeof(u32));
-            bulk_g2s(s_k, P.kin + base, TILE * sizeof(u32), &s_mbar[0]);
+            mbar_expect_tx(&s_mbar[0], TILE * sizeof(KT));
+            bulk_g2s(s_k, kin + base, TILE * sizeof(KT), &s_mbar[0]);
             mbar_expect_tx(&s_mbar[1], TILE * sizeof(VT));
             bulk_g2s(s_v, vin + base, TILE * sizeof(VT), &s_mbar[1]);
         }
@@ -155,7 +174,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     const u32 shift = P.shift;
     constexpr bool full = !TAIL;
 
-    u32 key[ITEMS];
+    KT key[ITEMS];
     if (full) {
         mbar_wait(&s_mbar[0], 0);
 #pragma unroll
@@ -164,14 +183,14 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
             const u32 i = wbase + j * 32 + lane;
-            key[j] = i < P.n ? __ldcs(P.kin + i) : 0u;
+            key[j] = i < P.n ? __ldcs(kin + i) : KT(0);
         }
     }
     if (IGD_SORT_EARLY) {
         // tile digit counts first, published before ranking (see fused.cuh)
 #pragma unroll
         for (int j = 0; j < ITEMS; j++)
-            if (full || wbase + j * 32 + lane < P.n) atomicAdd(&s_cnt[(key[j] >> shift) & 255u], 1u);
+            if (full || wbase + j * 32 + lane < P.n) atomicAdd(&s_cnt[(u32)(key[j] >> shift) & 255u], 1u);
         __syncthreads();
         st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
     }
@@ -181,7 +200,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     for (int j = 0; j < ITEMS; j++) {
         const bool valid = full || wbase + j * 32 + lane < P.n;
         const u32 vmask = full ? IGD_FULL : __ballot_sync(IGD_FULL, valid);
-        const u32 d = (key[j] >> shift) & 255u;
+        const u32 d = (u32)(key[j] >> shift) & 255u;
         // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set.
         // IGD_SORT_MIX = N: one row in N is ranked with match.any (MIO pipe), the others with the
         // 8 ballots (ALU / issue): the two bottleneck on different units
@@ -264,7 +283,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     // keys: reorder in shared memory (rank[] becomes the tile position), write digit runs
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
-        const u32 d = (key[j] >> shift) & 255u;
+        const u32 d = (u32)(key[j] >> shift) & 255u;
         rank[j] += s_tile_excl[d] + s_whist[warp][d];
         if (full || wbase + j * 32 + lane < P.n) s_k[rank[j]] = key[j];
     }
@@ -274,10 +293,10 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     for (int k = 0; k < ITEMS; k++) {
         const u32 i = t + k * THREADS;
         if (i < tile_n) {
-            const u32 kk = s_k[i];
-            const u32 d = (kk >> shift) & 255u;
+            const KT kk = s_k[i];
+            const u32 d = (u32)(kk >> shift) & 255u;
             s_dig[i] = (uint8_t)d;
-            __stcs(P.kout + (s_gbase[d] + i), kk);
+            __stcs(kout + (s_gbase[d] + i), kk);
         }
     }
     // values: same permutation, in place through the staged buffer

@@ -107,11 +107,21 @@ def igd_strerror(code: int) -> str:
 
 def igd_nccl_unique_id() -> bytes:
     """A fresh 128-byte NCCL unique id (rank 0 creates it, the caller shares it with the others)."""
+    _prefer_torch_nccl()
     buf = (ctypes.c_uint8 * 128)()
     rc = load_library().igd_nccl_unique_id(buf)
     if rc != IGD_OK:
         raise IgdError(rc, "igd_nccl_unique_id")
     return bytes(buf)
+
+
+def _prefer_torch_nccl():
+    """libigd resolves libnccl.so.2 at run time and reuses a copy already in the process: load
+    torch first so its NCCL (the one torch.distributed uses) is that copy."""
+    try:
+        import torch  # noqa: F401
+    except ImportError:
+        pass
 
 
 def igd_ctx_create(cuda_device: int, cuda_stream: int, alloc_fn=None, free_fn=None, nranks: int = 1,
@@ -120,6 +130,7 @@ def igd_ctx_create(cuda_device: int, cuda_stream: int, alloc_fn=None, free_fn=No
     ctx = ctypes.c_void_p()
     idbuf = None
     if nccl_id is not None:
+        _prefer_torch_nccl()
         assert len(nccl_id) == 128
         idbuf = (ctypes.c_uint8 * 128).from_buffer_copy(nccl_id)
     rc = lib.igd_ctx_create(ctypes.byref(ctx), cuda_device, ctypes.c_void_p(cuda_stream), nranks, rank,

@@ -117,16 +117,38 @@ def test_sparse_high_addresses(det):
     assert_same(det, ev, nb, bd, "high VA")
 
 
-def test_word_span_too_big(det):
-    import paper_conf_sosp_kamathb21_b200 as igd
-
-    b = tg.TraceBuilder(1, 32)
+def test_word_span_wide_keys(det):
+    # a4: accessed words spanning >= 2^32 words (sparse virtual addresses) take the u64-key path
+    b = tg.TraceBuilder(2, 64)
     b.st(0, 1)
-    b.st(0, 1 + (1 << 32))
-    det.load(b.events(), 1, 32)
-    with pytest.raises(igd.IgdError) as ei:
-        det.detect()
-    assert ei.value.code == igd.igd.IGD_ETOOBIG
+    b.st(0, 1 + (1 << 32))      # same low 32 bits, another word: must not collide
+    b.ld(64, 1)                 # R4 on word 1 only
+    b.ld(65, 1 + (1 << 32))     # R4 on the far word
+    b.fence(0)
+    b.ld(66, 7 << 40)
+    b.st(67, 7 << 40)
+    ev = b.events()
+    want = oracle.run(ev, 2, 64)
+    assert len(want) == 3
+    assert np.array_equal(gpu_run(det, ev, 2, 64), want)
+
+
+@pytest.mark.parametrize("seed,n,nb,bd,bits", [(41, 60_000, 4, 64, 45), (42, 300_000, 16, 128, 40),
+                                               (43, 120_000, 3, 96, 62), (44, 50_000, 2, 64, 33)])
+def test_wide_keys_vs_oracle(det, seed, n, nb, bd, bits):
+    # random traces whose words are spread over 2^bits words (up to ceil(bits/8) radix passes);
+    # lock words and data words both wide, few distinct words so histories are long
+    w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    ev, nb, bd = _fast_random(seed, n, 3_000, nb, bd, w, lock_words=12)
+    rng = np.random.default_rng(seed)
+    acc = ((ev["tk"] >> 24) & 0xF) <= 4
+    word = ev["addr"] >> np.uint64(2)
+    uniq, inv = np.unique(word[acc], return_inverse=True)
+    spread = rng.integers(0, 1 << bits, len(uniq), dtype=np.uint64)
+    spread[0] = 0
+    spread[-1] = (1 << bits) - 1
+    ev["addr"][acc] = (spread[inv] << np.uint64(2)) | (ev["addr"][acc] & np.uint64(3))
+    assert_same(det, ev, nb, bd, f"wide seed {seed}")
 
 
 @pytest.mark.parametrize("bad_at", [0, 5000, 99_999])
