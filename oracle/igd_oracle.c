@@ -152,6 +152,21 @@ static uint32_t o_fmix32(uint32_t h) {
 #define O_ETRACE (-2)
 #define O_ENOMEM (-4)
 
+/* Reading A34 (per-kernel geometry, "the number of warps per threadblock remains
+   constant for a kernel but can vary across kernels"): a KERNEL_BOUNDARY whose addr is
+   nonzero carries the next kernel's grid as (n_blocks << 32) | block_dim. */
+static int o_geom_code_ok(uint64_t code) {
+    uint64_t nb = code >> 32, bd = code & 0xFFFFFFFFu;
+    return nb >= 1 && bd >= 1 && nb * bd <= (1u << 24);
+}
+static void o_geom_set(o_geom* g, uint32_t n_blocks, uint32_t block_dim) {
+    g->D = block_dim;
+    g->Wb = (block_dim + 31) / 32;
+    g->blocks = n_blocks;
+    g->threads = n_blocks * block_dim;
+    g->warps = n_blocks * g->Wb;
+}
+
 /* Field rules per kind. Returns 1 when the event is well-formed. */
 static int o_valid(const o_event* e, const o_geom* g) {
     if (e->kind > O_KERNEL) return 0;
@@ -166,8 +181,10 @@ static int o_valid(const o_event* e, const o_geom* g) {
         return e->addr == 0 && (e->mask & lanebit) && e->scope != S_NONE;
     case O_SYNCWARP: case O_CG_TILE: case O_SYNCTHREADS: case O_CG_BLOCK:
         return e->addr == 0 && e->scope == S_NONE;
-    case O_GRID: case O_CG_GRID: case O_KERNEL:
+    case O_GRID: case O_CG_GRID:
         return e->addr == 0 && e->scope == S_NONE && e->tid == 0;
+    case O_KERNEL: /* addr: 0, or the next kernel's geometry (reading A34) */
+        return e->scope == S_NONE && e->tid == 0 && (e->addr == 0 || o_geom_code_ok(e->addr));
     }
     return 0;
 }
@@ -221,31 +238,43 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
     if (shard_K == 0 || shard_k >= shard_K) return O_EINVAL;
 
     o_geom g;
-    g.D = block_dim;
-    g.Wb = (block_dim + 31) / 32;
-    g.blocks = n_blocks;
-    g.threads = n_blocks * block_dim;
-    g.warps = n_blocks * g.Wb;
+    o_geom_set(&g, n_blocks, block_dim);
 
-    /* validate everything first (the oracle applies the 8(b) rules independently) */
+    /* validate everything first (the oracle applies the 8(b) rules independently), each event
+       against the geometry of its own kernel (A34) */
     for (uint64_t i = 0; i < n; i++) {
         o_event e;
         int ok = o_read_event(events + 16 * i, &e);
         if (!ok || !o_valid(&e, &g)) { *bad_index = i; return O_ETRACE; }
+        if (e.kind == O_KERNEL && e.addr != 0) o_geom_set(&g, (uint32_t)(e.addr >> 32), (uint32_t)e.addr);
     }
+    o_geom_set(&g, n_blocks, block_dim);
 
-    /* C.2 synchronization state: exact, unbounded counters */
-    uint64_t* devF = (uint64_t*)calloc(g.threads, sizeof(uint64_t));
-    uint64_t* anyF = (uint64_t*)calloc(g.threads, sizeof(uint64_t));
-    uint64_t* wbar = (uint64_t*)calloc(g.warps, sizeof(uint64_t));
-    uint64_t* bbar = (uint64_t*)calloc(g.blocks, sizeof(uint64_t));
+    /* C.2 synchronization state: exact, unbounded counters.  Sized for the largest grid of the
+       trace (A34: a kernel boundary may change the geometry) */
+    uint64_t maxT = g.threads, maxW = g.warps, maxB = g.blocks;
+    for (uint64_t i = 0; i < n; i++) {
+        o_event e;
+        o_read_event(events + 16 * i, &e);
+        if (e.kind == O_KERNEL && e.addr != 0) {
+            o_geom h;
+            o_geom_set(&h, (uint32_t)(e.addr >> 32), (uint32_t)e.addr);
+            if (h.threads > maxT) maxT = h.threads;
+            if (h.warps > maxW) maxW = h.warps;
+            if (h.blocks > maxB) maxB = h.blocks;
+        }
+    }
+    uint64_t* devF = (uint64_t*)calloc(maxT, sizeof(uint64_t));
+    uint64_t* anyF = (uint64_t*)calloc(maxT, sizeof(uint64_t));
+    uint64_t* wbar = (uint64_t*)calloc(maxW, sizeof(uint64_t));
+    uint64_t* bbar = (uint64_t*)calloc(maxB, sizeof(uint64_t));
     uint64_t G = 0;
     uint64_t kernel = 0; /* kernel boundaries so far (A31) */
-    o_table* wt = (o_table*)calloc(g.warps, sizeof(o_table));
-    o_table* tt = (o_table*)calloc(g.threads, sizeof(o_table));
-    uint8_t* isThread = (uint8_t*)calloc(g.warps, 1);
-    uint8_t* touched = (uint8_t*)calloc(g.warps, 1); /* warps whose tables were ever filled */
-    uint32_t* touched_list = (uint32_t*)calloc(g.warps, sizeof(uint32_t));
+    o_table* wt = (o_table*)calloc(maxW, sizeof(o_table));
+    o_table* tt = (o_table*)calloc(maxT, sizeof(o_table));
+    uint8_t* isThread = (uint8_t*)calloc(maxW, 1);
+    uint8_t* touched = (uint8_t*)calloc(maxW, 1); /* warps whose tables were ever filled */
+    uint32_t* touched_list = (uint32_t*)calloc(maxW, sizeof(uint32_t));
     uint32_t n_touched = 0;
     o_map map = {0, 0, 0};
     uint8_t* skip = (flags & 1u) ? (uint8_t*)calloc(n ? n : 1, 1) : NULL; /* A32 coalesced members */
@@ -319,6 +348,17 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
                 }
             }
             n_touched = 0;
+            if (e.addr != 0) {
+                /* A34: the next kernel runs on another grid.  Every shadow entry is discarded
+                   (above, by kernel number) and no counter snapshot survives the boundary, so
+                   the synchronization counters restart with the new thread / warp / block ids */
+                o_geom_set(&g, (uint32_t)(e.addr >> 32), (uint32_t)e.addr);
+                memset(devF, 0, maxT * sizeof(uint64_t));
+                memset(anyF, 0, maxT * sizeof(uint64_t));
+                memset(wbar, 0, maxW * sizeof(uint64_t));
+                memset(bbar, 0, maxB * sizeof(uint64_t));
+                G = 0;
+            }
             continue;
         }
 

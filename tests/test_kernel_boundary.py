@@ -196,3 +196,83 @@ def test_gpu_boundary_field_rules(det):
     with pytest.raises(igd.IgdError) as e:
         det.detect()
     assert e.value.code == igd.igd.IGD_ETRACE and e.value.bad_index == 20
+
+
+# ---- per-kernel geometry (reading A34: "the number of warps per threadblock remains
+# constant for a kernel but can vary across kernels") ----------------------------------------------
+def shifted_union_geo(parts, geoms):
+    out, base = [], 0
+    for t, (nb, bd) in zip(parts, geoms):
+        r = oracle.run(t, nb, bd).copy()
+        r["cur"] += np.uint64(base)
+        r["prev"] += np.uint64(base)
+        out.append(r)
+        base += len(t) + 1
+    allr = np.concatenate(out) if out else np.zeros(0, oracle.REPORT_DTYPE)
+    return allr[np.argsort(allr["cur"], kind="stable")]
+
+
+def mixed_geometry_kernels(seed, k, n):
+    rng = np.random.default_rng(seed)
+    parts, geoms = [], []
+    for j in range(k):
+        nb, bd = int(rng.integers(1, 5)), int(rng.choice([16, 32, 48, 64, 96, 128]))
+        kw = dict(weights=LOCKY, lock_words=3, p_lock_data=0.3) if (seed + j) % 2 else dict(n_words=6)
+        ev, _, _ = tg.random_trace(seed * 37 + j, int(rng.integers(1, n)), n_blocks=nb, block_dim=bd, **kw)
+        parts.append(ev)
+        geoms.append((nb, bd))
+    return parts, geoms
+
+
+@pytest.mark.parametrize("batch", range(4))
+def test_composition_law_mixed_geometry(batch):
+    # T1 on grid g1 | KB(g2) | T2 on grid g2 | ... == each kernel run alone on its own grid, shifted
+    for seed in range(batch * 50, (batch + 1) * 50):
+        parts, geoms = mixed_geometry_kernels(seed, 3, 150)
+        joined = tg.concat_kernels(parts, geoms)
+        got = full_tuples(oracle.run(joined, *geoms[0]))
+        assert got == full_tuples(shifted_union_geo(parts, geoms)), f"seed {seed}"
+
+
+def test_geometry_change_is_not_vacuous():
+    # the same events read under the first kernel's grid would be judged differently: with 64-thread
+    # blocks t0 and t40 share a block (R3 without a barrier); with 32-thread blocks they do not (R4)
+    b = tg.TraceBuilder(1, 64)
+    b.ld(0, 9)                      # kernel 1: nothing
+    b.kernel_boundary(4, 32)        # kernel 2: 4 blocks x 32 threads
+    b.st(0, 5)
+    b.ld(40, 5)
+    ev = b.events()
+    r = oracle.run(ev, 1, 64)
+    assert [(int(x["cur"]), int(x["prev"]), int(x["type"])) for x in r] == [(3, 2, 4)]
+    same = ev.copy()
+    same["addr"][1] = 0             # no geometry change: t40 is in t0's block -> R3
+    assert [int(x["type"]) for x in oracle.run(same, 1, 64)] == [3]
+
+
+@pytest.mark.parametrize("code,ok", [(0, True), ((2 << 32) | 64, True), ((1 << 32) | (1 << 24), True),
+                                      (64, False), (2 << 32, False), ((2 << 32) | (1 << 24), False)])
+def test_boundary_geometry_field_rule(code, ok):
+    b = tg.TraceBuilder(1, 64)
+    b.st(0, 1)
+    b.ev(tg.KERNEL_BOUNDARY, 0, 0, tg.NONE, 0xFFFFFFFF, addr=code)
+    b.st(0, 1)
+    if ok:
+        assert len(oracle.run(b.events(), 1, 64)) == 0
+    else:
+        with pytest.raises(oracle.OracleError) as e:
+            oracle.run(b.events(), 1, 64)
+        assert e.value.bad_index == 1
+
+
+def test_validation_uses_each_kernels_grid():
+    # tid 100 is out of range for 1 x 64 but valid after a boundary to 2 x 64, and vice versa
+    b = tg.TraceBuilder(1, 64)
+    b.st(0, 1)
+    b.kernel_boundary(2, 64)
+    b.st(100, 1)
+    b.kernel_boundary(1, 32)
+    b.st(40, 2)                     # 1 x 32 grid: tid 40 is invalid here
+    with pytest.raises(oracle.OracleError) as e:
+        oracle.run(b.events(), 1, 64)
+    assert e.value.bad_index == 4

@@ -115,8 +115,14 @@ class TraceBuilder:
     def grid_sync(self):
         return self.ev(GRID_SYNC, 0, 0, NONE, 0xFFFFFFFF)
 
-    def kernel_boundary(self):
-        return self.ev(KERNEL_BOUNDARY, 0, 0, NONE, 0xFFFFFFFF)
+    def kernel_boundary(self, n_blocks: int = None, block_dim: int = None):
+        """End the kernel.  With a grid, the next kernel runs on (n_blocks, block_dim): the
+        boundary's addr carries (n_blocks << 32) | block_dim (per-kernel geometry)."""
+        if n_blocks is None:
+            return self.ev(KERNEL_BOUNDARY, 0, 0, NONE, 0xFFFFFFFF)
+        i = self.ev(KERNEL_BOUNDARY, 0, 0, NONE, 0xFFFFFFFF, addr=geometry_code(n_blocks, block_dim))
+        self.geom = Geometry(n_blocks, block_dim)
+        return i
 
     def events(self):
         out = np.zeros(len(self.rows), EVENT_DTYPE)
@@ -191,22 +197,31 @@ def random_trace(seed: int, n: int, n_blocks: int = None, block_dim: int = None,
     return b.events(), n_blocks, block_dim
 
 
-def boundary_event() -> np.ndarray:
-    """One KERNEL_BOUNDARY event (addr 0, tid 0, scope NONE)."""
+def geometry_code(n_blocks: int, block_dim: int) -> int:
+    """A KERNEL_BOUNDARY's addr announcing the next kernel's grid: (n_blocks << 32) | block_dim."""
+    return (int(n_blocks) << 32) | int(block_dim)
+
+
+def boundary_event(n_blocks: int = None, block_dim: int = None) -> np.ndarray:
+    """One KERNEL_BOUNDARY event (tid 0, scope NONE); addr 0 keeps the geometry, else it carries
+    the next kernel's grid."""
     e = np.zeros(1, EVENT_DTYPE)
     e["tk"] = pack_tk(0, KERNEL_BOUNDARY, NONE)
     e["mask"] = 0xFFFFFFFF
+    if n_blocks is not None:
+        e["addr"] = geometry_code(n_blocks, block_dim)
     return e
 
 
-def concat_kernels(traces) -> np.ndarray:
-    """Join per-kernel traces (same geometry) into one multi-kernel trace, a KERNEL_BOUNDARY
-    between consecutive kernels.  Returns the trace; kernel k's events start at
-    sum(len(t) + 1 for t in traces[:k])."""
+def concat_kernels(traces, geoms=None) -> np.ndarray:
+    """Join per-kernel traces into one multi-kernel trace, a KERNEL_BOUNDARY between consecutive
+    kernels.  ``geoms``: per-kernel (n_blocks, block_dim); when given, each boundary announces the
+    next kernel's grid (the trace descriptor carries the first).  Returns the trace; kernel k's
+    events start at sum(len(t) + 1 for t in traces[:k])."""
     parts = []
     for k, t in enumerate(traces):
         if k:
-            parts.append(boundary_event())
+            parts.append(boundary_event(*geoms[k]) if geoms is not None else boundary_event())
         parts.append(np.asarray(t, EVENT_DTYPE))
     return np.concatenate(parts) if parts else np.zeros(0, EVENT_DTYPE)
 
