@@ -219,6 +219,12 @@ __device__ __forceinline__ u32 ev_kind(const uint4& e) { return (e.z >> 24) & 0x
 __device__ __forceinline__ u32 ev_scope(const uint4& e) { return (e.z >> 28) & 0x3u; }
 __device__ __forceinline__ u64 ev_addr(const uint4& e) { return (u64)e.x | ((u64)e.y << 32); }
 
+// Reading A34 (per-kernel geometry): a KERNEL_BOUNDARY's nonzero addr = (n_blocks << 32) |
+// block_dim of the next kernel; valid when both are >= 1 and the grid has <= 2^24 threads
+__host__ __device__ __forceinline__ bool geo_code_ok(u32 nb, u32 bd) {
+    return nb >= 1 && bd >= 1 && (u64)nb * bd <= (1ull << 24);
+}
+
 // normalised scope: SYSTEM == DEVICE (reading A12)
 __device__ __forceinline__ u32 norm_scope(u32 s) { return s == IGD_SCOPE_SYSTEM ? IGD_SCOPE_DEVICE : s; }
 

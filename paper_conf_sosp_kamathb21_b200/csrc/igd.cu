@@ -24,6 +24,7 @@
 #include "sync.cuh"
 #include <dlfcn.h>
 #include <nccl.h>  // types and prototypes only: the library is resolved at run time (NcclApi)
+#include <algorithm>
 #include <vector>
 
 namespace {
@@ -108,6 +109,13 @@ struct igd_ctx {
     int nranks = 1, rank = 0;
     ncclComm_t comm = nullptr;
     Buf cl_small, cl_mat, cl_recv, cl_sidx, cl_sev, cl_nrep, cl_rep;
+    // per-kernel geometry (reading A34): the trace runs as segments between grid-changing
+    // kernel boundaries, each on its own grid
+    bool in_segment = false;
+    const igd_event* seg_ev = nullptr;
+    u64 seg_n = 0, seg_first = 0;
+    u32 seg_nb = 0, seg_bd = 0;
+    Buf gkb, seg_rep;
     igd_alloc_fn afn = nullptr;
     igd_free_fn ffn = nullptr;
     void* auser = nullptr;
@@ -426,15 +434,22 @@ static int canon_reports(igd_ctx* ctx, const igd_report* in, u64 n, u64 n_time) 
 // The pipeline.  Single GPU: the trace is `ctx->events`.  Sharded (ctx->shard): the
 // synchronization side runs over the all-gathered sync stream (global timestamps in sh_sidx),
 // the access side over the records this rank received in the all-to-all.
+// Segment mode (ctx->in_segment, reading A34): the events [seg_first, seg_first + seg_n) of one
+// kernel run on their own grid; reports and error indices are shifted to global indices.
+constexpr int IGD_SEGMENTS_NEEDED = 1;  // internal: the trace changes grids, run it per segment
 static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const igd_trace_desc& D = ctx->desc;
     const bool SH = ctx->shard;
-    const u64 n = SH ? ctx->sh_ntotal : D.n_events;               // timestamp domain [0, n)
-    const igd_event* src_ev = SH ? (const igd_event*)ctx->sh_sev : ctx->events;
-    const u64 n_src = SH ? ctx->sh_ns : D.n_events;                // events the ingest reads
+    const bool SEG = ctx->in_segment && !SH;
+    const igd_event* ev0 = SEG ? ctx->seg_ev : ctx->events;
+    const u64 n_ev = SEG ? ctx->seg_n : D.n_events;
+    const u64 first = SEG ? ctx->seg_first : 0;
+    const u64 n = SH ? ctx->sh_ntotal : n_ev;                      // timestamp domain [0, n)
+    const igd_event* src_ev = SH ? (const igd_event*)ctx->sh_sev : ev0;
+    const u64 n_src = SH ? ctx->sh_ns : n_ev;                      // events the ingest reads
     ctx->n_reports = 0;
     ctx->bad_event = 0;
-    if (!SH) {  // sharded: keep igd_shard_prepare's launches in the same accounting
+    if (!SH && !SEG) {  // sharded / segments: keep the earlier launches in the same accounting
         ctx->launches = 0;
         ctx->nk = 0;
     }
@@ -445,7 +460,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         return IGD_OK;
     }
     Geo g;
-    geo_init(g, D.n_blocks, D.block_dim);
+    geo_init(g, SEG ? ctx->seg_nb : D.n_blocks, SEG ? ctx->seg_bd : D.block_dim);
     KeySpace ks;
     ks.init(g);
     const int sms = sm_count(ctx);
@@ -460,7 +475,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     RET(ensure(ctx, ctx->ctr, 64));
     RET(ensure(ctx, ctx->st_in_a, (in_tiles + 1) * sizeof(u32)));
     RET(ensure(ctx, ctx->st_in_s, (in_tiles + 1) * sizeof(u32)));
-    const u64 acc_cap = SH ? ctx->sh_nrec : D.n_events;
+    const u64 acc_cap = SH ? ctx->sh_nrec : n_ev;
+    RET(ensure(ctx, ctx->gkb, 1024 * sizeof(u64)));
     const int vbytes = SH ? 16 : 8;  // sorted payload: (index | tk) or {index, tk, mask, 0}
     for (int b = 0; b < 2; b++) {
         RET(ensure(ctx, ctx->acc_k[b], acc_cap * sizeof(u32)));
@@ -483,6 +499,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     ip.tile_sync = P_<u32>(ctx->st_in_s);
     ip.hist_acc = P_<u32>(ctx->hist);
     ip.hist_sync = P_<u32>(ctx->hist) + 1024;
+    ip.gkb = P_<u64>(ctx->gkb);
+    ip.gkb_cap = (u32)(ctx->gkb.cap / sizeof(u64));
     ip.stats = P_<u64>(ctx->stats);
     ip.n_tiles = (u32)in_tiles;
     ip.skip_bits = nullptr;
@@ -514,8 +532,11 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     CK(cudaMemcpyAsync(&ctx->h_small[0], P_<u32>(ctx->st_in_a) + in_tiles, sizeof(u32), cudaMemcpyDeviceToHost,
                        ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
+    // grid-changing kernel boundaries (A34): the caller reruns the trace segment by segment (the
+    // events of later kernels were validated against the first kernel's grid here)
+    if (!SH && !SEG && ctx->h_stats[6] > 0) return IGD_SEGMENTS_NEEDED;
     if (ctx->h_stats[2] != ~0ull) {
-        ctx->bad_event = ctx->h_stats[2];
+        ctx->bad_event = ctx->h_stats[2] + first;
         ctx->err = "invalid event at index " + std::to_string(ctx->bad_event);
         return IGD_ETRACE;
     }
@@ -751,7 +772,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.val = ctx->acc_v[acur].p;
             cp.wbase = key64 ? kbase : wbase;
             cp.n = (u32)n_acc;
-            cp.ev = ctx->events;
+            cp.ev = ev0;
             cp.g = g;
             cp.ks = ks;
             cp.desc = P_<uint4>(ctx->ldesc);
@@ -767,7 +788,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.rep = P_<igd_report>(ctx->rep_raw);
             cp.rep_cap = ctx->rep_cap;
             cp.rep_ctr = P_<unsigned long long>(ctx->rep_ctr);
-            cp.first_event = 0;
+            cp.first_event = first;
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
@@ -784,7 +805,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     }
     mark(ctx, 5);
     // ---------------- a7: canonical order (ascending cur) ----------------
-    RET(canon_reports(ctx, P_<igd_report>(ctx->rep_raw), n_rep, n));
+    RET(canon_reports(ctx, P_<igd_report>(ctx->rep_raw), n_rep, first + n));
     mark(ctx, 6);
     CK(cudaStreamSynchronize(ctx->stream));
     mark(ctx, 7);
@@ -842,6 +863,10 @@ static int shard_prepare_impl(igd_ctx* ctx, u32 P, u64* counts, u64* n_sync_stre
     bad[0] = ctx->h_stats[2];
     minmax[0] = ctx->h_stats[0];
     minmax[1] = ctx->h_stats[1];
+    if (ctx->h_stats[3] && bad[0] == ~0ull) {
+        ctx->err = "kernel boundaries that change the grid (reading A34) need a single-GPU context";
+        return IGD_EINVAL;
+    }
     std::vector<u64> ob(P + 1, 0);
     u64 nrec = 0;
     for (u32 o = 0; o < P; o++) {
@@ -867,6 +892,85 @@ static int shard_prepare_impl(igd_ctx* ctx, u32 P, u64* counts, u64* n_sync_stre
     }
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(ctx->stream));
+    return IGD_OK;
+}
+
+// ---------------- per-kernel geometry (reading A34) ----------------
+// A KERNEL_BOUNDARY with a nonzero addr starts a kernel on another grid.  Every word's shadow
+// state and every lock table end at a boundary (A31), so the trace is exactly the concatenation
+// of its segments between such boundaries, each checked on its own grid (the composition law the
+// oracle is pinned by).  Pass 0 of the whole-trace run listed the boundaries; each segment is then
+// a full pipeline run with shifted indices, its reports appended in order (canonical by
+// construction).  The boundary events themselves are validated here, in trace order with the
+// segments, so the first invalid index is the oracle's.
+static int segmented_detect(igd_ctx* ctx, u64* n_out) {
+    const u64 ng = ctx->h_stats[6];
+    const u64 cap = ctx->gkb.cap / sizeof(u64);
+    if (ng > cap) {  // more grid changes than the list holds: a larger list, one more pass 0
+        RET(ensure(ctx, ctx->gkb, (ng + 1) * sizeof(u64)));
+        ctx->in_segment = false;
+        u64 dummy = 0;
+        int rc = detect_impl(ctx, &dummy);
+        if (rc != IGD_SEGMENTS_NEEDED) return rc == IGD_OK ? IGD_ECUDA : rc;
+    }
+    std::vector<u64> kb(ng);
+    CK(cudaMemcpyAsync(kb.data(), ctx->gkb.p, ng * sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
+    std::vector<igd_event> kev(ng);
+    CK(cudaStreamSynchronize(ctx->stream));
+    std::sort(kb.begin(), kb.end());
+    for (u64 k = 0; k < ng; k++)
+        CK(cudaMemcpyAsync(&kev[k], ctx->events + kb[k], sizeof(igd_event), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    const u64 N = ctx->desc.n_events;
+    u32 nb = ctx->desc.n_blocks, bd = ctx->desc.block_dim;
+    u64 total = 0, start = 0;
+    for (u64 k = 0; k <= ng; k++) {
+        const u64 end = k < ng ? kb[k] : N;
+        if (end > start) {
+            ctx->in_segment = true;
+            ctx->seg_ev = ctx->events + start;
+            ctx->seg_n = end - start;
+            ctx->seg_first = start;
+            ctx->seg_nb = nb;
+            ctx->seg_bd = bd;
+            u64 nk = 0;
+            int rc = detect_impl(ctx, &nk);
+            ctx->in_segment = false;
+            if (rc != IGD_OK) return rc;
+            if (nk) {
+                // append (a grown buffer keeps the earlier segments' reports)
+                if (ctx->seg_rep.cap < (total + nk) * sizeof(igd_report)) {
+                    Buf nb2;
+                    std::swap(nb2, ctx->seg_rep);
+                    RET(ensure(ctx, ctx->seg_rep, (total + nk) * 2 * sizeof(igd_report)));
+                    if (total)
+                        CK(cudaMemcpyAsync(ctx->seg_rep.p, nb2.p, total * sizeof(igd_report), cudaMemcpyDeviceToDevice,
+                                           ctx->stream));
+                    RET(buf_free(ctx, nb2));
+                }
+                CK(cudaMemcpyAsync((char*)ctx->seg_rep.p + total * sizeof(igd_report), ctx->rep_out.p,
+                                   nk * sizeof(igd_report), cudaMemcpyDeviceToDevice, ctx->stream));
+                total += nk;
+            }
+        }
+        if (k == ng) break;
+        // the boundary itself: KERNEL_BOUNDARY, tid 0, scope NONE, a valid grid code
+        const igd_event& e = kev[k];
+        const u32 kind = (e.tk >> 24) & 0xFu, tid = e.tk & 0xFFFFFFu, scope = (e.tk >> 28) & 3u;
+        const u32 nnb = (u32)(e.addr >> 32), nbd = (u32)e.addr;
+        if ((e.tk >> 30) || kind != IGD_KERNEL_BOUNDARY || tid != 0 || scope != 0 || !geo_code_ok(nnb, nbd)) {
+            ctx->bad_event = kb[k];
+            ctx->err = "invalid event at index " + std::to_string(kb[k]);
+            return IGD_ETRACE;
+        }
+        nb = nnb;
+        bd = nbd;
+        start = kb[k] + 1;
+    }
+    std::swap(ctx->seg_rep, ctx->rep_out);  // rep_out: all segments' reports, ascending cur
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->n_reports = total;
+    *n_out = total;
     return IGD_OK;
 }
 
@@ -1138,7 +1242,9 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     ctx->coalesce = (flags & IGD_DETECT_COALESCE) != 0;
     ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
     ctx->shard = false;
+    ctx->in_segment = false;
     int rc = detect_impl(ctx, n_reports_global);
+    if (rc == IGD_SEGMENTS_NEEDED) rc = segmented_detect(ctx, n_reports_global);
     ctx->coalesce = false;
     ctx->paper_counters = false;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
@@ -1291,7 +1397,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf,
                   &ctx->cl_small,     &ctx->cl_mat,   &ctx->cl_recv,  &ctx->cl_sidx,  &ctx->cl_sev,
-                  &ctx->cl_nrep,      &ctx->cl_rep};
+                  &ctx->cl_nrep,      &ctx->cl_rep,   &ctx->gkb,      &ctx->seg_rep};
     for (Buf* b : all) buf_free(ctx, *b);
     cudaStreamSynchronize(ctx->stream);
     cudaFreeHost(ctx->h_stats);

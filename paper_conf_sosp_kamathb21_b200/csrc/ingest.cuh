@@ -43,7 +43,10 @@ struct Params {
     u32* tile_sync;  // [n_tiles + 1] pass 0: sync records per tile; scanned to bases
     u32* hist_acc;   // [4][256]
     u32* hist_sync;  // [4][256]
-    u64* stats;      // [0] min word, [1] max word, [2] bad index, [3] n_acc, [4] n_sync, [5] n_lock
+    u64* stats;      // [0] min word, [1] max word, [2] bad index, [3] n_acc, [4] n_sync, [5] n_lock,
+                     // [6] kernel boundaries that change the grid (reading A34)
+    u64* gkb;        // pass 0: indices of those boundaries (first gkb_cap of them, any order)
+    u32 gkb_cap;
     u32 n_tiles;
     const u32* skip_bits;  // coalesced mode (A32): bit i = event i is checked by its group's first lane
     int hist0;       // pass 0, fused pipeline: the 4 digit histograms of the access keys (digit 0 for
@@ -95,7 +98,10 @@ __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpa
             case IGD_CG_BLOCK_SYNC:
                 ok = addr0 && scope == IGD_SCOPE_NONE;
                 break;
-            default:  // GRID_SYNC, CG_GRID_SYNC, KERNEL_BOUNDARY
+            case IGD_KERNEL_BOUNDARY:  // addr 0, or the next kernel's grid (reading A34)
+                ok = scope == IGD_SCOPE_NONE && tid == 0 && (addr0 || geo_code_ok(e.y, e.x));
+                break;
+            default:  // GRID_SYNC, CG_GRID_SYNC
                 ok = addr0 && scope == IGD_SCOPE_NONE && tid == 0;
                 break;
         }
@@ -131,6 +137,7 @@ __device__ __forceinline__ Dec decode(const uint4& e, const Geo& g, const KeySpa
     } else {
         d.s0 = kind == IGD_KERNEL_BOUNDARY ? ks.kb : ks.grid;
         d.flags = 1u << 1;
+        if (kind == IGD_KERNEL_BOUNDARY && !addr0) d.flags |= 32u;  // the grid changes (A34)
     }
     return d;
 }
@@ -216,6 +223,10 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
             const u32 v = (acc ? 1u : 0u) | (ns << 16);
             if (PASS == 0) {
                 if (f & 16u) bad = min(bad, base + (u64)j * THREADS + tid);
+                if (f & 32u) {  // rare: a kernel boundary announcing another grid
+                    const unsigned long long slot = atomicAdd((unsigned long long*)&P.stats[6], 1ull);
+                    if (slot < P.gkb_cap) P.gkb[slot] = base + (u64)j * THREADS + tid;
+                }
                 // digit 0 of the access keys for the fused first radix pass (fused.cuh); the other
                 // digits: k_hist_keys over its output
                 // the low digit is nearly always distinct across lanes: plain shared atomics on

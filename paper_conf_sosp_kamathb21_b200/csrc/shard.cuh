@@ -52,7 +52,8 @@ struct Params {
     uint4* send;
     u32* sync_idx;
     uint4* sync_ev;
-    u64* stats;     // [0] min word, [1] max word, [2] first bad global index
+    u64* stats;     // [0] min word, [1] max word, [2] first bad global index, [3] grid-changing kernel
+                    // boundaries (reading A34; single-context only)
 };
 
 template <int PASS>
@@ -81,6 +82,8 @@ __global__ void __launch_bounds__(THREADS, IGD_SHARD_MINB) k_shard(Params P) {
                 if (d.flags & 16u) {
                     bad = min(bad, P.first + i);
                 } else {
+                    // a grid change (A34) is single-context only: counted, the host refuses it
+                    if (PASS == 0 && (d.flags & 32u)) atomicAdd((unsigned long long*)&P.stats[3], 1ull);
                     const u32 kind = ev_kind(e[j]);
                     if (d.flags & 1u) {
                         dst[j] = 0x100u | (NP == 1 ? 0u : fmix32(d.key) % NP);

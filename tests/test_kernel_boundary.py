@@ -276,3 +276,61 @@ def test_validation_uses_each_kernels_grid():
     with pytest.raises(oracle.OracleError) as e:
         oracle.run(b.events(), 1, 64)
     assert e.value.bad_index == 4
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("batch", range(3))
+def test_gpu_mixed_geometry_kernels(det, batch):
+    # libigd runs the segments between grid changes on their own grids: identical to the oracle
+    for seed in range(1000 + batch * 40, 1000 + (batch + 1) * 40):
+        parts, geoms = mixed_geometry_kernels(seed, int(np.random.default_rng(seed).integers(2, 5)), 200)
+        joined = tg.concat_kernels(parts, geoms)
+        det.load(joined, *geoms[0])
+        det.detect()
+        assert np.array_equal(det.reports(), oracle.run(joined, *geoms[0])), f"seed {seed}"
+
+
+@pytest.mark.gpu
+def test_gpu_mixed_geometry_multi_tile(det):
+    # large kernels on different grids (several check / sort tiles per segment), plain boundaries
+    # inside a segment too
+    from test_gpu_parity import _fast_random
+
+    w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    geoms = [(3, 96), (16, 128), (5, 48), (9, 16)]
+    parts = [_fast_random(60 + k, 40_000 + 10_000 * k, 300, nb, bd, w)[0] for k, (nb, bd) in enumerate(geoms)]
+    parts[1] = tg.concat_kernels([parts[1], parts[1][:5000]])  # a same-grid boundary inside
+    joined = tg.concat_kernels(parts, geoms)
+    det.load(joined, *geoms[0])
+    det.detect()
+    want = oracle.run(joined, *geoms[0])
+    assert len(want) > 0 and np.array_equal(det.reports(), want)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("where", ["boundary_code", "tid_in_later_kernel", "first_kernel"])
+def test_gpu_mixed_geometry_bad_event(det, where):
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    b = tg.TraceBuilder(1, 64)
+    b.st(0, 1)
+    b.st(60, 2)
+    b.kernel_boundary(2, 64)
+    b.st(100, 1)
+    b.kernel_boundary(1, 32)
+    b.st(20, 2)
+    ev = b.events()
+    if where == "boundary_code":
+        ev["addr"][4] = 1 << 32            # block_dim 0
+    elif where == "tid_in_later_kernel":
+        ev["tk"][5] = tg.pack_tk(40, tg.ST, 0)   # tid 40 on a 1 x 32 grid
+        ev["mask"][5] = 1 << 8
+    else:
+        ev["tk"][1] = tg.pack_tk(70, tg.ST, 0)   # tid 70 on the first 1 x 64 grid
+        ev["mask"][1] = 1 << 6
+    with pytest.raises(oracle.OracleError) as eo:
+        oracle.run(ev, 1, 64)
+    det.load(ev, 1, 64)
+    with pytest.raises(igd.IgdError) as eg:
+        det.detect()
+    assert eg.value.code == igd.igd.IGD_ETRACE and eg.value.bad_index == eo.value.bad_index
