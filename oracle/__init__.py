@@ -66,6 +66,11 @@ def _load():
         lib.igdo_run.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                  ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
                                  ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
+        lib.igdo_run_ex3.restype = ctypes.c_int
+        lib.igdo_run_ex3.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                     ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
+                                     ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
+                                     ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
         lib.igdo_run_ex.restype = ctypes.c_int
         lib.igdo_run_ex.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                     ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p,
@@ -75,11 +80,16 @@ def _load():
 
 
 def run(events: np.ndarray, n_blocks: int, block_dim: int, shard=(0, 1), cap: int = None,
-        coalesce: bool = False, paper_counters: bool = False):
+        coalesce: bool = False, paper_counters: bool = False, sticky_flags: bool = False,
+        tag_log2: int = 0, last_k: int = 1):
     """Replay ``events`` (EVENT_DTYPE, 16 B each) and return the report array (REPORT_DTYPE),
     ascending by ``cur``.  ``shard=(k, K)`` checks only words owned by shard k (C.7 5(b)).
     ``coalesce``: warp-coalesced check mode (§6.5, reading A32).  ``paper_counters``: the
-    synchronization IDs wrap at Fig. 4's widths (reading A33)."""
+    synchronization IDs wrap at Fig. 4's widths (reading A33).  Paper-fidelity modes (SURVEY
+    8(f) f3): ``sticky_flags`` -- P3-P5 gated on the word's sticky DevShared / BlkShared flags as
+    Table 2 is written (reading A35); ``tag_log2`` -- metadata table of 2^tag_log2 entries with a
+    10-bit Tag, aliasing words (reading A36); ``last_k`` -- the last k accessors / writers are
+    checked (reading A37)."""
     lib = _load()
     ev = np.ascontiguousarray(events)
     assert ev.dtype.itemsize == 16
@@ -90,8 +100,9 @@ def run(events: np.ndarray, n_blocks: int, block_dim: int, shard=(0, 1), cap: in
         out = np.zeros(cap, REPORT_DTYPE)
         nrep = ctypes.c_uint64(0)
         bad = ctypes.c_uint64(0)
-        rc = lib.igdo_run_ex(ev.ctypes.data if n else None, n, n_blocks, block_dim, shard[0], shard[1],
-                             (1 if coalesce else 0) | (2 if paper_counters else 0), out.ctypes.data, cap, ctypes.byref(nrep), ctypes.byref(bad))
+        flags = (1 if coalesce else 0) | (2 if paper_counters else 0) | (4 if sticky_flags else 0)
+        rc = lib.igdo_run_ex3(ev.ctypes.data if n else None, n, n_blocks, block_dim, shard[0], shard[1], flags,
+                              tag_log2, last_k, out.ctypes.data, cap, ctypes.byref(nrep), ctypes.byref(bad))
         if rc != O_OK:
             raise OracleError(rc, bad.value if rc == O_ETRACE else None)
         if nrep.value <= cap:

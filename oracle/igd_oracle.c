@@ -98,7 +98,10 @@ typedef struct {
     uint8_t used;                 /* hash slot occupied */
     uint8_t valid, modified, atomic, ascope, devShared, blkShared;
     uint16_t locks;               /* Bloom of the last accessor's held locks (A7) */
+    uint32_t tag;                 /* tag-aliasing mode (A36): the 10-bit Tag of the entry's word */
     o_rec LA, LW;                 /* last accessor, last writer */
+    o_rec* hist;                  /* last-k mode (A37): [0,8) accessors, [8,16) writers, newest first */
+    uint8_t nla, nlw;             /*   how many of each are held */
 } o_shadow;
 
 typedef struct {
@@ -228,14 +231,17 @@ static void o_mark_coalesced(const uint8_t* events, uint64_t n, const o_geom* g,
  * total is returned in *n_reports.  On an ill-formed event returns O_ETRACE and its index
  * in *bad_index.
  */
-int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,
-                uint32_t shard_k, uint32_t shard_K, uint32_t flags, o_report* out, uint64_t cap,
-                uint64_t* n_reports, uint64_t* bad_index) {
+int igdo_run_ex3(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,
+                 uint32_t shard_k, uint32_t shard_K, uint32_t flags, uint32_t tag_log2, uint32_t hist_k,
+                 o_report* out, uint64_t cap, uint64_t* n_reports, uint64_t* bad_index) {
     *n_reports = 0;
     *bad_index = 0;
     if (n_blocks == 0 || block_dim == 0) return O_EINVAL;
     if ((uint64_t)n_blocks * block_dim > (1u << 24)) return O_EINVAL;
     if (shard_K == 0 || shard_k >= shard_K) return O_EINVAL;
+    if (tag_log2 != 0 && (tag_log2 < 8 || tag_log2 > 22)) return O_EINVAL;
+    if (hist_k != 1 && hist_k != 2 && hist_k != 4 && hist_k != 8) return O_EINVAL;
+    const int sticky = (flags & 4u) != 0; /* A35: literal sticky sharing flags in P3-P5 */
 
     o_geom g;
     o_geom_set(&g, n_blocks, block_dim);
@@ -369,16 +375,28 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
         uint32_t w_c = g_warp(&g, c), b_c = g_block(&g, c);
         uint16_t L = o_held_of(TABLE(c));                        /* 3.1: before own update (A11) */
 
-        int owned = (shard_K == 1) || ((o_fmix32((uint32_t)word ^ (uint32_t)(word >> 32)) % shard_K) == shard_k);
+        /* A36 tag aliasing: the metadata entry of `word` is word mod 2^tag_log2, and the entry's
+           10-bit Tag (Fig. 4) is the next 10 bits of the word */
+        uint64_t mkey = tag_log2 ? (word & ((1ull << tag_log2) - 1)) : word;
+        uint32_t tag = tag_log2 ? (uint32_t)((word >> tag_log2) & 1023u) : 0;
+        int owned = (shard_K == 1) || ((o_fmix32((uint32_t)mkey ^ (uint32_t)(mkey >> 32)) % shard_K) == shard_k);
         if (skip && skip[i]) owned = 0; /* A32: checked by its group's first lane */
         if (owned) {
-            o_shadow* S = o_map_get(&map, word);
+            o_shadow* S = o_map_get(&map, mkey);
             if (!S) { rc = O_ENOMEM; goto done; }
-            if (S->valid && S->kernel != kernel) {                /* A31: from an earlier kernel */
+            if (S->valid && (S->kernel != kernel || S->tag != tag)) {
+                /* A31: from an earlier kernel; A36: the entry belongs to another word (Tag
+                   mismatch) -- the access claims it as a fresh entry */
                 uint64_t wd = S->word;
+                o_rec* hh = S->hist;
                 memset(S, 0, sizeof(*S));
                 S->used = 1;
                 S->word = wd;
+                S->hist = hh;
+            }
+            if (hist_k > 1 && !S->hist) {
+                S->hist = (o_rec*)calloc(16, sizeof(o_rec));
+                if (!S->hist) { rc = O_ENOMEM; goto done; }
             }
             if (!S->valid) goto writeback;                        /* P1: first access (this kernel) */
 
@@ -390,8 +408,19 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
             }
             if (k == O_LD && !S->modified) goto writeback;        /* P2: no write (A25) */
 
-            {
-                const o_rec* md = (k == O_LD) ? &S->LW : &S->LA; /* Table 2 definitions */
+            /* A37 last-k histories (§6.7): the candidates md_1..md_K are the last K
+               writers (loads) or accessors (stores, atomics), newest first; each is checked in
+               turn and the first racy one is reported.  K = 1 is Table 2 as written. */
+            const o_rec* cands[8];
+            int ncand = 1;
+            cands[0] = (k == O_LD) ? &S->LW : &S->LA; /* Table 2 definitions */
+            if (hist_k > 1) {
+                int have = (k == O_LD) ? S->nlw : S->nla;
+                ncand = have < (int)hist_k ? have : (int)hist_k;
+                for (int q = 0; q < ncand; q++) cands[q] = &S->hist[(k == O_LD ? 8 : 0) + q];
+            }
+            for (int cq = 0; cq < ncand; cq++) {
+                const o_rec* md = cands[cq];
                 uint32_t p = md->tid;
                 uint32_t w_p = g_warp(&g, p), b_p = g_block(&g, p);
                 /* preliminary checks (reading A4: md.* = relation between md and curr) */
@@ -413,8 +442,14 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
                     noDev = (dDev & 63u) == 0;
                     noAny = noDev && (dBlk & 63u) == 0;
                 }
+                if (sticky) {
+                    /* A35 literal reading: Table 2 gates P3 and P4 on !DevShared AND !BlkShared
+                       and P5 on !DevShared, taken as the word's sticky flags */
+                    if (S->devShared || S->blkShared) { P3 = 0; P4 = 0; }
+                    if (S->devShared) P5 = 0;
+                }
                 int P6 = S->atomic && isAtomic && (b_p == b_c || S->ascope == S_DEVICE);
-                if (P3 || P4 || P5 || P6) goto writeback;
+                if (P3 || P4 || P5 || P6) continue;
 
                 /* race checks in order; first true is reported */
                 int type = R_NONE;
@@ -435,6 +470,7 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
                         r->prev_kind = (uint8_t)md->kind;
                     }
                     (*n_reports)++;
+                    break; /* at most one report per access (A21) */
                 }
             }
         writeback: /* Fig. 6 "Race -> Writeback": always done (A11) */
@@ -444,9 +480,20 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
                 r.sDEV = DEV(c); r.sANY = ANY(c); r.sWB = WB(w_c); r.sBB = BB(b_c);
                 S->valid = 1;
                 S->kernel = kernel;
+                S->tag = tag;
                 S->LA = r;
                 S->locks = L;
                 if (isWrite) { S->modified = 1; S->LW = r; }
+                if (S->hist) { /* A37: push the record onto the histories */
+                    memmove(&S->hist[1], &S->hist[0], 7 * sizeof(o_rec));
+                    S->hist[0] = r;
+                    if (S->nla < 8) S->nla++;
+                    if (isWrite) {
+                        memmove(&S->hist[9], &S->hist[8], 7 * sizeof(o_rec));
+                        S->hist[8] = r;
+                        if (S->nlw < 8) S->nlw++;
+                    }
+                }
                 if (isAtomic) { S->atomic = 1; S->ascope = (uint8_t)s; }
             }
         }
@@ -484,9 +531,18 @@ int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t b
     }
 
 done:
+    for (uint64_t q = 0; q < map.cap; q++)
+        if (map.slot[q].used) free(map.slot[q].hist);
     free(devF); free(anyF); free(wbar); free(bbar); free(wt); free(tt);
     free(isThread); free(touched); free(touched_list); free(map.slot); free(skip);
     return rc;
+}
+
+int igdo_run_ex(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,
+                uint32_t shard_k, uint32_t shard_K, uint32_t flags, o_report* out, uint64_t cap,
+                uint64_t* n_reports, uint64_t* bad_index) {
+    return igdo_run_ex3(events, n, n_blocks, block_dim, shard_k, shard_K, flags, 0, 1, out, cap, n_reports,
+                        bad_index);
 }
 
 int igdo_run(const uint8_t* events, uint64_t n, uint32_t n_blocks, uint32_t block_dim,

@@ -20,6 +20,7 @@ import tracegen as tg
 LD, ST, ATOM, CAS, EXCH, FENCE = 0, 1, 2, 3, 4, 5
 SYNCWARP, SYNCTHREADS, GRID = 6, 7, 8
 CG_TILE, CG_BLOCK, CG_GRID = 9, 10, 11
+KERNEL_BOUNDARY = 12
 ACCESS = (LD, ST, ATOM, CAS, EXCH)
 ATOMICS = (ATOM, CAS, EXCH)
 
@@ -338,3 +339,85 @@ def closed_form_syncfree(events, nb, bd):
     ty = typ[sel]
     o = np.argsort(cur, kind="stable")
     return a[o], cur[o], prev[o], ty[o]
+
+
+def bf_scratch_modes(events, nb, bd, sticky=False, tag_log2=0, last_k=1):
+    """From-scratch evaluator of the paper-fidelity modes, same approach as
+    bf_scratch -- every access rescans the history of its metadata entry:
+
+    * ``sticky`` (reading A35): P3 and P4 also need the entry's sticky DevShared and BlkShared
+      clear, P5 DevShared clear, as Table 2 writes them (P:1110-1122);
+    * ``tag_log2`` (reading A36): word w uses entry w mod 2^tag_log2 whose 10-bit Tag is the next
+      bits of w; the entry's history is the longest run of its most recent accesses that carry
+      the current access's tag (an access with another tag claimed the entry, P1);
+    * ``last_k`` (reading A37): the candidates are the last k writers (loads) or accessors,
+      newest first; the first racy candidate is reported.
+    Kernel boundaries (A31) end every history.  Returns the same tuples as bf_scratch."""
+    geo = _Geo(nb, bd)
+    addr, tid, kind, scope, mask, rawkind = _decode(events)
+    L = lock_replay(events, nb, bd)
+    C = (1 << tag_log2) if tag_log2 else None
+    out = []
+    hist = {}  # entry -> list of (access index, tag)
+    for i in range(len(kind)):
+        k = kind[i]
+        if k == KERNEL_BOUNDARY:
+            hist = {}
+            continue
+        if k not in ACCESS:
+            continue
+        a = addr[i] >> 2
+        ent, tag = (a % C, (a // C) % 1024) if C else (a, 0)
+        seq_all = hist.setdefault(ent, [])
+        H = []
+        for j, tj in reversed(seq_all):
+            if tj != tag:
+                break
+            H.insert(0, j)
+        if H:
+            c = tid[i]
+            writes = [j for j in H if kind[j] != LD]
+            seq = H + [i]
+            devS = any(geo.block(tid[x]) != geo.block(tid[y]) for x, y in zip(seq, seq[1:]))
+            blkS = any(geo.block(tid[x]) == geo.block(tid[y]) and geo.warp(tid[x]) != geo.warp(tid[y])
+                       for x, y in zip(seq, seq[1:]))
+            ats = [j for j in H if kind[j] in ATOMICS]
+            atomic = bool(ats)
+            ascope = scope[ats[-1]] if ats else 0
+            locks = L[H[-1]]
+            LW = writes[-1] if writes else None
+            if not (k == LD and LW is None):
+                cands = (writes if k == LD else H)[::-1][:last_k]
+                for md in cands:
+                    p = tid[md]
+                    same_w = geo.warp(p) == geo.warp(c)
+                    same_b = geo.block(p) == geo.block(c)
+                    P3 = p == c
+                    P4 = same_w and (_sync_between(kind, tid, scope, geo, md, i, "warp_bar", geo.warp(c))
+                                     or (mask[i] >> geo.lane(p)) & 1 == 1)
+                    P5 = same_b and _sync_between(kind, tid, scope, geo, md, i, "block_bar", geo.block(c))
+                    if sticky:
+                        P3 = P3 and not devS and not blkS
+                        P4 = P4 and not devS and not blkS
+                        P5 = P5 and not devS
+                    P6 = atomic and k in ATOMICS and (same_b or ascope == 2)
+                    if P3 or P4 or P5 or P6:
+                        continue
+                    noAny = not _sync_between(kind, tid, scope, geo, md, i, "any_fence", p)
+                    noDev = not _sync_between(kind, tid, scope, geo, md, i, "dev_fence", p)
+                    typ = 0
+                    if atomic and ascope == 1 and geo.block(tid[LW]) != geo.block(c):
+                        typ = 1
+                    elif same_w and noAny and not devS and not blkS:
+                        typ = 2
+                    elif same_b and noAny and not devS:
+                        typ = 3
+                    elif not same_b and noDev:
+                        typ = 4
+                    elif (locks | L[i]) != 0 and (locks & L[i]) == 0:
+                        typ = 5
+                    if typ:
+                        out.append((a << 2, i, md, typ, rawkind[i], rawkind[md]))
+                        break
+        seq_all.append((i, tag))
+    return out

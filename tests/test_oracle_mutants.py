@@ -56,6 +56,45 @@ MUTANTS = {
 }
 
 
+# paper-fidelity modes (A35-A37): caught by the mode brute force of tests/pins.py
+MODE_MUTANTS = {
+    "A35_P5_gated_on_blkShared_too": ("if (S->devShared) P5 = 0;", "if (S->devShared || S->blkShared) P5 = 0;"),
+    "A35_P3_not_gated": ("if (S->devShared || S->blkShared) { P3 = 0; P4 = 0; }", "if (S->devShared || S->blkShared) { P4 = 0; }"),
+    "A36_tag_ignored": ("(S->kernel != kernel || S->tag != tag)", "(S->kernel != kernel)"),
+    "A36_tag_9_bits": ("(uint32_t)((word >> tag_log2) & 1023u)", "(uint32_t)((word >> tag_log2) & 511u)"),
+    "A37_oldest_first": ("cands[q] = &S->hist[(k == O_LD ? 8 : 0) + q];",
+                         "cands[q] = &S->hist[(k == O_LD ? 8 : 0) + ncand - 1 - q];"),
+    "A37_writers_for_stores": ("cands[q] = &S->hist[(k == O_LD ? 8 : 0) + q];", "cands[q] = &S->hist[8 + q];"),
+}
+
+
+def _run_mode(lib, ev, nb, bd, flags, tag_log2, last_k):
+    cap = 4096
+    out = np.zeros(cap, REPORT)
+    nrep, bad = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    rc = lib.igdo_run_ex3(ev.ctypes.data if len(ev) else None, len(ev), nb, bd, 0, 1, flags, tag_log2, last_k,
+                          out.ctypes.data, cap, ctypes.byref(nrep), ctypes.byref(bad))
+    assert rc == 0
+    return full_tuples(out[: nrep.value])
+
+
+def _caught_modes(lib):
+    from pins import bf_scratch_modes
+    from test_fidelity_modes import _tag_trace
+
+    for seed in range(150):
+        rng = np.random.default_rng(seed)
+        ev, nb, bd = tg.random_trace(seed, int(rng.integers(20, 150)), n_words=int(rng.integers(1, 6)))
+        if _run_mode(lib, ev, nb, bd, 4, 0, 1) != bf_scratch_modes(ev, nb, bd, sticky=True):
+            return f"sticky seed {seed}"
+        if _run_mode(lib, ev, nb, bd, 0, 0, 4) != bf_scratch_modes(ev, nb, bd, last_k=4):
+            return f"last-k seed {seed}"
+        ev, nb, bd = _tag_trace(seed, 120, 8)
+        if _run_mode(lib, ev, nb, bd, 0, 8, 1) != bf_scratch_modes(ev, nb, bd, tag_log2=8):
+            return f"tag seed {seed}"
+    return None
+
+
 def _build(mutant_src, d):
     c = os.path.join(d, "m.c")
     so = os.path.join(d, "m.so")
@@ -67,6 +106,10 @@ def _build(mutant_src, d):
     lib.igdo_run.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                              ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
                              ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
+    lib.igdo_run_ex3.restype = ctypes.c_int
+    lib.igdo_run_ex3.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
+                                 ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p,
+                                 ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
     lib.igdo_run_ex.restype = ctypes.c_int
     lib.igdo_run_ex.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                 ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64,
@@ -122,3 +165,13 @@ def test_mutant_is_caught(name):
     with tempfile.TemporaryDirectory() as d:
         lib = _build(src.replace(old, new, 1), d)
         assert _caught(lib) is not None, f"mutant {name} survived every pin"
+
+
+@pytest.mark.parametrize("name", sorted(MODE_MUTANTS))
+def test_mode_mutant_is_caught(name):
+    src = open(SRC).read()
+    old, new = MODE_MUTANTS[name]
+    assert src.count(old) >= 1, f"mutation anchor vanished: {old!r}"
+    with tempfile.TemporaryDirectory() as d:
+        lib = _build(src.replace(old, new, 1), d)
+        assert _caught_modes(lib) is not None, f"mutant {name} survived every pin"
