@@ -163,6 +163,19 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
    unchanged (the paper's bounded-counter false positives, §6.7).  Default: exact counters (A16).
    Also accepted by igd_shard_detect. */
 #define IGD_DETECT_PAPER_COUNTERS 4u
+/* Paper-fidelity modes (off by default, combinable):
+   IGD_DETECT_STICKY_FLAGS (reading A35): Table 2 as written -- P3 and P4 also need the word's
+     sticky DevShared and BlkShared flags clear, P5 DevShared clear.  The default
+     reading A4 derives them from md and the current access.  Also accepted by igd_shard_detect
+     and collective contexts.
+   IGD_DETECT_TAG_LOG2(b), 8 <= b <= 22 (reading A36): the metadata of Fig. 4 as a table of 2^b
+     entries with a 10-bit Tag: word w uses entry w mod 2^b with Tag
+     (w >> b) mod 2^10; an access whose Tag differs from the entry's claims it (a first access),
+     words with equal entry and Tag share it.  Reports carry the accessed word's address.
+     Single-GPU contexts only (IGD_EINVAL otherwise). */
+#define IGD_DETECT_STICKY_FLAGS 8u
+#define IGD_DETECT_TAG_SHIFT 8
+#define IGD_DETECT_TAG_LOG2(b) ((uint32_t)(b) << IGD_DETECT_TAG_SHIFT)
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global);
 /* Collective contexts (created with an NCCL id): every rank calls igd_detect after loading its
    contiguous chunk [desc.first_event, desc.first_event + desc.n_events) of one global trace of

@@ -132,6 +132,7 @@ struct Params {
     u64 rep_cap;
     unsigned long long* rep_ctr;
     u64 first_event; // global index offset (multi-rank)
+    u32 addr_from_ev;  // tag-aliasing mode (A36): keys hold entry + tag, report addresses come from the trace
 };
 
 // Grid-sync bucket table: gtab[b] = {index, timestamp} of the first grid sync with timestamp >=

@@ -88,8 +88,12 @@ __device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, co
 // KB: the trace has kernel boundaries (a separate instantiation: the boundary test costs
 // registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
 // KT: u32 word keys (low 32 bits; spans < 2^32 words) or u64 keys (word - wbase, a4's wide path)
-template <bool MV, bool KB, bool WRAP, bool GEO2, typename KT = u32>
+// FID: paper-fidelity bits -- 1 = Fig. 4-width synchronization IDs (reading A33), 2 = sticky
+// sharing flags gate P3-P5 as Table 2 is written (reading A35)
+template <bool MV, bool KB, int FID, bool GEO2, typename KT = u32>
 __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
+    constexpr bool WRAP = (FID & 1) != 0;
+    constexpr bool STK = (FID & 2) != 0;
     __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
     __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
     __shared__ uint8_t q_f[C4_TILE];              // queue flags
@@ -335,7 +339,9 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                     same_b = bp == bc;
                     same_w = same_b && (GEO2 ? (p >> 5) == (c >> 5) : ((p - bp * g.D) >> 5) == ((c - bc * g.D) >> 5));
                 }
-                if (same_t) {  // P3: program order
+                // A35 (sticky mode): P3 / P4 need the word never shared across warps or blocks
+                const bool unshared = !STK || (!dev && !blk);
+                if (same_t && unshared) {  // P3: program order
                     CSTAT(2);
                     break;
                 }
@@ -346,8 +352,8 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 // P4 lockstep clause: md's lane in this instruction's active mask (tk bit 31: full
                 // warp; bit 30: own lane only; otherwise the mask itself, from the payload in MV
                 // mode, else gathered from the trace)
-                if (same_w && (Z[j] >> 31)) break;
-                if (same_w && !(Z[j] >> 30)) {
+                if (same_w && unshared && (Z[j] >> 31)) break;
+                if (same_w && unshared && !(Z[j] >> 30)) {
                     if (p == IGD_NONE32) p = tk_at(mdp) & 0xFFFFFFu;
                     // prefetched unless md is an earlier writer (M[j] is the mask then only
                     // if the previous access was also a same-warp candidate)
@@ -405,13 +411,16 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         }
         const u32 p = mdz & 0xFFFFFFu;
         const bool same_w = flags & QF_SAME_W, same_b = flags & QF_SAME_B;
+        // A35 (sticky mode): P4 needs neither sharing flag, P5 no DevShared
+        const bool p4w = same_w && (!STK || !(flags & (QF_DEV | QF_BLK)));
+        const bool p5b = same_b && (!STK || !(flags & QF_DEV));
         u32 type;
         if (WRAP) {
             // reading A33: an ID moved iff the number of its events since md is not a multiple of
             // 2^width (Fig. 4: WarpBarID 6, BlkBarID 8, DevFenceID 6, BlkFenceID 6 bits)
             const u32 gcnt = P.glo != P.ghi ? q_count(P.desc, P.sts, ks.grid, mdIdx, i) : 0u;
-            if (same_w && (q_count(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i) & 63u)) continue;  // P4
-            if (same_b && ((q_count(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i) + gcnt) & 255u)) continue;  // P5
+            if (p4w && (q_count(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i) & 63u)) continue;  // P4
+            if (p5b && ((q_count(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i) + gcnt) & 255u)) continue;  // P5
             type = (flags & QF_R1) ? IGD_R1 : 0u;
             if (!type) {
                 const u32 dfen = q_count(P.desc, P.sts, ks.dev + p, mdIdx, i);  // device fences of md's thread
@@ -426,9 +435,9 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 }
             }
         } else {
-        if (same_w && q_between(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i)) continue;  // P4: syncwarp
+        if (p4w && q_between(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i)) continue;  // P4: syncwarp
         const bool grid = q_grid(P, mdIdx, i);
-        if (same_b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) continue;  // P5
+        if (p5b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) continue;  // P5
         type = (flags & QF_R1) ? IGD_R1 : 0u;
         if (!type) {
             if (same_b) {
@@ -461,7 +470,8 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             if (slot < P.rep_cap) {
                 igd_report r;
                 // full word from the 32-bit key: the accessed words span < 2^32 from wbase
-                if (sizeof(KT) == 8) r.addr = (P.wbase + (u64)__ldg(keys + x)) << 2;  // key = word - wbase
+                if (P.addr_from_ev) r.addr = ev_addr(ld_event(P.ev, i)) & ~3ull;  // tag mode (A36): the key is the entry
+                else if (sizeof(KT) == 8) r.addr = (P.wbase + (u64)__ldg(keys + x)) << 2;  // key = word - wbase
                 else r.addr = (P.wbase + (u32)((u32)__ldg(keys + x) - (u32)P.wbase)) << 2;
                 r.cur = P.first_event + i;
                 r.prev = P.first_event + mdIdx;

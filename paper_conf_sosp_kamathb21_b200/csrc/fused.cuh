@@ -53,6 +53,8 @@ struct Params {
     u32* tile_ctr;          // zeroed: tile tickets (CTA start order, see rsort::k_onesweep)
     void* kout;             // access keys (u32 or u64, template KT), sorted by digit 0
     u64 kbase;              // KT = u64: key = word - kbase (kbase's low 8 bits are 0)
+    u32 keymask;            // KT = u32: key = low 32 bits of the word & keymask (tag mode, A36:
+                            // entry + 10-bit Tag); all ones otherwise
     u64* vout;              // access payload (event index | tk << 32), same order
     const u32* skip_bits;   // coalesced mode (A32): bit i = event i is not an access record
 };
@@ -171,7 +173,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
         if (COAL && d.acc && in && ((__ldg(P.skip_bits + ((base + p) >> 5)) >> (p & 31u)) & 1u))
             d.acc = false;  // A32: checked by its coalesced group's first lane
         if (sizeof(KT) == 8) key[j] = (KT)((((u64)ev.y << 32) | ev.x) >> 2) - (KT)P.kbase;
-        else key[j] = (KT)d.key;
+        else key[j] = (KT)(d.key & P.keymask);
         tk[j] = d.tk;
         amask |= ((in && d.acc) ? 1u : 0u) << j;
         if (IGD_FUSED_EARLY && in && d.acc) atomicAdd(&s_cnt[(u32)key[j] & 255u], 1u);

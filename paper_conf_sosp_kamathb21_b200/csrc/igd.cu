@@ -134,6 +134,8 @@ struct igd_ctx {
     u64 rep_cap = 0;
     bool coalesce = false;  // IGD_DETECT_COALESCE of the running igd_detect (reading A32)
     bool paper_counters = false;  // IGD_DETECT_PAPER_COUNTERS (reading A33)
+    bool sticky = false;          // IGD_DETECT_STICKY_FLAGS (reading A35)
+    u32 tag_log2 = 0;             // IGD_DETECT_TAG_LOG2 (reading A36): 0 = exact per-word state
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
     bool shard = false;
@@ -322,6 +324,7 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         pp.vout = v[cur ^ 1].p;
         pp.n = (u32)n;
         pp.shift = p * 8;
+        pp.dmask = max_bits >= p * 8 + 8 ? 255u : (1u << (max_bits - p * 8)) - 1u;
         pp.digit_base = P_<u32>(ctx->base) + p * 256;
         pp.status = P_<u64>(ctx->status);
         pp.tile_ctr = P_<u32>(ctx->ctr);
@@ -342,35 +345,44 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
     return IGD_OK;
 }
 
-// a6 kernel instantiation: sharded payload (MV), kernel boundaries (KB), paper-width IDs (WRAP)
+// a6 kernel instantiation: sharded payload (MV), kernel boundaries (KB), paper-fidelity bits
+// (FID: 1 = Fig. 4-width IDs, A33; 2 = sticky sharing flags, A35), power-of-two geometry (GEO2),
+// u64 keys (a4's wide path).  The fidelity modes and the wide path use the general-geometry
+// instantiation only (fewer kernels to build; they are not the timed path).
 template <bool MV, bool KB>
-static void launch_check_w(bool wrap, unsigned tb, cudaStream_t st, const check::Params& cp) {
+static void launch_check_w(int fid, unsigned tb, cudaStream_t st, const check::Params& cp) {
     // power-of-two geometry (block_dim >= 32): shift / mask instead of divisions (common case)
     const bool geo2 = cp.g.dlog < 32 && cp.g.D >= 32;
-    if (wrap) {
-        if (geo2) check::k_check4<MV, KB, true, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
-        else check::k_check4<MV, KB, true, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
-    } else {
-        if (geo2) check::k_check4<MV, KB, false, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
-        else check::k_check4<MV, KB, false, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+    switch (fid) {
+        case 0:
+            if (geo2) check::k_check4<MV, KB, 0, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
+            else check::k_check4<MV, KB, 0, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+            break;
+        case 1: check::k_check4<MV, KB, 1, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 2: check::k_check4<MV, KB, 2, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        default: check::k_check4<MV, KB, 3, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
     }
 }
-static void launch_check(bool mv, bool kb, bool wrap, bool key64, unsigned tb, cudaStream_t st,
+template <bool KB>
+static void launch_check_64(int fid, unsigned tb, cudaStream_t st, const check::Params& cp) {
+    switch (fid) {
+        case 0: check::k_check4<false, KB, 0, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 1: check::k_check4<false, KB, 1, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 2: check::k_check4<false, KB, 2, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        default: check::k_check4<false, KB, 3, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+    }
+}
+static void launch_check(bool mv, bool kb, int fid, bool key64, unsigned tb, cudaStream_t st,
                          const check::Params& cp) {
-    if (key64) {  // a4's wide path (single GPU): general geometry instantiation
-        if (kb) {
-            if (wrap) check::k_check4<false, true, true, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
-            else check::k_check4<false, true, false, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
-        } else {
-            if (wrap) check::k_check4<false, false, true, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
-            else check::k_check4<false, false, false, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp);
-        }
+    if (key64) {  // a4's wide path (single GPU)
+        if (kb) launch_check_64<true>(fid, tb, st, cp);
+        else launch_check_64<false>(fid, tb, st, cp);
         return;
     }
-    if (mv && kb) launch_check_w<true, true>(wrap, tb, st, cp);
-    else if (mv) launch_check_w<true, false>(wrap, tb, st, cp);
-    else if (kb) launch_check_w<false, true>(wrap, tb, st, cp);
-    else launch_check_w<false, false>(wrap, tb, st, cp);
+    if (mv && kb) launch_check_w<true, true>(fid, tb, st, cp);
+    else if (mv) launch_check_w<true, false>(fid, tb, st, cp);
+    else if (kb) launch_check_w<false, true>(fid, tb, st, cp);
+    else launch_check_w<false, false>(fid, tb, st, cp);
 }
 
 static int scan_excl(igd_ctx* ctx, u32* data, u64 n) {
@@ -547,7 +559,13 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     if (n_sync + 64 > 0xFFFFFFFFull) return IGD_ETOOBIG;  // 32-bit record positions
     // a4: accessed words spanning >= 2^32 words (sparse virtual addresses) take the wide path:
     // u64 keys word - kbase, sorted over ceil(bits(span) / 8) digit passes
-    const bool key64 = !SH && n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32);
+    // A36 tag mode: keys = low (tag_log2 + 10) bits of the word (entry + Tag), sorted by the entry
+    const u32 TG = SH ? 0u : ctx->tag_log2;
+    const bool key64 = !SH && !TG && n_acc > 0 && ctx->h_stats[1] - ctx->h_stats[0] >= (1ull << 32);
+    if (TG && !FUSED) {
+        ctx->err = "the tag-aliasing mode needs the fused ingest pipeline";
+        return IGD_EINVAL;
+    }
     const u64 kbase = key64 ? (ctx->h_stats[0] & ~255ull) : 0;  // low digit unchanged: pass 0's histogram holds
     if (key64) {
         if (!FUSED) {
@@ -591,6 +609,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         fp.tile_ctr = P_<u32>(ctx->ctr);
         fp.kout = ctx->acc_k[1].p;
         fp.kbase = kbase;
+        fp.keymask = TG ? (u32)((1ull << (TG + 10)) - 1) : 0xFFFFFFFFu;
         fp.vout = P_<u64>(ctx->acc_v[1]);
         fp.skip_bits = ip.skip_bits;
         {
@@ -636,6 +655,14 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         KTimer kt(ctx, KC_INGEST, 8.0 * (double)n_acc);
         const unsigned hb = (unsigned)std::min<u64>((n_acc + 255) / 256, (u64)sms * 8);
         rsort::k_hist8<<<hb, 256, 0, ctx->stream>>>(P_<u64>(ctx->acc_k[1]), n_acc, P_<u32>(ctx->hist) + 2048, 1);
+    }
+    if (TG && n_acc > 0) {
+        // tag mode: the sort runs over the entry bits only; digits 1..3 of the masked keys
+        CK(cudaMemsetAsync(P_<u32>(ctx->hist) + 256, 0, 768 * sizeof(u32), ctx->stream));
+        KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);
+        const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
+        ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[1]), (u32)n_acc, P_<u32>(ctx->hist), 1,
+                                                         (u32)((1ull << TG) - 1));
     }
     if (FUSED && n_sync > 0) {
         // sync-key digit histograms over the records the fused pass wrote (trace order)
@@ -748,8 +775,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist) + 2048, h_hist64.data(),
                        bits_needed(ctx->h_stats[1] - kbase), &acur, vbytes, 1, 1, nullptr, 8));
     else
-        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc, 32, &acur,
-                       vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0, SH ? ctx->sh_rec : nullptr));
+        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc,
+                       TG ? TG : 32u, &acur, vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0, SH ? ctx->sh_rec : nullptr));
     ctx->last_acur = acur;
     ctx->last_nacc = SH ? 0 : n_acc;
     mark(ctx, 4);
@@ -789,10 +816,12 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.rep_cap = ctx->rep_cap;
             cp.rep_ctr = P_<unsigned long long>(ctx->rep_ctr);
             cp.first_event = first;
+            cp.addr_from_ev = TG ? 1u : 0u;
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
-                launch_check(SH, cp.has_kb != 0, ctx->paper_counters, key64, (unsigned)tiles, ctx->stream, cp);
+                launch_check(SH, cp.has_kb != 0, (ctx->paper_counters ? 1 : 0) | (ctx->sticky ? 2 : 0), key64,
+                             (unsigned)tiles, ctx->stream, cp);
             }
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
@@ -1219,16 +1248,27 @@ static void collect_timing(igd_ctx* ctx);
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     if (!ctx || !n_reports_global) return IGD_EINVAL;
     if (!ctx->loaded) return IGD_ESTATE;
+    const u32 tag_log2 = (flags >> IGD_DETECT_TAG_SHIFT) & 31u;
+    if (tag_log2 && (tag_log2 < 8 || tag_log2 > 22)) {
+        ctx->err = "IGD_DETECT_TAG_LOG2 must be 8..22";
+        return IGD_EINVAL;
+    }
     if (ctx->comm) {  // collective over the communicator's ranks
         if (flags & IGD_DETECT_COALESCE) {  // reading A32: a group may straddle two ranks' chunks
             ctx->err = "IGD_DETECT_COALESCE is a single-context mode";
             return IGD_EINVAL;
         }
+        if (tag_log2) {  // A36: the owner hash would have to be over metadata entries
+            ctx->err = "the tag-aliasing mode is a single-context mode";
+            return IGD_EINVAL;
+        }
         cudaSetDevice(ctx->device);
         ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
         ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
+        ctx->sticky = (flags & IGD_DETECT_STICKY_FLAGS) != 0;
         int rc = collective_detect(ctx, n_reports_global);
         ctx->paper_counters = false;
+        ctx->sticky = false;
         if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
         return rc;
     }
@@ -1241,12 +1281,16 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
     ctx->coalesce = (flags & IGD_DETECT_COALESCE) != 0;
     ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
+    ctx->sticky = (flags & IGD_DETECT_STICKY_FLAGS) != 0;
+    ctx->tag_log2 = tag_log2;
     ctx->shard = false;
     ctx->in_segment = false;
     int rc = detect_impl(ctx, n_reports_global);
     if (rc == IGD_SEGMENTS_NEEDED) rc = segmented_detect(ctx, n_reports_global);
     ctx->coalesce = false;
     ctx->paper_counters = false;
+    ctx->sticky = false;
+    ctx->tag_log2 = 0;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
     return rc;
 }
@@ -1288,6 +1332,11 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     cudaSetDevice(ctx->device);
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
     ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
+    ctx->sticky = (flags & IGD_DETECT_STICKY_FLAGS) != 0;
+    if ((flags >> IGD_DETECT_TAG_SHIFT) & 31u) {
+        ctx->err = "the tag-aliasing mode is a single-context mode";
+        return IGD_EINVAL;
+    }
     ctx->shard = true;
     ctx->sh_rec = d_records;
     ctx->sh_nrec = n_records;
@@ -1306,6 +1355,7 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     if (aliased) buf_free(ctx, ctx->sh_send);
     ctx->shard = false;
     ctx->paper_counters = false;
+    ctx->sticky = false;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
     return rc;
 }

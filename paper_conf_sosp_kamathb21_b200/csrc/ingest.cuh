@@ -388,7 +388,7 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
 // Digit histograms (4 x 8-bit) of the compacted access keys: a light, high-occupancy pass over
 // 4 bytes per access, with warp-uniform digits aggregated into one shared atomic.
 __global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys, u32 n, u32* __restrict__ hist,
-                                                   int first_digit) {
+                                                   int first_digit, u32 kmask = 0xFFFFFFFFu) {
     __shared__ u32 s[4][256];
     const u32 lane = threadIdx.x & 31u;
     for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&s[0][0])[i] = 0;
@@ -397,7 +397,7 @@ __global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys,
     for (u32 q = blockIdx.x * blockDim.x + threadIdx.x; q - lane < n4; q += gridDim.x * blockDim.x) {
         const bool in = q < n4;
         const uint4 k4 = in ? __ldcs(reinterpret_cast<const uint4*>(keys) + q) : make_uint4(0, 0, 0, 0);
-        const u32 kk[4] = {k4.x, k4.y, k4.z, k4.w};
+        const u32 kk[4] = {k4.x & kmask, k4.y & kmask, k4.z & kmask, k4.w & kmask};
 #pragma unroll
         for (int e = 0; e < 4; e++)
 #pragma unroll
@@ -406,7 +406,7 @@ __global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys,
     }
     if (blockIdx.x == 0)  // the n % 4 tail
         for (u32 i = n4 * 4 + threadIdx.x; i < n; i += blockDim.x) {
-            const u32 k = keys[i];
+            const u32 k = keys[i] & kmask;
 #pragma unroll
             for (int p = 0; p < 4; p++)
                 if (p >= first_digit) atomicAdd(&s[p][(k >> (8 * p)) & 255u], 1u);

@@ -94,6 +94,7 @@ struct PassParams {
     void* vout;
     u32 n;
     u32 shift;
+    u32 dmask;              // 255, or fewer bits for the top digit of a masked key (tag mode, A36)
     const u32* digit_base;  // [256] exclusive global offsets of this pass's digits
     u64* status;            // [n_tiles * 256], zeroed
     u32* tile_ctr;          // zeroed before the pass: tile tickets (the TAIL launch follows the full one)
@@ -171,7 +172,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     const u32 base = tile * TILE;  // n <= 2^32 - 2^13 (checked by the host)
     const u32 wofs = warp * 32 * ITEMS;
     const u32 wbase = base + wofs;
-    const u32 shift = P.shift;
+    const u32 shift = P.shift, dmask = P.dmask;
     constexpr bool full = !TAIL;
 
     KT key[ITEMS];
@@ -190,7 +191,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         // tile digit counts first, published before ranking (see fused.cuh)
 #pragma unroll
         for (int j = 0; j < ITEMS; j++)
-            if (full || wbase + j * 32 + lane < P.n) atomicAdd(&s_cnt[(u32)(key[j] >> shift) & 255u], 1u);
+            if (full || wbase + j * 32 + lane < P.n) atomicAdd(&s_cnt[(u32)(key[j] >> shift) & dmask], 1u);
         __syncthreads();
         st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
     }
@@ -200,7 +201,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     for (int j = 0; j < ITEMS; j++) {
         const bool valid = full || wbase + j * 32 + lane < P.n;
         const u32 vmask = full ? IGD_FULL : __ballot_sync(IGD_FULL, valid);
-        const u32 d = (u32)(key[j] >> shift) & 255u;
+        const u32 d = (u32)(key[j] >> shift) & dmask;
         // invalid lanes (last tile) get a unique out-of-range digit; masked out of every peer set.
         // IGD_SORT_MIX = N: one row in N is ranked with match.any (MIO pipe), the others with the
         // 8 ballots (ALU / issue): the two bottleneck on different units
@@ -283,7 +284,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     // keys: reorder in shared memory (rank[] becomes the tile position), write digit runs
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
-        const u32 d = (u32)(key[j] >> shift) & 255u;
+        const u32 d = (u32)(key[j] >> shift) & dmask;
         rank[j] += s_tile_excl[d] + s_whist[warp][d];
         if (full || wbase + j * 32 + lane < P.n) s_k[rank[j]] = key[j];
     }
@@ -294,7 +295,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         const u32 i = t + k * THREADS;
         if (i < tile_n) {
             const KT kk = s_k[i];
-            const u32 d = (u32)(kk >> shift) & 255u;
+            const u32 d = (u32)(kk >> shift) & dmask;
             s_dig[i] = (uint8_t)d;
             __stcs(kout + (s_gbase[d] + i), kk);
         }

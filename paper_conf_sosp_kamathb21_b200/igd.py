@@ -21,6 +21,8 @@ IGD_TRACE_DEVICE_PTR = 1
 IGD_DETECT_TIMING = 1
 IGD_DETECT_COALESCE = 2
 IGD_DETECT_PAPER_COUNTERS = 4
+IGD_DETECT_STICKY_FLAGS = 8
+IGD_DETECT_TAG_SHIFT = 8
 IGD_N_STAGES = 8
 IGD_N_KCLASS = 9
 
@@ -235,11 +237,15 @@ class Detector:
             igd_trace_load(self.ctx, n_blocks, block_dim, ev.ctypes.data if len(ev) else 0, len(ev), False,
                            first_event, n_events_total)
 
-    def detect(self, timing: bool = False, coalesce: bool = False, paper_counters: bool = False) -> int:
+    def detect(self, timing: bool = False, coalesce: bool = False, paper_counters: bool = False,
+               sticky_flags: bool = False, tag_log2: int = 0) -> int:
         """igd_detect; ``coalesce``: warp-coalesced check mode (IGD_DETECT_COALESCE, reading A32);
-        ``paper_counters``: Fig. 4-width synchronization IDs (IGD_DETECT_PAPER_COUNTERS, A33)."""
+        ``paper_counters``: Fig. 4-width synchronization IDs (IGD_DETECT_PAPER_COUNTERS, A33);
+        ``sticky_flags``: Table 2's sticky sharing flags in P3-P5 (IGD_DETECT_STICKY_FLAGS, A35);
+        ``tag_log2``: a 2^tag_log2-entry metadata table with 10-bit Tags (IGD_DETECT_TAG_LOG2, A36)."""
         flags = ((IGD_DETECT_TIMING if timing else 0) | (IGD_DETECT_COALESCE if coalesce else 0)
-                 | (IGD_DETECT_PAPER_COUNTERS if paper_counters else 0))
+                 | (IGD_DETECT_PAPER_COUNTERS if paper_counters else 0)
+                 | (IGD_DETECT_STICKY_FLAGS if sticky_flags else 0) | (int(tag_log2) << IGD_DETECT_TAG_SHIFT))
         self.n_reports = igd_detect(self.ctx, flags)
         return self.n_reports
 

@@ -167,3 +167,73 @@ def test_modes_reject_bad_parameters():
     for kw in (dict(tag_log2=7), dict(tag_log2=23), dict(last_k=3)):
         with pytest.raises(oracle.OracleError):
             oracle.run(ev, 1, 32, **kw)
+
+
+# ---------------- GPU parity of the modes (libigd through the C ABI) ----------------
+@pytest.fixture(scope="module")
+def det():
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    d = igd.Detector(0)
+    yield d
+    d.close()
+
+
+def _gpu(det, ev, nb, bd, **kw):
+    det.load(ev, nb, bd)
+    det.detect(**kw)
+    return det.reports()
+
+
+@pytest.mark.gpu
+def test_gpu_w8_sticky(det):
+    ev, nb, bd, _ = parse(os.path.join(GOLDEN_DIR, "W8_sharing_flag_reading.trace"))
+    assert np.array_equal(_gpu(det, ev, nb, bd, sticky_flags=True), oracle.run(ev, nb, bd, sticky_flags=True))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", [dict(sticky_flags=True), dict(sticky_flags=True, paper_counters=True),
+                                  dict(tag_log2=8), dict(tag_log2=12), dict(tag_log2=22),
+                                  dict(tag_log2=10, sticky_flags=True)],
+                         ids=["sticky", "sticky+paper", "tag8", "tag12", "tag22", "tag10+sticky"])
+def test_gpu_modes_vs_oracle(det, mode):
+    from test_gpu_parity import _fast_random
+
+    w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    for seed, n, words, nb, bd in [(71, 30_000, 40, 3, 96), (72, 150_000, 3_000, 8, 128), (73, 80_000, 5, 2, 64),
+                                   (74, 60_000, 700, 5, 48)]:
+        ev, nb, bd = _fast_random(seed, n, words, nb, bd, w)
+        if "tag_log2" in mode:
+            # spread words over several tags / aliases of each entry
+            rng = np.random.default_rng(seed)
+            acc = ((ev["tk"] >> 24) & 0xF) <= 2
+            bump = rng.choice([0, 1, 3, 1 << 9, 1 << 10, (1 << 10) | 1], size=len(ev)).astype(np.uint64)
+            w_ = ev["addr"] >> np.uint64(2)
+            ev["addr"] = np.where(acc, (w_ + (bump << np.uint64(mode["tag_log2"]))) << np.uint64(2), ev["addr"])
+        want = oracle.run(ev, nb, bd, **mode)
+        got = _gpu(det, ev, nb, bd, **mode)
+        assert len(want) > 0 and np.array_equal(got, want), f"{mode} seed {seed}"
+
+
+@pytest.mark.gpu
+def test_gpu_sticky_lock_heavy_and_goldens(det):
+    from golden_io import all_golden
+    from test_gpu_parity import _fast_random
+
+    for path in all_golden():
+        ev, nb, bd, _ = parse(path)
+        assert np.array_equal(_gpu(det, ev, nb, bd, sticky_flags=True), oracle.run(ev, nb, bd, sticky_flags=True)), path
+    ev, nb, bd = _fast_random(75, 120_000, 300, 4, 64, LOCKY, lock_words=40)
+    assert np.array_equal(_gpu(det, ev, nb, bd, sticky_flags=True), oracle.run(ev, nb, bd, sticky_flags=True))
+
+
+@pytest.mark.gpu
+def test_gpu_tag_mode_rejects_bad_sizes(det):
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    ev, nb, bd, _ = parse(os.path.join(GOLDEN_DIR, "W1_mp_block_fence.trace"))
+    det.load(ev, nb, bd)
+    for b in (7, 23):
+        with pytest.raises(igd.IgdError) as e:
+            det.detect(tag_log2=b)
+        assert e.value.code == igd.igd.IGD_EINVAL
