@@ -173,6 +173,11 @@ int igd_trace_load(igd_ctx* ctx, const igd_trace_desc* desc, const igd_event* ev
      (w >> b) mod 2^10; an access whose Tag differs from the entry's claims it (a first access),
      words with equal entry and Tag share it.  Reports carry the accessed word's address.
      Single-GPU contexts only (IGD_EINVAL otherwise). */
+/* IGD_DETECT_LAST_K(k), k in {2, 4, 8} (reading A37, §6.7): the last k writers (loads)
+     or accessors (stores, atomics) of the word are checked newest first with Table 2, and the
+     first racy one is reported.  k = 1 (or 0) is the default.  Single-GPU contexts only. */
+#define IGD_DETECT_LAST_K_SHIFT 16
+#define IGD_DETECT_LAST_K(k) ((uint32_t)(k) << IGD_DETECT_LAST_K_SHIFT)
 #define IGD_DETECT_STICKY_FLAGS 8u
 #define IGD_DETECT_TAG_SHIFT 8
 #define IGD_DETECT_TAG_LOG2(b) ((uint32_t)(b) << IGD_DETECT_TAG_SHIFT)

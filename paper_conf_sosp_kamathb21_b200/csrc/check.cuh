@@ -31,6 +31,7 @@ __device__ __forceinline__ u32 st_dev(u64 s) { return (u32)(s >> 34) & 1u; }
 __device__ __forceinline__ u32 st_blk(u64 s) { return (u32)(s >> 35) & 1u; }
 __device__ __forceinline__ u32 st_head(u64 s) { return (u32)(s >> 36) & 1u; }
 #define ST_IDENTITY (0xFFFFFFFFull)
+#define ST_HEAD_MARK (ST_IDENTITY | (1ull << 36))  // last-k mode: the access starts its segment
 
 // a then b (b later): segmented "last-of" / OR combine
 __device__ __forceinline__ u64 combine(u64 a, u64 b) {
@@ -133,6 +134,7 @@ struct Params {
     unsigned long long* rep_ctr;
     u64 first_event; // global index offset (multi-rank)
     u32 addr_from_ev;  // tag-aliasing mode (A36): keys hold entry + tag, report addresses come from the trace
+    u64* st_out;       // last-k mode (A37): per-access scan state out, no checks here (NULL otherwise)
 };
 
 // Grid-sync bucket table: gtab[b] = {index, timestamp} of the first grid sync with timestamp >=

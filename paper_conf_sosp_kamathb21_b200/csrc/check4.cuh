@@ -288,6 +288,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         const bool isHead = (hm[j] >> lane) & 1u;
         bool queue = false;
         u32 mdp = 0, fl = 0;
+        if (isHead && P.st_out && x < n) P.st_out[x] = ST_HEAD_MARK;  // a first access (P1)
         if (!isHead) {
             u32 m = hm[j] & le;
             const int sH = m ? j * 32 + hib(m) : cH;
@@ -314,7 +315,9 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 blk = lbv >= 0 || st_blk(carry);
             }
             const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
-            do {
+            if (P.st_out) {  // last-k mode (A37): the scan state goes to k_lastk, which decides
+                if (x < n) P.st_out[x] = st_make(lastW, as, dev ? 1u : 0u, blk ? 1u : 0u, 0u);
+            } else do {
                 CSTAT(0);
                 if (kind == IGD_LD && lastW == IGD_NONE32) {  // P2: never written
                     CSTAT(1);

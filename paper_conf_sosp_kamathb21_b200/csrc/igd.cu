@@ -19,6 +19,7 @@
 #include "common.cuh"
 #include "fused.cuh"
 #include "ingest.cuh"
+#include "lastk.cuh"
 #include "sort.cuh"
 #include "shard.cuh"
 #include "sync.cuh"
@@ -136,6 +137,8 @@ struct igd_ctx {
     bool paper_counters = false;  // IGD_DETECT_PAPER_COUNTERS (reading A33)
     bool sticky = false;          // IGD_DETECT_STICKY_FLAGS (reading A35)
     u32 tag_log2 = 0;             // IGD_DETECT_TAG_LOG2 (reading A36): 0 = exact per-word state
+    u32 last_k = 1;               // IGD_DETECT_LAST_K (reading A37): history depth
+    Buf lk_state;
     int fused = 1;      // single GPU: ingest write pass fused with radix pass 0 (IGD_FUSED=0: unfused)
     // sharded mode: stage-1 outputs, stage-2 inputs
     bool shard = false;
@@ -817,6 +820,11 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             cp.rep_ctr = P_<unsigned long long>(ctx->rep_ctr);
             cp.first_event = first;
             cp.addr_from_ev = TG ? 1u : 0u;
+            const u32 LK = SH ? 1u : ctx->last_k;
+            if (LK > 1) {  // A37: the scan state per access, then the candidates per access
+                RET(ensure(ctx, ctx->lk_state, n_acc * sizeof(u64)));
+                cp.st_out = P_<u64>(ctx->lk_state);
+            }
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
@@ -824,6 +832,28 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
                              (unsigned)tiles, ctx->stream, cp);
             }
             CK(cudaGetLastError());
+            if (LK > 1) {
+                lastk::Params lp2;
+                lp2.C = cp;
+                lp2.C.st_out = nullptr;
+                lp2.st = P_<u64>(ctx->lk_state);
+                lp2.k = LK;
+                const unsigned lb = (unsigned)((n_acc + 255) / 256);
+                KTimer kt(ctx, KC_CHECK, 20.0 * (double)n_acc);
+                const bool W = ctx->paper_counters, T = ctx->sticky;
+                if (key64) {
+                    if (W && T) lastk::k_lastk<true, true, u64><<<lb, 256, 0, ctx->stream>>>(lp2);
+                    else if (W) lastk::k_lastk<true, false, u64><<<lb, 256, 0, ctx->stream>>>(lp2);
+                    else if (T) lastk::k_lastk<false, true, u64><<<lb, 256, 0, ctx->stream>>>(lp2);
+                    else lastk::k_lastk<false, false, u64><<<lb, 256, 0, ctx->stream>>>(lp2);
+                } else {
+                    if (W && T) lastk::k_lastk<true, true, u32><<<lb, 256, 0, ctx->stream>>>(lp2);
+                    else if (W) lastk::k_lastk<true, false, u32><<<lb, 256, 0, ctx->stream>>>(lp2);
+                    else if (T) lastk::k_lastk<false, true, u32><<<lb, 256, 0, ctx->stream>>>(lp2);
+                    else lastk::k_lastk<false, false, u32><<<lb, 256, 0, ctx->stream>>>(lp2);
+                }
+                CK(cudaGetLastError());
+            }
             CK(cudaMemcpyAsync(ctx->h_small, ctx->rep_ctr.p, sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
             CK(cudaStreamSynchronize(ctx->stream));
             n_rep = ctx->h_small[0];
@@ -1253,13 +1283,19 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
         ctx->err = "IGD_DETECT_TAG_LOG2 must be 8..22";
         return IGD_EINVAL;
     }
+    u32 last_k = (flags >> IGD_DETECT_LAST_K_SHIFT) & 15u;
+    if (last_k == 0) last_k = 1;
+    if (last_k != 1 && last_k != 2 && last_k != 4 && last_k != 8) {
+        ctx->err = "IGD_DETECT_LAST_K must be 1, 2, 4 or 8";
+        return IGD_EINVAL;
+    }
     if (ctx->comm) {  // collective over the communicator's ranks
         if (flags & IGD_DETECT_COALESCE) {  // reading A32: a group may straddle two ranks' chunks
             ctx->err = "IGD_DETECT_COALESCE is a single-context mode";
             return IGD_EINVAL;
         }
-        if (tag_log2) {  // A36: the owner hash would have to be over metadata entries
-            ctx->err = "the tag-aliasing mode is a single-context mode";
+        if (tag_log2 || last_k > 1) {  // A36: the owner hash would have to be over metadata entries
+            ctx->err = "the tag-aliasing and last-k modes are single-context modes";
             return IGD_EINVAL;
         }
         cudaSetDevice(ctx->device);
@@ -1283,6 +1319,7 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
     ctx->sticky = (flags & IGD_DETECT_STICKY_FLAGS) != 0;
     ctx->tag_log2 = tag_log2;
+    ctx->last_k = last_k;
     ctx->shard = false;
     ctx->in_segment = false;
     int rc = detect_impl(ctx, n_reports_global);
@@ -1291,6 +1328,7 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     ctx->paper_counters = false;
     ctx->sticky = false;
     ctx->tag_log2 = 0;
+    ctx->last_k = 1;
     if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
     return rc;
 }
@@ -1333,8 +1371,8 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
     ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
     ctx->sticky = (flags & IGD_DETECT_STICKY_FLAGS) != 0;
-    if ((flags >> IGD_DETECT_TAG_SHIFT) & 31u) {
-        ctx->err = "the tag-aliasing mode is a single-context mode";
+    if (((flags >> IGD_DETECT_TAG_SHIFT) & 31u) || ((flags >> IGD_DETECT_LAST_K_SHIFT) & 15u) > 1) {
+        ctx->err = "the tag-aliasing and last-k modes are single-context modes";
         return IGD_EINVAL;
     }
     ctx->shard = true;
@@ -1447,7 +1485,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf,
                   &ctx->cl_small,     &ctx->cl_mat,   &ctx->cl_recv,  &ctx->cl_sidx,  &ctx->cl_sev,
-                  &ctx->cl_nrep,      &ctx->cl_rep,   &ctx->gkb,      &ctx->seg_rep};
+                  &ctx->cl_nrep,      &ctx->cl_rep,   &ctx->gkb,      &ctx->seg_rep,  &ctx->lk_state};
     for (Buf* b : all) buf_free(ctx, *b);
     cudaStreamSynchronize(ctx->stream);
     cudaFreeHost(ctx->h_stats);

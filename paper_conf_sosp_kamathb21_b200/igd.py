@@ -23,6 +23,7 @@ IGD_DETECT_COALESCE = 2
 IGD_DETECT_PAPER_COUNTERS = 4
 IGD_DETECT_STICKY_FLAGS = 8
 IGD_DETECT_TAG_SHIFT = 8
+IGD_DETECT_LAST_K_SHIFT = 16
 IGD_N_STAGES = 8
 IGD_N_KCLASS = 9
 
@@ -238,14 +239,16 @@ class Detector:
                            first_event, n_events_total)
 
     def detect(self, timing: bool = False, coalesce: bool = False, paper_counters: bool = False,
-               sticky_flags: bool = False, tag_log2: int = 0) -> int:
+               sticky_flags: bool = False, tag_log2: int = 0, last_k: int = 1) -> int:
         """igd_detect; ``coalesce``: warp-coalesced check mode (IGD_DETECT_COALESCE, reading A32);
         ``paper_counters``: Fig. 4-width synchronization IDs (IGD_DETECT_PAPER_COUNTERS, A33);
         ``sticky_flags``: Table 2's sticky sharing flags in P3-P5 (IGD_DETECT_STICKY_FLAGS, A35);
-        ``tag_log2``: a 2^tag_log2-entry metadata table with 10-bit Tags (IGD_DETECT_TAG_LOG2, A36)."""
+        ``tag_log2``: a 2^tag_log2-entry metadata table with 10-bit Tags (IGD_DETECT_TAG_LOG2, A36);
+        ``last_k``: the last k writers / accessors are checked (IGD_DETECT_LAST_K, A37)."""
         flags = ((IGD_DETECT_TIMING if timing else 0) | (IGD_DETECT_COALESCE if coalesce else 0)
                  | (IGD_DETECT_PAPER_COUNTERS if paper_counters else 0)
-                 | (IGD_DETECT_STICKY_FLAGS if sticky_flags else 0) | (int(tag_log2) << IGD_DETECT_TAG_SHIFT))
+                 | (IGD_DETECT_STICKY_FLAGS if sticky_flags else 0) | (int(tag_log2) << IGD_DETECT_TAG_SHIFT)
+                 | ((int(last_k) if last_k > 1 else 0) << IGD_DETECT_LAST_K_SHIFT))
         self.n_reports = igd_detect(self.ctx, flags)
         return self.n_reports
 

@@ -194,8 +194,11 @@ def test_gpu_w8_sticky(det):
 @pytest.mark.gpu
 @pytest.mark.parametrize("mode", [dict(sticky_flags=True), dict(sticky_flags=True, paper_counters=True),
                                   dict(tag_log2=8), dict(tag_log2=12), dict(tag_log2=22),
-                                  dict(tag_log2=10, sticky_flags=True)],
-                         ids=["sticky", "sticky+paper", "tag8", "tag12", "tag22", "tag10+sticky"])
+                                  dict(tag_log2=10, sticky_flags=True), dict(last_k=2), dict(last_k=4),
+                                  dict(last_k=8), dict(last_k=4, sticky_flags=True),
+                                  dict(last_k=2, paper_counters=True), dict(last_k=4, tag_log2=12)],
+                         ids=["sticky", "sticky+paper", "tag8", "tag12", "tag22", "tag10+sticky", "last2", "last4",
+                              "last8", "last4+sticky", "last2+paper", "last4+tag12"])
 def test_gpu_modes_vs_oracle(det, mode):
     from test_gpu_parity import _fast_random
 
@@ -237,3 +240,23 @@ def test_gpu_tag_mode_rejects_bad_sizes(det):
         with pytest.raises(igd.IgdError) as e:
             det.detect(tag_log2=b)
         assert e.value.code == igd.igd.IGD_EINVAL
+
+
+@pytest.mark.gpu
+def test_gpu_last_k_worked_example_and_kernels(det):
+    b = tg.TraceBuilder(2, 64)
+    b.st(0, 3)
+    b.st(1, 3, mask=0x3)
+    b.fence(1)
+    b.ld(64, 3)
+    ev = b.events()
+    assert np.array_equal(_gpu(det, ev, 2, 64, last_k=2), oracle.run(ev, 2, 64, last_k=2))
+    assert len(_gpu(det, ev, 2, 64, last_k=2)) == 1
+    # kernel boundaries end the histories (A31)
+    from test_gpu_parity import _fast_random
+
+    w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1, 1]
+    ev, nb, bd = _fast_random(76, 90_000, 60, 3, 64, w[:12])
+    joined = tg.concat_kernels([ev[:40_000], ev[40_000:]])
+    for k in (2, 8):
+        assert np.array_equal(_gpu(det, joined, nb, bd, last_k=k), oracle.run(joined, nb, bd, last_k=k))
