@@ -150,6 +150,9 @@ struct igd_ctx {
     const void* sh_sev = nullptr;
     u64 sh_ns = 0, sh_wbase = 0, sh_ntotal = 0;
     int last_acur = 0;  // buffer holding the sorted accesses of the last igd_detect (debug hooks)
+    int last_scur = 0;  // ... the sorted sync records
+    u64 last_nsync = 0, last_npts = 0;  // sync records, lock change points
+    u32 last_E = 0, last_T = 0;         // entities, threads
     u64 last_nacc = 0;
     u64 n_reports = 0;
     u64 bad_event = 0;
@@ -698,6 +701,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
 
     // ---------------- a2: sync records sorted by entity, CSR offsets ----------------
     int scur = 0;
+    ctx->last_nsync = 0;
+    ctx->last_npts = 0;
     RET(radix_sort(ctx, KC_SORT_SYNC, ctx->syn_k, ctx->syn_v, n_sync, P_<u32>(ctx->hist) + 1024, h_hist_sync,
                    bits_needed(ks.E), &scur));
     mark(ctx, 2);
@@ -770,6 +775,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lv.toff = P_<u32>(ctx->tcnt);
         lv.tpts = P_<u64>(ctx->tpts);
         lv.any = 1;
+        ctx->last_npts = tot;
     }
     mark(ctx, 3);
     // ---------------- a5: accesses sorted by word, stable ----------------
@@ -781,6 +787,10 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc,
                        TG ? TG : 32u, &acur, vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0, SH ? ctx->sh_rec : nullptr));
     ctx->last_acur = acur;
+    ctx->last_scur = scur;
+    ctx->last_nsync = n_sync;
+    ctx->last_E = ks.E;
+    ctx->last_T = g.T;
     ctx->last_nacc = SH ? 0 : n_acc;
     mark(ctx, 4);
     // ---------------- a6: segmented shadow pass + check ----------------
@@ -1520,6 +1530,33 @@ int igd_debug_check_stats(igd_ctx* ctx, int enable, uint64_t* out16) {
     const unsigned long long zero[16] = {0};
     CK(cudaMemcpyToSymbol(check::g_chk_stats, zero, sizeof(zero)));
     CK(cudaMemcpyToSymbol(check::g_chk_stats_on, &enable, sizeof(int)));
+    return IGD_OK;
+}
+
+int igd_debug_sync_tables(igd_ctx* ctx, uint64_t* sizes, uint32_t* off, uint32_t* ts, uint32_t* toff,
+                          uint64_t* tpts) {
+    if (!ctx || !sizes) return IGD_EINVAL;
+    if (!ctx->loaded) return IGD_ESTATE;
+    sizes[0] = ctx->last_E;
+    sizes[1] = ctx->last_nsync;
+    sizes[2] = ctx->last_T;
+    sizes[3] = ctx->last_npts;
+    cudaSetDevice(ctx->device);
+    if (off && ctx->last_E) CK(cudaMemcpy(off, ctx->off.p, ((u64)ctx->last_E + 1) * sizeof(u32), cudaMemcpyDeviceToHost));
+    if (ts && ctx->last_nsync)
+        CK(cudaMemcpy(ts, ctx->syn_v[ctx->last_scur].p, ctx->last_nsync * sizeof(u32), cudaMemcpyDeviceToHost));
+    if (toff && ctx->last_npts)
+        CK(cudaMemcpy(toff, ctx->tcnt.p, ((u64)ctx->last_T + 1) * sizeof(u32), cudaMemcpyDeviceToHost));
+    if (tpts && ctx->last_npts) CK(cudaMemcpy(tpts, ctx->tpts.p, ctx->last_npts * sizeof(u64), cudaMemcpyDeviceToHost));
+    return IGD_OK;
+}
+
+int igd_debug_scan_state(igd_ctx* ctx, uint64_t n, uint64_t* state, uint32_t* keys, uint64_t* payload) {
+    if (!ctx || n != ctx->last_nacc) return IGD_EINVAL;
+    cudaSetDevice(ctx->device);
+    if (state && n) CK(cudaMemcpy(state, ctx->lk_state.p, n * sizeof(u64), cudaMemcpyDeviceToHost));
+    if (keys && n) CK(cudaMemcpy(keys, ctx->acc_k[ctx->last_acur].p, n * sizeof(u32), cudaMemcpyDeviceToHost));
+    if (payload && n) CK(cudaMemcpy(payload, ctx->acc_v[ctx->last_acur].p, n * sizeof(u64), cudaMemcpyDeviceToHost));
     return IGD_OK;
 }
 

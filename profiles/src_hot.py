@@ -9,7 +9,7 @@ import sys
 rep, kre = sys.argv[1], sys.argv[2]
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 40
 raw = subprocess.check_output(["ncu", "-i", rep, "--page", "source", "--csv", "--kernel-name", f"regex:{kre}",
-                               "--launch-count", "1", "--print-source", "cuda,sass"], text=True,
+                               "--launch-skip", str(int(sys.argv[4]) if len(sys.argv) > 4 else 0), "--launch-count", "1", "--print-source", "cuda,sass"], text=True,
                               stderr=subprocess.DEVNULL)
 rows = list(csv.reader(io.StringIO(raw)))
 out = []
