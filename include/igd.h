@@ -228,6 +228,27 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
                      const void* d_sync_events, uint64_t n_sync_stream, uint64_t min_word, uint32_t flags,
                      uint64_t* n_reports);
 
+/* ---- streaming sessions (the paper's online setting) ----
+   A trace arrives in consecutive chunks (e.g. drained from an instrumentation buffer) and each
+   chunk is checked on arrival: its reports (global trace indices, ascending cur, read with
+   igd_reports) are final, and their union over the session equals igd_detect of the whole trace.
+   The context carries the synchronization stream so far and, per accessed word, its last writer,
+   last accessor, sticky sharing flags and scope of its last atomic.  Single-GPU contexts; the
+   session's words must span < 2^32 words (IGD_ETOOBIG); grid-changing kernel boundaries are
+   rejected (IGD_EINVAL).
+   igd_stream_begin: start (or restart) a session for kernels of grid (n_blocks, block_dim).
+   igd_stream_feed: check the next n_events events (event_flags: IGD_TRACE_DEVICE_PTR for a
+     device pointer, borrowed for the call, else host memory, copied); detect_flags:
+     IGD_DETECT_TIMING | IGD_DETECT_PAPER_COUNTERS | IGD_DETECT_STICKY_FLAGS.  *n_reports = this
+     chunk's reports.  IGD_ETRACE (igd_bad_event = global index) and other errors end the session.
+     IGD_ESTATE without an active session.  igd_detect / igd_shard_detect return IGD_ESTATE
+     while a session is active.
+   igd_stream_end: end the session and release its carried state. */
+int igd_stream_begin(igd_ctx* ctx, uint32_t n_blocks, uint32_t block_dim);
+int igd_stream_feed(igd_ctx* ctx, const igd_event* events, uint64_t n_events, uint32_t event_flags,
+                    uint32_t detect_flags, uint64_t* n_reports);
+int igd_stream_end(igd_ctx* ctx);
+
 /* Copy min(cap, total) reports, ascending by `cur` (at most one report per access, so the
    order is total), to host memory `host_out`; *n_written = number copied. */
 int igd_reports(igd_ctx* ctx, igd_report* host_out, uint64_t cap, uint64_t* n_written);

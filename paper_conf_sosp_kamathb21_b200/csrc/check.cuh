@@ -135,7 +135,24 @@ struct Params {
     u64 first_event; // global index offset (multi-rank)
     u32 addr_from_ev;  // tag-aliasing mode (A36): keys hold entry + tag, report addresses come from the trace
     u64* st_out;       // last-k mode (A37): per-access scan state out, no checks here (NULL otherwise)
+    u32 carry_before;  // streaming mode (f4): records with index < carry_before are carried state
+    void* carry_out;   // streaming mode: 2 uint4 per access (carried pair at each word's last access)
 };
+
+// Streaming mode: keep the carried pairs written at each word's last access (compaction by
+// flag, exclusive scan, scatter; the survivors stay in key order)
+__global__ void k_carry_flags(const uint4* __restrict__ co, u32 n, u32* __restrict__ flags) {
+    for (u32 x = blockIdx.x * blockDim.x + threadIdx.x; x <= n; x += gridDim.x * blockDim.x)
+        flags[x] = x < n && co[2 * (u64)x + 1].y != IGD_NONE32 ? 1u : 0u;
+}
+__global__ void k_carry_scatter(const uint4* __restrict__ co, const u32* __restrict__ pos, u32 n,
+                                uint4* __restrict__ out) {
+    for (u32 x = blockIdx.x * blockDim.x + threadIdx.x; x < n; x += gridDim.x * blockDim.x)
+        if (pos[x + 1] != pos[x]) {
+            out[2 * (u64)pos[x]] = co[2 * (u64)x];
+            out[2 * (u64)pos[x] + 1] = co[2 * (u64)x + 1];
+        }
+}
 
 // Grid-sync bucket table: gtab[b] = {index, timestamp} of the first grid sync with timestamp >=
 // b << shift (timestamp NONE past the last).  The grid list is global and short, so "a grid sync

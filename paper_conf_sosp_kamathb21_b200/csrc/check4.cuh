@@ -89,11 +89,17 @@ __device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, co
 // registers, 8% of the kernel, ncu r01s3, when compiled into the common case)
 // KT: u32 word keys (low 32 bits; spans < 2^32 words) or u64 keys (word - wbase, a4's wide path)
 // FID: paper-fidelity bits -- 1 = Fig. 4-width synchronization IDs (reading A33), 2 = sticky
-// sharing flags gate P3-P5 as Table 2 is written (reading A35)
+// sharing flags gate P3-P5 as Table 2 is written (reading A35), 4 = last-k state out (A37)
 template <bool MV, bool KB, int FID, bool GEO2, typename KT = u32>
 __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
     constexpr bool WRAP = (FID & 1) != 0;
     constexpr bool STK = (FID & 2) != 0;
+    constexpr bool LKO = (FID & 4) != 0;  // last-k mode (A37): scan state out, decisions in k_lastk
+    // streaming mode (sharded payload only): records with an index below
+    // P.carry_before are carried state of earlier chunks -- per word a head record and the last
+    // accessor, whose mask field holds the word's sticky flags and the scope of its last atomic --
+    // and are never checked; the state after each word's last access goes to P.carry_out
+    constexpr bool CARRY = MV && (FID & 8) != 0;
     __shared__ u32 s_v[C4_TILE], s_z[C4_TILE];    // staged payload: trace index, tk
     __shared__ u32 q_x[C4_TILE], q_md[C4_TILE];   // per-warp queues: sorted position, md position
     __shared__ uint8_t q_f[C4_TILE];              // queue flags
@@ -161,6 +167,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
 
     // ---- predicates and ballots ----
     u32 hm[C4_ITEMS], wm[C4_ITEMS], am[C4_ITEMS], bsm[C4_ITEMS], dm[C4_ITEMS], bm[C4_ITEMS], tm[C4_ITEMS];
+    u32 pm[C4_ITEMS], kc[C4_ITEMS];  // CARRY: carried records, key changes
 #pragma unroll
     for (int j = 0; j < C4_ITEMS; j++) {
         const u32 x = wbase + j * 32 + lane;
@@ -191,11 +198,24 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             blk = !dev && (GEO2 ? (pt >> 5) != (c >> 5) : ((pt - bp * g.D) >> 5) != ((c - bc * g.D) >> 5));
             same_t = pt == c;
         }
-        const bool isA = in && kind >= IGD_ATOM && kind <= IGD_EXCH;
+        bool isA = in && kind >= IGD_ATOM && kind <= IGD_EXCH;
+        u32 ascp = norm_scope((Z[j] >> 28) & 3u);
+        if (CARRY) {
+            const bool pseudo = in && V[j] < P.carry_before;
+            pm[j] = __ballot_sync(IGD_FULL, pseudo);
+            kc[j] = __ballot_sync(IGD_FULL, in && (!pvalid || pK != K[j]));
+            if (pseudo && !head) {  // the carried last accessor: the word's state before the chunk
+                dev = M[j] & 1u;
+                blk = (M[j] >> 1) & 1u;
+                same_t = false;
+                ascp = (M[j] >> 2) & 3u;
+                isA = ascp != 0;
+            }
+        }
         hm[j] = __ballot_sync(IGD_FULL, head);
         wm[j] = __ballot_sync(IGD_FULL, in && kind != IGD_LD);
         am[j] = __ballot_sync(IGD_FULL, isA);
-        bsm[j] = __ballot_sync(IGD_FULL, isA && norm_scope((Z[j] >> 28) & 3u) == IGD_SCOPE_BLOCK);
+        bsm[j] = __ballot_sync(IGD_FULL, isA && ascp == IGD_SCOPE_BLOCK);
         dm[j] = __ballot_sync(IGD_FULL, dev);
         bm[j] = __ballot_sync(IGD_FULL, blk);
         tm[j] = __ballot_sync(IGD_FULL, same_t);
@@ -288,7 +308,9 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         const bool isHead = (hm[j] >> lane) & 1u;
         bool queue = false;
         u32 mdp = 0, fl = 0;
-        if (isHead && P.st_out && x < n) P.st_out[x] = ST_HEAD_MARK;  // a first access (P1)
+        if (LKO && isHead && x < n) P.st_out[x] = ST_HEAD_MARK;  // a first access (P1)
+        u32 cw_lastW = IGD_NONE32, cw_as = 0;  // CARRY: the state before x (heads: none)
+        bool cw_dev = false, cw_blk = false;
         if (!isHead) {
             u32 m = hm[j] & le;
             const int sH = m ? j * 32 + hib(m) : cH;
@@ -315,7 +337,15 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 blk = lbv >= 0 || st_blk(carry);
             }
             const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
-            if (P.st_out) {  // last-k mode (A37): the scan state goes to k_lastk, which decides
+            if (CARRY) {
+                cw_lastW = lastW;
+                cw_as = as;
+                cw_dev = dev;
+                cw_blk = blk;
+            }
+            if (CARRY && ((pm[j] >> lane) & 1u)) {
+                // a carried record: history only, decided in an earlier chunk
+            } else if (LKO) {  // last-k mode (A37): the scan state goes to k_lastk, which decides
                 if (x < n) P.st_out[x] = st_make(lastW, as, dev ? 1u : 0u, blk ? 1u : 0u, 0u);
             } else do {
                 CSTAT(0);
@@ -373,6 +403,32 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 queue = true;
                 CSTAT(6);
             } while (0);
+        }
+        if (CARRY && P.carry_out && x < n) {
+            // streaming mode: after a word's last access of this run, its state goes out as the next
+            // chunk's carried pair {head record, last accessor + flags}
+            bool last;
+            if (x + 1 >= n) last = true;
+            else if (lane < 31) last = (kc[j] >> (lane + 1)) & 1u;
+            else if (j + 1 < C4_ITEMS) last = kc[(j + 1) % C4_ITEMS] & 1u;
+            else last = __ldg(keys + x + 1) != K[j];
+            uint4* co = reinterpret_cast<uint4*>(P.carry_out) + 2 * (u64)x;
+            if (last) {
+                const u32 kd = (Z[j] >> 24) & 0xFu;
+                const u32 sX = ((bsm[j] >> lane) & 1u) ? IGD_SCOPE_BLOCK : IGD_SCOPE_DEVICE;
+                const u32 lw = kd != IGD_LD ? x : cw_lastW;
+                const u32 asA = ((am[j] >> lane) & 1u) ? sX : cw_as;
+                const u32 k32 = (u32)K[j];
+                if (lw != IGD_NONE32 && lw != x) {
+                    const u32 li = (lw - tbase < (u32)C4_TILE) ? s_v[lw - tbase] : acc_at<MV>(P.val, lw).idx;
+                    co[0] = make_uint4(k32, li, tk_at(lw), 0u);
+                } else {  // no earlier writer to keep: a neutral head (a load, never a writer)
+                    co[0] = make_uint4(k32, V[j], (Z[j] & 0xFFFFFFu) | ((u32)IGD_LD << 24), 0u);
+                }
+                co[1] = make_uint4(k32, V[j], Z[j], (cw_dev ? 1u : 0u) | (cw_blk ? 2u : 0u) | (asA << 2));
+            } else {
+                co[1] = make_uint4(0u, IGD_NONE32, 0u, 0u);
+            }
         }
         const u32 qmask = __ballot_sync(IGD_FULL, queue);
         if (queue) {

@@ -28,6 +28,10 @@
 #include <algorithm>
 #include <vector>
 
+#ifndef IGD_PASS0_GENERIC
+#define IGD_PASS0_GENERIC 0  // 1: the fused pipeline's pass 0 through the generic k_ingest<0> (A/B)
+#endif
+
 namespace {
 
 enum KClass { KC_INGEST = 0, KC_SORT_SYNC, KC_CSR, KC_LOCK, KC_SORT_ACC, KC_CHECK, KC_REPORT, KC_MISC, KC_FUSED };
@@ -117,6 +121,13 @@ struct igd_ctx {
     u64 seg_n = 0, seg_first = 0;
     u32 seg_nb = 0, seg_bd = 0;
     Buf gkb, seg_rep;
+    // streaming sessions: chunks of one trace checked in order, the shadow state
+    // carried between them as two records per word, the synchronization stream accumulated
+    bool str_active = false;
+    u64 str_n = 0, str_wmin = ~0ull, str_wmax = 0, str_nsync = 0, str_ncarry = 0;
+    u32 str_nb = 0, str_bd = 0;
+    Buf str_sidx, str_sev, str_carry[2], str_rec, str_co, str_flags;
+    int str_cur = 0;
     igd_alloc_fn afn = nullptr;
     igd_free_fn ffn = nullptr;
     void* auser = nullptr;
@@ -359,6 +370,17 @@ template <bool MV, bool KB>
 static void launch_check_w(int fid, unsigned tb, cudaStream_t st, const check::Params& cp) {
     // power-of-two geometry (block_dim >= 32): shift / mask instead of divisions (common case)
     const bool geo2 = cp.g.dlog < 32 && cp.g.D >= 32;
+    if constexpr (MV) {
+        if (fid & 8) {  // streaming mode (f4): carried records, state out
+            switch (fid & 3) {
+                case 0: check::k_check4<MV, KB, 8, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+                case 1: check::k_check4<MV, KB, 9, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+                case 2: check::k_check4<MV, KB, 10, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+                default: check::k_check4<MV, KB, 11, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+            }
+            return;
+        }
+    }
     switch (fid) {
         case 0:
             if (geo2) check::k_check4<MV, KB, 0, true><<<tb, check::C4_THREADS, 0, st>>>(cp);
@@ -366,7 +388,15 @@ static void launch_check_w(int fid, unsigned tb, cudaStream_t st, const check::P
             break;
         case 1: check::k_check4<MV, KB, 1, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
         case 2: check::k_check4<MV, KB, 2, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
-        default: check::k_check4<MV, KB, 3, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 3: check::k_check4<MV, KB, 3, false><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        default:  // last-k state out (single context only)
+            if constexpr (!MV) {
+                if (fid == 4) check::k_check4<MV, KB, 4, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+                else if (fid == 5) check::k_check4<MV, KB, 5, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+                else if (fid == 6) check::k_check4<MV, KB, 6, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+                else check::k_check4<MV, KB, 7, false><<<tb, check::C4_THREADS, 0, st>>>(cp);
+            }
+            break;
     }
 }
 template <bool KB>
@@ -375,7 +405,11 @@ static void launch_check_64(int fid, unsigned tb, cudaStream_t st, const check::
         case 0: check::k_check4<false, KB, 0, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
         case 1: check::k_check4<false, KB, 1, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
         case 2: check::k_check4<false, KB, 2, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
-        default: check::k_check4<false, KB, 3, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 3: check::k_check4<false, KB, 3, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 4: check::k_check4<false, KB, 4, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 5: check::k_check4<false, KB, 5, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        case 6: check::k_check4<false, KB, 6, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
+        default: check::k_check4<false, KB, 7, false, u64><<<tb, check::C4_THREADS, 0, st>>>(cp); break;
     }
 }
 static void launch_check(bool mv, bool kb, int fid, bool key64, unsigned tb, cudaStream_t st,
@@ -540,7 +574,16 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     const u64 grid = std::max<u64>(1, std::min<u64>((u64)sms * (occ > 0 ? occ : 1), in_tiles));
     if (n_src > 0) {
         KTimer kt(ctx, KC_INGEST, 16.0 * (double)n_src);  // pass 0 reads every event
-        ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+        if (FUSED && !IGD_PASS0_GENERIC) {
+            // the timed path: branch-free rules, compile-time geometry / coalescing variants
+            const bool geo2 = g.dlog < 32 && g.D >= 32;
+            if (geo2 && !ip.skip_bits) ingest::k_count_fused<true, false><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+            else if (geo2) ingest::k_count_fused<true, true><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+            else if (!ip.skip_bits) ingest::k_count_fused<false, false><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+            else ingest::k_count_fused<false, true><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+        } else {
+            ingest::k_ingest<0><<<(unsigned)grid, ingest::THREADS, 0, ctx->stream>>>(ip);
+        }
     }
     CK(cudaGetLastError());
     RET(scan_excl(ctx, P_<u32>(ctx->st_in_a), in_tiles + 1));
@@ -838,8 +881,14 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             {
                 // key + payload streamed (12 or 20 bytes per access)
                 KTimer kt(ctx, KC_CHECK, (4.0 + vbytes) * (double)n_acc);
-                launch_check(SH, cp.has_kb != 0, (ctx->paper_counters ? 1 : 0) | (ctx->sticky ? 2 : 0), key64,
-                             (unsigned)tiles, ctx->stream, cp);
+                if (SH && ctx->str_active) {  // streaming mode (f4)
+                    cp.carry_before = (u32)ctx->str_n;
+                    cp.carry_out = ctx->str_co.p;
+                }
+                launch_check(SH, cp.has_kb != 0,
+                             (ctx->paper_counters ? 1 : 0) | (ctx->sticky ? 2 : 0) | (LK > 1 ? 4 : 0) |
+                                 (SH && ctx->str_active ? 8 : 0),
+                             key64, (unsigned)tiles, ctx->stream, cp);
             }
             CK(cudaGetLastError());
             if (LK > 1) {
@@ -1040,6 +1089,122 @@ static int segmented_detect(igd_ctx* ctx, u64* n_out) {
     CK(cudaStreamSynchronize(ctx->stream));
     ctx->n_reports = total;
     *n_out = total;
+    return IGD_OK;
+}
+
+// ---------------- streaming sessions ----------------
+// A producer (e.g. an instrumentation runtime draining per-warp buffers)
+// hands over a trace in consecutive chunks.  Each chunk is checked as soon as it arrives and its
+// reports are final: the union over the chunks is exactly the whole-trace result.  Carried
+// between chunks: the synchronization stream so far (epoch tables and lock replay are rebuilt
+// over it, so interval queries reaching into earlier chunks stay exact), and per accessed word
+// two records {a head record (its last writer when that is not its last accessor, else a
+// neutral load), its last accessor with the word's sticky DevShared / BlkShared and the scope of
+// its last atomic}.  The chunk's access records follow the carried ones into the sharded-mode
+// pipeline (stable sort by word keeps carried state before new accesses), the check skips the
+// carried records and writes the next carried pairs.
+static int grow_keep(igd_ctx* ctx, Buf& b, size_t used, size_t want) {
+    if (b.cap >= want) return IGD_OK;
+    Buf nb;
+    RET(ensure(ctx, nb, want + want / 2));
+    if (used) CK(cudaMemcpyAsync(nb.p, b.p, used, cudaMemcpyDeviceToDevice, ctx->stream));
+    RET(buf_free(ctx, b));
+    b = nb;
+    return IGD_OK;
+}
+
+static int stream_feed_impl(igd_ctx* ctx, const igd_event* events, u64 n, u32 ev_flags, u64* n_out) {
+    *n_out = 0;
+    ctx->n_reports = 0;
+    ctx->launches = 0;
+    ctx->nk = 0;
+    igd_trace_desc d{};
+    d.n_blocks = ctx->str_nb;
+    d.block_dim = ctx->str_bd;
+    d.first_event = ctx->str_n;
+    d.n_events = n;
+    d.n_events_total = ctx->str_n + n;
+    d.flags = ev_flags;
+    if (d.n_events_total > 0xFFFFFFFFull - 2 * rsort::TILE) return IGD_ETOOBIG;
+    RET(igd_trace_load(ctx, &d, events));
+    u64 counts[2] = {0, 0}, nsync = 0, bad = ~0ull, mm[2] = {~0ull, 0};
+    RET(shard_prepare_impl(ctx, 1, counts, &nsync, &bad, mm));
+    if (bad != ~0ull) {
+        ctx->bad_event = bad;
+        ctx->err = "invalid event at index " + std::to_string(bad);
+        return IGD_ETRACE;
+    }
+    const u64 nrec = counts[0];
+    const u64 wmin = std::min(ctx->str_wmin, mm[0]), wmax = nrec ? std::max(ctx->str_wmax, mm[1]) : ctx->str_wmax;
+    if (wmin != ~0ull && wmax - wmin >= (1ull << 32)) {
+        ctx->err = "a streaming session's words must span < 2^32 words";
+        return IGD_ETOOBIG;
+    }
+    // the synchronization stream so far
+    RET(grow_keep(ctx, ctx->str_sidx, ctx->str_nsync * sizeof(u32), (ctx->str_nsync + nsync + 1) * sizeof(u32)));
+    RET(grow_keep(ctx, ctx->str_sev, ctx->str_nsync * 16, (ctx->str_nsync + nsync + 1) * 16));
+    if (nsync) {
+        CK(cudaMemcpyAsync(P_<u32>(ctx->str_sidx) + ctx->str_nsync, ctx->sh_sidx_buf.p, nsync * sizeof(u32),
+                           cudaMemcpyDeviceToDevice, ctx->stream));
+        CK(cudaMemcpyAsync((char*)ctx->str_sev.p + ctx->str_nsync * 16, ctx->sh_sev_buf.p, nsync * 16,
+                           cudaMemcpyDeviceToDevice, ctx->stream));
+    }
+    const u64 nsy = ctx->str_nsync + nsync;
+    // carried records, then the chunk's records (trace order)
+    const u64 nc = ctx->str_ncarry, nall = nc + nrec;
+    if (nall > 0xFFFFFFFFull - 2 * rsort::TILE || nsy + 64 > 0xFFFFFFFFull) return IGD_ETOOBIG;
+    RET(ensure(ctx, ctx->str_rec, (nall + 1) * 16));
+    if (nc) CK(cudaMemcpyAsync(ctx->str_rec.p, ctx->str_carry[ctx->str_cur].p, nc * 16, cudaMemcpyDeviceToDevice,
+                               ctx->stream));
+    if (nrec) CK(cudaMemcpyAsync((char*)ctx->str_rec.p + nc * 16, ctx->sh_send.p, nrec * 16, cudaMemcpyDeviceToDevice,
+                                 ctx->stream));
+    RET(buf_free(ctx, ctx->sh_send));
+    RET(ensure(ctx, ctx->str_co, (2 * nall + 2) * 16));
+    ctx->shard = true;
+    ctx->sh_rec = ctx->str_rec.p;
+    ctx->sh_nrec = nall;
+    ctx->sh_sidx = P_<u32>(ctx->str_sidx);
+    ctx->sh_sev = ctx->str_sev.p;
+    ctx->sh_ns = nsy;
+    ctx->sh_wbase = wmin == ~0ull ? 0 : wmin;
+    ctx->sh_ntotal = d.n_events_total;
+    u64 nrep = 0;
+    int rc = detect_impl(ctx, &nrep);
+    ctx->shard = false;
+    if (rc != IGD_OK) return rc;
+    // the next carried pairs (in key order)
+    if (nall) {
+        RET(ensure(ctx, ctx->str_flags, (nall + 1) * sizeof(u32)));
+        const int sms = sm_count(ctx);
+        const unsigned blocks = (unsigned)std::min<u64>((nall + 256) / 256, (u64)sms * 16);
+        {
+            KTimer kt(ctx, KC_MISC, 0);
+            check::k_carry_flags<<<blocks, 256, 0, ctx->stream>>>(reinterpret_cast<const uint4*>(ctx->str_co.p),
+                                                                 (u32)nall, P_<u32>(ctx->str_flags));
+        }
+        RET(scan_excl(ctx, P_<u32>(ctx->str_flags), nall + 1));
+        u32 kept = 0;
+        CK(cudaMemcpyAsync(&kept, P_<u32>(ctx->str_flags) + nall, sizeof(u32), cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        Buf& out = ctx->str_carry[ctx->str_cur ^ 1];
+        RET(ensure(ctx, out, ((u64)kept * 2 + 1) * 16));
+        {
+            KTimer kt(ctx, KC_MISC, 0);
+            check::k_carry_scatter<<<blocks, 256, 0, ctx->stream>>>(reinterpret_cast<const uint4*>(ctx->str_co.p),
+                                                                   P_<u32>(ctx->str_flags), (u32)nall,
+                                                                   reinterpret_cast<uint4*>(out.p));
+        }
+        CK(cudaGetLastError());
+        ctx->str_cur ^= 1;
+        ctx->str_ncarry = (u64)kept * 2;
+    }
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->str_nsync = nsy;
+    ctx->str_n += n;
+    ctx->str_wmin = wmin;
+    ctx->str_wmax = wmax;
+    ctx->n_reports = nrep;
+    *n_out = nrep;
     return IGD_OK;
 }
 
@@ -1287,7 +1452,7 @@ static void collect_timing(igd_ctx* ctx);
 
 int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
     if (!ctx || !n_reports_global) return IGD_EINVAL;
-    if (!ctx->loaded) return IGD_ESTATE;
+    if (!ctx->loaded || ctx->str_active) return IGD_ESTATE;
     const u32 tag_log2 = (flags >> IGD_DETECT_TAG_SHIFT) & 31u;
     if (tag_log2 && (tag_log2 < 8 || tag_log2 > 22)) {
         ctx->err = "IGD_DETECT_TAG_LOG2 must be 8..22";
@@ -1377,6 +1542,7 @@ int igd_shard_detect(igd_ctx* ctx, const void* d_records, uint64_t n_records, co
         ctx->err = "IGD_DETECT_COALESCE is a single-context mode";
         return IGD_EINVAL;
     }
+    if (ctx->str_active) return IGD_ESTATE;  // a streaming session owns the sharded-mode state
     cudaSetDevice(ctx->device);
     ctx->timing = (flags & IGD_DETECT_TIMING) != 0;
     ctx->paper_counters = (flags & IGD_DETECT_PAPER_COUNTERS) != 0;
@@ -1470,6 +1636,52 @@ int igd_kernel_stats(const igd_ctx* ctx, int kclass, const char** name, uint32_t
     return IGD_OK;
 }
 
+int igd_stream_begin(igd_ctx* ctx, uint32_t n_blocks, uint32_t block_dim) {
+    if (!ctx || n_blocks == 0 || block_dim == 0 || (u64)n_blocks * block_dim > (1ull << 24)) return IGD_EINVAL;
+    if (ctx->comm) {
+        ctx->err = "streaming sessions are single-context";
+        return IGD_EINVAL;
+    }
+    ctx->str_active = true;
+    ctx->str_n = ctx->str_nsync = ctx->str_ncarry = 0;
+    ctx->str_wmin = ~0ull;
+    ctx->str_wmax = 0;
+    ctx->str_nb = n_blocks;
+    ctx->str_bd = block_dim;
+    ctx->str_cur = 0;
+    return IGD_OK;
+}
+
+int igd_stream_feed(igd_ctx* ctx, const igd_event* events, uint64_t n_events, uint32_t event_flags,
+                    uint32_t detect_flags, uint64_t* n_reports) {
+    if (!ctx || !n_reports) return IGD_EINVAL;
+    if (!ctx->str_active) return IGD_ESTATE;
+    if (detect_flags & (IGD_DETECT_COALESCE | (31u << IGD_DETECT_TAG_SHIFT) | (15u << IGD_DETECT_LAST_K_SHIFT))) {
+        ctx->err = "streaming sessions support IGD_DETECT_TIMING, _PAPER_COUNTERS and _STICKY_FLAGS";
+        return IGD_EINVAL;
+    }
+    cudaSetDevice(ctx->device);
+    ctx->timing = (detect_flags & IGD_DETECT_TIMING) != 0;
+    ctx->paper_counters = (detect_flags & IGD_DETECT_PAPER_COUNTERS) != 0;
+    ctx->sticky = (detect_flags & IGD_DETECT_STICKY_FLAGS) != 0;
+    int rc = stream_feed_impl(ctx, events, n_events, event_flags, n_reports);
+    ctx->paper_counters = false;
+    ctx->sticky = false;
+    if (rc != IGD_OK) ctx->str_active = false;  // a failed chunk ends the session
+    if (rc == IGD_OK && ctx->timing) collect_timing(ctx);
+    return rc;
+}
+
+int igd_stream_end(igd_ctx* ctx) {
+    if (!ctx) return IGD_EINVAL;
+    cudaSetDevice(ctx->device);
+    ctx->str_active = false;
+    Buf* all[] = {&ctx->str_sidx, &ctx->str_sev, &ctx->str_carry[0], &ctx->str_carry[1], &ctx->str_rec,
+                  &ctx->str_co, &ctx->str_flags};
+    for (Buf* b : all) RET(buf_free(ctx, *b));
+    return IGD_OK;
+}
+
 int igd_nccl_unique_id(uint8_t* out128) {
     if (!out128) return IGD_EINVAL;
     NcclApi& N = nccl();
@@ -1495,7 +1707,9 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf,
                   &ctx->cl_small,     &ctx->cl_mat,   &ctx->cl_recv,  &ctx->cl_sidx,  &ctx->cl_sev,
-                  &ctx->cl_nrep,      &ctx->cl_rep,   &ctx->gkb,      &ctx->seg_rep,  &ctx->lk_state};
+                  &ctx->cl_nrep,      &ctx->cl_rep,   &ctx->gkb,      &ctx->seg_rep,  &ctx->lk_state,
+                  &ctx->str_sidx,     &ctx->str_sev,  &ctx->str_carry[0], &ctx->str_carry[1], &ctx->str_rec,
+                  &ctx->str_co,       &ctx->str_flags};
     for (Buf* b : all) buf_free(ctx, *b);
     cudaStreamSynchronize(ctx->stream);
     cudaFreeHost(ctx->h_stats);

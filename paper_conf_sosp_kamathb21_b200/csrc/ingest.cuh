@@ -385,6 +385,124 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_ingest(Params P) {
     if (tid == 0 && cta_sync) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cta_sync);
 }
 
+// ---- pass 0 of the fused single-GPU pipeline (the timed path) ----------------------------------
+// The same outputs as k_ingest<0> with hist0 = 1 (field rules -> first invalid index, per-tile
+// access / sync-record counts, digit histograms of the access keys, word range, lock events,
+// grid-changing kernel boundaries), with a branch-free rule check: one 4-bit rule word per kind
+// (lane in mask / scope set or NONE / addr 0 / tid 0) instead of the switch, which was the
+// kernel's most divergent line (ncu r02h: 8 % of instructions, 11 % of stall samples), and
+// compile-time geometry (GEO2: power-of-two block_dim >= 32) and coalesced-mode (COAL) variants.
+//   rule bits: 1 = lane(tid) in mask, 2 = scope != NONE (else == NONE), 4 = addr == 0, 8 = tid == 0
+constexpr u64 kRules = 0x1ull | (0x1ull << 4) | (0x3ull << 8) | (0x3ull << 12) | (0x3ull << 16) |
+                       (0x7ull << 20) | (0x4ull << 24) | (0x4ull << 28) | (0xCull << 32) | (0x4ull << 36) |
+                       (0x4ull << 40) | (0xCull << 44) | (0x8ull << 48);
+// sync records per kind (2 bits each): CAS / EXCH 1 (lock list), FENCE 1 (+1 when device scope),
+// the barriers, grid syncs and kernel boundaries 1
+constexpr u32 kSyncRecs = (1u << 6) | (1u << 8) | (1u << 10) | (1u << 12) | (1u << 14) | (1u << 16) |
+                          (1u << 18) | (1u << 20) | (1u << 22) | (1u << 24);
+
+template <bool GEO2, bool COAL>
+__global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_count_fused(Params P) {
+    __shared__ u32 s_hacc[4][256];
+    __shared__ u32 s_hup[3][256];
+    __shared__ u32 s_wtot[WARPS];
+    const u32 tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    for (int i = tid; i < 4 * 256; i += THREADS) {
+        (&s_hacc[0][0])[i] = 0;
+        if (i < 3 * 256) (&s_hup[0][0])[i] = 0;
+    }
+    __syncthreads();
+    u64 wmin = ~0ull, wmax = 0, bad = ~0ull;
+    u32 cnt_lock = 0;
+    u64 cta_sync = 0;
+    const Geo g = P.g;
+    for (u32 tile = blockIdx.x; tile < P.n_tiles; tile += gridDim.x) {
+        const u64 base = (u64)tile * TILE;
+        uint4 e[ITEMS];
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const u64 i = base + (u64)j * THREADS + tid;
+            e[j] = (i < P.n) ? ld_event_stream(P.ev, i) : make_uint4(0, 0, 0, 0);
+        }
+        u32 wsum = 0;
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const u64 i = base + (u64)j * THREADS + tid;
+            const bool in = i < P.n;
+            const u32 t = e[j].z & 0xFFFFFFu, kind = (e[j].z >> 24) & 0xFu, scope = (e[j].z >> 28) & 3u;
+            const bool addr0 = (e[j].x | e[j].y) == 0;
+            const u32 r = (u32)(kRules >> (4 * (kind & 15u))) & 15u;
+            const u32 ln = GEO2 ? (t & 31u) : ((t - g.block(t) * g.D) & 31u);
+            bool ok = (e[j].z >> 30) == 0 && kind <= IGD_KERNEL_BOUNDARY && t < g.T;
+            ok = ok && (!(r & 1u) || ((e[j].w >> ln) & 1u)) && ((r & 2u) ? scope != 0u : scope == 0u) &&
+                 (!(r & 4u) || addr0) && (!(r & 8u) || t == 0u) &&
+                 (kind != IGD_KERNEL_BOUNDARY || addr0 || geo_code_ok(e[j].y, e[j].x));
+            bool acc = in && ok && kind <= IGD_EXCH;
+            if (COAL && acc && ((__ldg(P.skip_bits + (i >> 5)) >> (i & 31u)) & 1u)) acc = false;  // A32
+            const u32 ns = (in && ok) ? ((kSyncRecs >> (2 * kind)) & 3u) + (kind == IGD_FENCE && scope >= 2u ? 1u : 0u)
+                                      : 0u;
+            if (in && !ok) bad = min(bad, i);
+            if (in && ok && kind == IGD_KERNEL_BOUNDARY && !addr0) {  // rare: another grid (A34)
+                const unsigned long long slot = atomicAdd((unsigned long long*)&P.stats[6], 1ull);
+                if (slot < P.gkb_cap) P.gkb[slot] = i;
+            }
+            cnt_lock += (in && ok && (kind == IGD_CAS || kind == IGD_EXCH)) ? 1u : 0u;
+            const u32 key = (e[j].x >> 2) | (e[j].y << 30);
+            if (acc) {
+                const u64 word = ev_addr(e[j]) >> 2;
+                wmin = min(wmin, word);
+                wmax = max(wmax, word);
+                atomicAdd(&s_hacc[warp & 3u][key & 255u], 1u);
+            }
+            // digits 1..3: one set of atomics per distinct upper-24-bit value among the lanes
+            const u32 am = __ballot_sync(IGD_FULL, acc);
+            if (am) {
+                const u32 hi = key >> 8;
+                const u32 peers = __match_any_sync(IGD_FULL, acc ? hi : (0x1000000u | lane)) & am;
+                const u32 c = (acc && lane == (u32)(__ffs(peers) - 1)) ? __popc(peers) : 0u;
+                if (c) {
+                    atomicAdd(&s_hup[0][hi & 255u], c);
+                    atomicAdd(&s_hup[1][(hi >> 8) & 255u], c);
+                    atomicAdd(&s_hup[2][hi >> 16], c);
+                }
+            }
+            wsum += __reduce_add_sync(IGD_FULL, (acc ? 1u : 0u) | (ns << 16));
+        }
+        if (lane == 0) s_wtot[warp] = wsum;
+        __syncthreads();
+        if (warp == 0) {
+            const u32 x = lane < WARPS ? s_wtot[lane] : 0u;
+            const u32 ta = __reduce_add_sync(IGD_FULL, x & 0xFFFFu);
+            const u32 ts = __reduce_add_sync(IGD_FULL, x >> 16);
+            if (lane == 0) {
+                P.tile_acc[tile] = ta;
+                P.tile_sync[tile] = ts;
+                cta_sync += ts;
+            }
+        }
+        __syncthreads();
+    }
+    for (int i = tid; i < 4 * 256; i += THREADS) {
+        const u32 a = i < 256 ? s_hacc[0][i] + s_hacc[1][i] + s_hacc[2][i] + s_hacc[3][i] : (&s_hup[0][0])[i - 256];
+        if (a) atomicAdd(&P.hist_acc[i], a);
+    }
+    u64 cl = cnt_lock;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        wmin = min(wmin, __shfl_xor_sync(IGD_FULL, wmin, o));
+        wmax = max(wmax, __shfl_xor_sync(IGD_FULL, wmax, o));
+        bad = min(bad, __shfl_xor_sync(IGD_FULL, bad, o));
+        cl += __shfl_xor_sync(IGD_FULL, cl, o);
+    }
+    if (lane == 0) {
+        if (wmin != ~0ull) atomicMin((unsigned long long*)&P.stats[0], (unsigned long long)wmin);
+        if (wmin != ~0ull) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
+        if (bad != ~0ull) atomicMin((unsigned long long*)&P.stats[2], (unsigned long long)bad);
+        if (cl) atomicAdd((unsigned long long*)&P.stats[5], (unsigned long long)cl);
+    }
+    if (tid == 0 && cta_sync) atomicAdd((unsigned long long*)&P.stats[4], (unsigned long long)cta_sync);
+}
+
 // Digit histograms (4 x 8-bit) of the compacted access keys: a light, high-occupancy pass over
 // 4 bytes per access, with warp-uniform digits aggregated into one shared atomic.
 __global__ void __launch_bounds__(256) k_hist_keys(const u32* __restrict__ keys, u32 n, u32* __restrict__ hist,

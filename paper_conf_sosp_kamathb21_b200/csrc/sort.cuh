@@ -123,6 +123,35 @@ constexpr size_t onesweep_smem() {
     return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT) + TILE;
 }
 
+#ifndef IGD_SORT_LB_EARLY
+#define IGD_SORT_LB_EARLY 0  // 1: look-back before ranking (measured slower: C5 access sort 80.3 -> 86.7 ms, r02j)
+#endif
+// Decoupled look-back for digit d of `tile`: the sum of the digit's counts over all earlier tiles.
+// LB predecessor statuses are requested at once, so a walk back over tiles that have published
+// only their aggregate costs one L2 round trip per LB tiles instead of one per tile.
+__device__ __forceinline__ u64 lookback_digit(const PassParams& P, u32 tile, u32 d) {
+    u64 excl = 0;
+    if (tile == 0) return 0;
+    long tt = (long)tile - 1;
+    bool done = false;
+    while (!done) {
+        u64 s[IGD_SORT_LB];
+#pragma unroll
+        for (int q = 0; q < IGD_SORT_LB; q++)
+            s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + d) : ST_INC;
+#pragma unroll
+        for (int q = 0; q < IGD_SORT_LB; q++) {
+            if (!done) {
+                s[q] = spin_status(P.status + (u64)(tt - q) * RADIX + d, s[q]);
+                excl += s[q] & ST_VAL_MASK;
+                done = (s[q] >> 62) == 2;
+            }
+        }
+        tt -= IGD_SORT_LB;
+    }
+    return excl;
+}
+
 // TAIL = false: every tile of the launch is full (no bounds tests on the hot path); TAIL = true:
 // the one partial last tile, launched after the full ones (its look-back finds them published).
 // KT = u32 (word spans < 2^32 words) or u64 keys (reading a4's wide path: up to 8 digit passes)
@@ -195,6 +224,14 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         __syncthreads();
         st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
     }
+    u64 excl_early = 0;
+    if (IGD_SORT_EARLY && IGD_SORT_LB_EARLY) {
+        // the look-back right after the aggregate, before ranking: this tile's inclusive prefix is
+        // published early, so successors' walks stop sooner (ncu r02h: look-back spins were a
+        // quarter of the stall samples when it followed the ranking)
+        excl_early = lookback_digit(P, tile, t);
+        if (tile > 0) st_relaxed(P.status + (u64)tile * RADIX + t, ST_INC | (excl_early + s_cnt[t]));
+    }
     u32 rank[ITEMS];
     const u32 lt = lanemask_lt();
 #pragma unroll
@@ -256,24 +293,10 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     {
         const u32 d = t;
         u64 excl = 0;
-        if (tile > 0) {
-            long tt = (long)tile - 1;
-            bool done = false;
-            while (!done) {
-                u64 s[IGD_SORT_LB];
-#pragma unroll
-                for (int q = 0; q < IGD_SORT_LB; q++)
-                    s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + d) : ST_INC;
-#pragma unroll
-                for (int q = 0; q < IGD_SORT_LB; q++) {
-                    if (!done) {
-                        s[q] = spin_status(P.status + (u64)(tt - q) * RADIX + d, s[q]);
-                        excl += s[q] & ST_VAL_MASK;
-                        done = (s[q] >> 62) == 2;
-                    }
-                }
-                tt -= IGD_SORT_LB;
-            }
+        if (IGD_SORT_EARLY && IGD_SORT_LB_EARLY) {
+            excl = excl_early;
+        } else if (tile > 0) {
+            excl = lookback_digit(P, tile, d);
             st_relaxed(P.status + (u64)tile * RADIX + d, ST_INC | (excl + cnt));
         }
         // output position of tile position i with digit d = s_gbase[d] + i (u32 arithmetic wraps

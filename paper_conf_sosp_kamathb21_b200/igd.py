@@ -84,6 +84,12 @@ def load_library(build_if_missing: bool = True):
     lib.igd_shard_buffers.restype = i32
     lib.igd_shard_detect.argtypes = [vp, vp, u64, vp, vp, u64, u64, u32, ctypes.POINTER(u64)]
     lib.igd_shard_detect.restype = i32
+    lib.igd_stream_begin.argtypes = [vp, u32, u32]
+    lib.igd_stream_begin.restype = i32
+    lib.igd_stream_feed.argtypes = [vp, vp, u64, u32, u32, ctypes.POINTER(u64)]
+    lib.igd_stream_feed.restype = i32
+    lib.igd_stream_end.argtypes = [vp]
+    lib.igd_stream_end.restype = i32
     lib.igd_nccl_unique_id.argtypes = [vp]
     lib.igd_nccl_unique_id.restype = i32
     lib.igd_ctx_destroy.argtypes = [vp]
@@ -254,6 +260,39 @@ class Detector:
 
     def reports(self) -> np.ndarray:
         return igd_reports(self.ctx, self.n_reports)
+
+    # ---- streaming sessions (igd_stream_*) ----
+    def stream_begin(self, n_blocks: int, block_dim: int):
+        rc = load_library().igd_stream_begin(self.ctx, n_blocks, block_dim)
+        if rc != IGD_OK:
+            raise IgdError(rc, load_library().igd_last_error(self.ctx).decode())
+
+    def stream_feed(self, events, paper_counters: bool = False, sticky_flags: bool = False,
+                    timing: bool = False) -> np.ndarray:
+        """Check the next chunk (host EVENT_DTYPE array or CUDA tensor); returns its reports."""
+        lib = load_library()
+        torch = self._torch
+        if isinstance(events, torch.Tensor):
+            assert events.is_cuda and events.is_contiguous() and events.data_ptr() % 16 == 0
+            n = events.numel() * events.element_size() // 16
+            ptr, fl, keep = events.data_ptr() if n else 0, IGD_TRACE_DEVICE_PTR, events
+        else:
+            keep = np.ascontiguousarray(events)
+            n = len(keep)
+            ptr, fl = keep.ctypes.data if n else 0, 0
+        flags = ((IGD_DETECT_TIMING if timing else 0) | (IGD_DETECT_PAPER_COUNTERS if paper_counters else 0)
+                 | (IGD_DETECT_STICKY_FLAGS if sticky_flags else 0))
+        nr = ctypes.c_uint64(0)
+        rc = lib.igd_stream_feed(self.ctx, ctypes.c_void_p(ptr or None), n, fl, flags, ctypes.byref(nr))
+        del keep
+        if rc != IGD_OK:
+            bad = lib.igd_bad_event(self.ctx) if rc == IGD_ETRACE else None
+            raise IgdError(rc, lib.igd_last_error(self.ctx).decode(), bad)
+        self.n_reports = int(nr.value)
+        return self.reports()
+
+    def stream_end(self):
+        load_library().igd_stream_end(self.ctx)
 
     def stage_times(self) -> dict:
         lib = load_library()
