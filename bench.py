@@ -94,10 +94,49 @@ def peaks():
         return 6650.0, "fallback"
 
 
+def host_info():
+    """The host the oracle baseline ran on (nproc, CPU model, RAM)."""
+    model, ram = None, None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal"):
+                ram = round(int(line.split()[1]) / 1024 / 1024, 1)
+                break
+    except OSError:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count(), "ram_gib": ram}
+
+
+def pin_one_core():
+    """Pin this process to one host core for the oracle timing (the `taskset -c` of SURVEY 8(d));
+    returns the previous affinity to restore, or None."""
+    try:
+        prev = os.sched_getaffinity(0)
+        core = sorted(prev)[min(1, len(prev) - 1)]
+        os.sched_setaffinity(0, {core})
+        return prev
+    except (AttributeError, OSError):
+        return None
+
+
 def oracle_baseline(ev, nb, bd, budget_s=15.0, coalesce=False, paper_counters=False):
-    """Time the CPU oracle (as it stands, single-threaded) on a bounded prefix of the trace."""
+    """Time the CPU oracle (as it stands, single-threaded, pinned to one core) on a bounded prefix
+    of the trace."""
     import oracle
 
+    prev = pin_one_core()
+    try:
+        return _oracle_baseline(oracle, ev, nb, bd, budget_s, coalesce, paper_counters)
+    finally:
+        if prev is not None:
+            os.sched_setaffinity(0, prev)
+
+
+def _oracle_baseline(oracle, ev, nb, bd, budget_s, coalesce, paper_counters):
     n = min(len(ev), 2_000_000)
     t0 = time.perf_counter()
     oracle.run(ev[:n], nb, bd, coalesce=coalesce, paper_counters=paper_counters)
@@ -125,6 +164,7 @@ def run_reference(args, fam, rank, world):
     ev = plan.fill(0, sample)
     nb, bd, n_total = plan.n_blocks, plan.block_dim, plan.n_events
     plan.close()
+    pin_one_core()
     for _ in range(args.warmup):
         oracle.run(ev[: min(sample, 1_000_000)], nb, bd)
     times = []
@@ -141,7 +181,7 @@ def run_reference(args, fam, rank, world):
             "config": {"workload": F.FAMILY_NAMES[fam], "events": n_total, "sample_events": sample,
                        "n_blocks": nb, "block_dim": bd},
             "cpu_baseline": {"value": value, "unit": "G events/s", "cores": 1, "kind": "oracle",
-                             "sample": sample_desc},
+                             "sample": sample_desc, "host": host_info()},
             "e2e": {"value": value, "unit": "G events/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -273,9 +313,20 @@ def run_sharded(args, fam, rank, world, local):
 
 
 # kernel class -> the kernel ncu names for it (classes made of one kernel)
-CLASS_KERNEL = {"sort_access": "rsort::k_onesweep<1, unsigned long, 0>", "check": "check::k_check4<0, 0, 0>",
-                "ingest_sort0": "fused::k_ingest_sort0", "ingest": "ingest::k_ingest<0>"}
-TRAFFIC_JSON = os.path.join(ROOT, "profiles", "traffic_r01.json")
+CLASS_KERNEL = {"sort_access": "rsort::k_onesweep<unsigned long, 0, unsigned int>",
+                "check": "check::k_check4<0, 0, 0, 1, unsigned int>",
+                "ingest_sort0": "fused::k_ingest_sort0<0, unsigned int>", "ingest": "ingest::k_count_fused<1, 0>"}
+TRAFFIC_JSON = os.path.join(ROOT, "profiles", "traffic_r02.json")
+
+
+def ncu_path_bytes(workload, n):
+    """DRAM bytes of one whole igd_detect (every kernel) from the committed ncu launch list of this
+    workload at this size (profiles/summarize_launches.py --detects), or None."""
+    try:
+        d = json.load(open(TRAFFIC_JSON)).get(f"{workload}@{n}", {})
+    except (OSError, ValueError):
+        return None
+    return d.get("__dram_per_detect__")
 
 
 def ncu_traffic(workload, n, kclass):
@@ -397,10 +448,24 @@ def main():
     path_gbs = total_alg / (ms / 1e3) / 1e9
     f_acc = None
     traffic, tsrc = ncu_traffic(F.FAMILY_NAMES[fam], n, dom)
-    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "peak_source": peak_kind, "traffic": traffic, "traffic_source": tsrc,
+    path_bytes = ncu_path_bytes(F.FAMILY_NAMES[fam], n)
+    # achieved = SURVEY 8(d)'s algorithmic bytes per unit x the units one launch processes:
+    # a radix pass reads and writes 8 B per access; the check reads 8 B and gathers one 32-B sector
+    # per access; the ingest reads every 16-B event and writes an 8-B key per access.  The design's
+    # own element bytes (12-B sort elements) are reported beside it.
+    kinds_all = np.bincount(((host["tk"] >> 24) & 0xF).astype(np.int64), minlength=13)
+    n_acc = int(kinds_all[:5].sum())
+    survey_bytes = {"sort_access": 16.0 * n_acc, "check": 40.0 * n_acc, "ingest_sort0": 16.0 * n + 8.0 * n_acc,
+                    "ingest": 16.0 * n}
+    per_launch = survey_bytes.get(dom)
+    s_achieved = per_launch / (kms / max(cnt, 1) / 1e3) / 1e9 if (per_launch and kms > 0) else achieved
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": s_achieved, "peak": peak, "unit": "GB/s",
+                "frac": s_achieved / peak, "peak_source": peak_kind, "traffic": traffic, "traffic_source": tsrc,
+                "alg_bytes_basis": "SURVEY 8(d) per-unit bytes" if per_launch else "design bytes",
+                "alg_bytes_per_launch": per_launch if per_launch else kbytes / max(cnt, 1),
                 "launches_per_step": cnt / args.steps, "ms_per_launch": kms / max(cnt, 1),
-                "alg_bytes_per_launch": kbytes / max(cnt, 1)}
+                "achieved_design_bytes": achieved, "frac_design_bytes": achieved / peak,
+                "design_bytes_per_launch": kbytes / max(cnt, 1)}
     breakdown = {k: {"launches": v[0] // args.steps, "ms": v[1] / args.steps,
                      "alg_GBps": (v[2] / (v[1] / 1e3) / 1e9) if v[1] > 0 else None}
                  for k, v in kstats.items() if v[0]}
@@ -441,7 +506,8 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         sn, sdt = oracle_baseline(host, nb, bd, coalesce=co, paper_counters=pc)
         cpu = {"value": sn / sdt / 1e9, "unit": "G events/s", "cores": 1, "kind": "oracle",
-               "sample": f"first {sn} events of {F.FAMILY_NAMES[fam]} ({sdt:.1f}s, single-threaded C oracle)"}
+               "sample": f"first {sn} events of {F.FAMILY_NAMES[fam]} ({sdt:.1f}s, single-threaded C oracle "
+                         f"pinned to one core)", "host": host_info()}
     if pinned:
         cudart.cudaHostUnregister(host.ctypes.data)
 
@@ -471,6 +537,11 @@ def main():
                 "roofline": roofline,
                 "path": {"alg_bytes_per_event_B_alg": b_alg, "alg_GBps_B_alg": value * b_alg,
                          "frac_B_alg": value * b_alg / peak, "kernel_alg_GBps": path_gbs,
+                         # SURVEY 8(d) fraction 1 (north_star's gate): ncu DRAM bytes of a whole detect
+                         # (committed launch list) over this run's step time
+                         "ncu_dram_bytes_per_step": path_bytes,
+                         "achieved_dram_GBps": (path_bytes / (ms / 1e3) / 1e9) if path_bytes else None,
+                         "achieved_dram_frac": (path_bytes / (ms / 1e3) / 1e9 / peak) if path_bytes else None,
                          "stages_ms": stages, "kernels": breakdown},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk}
         print(json.dumps(line), flush=True)

@@ -24,6 +24,7 @@
 #include "shard.cuh"
 #include "sync.cuh"
 #include <dlfcn.h>
+#include <nvtx3/nvToolsExt.h>
 #include <nccl.h>  // types and prototypes only: the library is resolved at run time (NcclApi)
 #include <algorithm>
 #include <vector>
@@ -175,6 +176,7 @@ struct igd_ctx {
     u64* h_small = nullptr;  // 8
 
     bool timing = false;
+    int nvtx_depth = 0;
     cudaEvent_t ev[IGD_N_STAGES + 1];
     float stage_ms[IGD_N_STAGES];
     // per-launch timing (IGD_DETECT_TIMING): events around every kernel launch
@@ -281,8 +283,21 @@ static int sm_count(igd_ctx* ctx) {
     return v;
 }
 
+// Stage boundaries: CUDA events (IGD_DETECT_TIMING) and an NVTX range per stage
+// ("igd:<stage>", visible to Nsight Systems / ncu --nvtx; a no-op without a tool attached).
 static void mark(igd_ctx* ctx, int stage) {
     if (ctx->timing) cudaEventRecord(ctx->ev[stage], ctx->stream);
+    while (ctx->nvtx_depth > 0) {
+        nvtxRangePop();
+        ctx->nvtx_depth--;
+    }
+    if (stage < IGD_N_STAGES - 1) {
+        static const char* names[IGD_N_STAGES - 1] = {"igd:a1-a4 ingest", "igd:a2 sync sort", "igd:a2-a3 tables+locks",
+                                                      "igd:a5 access sort", "igd:a6 check", "igd:a7 reports",
+                                                      "igd:host sync"};
+        nvtxRangePushA(names[stage]);
+        ctx->nvtx_depth++;
+    }
 }
 
 // One radix pass over n keys: the full tiles, then (if any) the partial last tile (same tile

@@ -15,6 +15,11 @@ BSCALE = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12, 
 
 args = sys.argv[1:]
 tj = None
+detects = None
+if "--detects" in args:  # igd_detect calls the launch list covers (warmup + steps of the bench run)
+    i = args.index("--detects")
+    detects = int(args[i + 1])
+    args = args[:i] + args[i + 2:]
 if "--traffic-json" in args:
     i = args.index("--traffic-json")
     tj = (args[i + 1], args[i + 2])
@@ -52,4 +57,6 @@ if tj:
     out, workload = tj
     d = json.load(open(out)) if os.path.exists(out) else {}
     d[workload] = {k: dram[k] / cnt[k] for k in dram if dram[k]}
+    if detects:
+        d[workload]["__dram_per_detect__"] = sum(dram.values()) / detects
     json.dump(d, open(out, "w"), indent=1, sort_keys=True)
