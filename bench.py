@@ -35,6 +35,18 @@ METRIC = "G events race-checked/s at 1/2/4/8 B200; achieved HBM GB/s vs peak"
 CONFIGS = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5}
 
 
+def gen_kw(args):
+    import tracegen.families as F
+
+    return dict(F.SYNC_HEAVY) if getattr(args, "sync_heavy", False) else {}
+
+
+def workload_name(args, fam):
+    import tracegen.families as F
+
+    return F.FAMILY_NAMES[fam] + ("-sync-heavy" if getattr(args, "sync_heavy", False) else "")
+
+
 def log(*a):
     print(*a, file=sys.stderr, flush=True)
 
@@ -158,7 +170,7 @@ def run_reference(args, fam, rank, world):
     import tracegen.families as F
     import oracle
 
-    plan = F.Plan(fam)
+    plan = F.Plan(fam, **gen_kw(args))
     # each step checks a bounded prefix sample of the workload so the run ends in minutes
     sample = min(plan.n_events, args.oracle_events or 12_000_000)
     ev = plan.fill(0, sample)
@@ -174,11 +186,11 @@ def run_reference(args, fam, rank, world):
         times.append(time.perf_counter() - t0)
     t = sum(times) / len(times)
     value = sample / t / 1e9
-    sample_desc = f"first {sample} of {n_total} events of {F.FAMILY_NAMES[fam]} (single-threaded oracle)"
+    sample_desc = f"first {sample} of {n_total} events of {workload_name(args, fam)} (single-threaded oracle)"
     line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic", "impl": "reference",
-            "config": {"workload": F.FAMILY_NAMES[fam], "events": n_total, "sample_events": sample,
+            "config": {"workload": workload_name(args, fam), "events": n_total, "sample_events": sample,
                        "n_blocks": nb, "block_dim": bd},
             "cpu_baseline": {"value": value, "unit": "G events/s", "cores": 1, "kind": "oracle",
                              "sample": sample_desc, "host": host_info()},
@@ -219,7 +231,7 @@ def run_sharded(args, fam, rank, world, local):
     nccl_id = bytes(idt.cpu().numpy().tobytes())
 
     t0 = time.time()
-    plan = F.Plan(fam, args.events or None)
+    plan = F.Plan(fam, args.events or None, **gen_kw(args))
     n, nb, bd = plan.n_events, plan.n_blocks, plan.block_dim
     lo = n * rank // world
     cnt = n * (rank + 1) // world - lo
@@ -228,7 +240,7 @@ def run_sharded(args, fam, rank, world, local):
     lg = plan.ledger()
     plan.close()
     if rank == 0:
-        log(f"[bench] {F.FAMILY_NAMES[fam]}: {n} events over {world} ranks, chunk {cnt}, {time.time() - t0:.1f}s")
+        log(f"[bench] {workload_name(args, fam)}: {n} events over {world} ranks, chunk {cnt}, {time.time() - t0:.1f}s")
     cudart = torch.cuda.cudart()
     pinned = cudart.cudaHostRegister(host.ctypes.data, host.nbytes, 0) == 0
     chunk = torch.from_numpy(host.view(np.uint8)).to(f"cuda:{dev_index}")
@@ -293,7 +305,7 @@ def run_sharded(args, fam, rank, world, local):
         line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-                "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
+                "config": {"workload": workload_name(args, fam), "events": n, "n_blocks": nb, "block_dim": bd,
                            "reports": int(nrep), "ledger_reports": int(len(lg)), "ledger_match": ledger_match,
                            "l2": "inputs larger than L2 (no flush)",
                            "parallelism": f"{world} ranks: contiguous trace chunks, words hash-sharded "
@@ -360,6 +372,8 @@ def main():
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"], help="N>1 collectives")
     ap.add_argument("--paper-counters", action="store_true",
                     help="Fig. 4-width synchronization IDs (IGD_DETECT_PAPER_COUNTERS, reading A33)")
+    ap.add_argument("--sync-heavy", action="store_true",
+                    help="C2 / C5 sync-heavy variant (spin-lock sections ~8 %%, fences ~5 %%; SURVEY 8(d))")
     ap.add_argument("--coalesce", action="store_true",
                     help="warp-coalesced check mode (IGD_DETECT_COALESCE, reading A32; 1 GPU)")
     args = ap.parse_args()
@@ -387,14 +401,14 @@ def main():
 
     # ---------------- workload ----------------
     t0 = time.time()
-    plan = F.Plan(fam, args.events or None)
+    plan = F.Plan(fam, args.events or None, **gen_kw(args))
     n, nb, bd = plan.n_events, plan.n_blocks, plan.block_dim
     host = np.empty(n, igd.EVENT_DTYPE)
     plan.fill(out=host, threads=args.threads)
     lg = plan.ledger()
     ledger_n = len(lg)
     plan.close()
-    log(f"[bench] {F.FAMILY_NAMES[fam]}: {n} events, {nb}x{bd} threads, generated in {time.time() - t0:.1f}s")
+    log(f"[bench] {workload_name(args, fam)}: {n} events, {nb}x{bd} threads, generated in {time.time() - t0:.1f}s")
     cudart = torch.cuda.cudart()
     pinned = cudart.cudaHostRegister(host.ctypes.data, host.nbytes, 0) == 0
     dev = torch.empty(host.nbytes, dtype=torch.uint8, device="cuda")
@@ -447,8 +461,8 @@ def main():
     total_alg = sum(v[2] for v in kstats.values()) / args.steps
     path_gbs = total_alg / (ms / 1e3) / 1e9
     f_acc = None
-    traffic, tsrc = ncu_traffic(F.FAMILY_NAMES[fam], n, dom)
-    path_bytes = ncu_path_bytes(F.FAMILY_NAMES[fam], n)
+    traffic, tsrc = ncu_traffic(workload_name(args, fam), n, dom)
+    path_bytes = ncu_path_bytes(workload_name(args, fam), n)
     # achieved = SURVEY 8(d)'s algorithmic bytes per unit x the units one launch processes:
     # a radix pass reads and writes 8 B per access; the check reads 8 B and gathers one 32-B sector
     # per access; the ingest reads every 16-B event and writes an 8-B key per access.  The design's
@@ -506,7 +520,7 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         sn, sdt = oracle_baseline(host, nb, bd, coalesce=co, paper_counters=pc)
         cpu = {"value": sn / sdt / 1e9, "unit": "G events/s", "cores": 1, "kind": "oracle",
-               "sample": f"first {sn} events of {F.FAMILY_NAMES[fam]} ({sdt:.1f}s, single-threaded C oracle "
+               "sample": f"first {sn} events of {workload_name(args, fam)} ({sdt:.1f}s, single-threaded C oracle "
                          f"pinned to one core)", "host": host_info()}
     if pinned:
         cudart.cudaHostUnregister(host.ctypes.data)
@@ -526,7 +540,7 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": "G events/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-                "config": {"workload": F.FAMILY_NAMES[fam], "events": n, "n_blocks": nb, "block_dim": bd,
+                "config": {"workload": workload_name(args, fam), "events": n, "n_blocks": nb, "block_dim": bd,
                            "f_acc": f_acc, "reports": int(nrep),
                            "ledger_reports": None if (co or pc) else ledger_n,  # ledger: per-lane, exact IDs
                            "ledger_match": ledger_match,

@@ -84,3 +84,20 @@ def test_c5_exercises_every_radix_digit():
     for d in range(4):
         digits = np.unique(((w >> np.uint64(8 * d)) & np.uint64(255)))
         assert len(digits) >= (48 if d == 3 else 256)
+
+
+# ---- the sync-heavy variant (f_acc ~0.9-0.95, fences ~5 %, spin-lock sections ~8 %) ----
+@pytest.mark.parametrize("fam,n,rate", [(2, 3_000_000, 3.0), (5, 14_000_000, 30.0)])
+def test_sync_heavy_ledger_equals_oracle(fam, n, rate):
+    ev, nb, bd, led = F.generate(fam, n, rate=rate, **F.SYNC_HEAVY)
+    kinds = np.bincount(((ev["tk"] >> 24) & 0xF).astype(np.int64), minlength=13)
+    if fam == 2:
+        assert kinds[5] / n > 0.04 and kinds[:5].sum() / n < 0.96  # fences, f_acc
+        assert (kinds[3] + kinds[4]) / n > 0.02                      # lock CAS / EXCH
+    rep = oracle.run(ev, nb, bd)
+    assert len(led) > 0 and key4(rep) == key4(led)
+
+
+def test_sync_heavy_race_free():
+    ev, nb, bd, led = F.generate(2, 2_000_000, fixed=True, **F.SYNC_HEAVY)
+    assert len(led) == 0 and len(oracle.run(ev, nb, bd)) == 0

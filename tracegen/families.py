@@ -28,7 +28,7 @@ DEFAULT_N = {1: 10_000, 2: 10_000_000, 3: 100_000_000, 4: 500_000_000, 5: 4_000_
 class _Cfg(ctypes.Structure):
     _fields_ = [("family", ctypes.c_uint32), ("fixed", ctypes.c_uint32), ("n_blocks", ctypes.c_uint32),
                 ("block_dim", ctypes.c_uint32), ("seed", ctypes.c_uint64), ("n_target", ctypes.c_uint64),
-                ("rate", ctypes.c_double)]
+                ("rate", ctypes.c_double), ("lock_frac", ctypes.c_double), ("fence_frac", ctypes.c_double)]
 
 
 def build(force=False):
@@ -62,10 +62,13 @@ def _load():
 class Plan:
     """A planned trace: sizes and ledger known, events generated on demand (any range)."""
 
-    def __init__(self, family: int, n: int = None, seed: int = None, fixed: bool = False, rate: float = 1.0):
+    def __init__(self, family: int, n: int = None, seed: int = None, fixed: bool = False, rate: float = 1.0,
+                 lock_frac: float = 0.0, fence_frac: float = 0.0):
+        """``lock_frac`` / ``fence_frac`` (C2, C5): the sync-heavy variant's share of spin-locked
+        vertices (default 1 %) and per-warp release fences after each update round (default none)."""
         lib = _load()
         cfg = _Cfg(family, 1 if fixed else 0, 0, 0, FAMILY_SEED[family] if seed is None else seed,
-                   0 if n is None else n, rate)
+                   0 if n is None else n, rate, lock_frac, fence_frac)
         ne, nb, bd = ctypes.c_uint64(), ctypes.c_uint32(), ctypes.c_uint32()
         self._p = lib.igdgen_plan(ctypes.byref(cfg), ctypes.byref(ne), ctypes.byref(nb), ctypes.byref(bd))
         if not self._p:
@@ -105,9 +108,13 @@ class Plan:
             pass
 
 
-def generate(family: int, n: int = None, seed: int = None, fixed: bool = False, rate: float = 1.0):
+# the sync-heavy variant of C2 / C5 (fences ~5 %, spin-lock sections ~8 %)
+SYNC_HEAVY = {"lock_frac": 0.25, "fence_frac": 1.0}
+
+
+def generate(family: int, n: int = None, seed: int = None, fixed: bool = False, rate: float = 1.0, **kw):
     """Whole trace in host memory: (events, n_blocks, block_dim, ledger)."""
-    p = Plan(family, n, seed, fixed, rate)
+    p = Plan(family, n, seed, fixed, rate, **kw)
     ev = p.fill()
     led = p.ledger()
     nb, bd = p.n_blocks, p.block_dim
