@@ -763,6 +763,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     ctx->last_npts = 0;
     RET(radix_sort(ctx, KC_SORT_SYNC, ctx->syn_k, ctx->syn_v, n_sync, P_<u32>(ctx->hist) + 1024, h_hist_sync,
                    bits_needed(ks.E), &scur));
+    // the check's 32-byte timestamp probes may read up to 64 entries past the last list: defined
+    // values there (they are masked out of every decision; compute-sanitizer initcheck is clean)
+    CK(cudaMemsetAsync(P_<u32>(ctx->syn_v[scur]) + n_sync, 0xFF, 64 * sizeof(u32), ctx->stream));
     mark(ctx, 2);
     RET(ensure(ctx, ctx->off, ((u64)ks.E + 2) * sizeof(u32)));
     {
