@@ -498,15 +498,12 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         const bool grid = q_grid(P, mdIdx, i);
         if (p5b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) continue;  // P5
         type = (flags & QF_R1) ? IGD_R1 : 0u;
-        if (!type) {
-            if (same_b) {
-                // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread must
-                // not have fenced since md (A1, A30)
-                if (!(flags & QF_DEV) && !grid && !q_between(P.desc, P.sts, ks.any + p, mdIdx, i))
-                    type = (same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3;
-            } else if (!grid && !q_between(P.desc, P.sts, ks.dev + p, mdIdx, i)) {
-                type = IGD_R4;  // R4: other block, no device fence by md's thread
-            }
+        // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread has not fenced
+        // (any scope) since md (A1, A30); R4 (other block): no device fence by md's thread.  One
+        // query call site for both (divergent lanes would otherwise run two in turn).
+        if (!type && !grid && (!same_b || !(flags & QF_DEV))) {
+            if (!q_between(P.desc, P.sts, (same_b ? ks.any : ks.dev) + p, mdIdx, i))
+                type = same_b ? ((same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3) : IGD_R4;
         }
         }
         if (!type && P.lv.any) {  // R5: lock sets of the last accessor and of this access
@@ -519,9 +516,11 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 laIdx = a.idx;
                 laz = a.tk;
             }
-            u32 L, locks;
-            syncx::held_before2(P.lv, c, i, laz & 0xFFFFFFu, laIdx, L, locks);
-            if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
+            if (syncx::may_hold(P.lv, c) || syncx::may_hold(P.lv, laz & 0xFFFFFFu)) {
+                u32 L, locks;
+                syncx::held_before2(P.lv, c, i, laz & 0xFFFFFFu, laIdx, L, locks);
+                if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;
+            }
         }
         if (type) {
             CSTAT(11);

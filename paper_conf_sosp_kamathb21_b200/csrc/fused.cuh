@@ -65,10 +65,14 @@ struct FDec {
     u32 key, tk, ns, s0, s1;
     bool acc;
 };
+// GEO2: block_dim is a power of two >= 32 (block / warp / lane by shifts and masks)
+template <bool GEO2>
 __device__ __forceinline__ FDec fdecode(const uint4& e, const Geo& g, const KeySpace& ks) {
     FDec d;
     const u32 tid = ev_tid(e), kind = ev_kind(e);
-    const u32 b = g.block(tid), off = tid - b * g.D, w = b * g.Wb + (off >> 5);
+    const u32 b = GEO2 ? tid >> g.dlog : g.block(tid);
+    const u32 off = GEO2 ? (tid & (g.D - 1u)) : tid - b * g.D;
+    const u32 w = GEO2 ? tid >> 5 : b * g.Wb + (off >> 5);
     d.key = (e.x >> 2) | (e.y << 30);
     d.tk = e.z;
     d.ns = 1;
@@ -108,7 +112,7 @@ constexpr size_t smem_bytes() {
 // skip-bit test (ncu r02b: 6% of the kernel's instructions)
 // KT: u32 keys (low 32 bits of the word; spans < 2^32 words) or u64 keys (word - kbase, the wide
 // path of a4)
-template <bool COAL, typename KT = u32>
+template <bool COAL, typename KT = u32, bool GEO2 = false>
 __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params P) {
     __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
@@ -168,7 +172,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     for (int j = 0; j < ITEMS; j++) {
         const u32 p = wofs + j * 32 + lane;
         const uint4 ev = s_ev[p];
-        FDec d = fdecode(ev, g, ks);  // valid: ingest pass 0 checked every event
+        FDec d = fdecode<GEO2>(ev, g, ks);  // valid: ingest pass 0 checked every event
         const bool in = p < tile_e;
         if (COAL && d.acc && in && ((__ldg(P.skip_bits + ((base + p) >> 5)) >> (p & 31u)) & 1u))
             d.acc = false;  // A32: checked by its coalesced group's first lane
@@ -181,7 +185,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
         nsbits |= ns << (2 * j);
         // the event's own slot now holds its sync record keys (read back by this thread only)
         if (ns) *reinterpret_cast<uint2*>(&s_ev[p]) = make_uint2(d.s0, d.s1);
-        nsync_w += __popc(__ballot_sync(IGD_FULL, ns >= 1)) + __popc(__ballot_sync(IGD_FULL, ns == 2));
+        nsync_w += __reduce_add_sync(IGD_FULL, ns);
     }
     if (lane == 0) s_wsync[warp] = nsync_w;
     __syncthreads();

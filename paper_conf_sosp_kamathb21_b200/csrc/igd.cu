@@ -141,7 +141,7 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
-    Buf off, ldesc, gtab, tcnt, tpts, skipb;
+    Buf off, ldesc, gtab, tcnt, tpts, tbits, skipb;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
@@ -685,6 +685,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
                 else fused::k_ingest_sort0<false, u64><<<(unsigned)ft, fused::THREADS, sm64, ctx->stream>>>(fp);
             } else if (fp.skip_bits) {
                 fused::k_ingest_sort0<true><<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
+            } else if (g.dlog < 32 && g.D >= 32) {  // power-of-two geometry (common case)
+                fused::k_ingest_sort0<false, u32, true><<<(unsigned)ft, fused::THREADS, fused::smem_bytes(),
+                                                          ctx->stream>>>(fp);
             } else {
                 fused::k_ingest_sort0<false><<<(unsigned)ft, fused::THREADS, fused::smem_bytes(), ctx->stream>>>(fp);
             }
@@ -836,6 +839,14 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lv.toff = P_<u32>(ctx->tcnt);
         lv.tpts = P_<u64>(ctx->tpts);
         lv.any = 1;
+        RET(ensure(ctx, ctx->tbits, ((u64)g.T / 32 + 1) * sizeof(u32)));
+        {
+            KTimer kt(ctx, KC_LOCK, 4.0 * (double)g.T);
+            const u32 nw = (g.T + 31) / 32;
+            syncx::k_lock_bits<<<(nw + 255) / 256, 256, 0, ctx->stream>>>(P_<u32>(ctx->tcnt), g.T, P_<u32>(ctx->tbits));
+        }
+        CK(cudaGetLastError());
+        lv.tbits = P_<u32>(ctx->tbits);
         ctx->last_npts = tot;
     }
     mark(ctx, 3);
@@ -1389,6 +1400,8 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
                          (int)fused::smem_bytes());
     cudaFuncSetAttribute(fused::k_ingest_sort0<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes());
+    cudaFuncSetAttribute(fused::k_ingest_sort0<false, u32, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)fused::smem_bytes());
     cudaFuncSetAttribute(fused::k_ingest_sort0<false, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes<u64>());
     cudaFuncSetAttribute(fused::k_ingest_sort0<true, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1721,7 +1734,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
                   &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->tcnt,
-                  &ctx->tpts,         &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
+                  &ctx->tpts,         &ctx->tbits,    &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf,
                   &ctx->cl_small,     &ctx->cl_mat,   &ctx->cl_recv,  &ctx->cl_sidx,  &ctx->cl_sev,

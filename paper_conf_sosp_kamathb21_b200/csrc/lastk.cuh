@@ -54,7 +54,8 @@ __global__ void __launch_bounds__(256) k_lastk(Params L) {
     u32 Lc = 0, locks = 0;
     if (P.lv.any) {
         const check::Acc la = at<false>(P, x - 1);
-        syncx::held_before2(P.lv, c, i, la.tk & 0xFFFFFFu, la.idx, Lc, locks);
+        if (syncx::may_hold(P.lv, c) || syncx::may_hold(P.lv, la.tk & 0xFFFFFFu))
+            syncx::held_before2(P.lv, c, i, la.tk & 0xFFFFFFu, la.idx, Lc, locks);
     }
     u32 mask = 0;
     bool have_mask = false;

@@ -93,6 +93,7 @@ struct LockParams {
 // The event with timestamp ts: ev[ts] on one GPU; in sharded mode `ev` is the all-gathered
 // synchronization stream and its position is found by binary search on the timestamps.
 __device__ __forceinline__ uint4 event_at(const LockParams& P, u32 ts) {
+    if (ts == IGD_NONE32) return make_uint4(0, 0, 0, 0);
     if (!P.gidx) return ld_event(P.ev, ts);
     u32 lo = 0, hi = P.gn;
     while (lo < hi) {
@@ -104,6 +105,11 @@ __device__ __forceinline__ uint4 event_at(const LockParams& P, u32 ts) {
 }
 
 // One warp per traced warp.  WRITE = false: count change points; true: write them.
+// The replay is a serial chain per traced warp (one iteration per lock / fence / grid event), so
+// every load it depends on is issued ahead: each lane keeps its next two fence timestamps and its
+// next device-fence timestamp (a fence is device scope iff it heads the thread's DevF list too --
+// no event load), and the warp keeps its next two lock events' timestamps and the next lock event
+// itself (ncu r02m, sync-heavy C5: the chained event loads made this kernel 43 ms).
 template <bool WRITE>
 __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     const u32 lane = threadIdx.x & 31u;
@@ -120,10 +126,12 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
         if (!WRITE && has_thread) P.tcnt[my_t] = 0;
         return;
     }
-    u32 f_lo = 0, f_hi = 0;
+    u32 f_lo = 0, f_hi = 0, d_lo = 0, d_hi = 0;
     if (has_thread) {
         f_lo = P.off[ks.any + my_t];
         f_hi = P.off[ks.any + my_t + 1];
+        d_lo = P.off[ks.dev + my_t];
+        d_hi = P.off[ks.dev + my_t + 1];
     }
     u32 g_lo = P.off[ks.grid], g_hi = P.off[ks.grid + 1];
     u32 k_lo = P.off[ks.kb], k_hi = P.off[ks.kb + 1];
@@ -136,13 +144,16 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     u32 nt = 0;
     u32 tout = (WRITE && has_thread) ? P.toff[my_t] : 0;
 
-    u32 my_next = (f_lo < f_hi) ? __ldg(P.sts + f_lo) : IGD_NONE32;
-    u32 lk_next = __ldg(P.sts + lk_lo);
-    u32 g_next = (g_lo < g_hi) ? __ldg(P.sts + g_lo) : IGD_NONE32;
-    u32 k_next = (k_lo < k_hi) ? __ldg(P.sts + k_lo) : IGD_NONE32;
+    auto ts_at = [&](u32 pos, u32 hi) -> u32 { return pos < hi ? __ldg(P.sts + pos) : IGD_NONE32; };
+    u32 fA = ts_at(f_lo, f_hi), fB = ts_at(f_lo + 1, f_hi);  // this lane's next two fences
+    u32 dN = ts_at(d_lo, d_hi);                               // ... and next device fence
+    u32 lA = ts_at(lk_lo, lk_hi), lB = ts_at(lk_lo + 1, lk_hi);
+    uint4 eA = event_at(P, lA);                                // the next lock event
+    u32 g_next = ts_at(g_lo, g_hi);
+    u32 k_next = ts_at(k_lo, k_hi);
     while (true) {
-        const u32 f_min = __reduce_min_sync(IGD_FULL, my_next);
-        const u32 ts = min(min(f_min, k_next), min(lk_next, g_next));
+        const u32 f_min = __reduce_min_sync(IGD_FULL, fA);
+        const u32 ts = min(min(f_min, k_next), min(lA, g_next));
         if (ts == IGD_NONE32) break;
         if (ts == k_next) {
             // kernel boundary: the next kernel's locking protocol is inferred afresh (A31)
@@ -150,15 +161,20 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
             tt.clear();
             isThread = false;
             k_lo++;
-            k_next = (k_lo < k_hi) ? __ldg(P.sts + k_lo) : IGD_NONE32;
+            k_next = ts_at(k_lo, k_hi);
         } else if (ts == g_next) {
             // grid sync: every thread fences at device scope (A15)
             wt.activate(IGD_SCOPE_DEVICE);
             tt.activate(IGD_SCOPE_DEVICE);
             g_lo++;
-            g_next = (g_lo < g_hi) ? __ldg(P.sts + g_lo) : IGD_NONE32;
-        } else if (ts == lk_next) {
-            const uint4 e = event_at(P, ts);
+            g_next = ts_at(g_lo, g_hi);
+        } else if (ts == lA) {
+            const uint4 e = eA;
+            // advance the lock stream first: the next event's load overlaps this one's work
+            lk_lo++;
+            lA = lB;
+            lB = ts_at(lk_lo + 1, lk_hi);
+            if (lA != IGD_NONE32) eA = event_at(P, lA);
             const u32 kind = ev_kind(e), s = norm_scope(ev_scope(e));
             const u32 h = lock_h18(ev_addr(e) >> 2);
             const u32 el = P.g.lane(ev_tid(e));
@@ -176,16 +192,17 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
                     wt.remove(h, s);
                 }
             }
-            lk_lo++;
-            lk_next = (lk_lo < lk_hi) ? __ldg(P.sts + lk_lo) : IGD_NONE32;
         } else {
-            // a fence by the lane whose next fence is ts
-            const u32 owner = __ffs(__ballot_sync(IGD_FULL, my_next == ts)) - 1;
+            // a fence by the lane whose next fence is ts: device scope iff it also heads the lane's
+            // device-fence list (a device fence is on both lists, A12)
+            const u32 owner = __ffs(__ballot_sync(IGD_FULL, fA == ts)) - 1;
             u32 s = 0;
             if (lane == owner) {
-                s = norm_scope(ev_scope(event_at(P, ts)));
+                s = (dN == ts) ? IGD_SCOPE_DEVICE : IGD_SCOPE_BLOCK;
+                if (dN == ts) dN = ts_at(++d_lo, d_hi);
                 f_lo++;
-                my_next = (f_lo < f_hi) ? __ldg(P.sts + f_lo) : IGD_NONE32;
+                fA = fB;
+                fB = ts_at(f_lo + 1, f_hi);
             }
             s = __shfl_sync(IGD_FULL, s, owner);
             if (isThread) {
@@ -210,8 +227,20 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
 struct LockView {
     const u32* toff;  // [T+1] per-thread change-point offsets
     const u64* tpts;  // change points (ts << 16 | bloom)
+    const u32* tbits; // [ceil(T/32)] bit t: thread t ever holds a lock (has change points)
     u32 any;          // 0 when the trace has no CAS/EXCH at all
 };
+// A thread that never holds a lock has an empty Bloom at every time: R5 needs one of the two
+// threads to have change points (a 1-bit-per-thread table, L1-resident, in front of the searches)
+__device__ __forceinline__ bool may_hold(const LockView& V, u32 t) { return (__ldg(V.tbits + (t >> 5)) >> (t & 31u)) & 1u; }
+
+__global__ void k_lock_bits(const u32* __restrict__ toff, u32 T, u32* __restrict__ bits) {
+    const u32 w = blockIdx.x * blockDim.x + threadIdx.x;
+    if (w * 32 >= T) return;
+    u32 b = 0;
+    for (u32 k = 0; k < 32 && w * 32 + k < T; k++) b |= (toff[w * 32 + k + 1] > toff[w * 32 + k] ? 1u : 0u) << k;
+    bits[w] = b;
+}
 
 // Lock sets of two (thread, time) pairs at once -- R5's L(c, i) and the last accessor's -- with
 // the two binary searches interleaved (independent L2 chains).
