@@ -108,8 +108,8 @@ __device__ __forceinline__ uint4 event_at(const LockParams& P, u32 ts) {
 // The replay is a serial chain per traced warp (one iteration per lock / fence / grid event), so
 // every load it depends on is issued ahead: each lane keeps its next two fence timestamps and its
 // next device-fence timestamp (a fence is device scope iff it heads the thread's DevF list too --
-// no event load), and the warp keeps its next two lock events' timestamps and the next lock event
-// itself (ncu r02m, sync-heavy C5: the chained event loads made this kernel 43 ms).
+// no event load), and the warp holds a window of its next 32 lock events, loaded in parallel and
+// read by shuffles (sync-heavy C5: chained per-event loads made this kernel 43 ms).
 template <bool WRITE>
 __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     const u32 lane = threadIdx.x & 31u;
@@ -147,8 +147,12 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     auto ts_at = [&](u32 pos, u32 hi) -> u32 { return pos < hi ? __ldg(P.sts + pos) : IGD_NONE32; };
     u32 fA = ts_at(f_lo, f_hi), fB = ts_at(f_lo + 1, f_hi);  // this lane's next two fences
     u32 dN = ts_at(d_lo, d_hi);                               // ... and next device fence
-    u32 lA = ts_at(lk_lo, lk_hi), lB = ts_at(lk_lo + 1, lk_hi);
-    uint4 eA = event_at(P, lA);                                // the next lock event
+    // the warp's lock events come in bursts (a lock section's CAS / EXCH of every locked lane):
+    // a window of the next 32, lane i holding event lk_lo + i, loaded in parallel
+    u32 win = lk_lo;  // lock index held by lane 0
+    u32 w_ts = ts_at(win + lane, lk_hi);
+    uint4 w_ev = event_at(P, w_ts);
+    u32 lA = __shfl_sync(IGD_FULL, w_ts, 0);
     u32 g_next = ts_at(g_lo, g_hi);
     u32 k_next = ts_at(k_lo, k_hi);
     while (true) {
@@ -169,12 +173,19 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
             g_lo++;
             g_next = ts_at(g_lo, g_hi);
         } else if (ts == lA) {
-            const uint4 e = eA;
-            // advance the lock stream first: the next event's load overlaps this one's work
+            const u32 q = lk_lo - win;
+            uint4 e;
+            e.x = __shfl_sync(IGD_FULL, w_ev.x, q);
+            e.y = __shfl_sync(IGD_FULL, w_ev.y, q);
+            e.z = __shfl_sync(IGD_FULL, w_ev.z, q);
+            e.w = __shfl_sync(IGD_FULL, w_ev.w, q);
             lk_lo++;
-            lA = lB;
-            lB = ts_at(lk_lo + 1, lk_hi);
-            if (lA != IGD_NONE32) eA = event_at(P, lA);
+            if (lk_lo - win == 32u) {  // window consumed: the next 32
+                win = lk_lo;
+                w_ts = ts_at(win + lane, lk_hi);
+                w_ev = event_at(P, w_ts);
+            }
+            lA = lk_lo < lk_hi ? __shfl_sync(IGD_FULL, w_ts, lk_lo - win) : IGD_NONE32;
             const u32 kind = ev_kind(e), s = norm_scope(ev_scope(e));
             const u32 h = lock_h18(ev_addr(e) >> 2);
             const u32 el = P.g.lane(ev_tid(e));
