@@ -328,6 +328,62 @@ def run_sharded(args, fam, rank, world, local):
     dist.destroy_process_group()
 
 
+def run_stream(args, fam):
+    """--stream-chunks K: each step is one streaming session over the device-resident
+    trace cut into K equal chunks (igd_stream_begin / feed x K / end); the union of the chunks'
+    reports is compared with the injection ledger."""
+    import torch
+
+    import paper_conf_sosp_kamathb21_b200 as igd
+    import tracegen.families as F
+
+    torch.cuda.set_device(0)
+    plan = F.Plan(fam, args.events or None, **gen_kw(args))
+    n, nb, bd = plan.n_events, plan.n_blocks, plan.block_dim
+    host = np.empty(n, igd.EVENT_DTYPE)
+    plan.fill(out=host, threads=args.threads)
+    lg = plan.ledger()
+    plan.close()
+    dev = torch.from_numpy(host.view(np.uint8)).cuda()
+    K = args.stream_chunks
+    cuts = [n * k // K for k in range(K + 1)]
+    chunks = [dev[cuts[k] * 16: cuts[k + 1] * 16] for k in range(K)]
+    det = igd.Detector(0)
+
+    def session():
+        det.stream_begin(nb, bd)
+        parts = [det.stream_feed(c) for c in chunks]
+        det.stream_end()
+        return np.concatenate(parts) if parts else np.zeros(0, igd.REPORT_DTYPE)
+
+    for _ in range(args.warmup):
+        rep = session()
+    clocks = ClockSampler(0)
+    clocks.start()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(det.stream)
+    for _ in range(args.steps):
+        rep = session()
+    e1.record(det.stream)
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    ledger_match = bool(len(lg) == len(rep) and np.array_equal(lg["cur"], rep["cur"])
+                        and np.array_equal(lg["addr"], rep["addr"]) and np.array_equal(lg["prev"], rep["prev"])
+                        and np.array_equal(lg["type"].astype(np.uint8), rep["type"]))
+    line = {"metric": METRIC, "value": n / (ms / 1e3) / 1e9, "unit": "G events/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": workload_name(args, fam), "events": n, "n_blocks": nb, "block_dim": bd,
+                       "check_mode": f"streaming session, {K} chunks (igd_stream_*)", "reports": int(len(rep)),
+                       "ledger_reports": int(len(lg)), "ledger_match": ledger_match,
+                       "l2": "inputs larger than L2 (no flush)" if n * 16 > 126e6 else "inputs smaller than L2"},
+            "roofline": None, "cpu_baseline": None, "e2e": None, "gpu_launches": None, "clocks": clk}
+    print(json.dumps(line), flush=True)
+    det.close()
+
+
 # kernel class -> the kernel ncu names for it (classes made of one kernel)
 CLASS_KERNEL = {"sort_access": "rsort::k_onesweep<unsigned long, 0, unsigned int>",
                 "check": "check::k_check4<0, 0, 0, 1, unsigned int>",
@@ -376,6 +432,8 @@ def main():
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"], help="N>1 collectives")
     ap.add_argument("--paper-counters", action="store_true",
                     help="Fig. 4-width synchronization IDs (IGD_DETECT_PAPER_COUNTERS, reading A33)")
+    ap.add_argument("--stream-chunks", type=int, default=0,
+                    help="f4: time streaming sessions of this many chunks instead of igd_detect (1 GPU)")
     ap.add_argument("--sync-heavy", action="store_true",
                     help="C2 / C5 sync-heavy variant (spin-lock sections ~8 %%, fences ~5 %%; SURVEY 8(d))")
     ap.add_argument("--coalesce", action="store_true",
@@ -391,6 +449,8 @@ def main():
         return run_reference(args, fam, rank, world)
     if args.coalesce and (world > 1 or args.sharded):
         raise SystemExit("--coalesce is a single-context mode (reading A32)")
+    if args.stream_chunks:
+        return run_stream(args, fam)
     if world > 1 or args.sharded:
         return run_sharded(args, fam, rank, world, local)
 
