@@ -222,7 +222,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         // P4's lockstep clause will need this instruction's active mask when md is likely the
         // previous access, from another lane of the same warp, and the mask is partial: gather
         // it now so the trace read overlaps the scans (phase 1 re-checks the exact condition)
-        if (!MV && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) M[j] = ld_event(P.ev, V[j]).w;
+        if (!MV && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) {
+            M[j] = ld_event(P.ev, V[j]).w;
+            CSTAT(5);
+        }
     }
 
     // ---- warp aggregate in the packed state of check.cuh (state after the warp's last access) ----
@@ -385,7 +388,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 // P4 lockstep clause: md's lane in this instruction's active mask (tk bit 31: full
                 // warp; bit 30: own lane only; otherwise the mask itself, from the payload in MV
                 // mode, else gathered from the trace)
-                if (same_w && unshared && (Z[j] >> 31)) break;
+                if (same_w && unshared && (Z[j] >> 31)) {
+                    CSTAT(4);
+                    break;
+                }
                 if (same_w && unshared && !(Z[j] >> 30)) {
                     if (p == IGD_NONE32) p = tk_at(mdp) & 0xFFFFFFu;
                     // prefetched unless md is an earlier writer (M[j] is the mask then only
@@ -494,14 +500,21 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 }
             }
         } else {
-        if (p4w && q_between(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i)) continue;  // P4: syncwarp
+        if (p4w && q_between(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i)) {  // P4: syncwarp
+            CSTAT(12);
+            continue;
+        }
         const bool grid = q_grid(P, mdIdx, i);
-        if (p5b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) continue;  // P5
+        if (p5b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) {  // P5
+            CSTAT(13);
+            continue;
+        }
         type = (flags & QF_R1) ? IGD_R1 : 0u;
         // R2 (same warp, no sharing) then R3 (same block, no DevShared): md's thread has not fenced
         // (any scope) since md (A1, A30); R4 (other block): no device fence by md's thread.  One
         // query call site for both (divergent lanes would otherwise run two in turn).
         if (!type && !grid && (!same_b || !(flags & QF_DEV))) {
+            CSTAT(14);
             if (!q_between(P.desc, P.sts, (same_b ? ks.any : ks.dev) + p, mdIdx, i))
                 type = same_b ? ((same_w && !(flags & QF_BLK)) ? IGD_R2 : IGD_R3) : IGD_R4;
         }
@@ -517,6 +530,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                 laz = a.tk;
             }
             if (syncx::may_hold(P.lv, c) || syncx::may_hold(P.lv, laz & 0xFFFFFFu)) {
+                CSTAT(15);
                 u32 L, locks;
                 syncx::held_before2(P.lv, c, i, laz & 0xFFFFFFu, laIdx, L, locks);
                 if ((locks | L) != 0 && (locks & L) == 0) type = IGD_R5;

@@ -68,6 +68,13 @@ struct Table {
         for (int k = 0; k < 3; k++)
             if (le_valid(e[k]) && le_hash(e[k]) == h && le_scope(e[k]) == s) e[k] = 0;
     }
+    // an entry a fence could still activate (valid, not active)
+    __device__ __forceinline__ bool pending() const {
+        bool p = false;
+#pragma unroll
+        for (int k = 0; k < 3; k++) p |= le_valid(e[k]) && !le_active(e[k]);
+        return p;
+    }
     __device__ __forceinline__ u32 held() const {
         u32 b = 0;
 #pragma unroll
@@ -155,7 +162,40 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     u32 lA = __shfl_sync(IGD_FULL, w_ts, 0);
     u32 g_next = ts_at(g_lo, g_hi);
     u32 k_next = ts_at(k_lo, k_hi);
+    auto lower = [&](u32 lo, u32 hi, u32 v) -> u32 {  // first position in [lo, hi) with ts >= v
+        while (lo < hi) {
+            const u32 mid = (lo + hi) >> 1;
+            if (__ldg(P.sts + mid) < v) lo = mid + 1;
+            else hi = mid;
+        }
+        return lo;
+    };
+    // first position >= lo with ts >= v, given ts[lo] < v: exponential probes, then a binary search
+    // (the target is usually a few entries ahead)
+    auto gallop = [&](u32 lo, u32 hi, u32 v) -> u32 {
+        u32 prev = lo, step = 1;
+        while (true) {
+            const u32 q = prev + step;
+            if (q >= hi || __ldg(P.sts + q) >= v) return lower(prev + 1, q < hi ? q : hi, v);
+            prev = q;
+            step <<= 1;
+        }
+    };
     while (true) {
+        // A fence can only change the lock state by activating a valid, inactive entry of the
+        // fencing thread's table (the warp's until isThread).  Without one, this lane's fences up
+        // to the next lock event / grid sync / kernel boundary are no-ops: jump over them (a lock
+        // section's later fences and release fences are the bulk of a lock-heavy warp's stream).
+        const u32 next_rel = min(min(lA, g_next), k_next);
+        if (fA < next_rel && !(isThread ? tt.pending() : wt.pending())) {
+            f_lo = fB >= next_rel ? f_lo + 1 : gallop(f_lo + 1, f_hi, next_rel);
+            fA = ts_at(f_lo, f_hi);
+            fB = ts_at(f_lo + 1, f_hi);
+            if (dN < next_rel) {
+                d_lo = gallop(d_lo, d_hi, next_rel);
+                dN = ts_at(d_lo, d_hi);
+            }
+        }
         const u32 f_min = __reduce_min_sync(IGD_FULL, fA);
         const u32 ts = min(min(f_min, k_next), min(lA, g_next));
         if (ts == IGD_NONE32) break;

@@ -16,7 +16,7 @@ import paper_conf_sosp_kamathb21_b200 as igd  # noqa: E402
 import tracegen.families as F  # noqa: E402
 
 NAMES = ["checked", "P2", "P3", "P6", "P4_lockstep", "mask_gather", "queued", "q_calls", "q_fast", "q_probe_hit",
-         "q_bsearch", "reports", "prefix_waits", "md_lw_load"]
+         "q_bsearch", "reports", "ph2_P4_syncwarp", "ph2_P5", "ph2_fence_query", "ph2_R5_search"]
 fam = int(sys.argv[1][1:]) if len(sys.argv) > 1 else 4
 plan = F.Plan(fam, n=int(float(sys.argv[2])) if len(sys.argv) > 2 else None)
 ev = plan.fill()
