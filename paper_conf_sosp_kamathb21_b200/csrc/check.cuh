@@ -195,6 +195,7 @@ __device__ __forceinline__ bool q_grid(const PP& P, u32 a, u32 b) {
 #define QF_DEV 4u
 #define QF_BLK 8u
 #define QF_R1 16u
+#define QF_MASK 32u  // P4's lockstep clause still needs the active mask (read from the trace)
 
 // Sorted payload of one access: single GPU = u64 (trace index | tk << 32), the active mask is
 // gathered from the trace when needed; sharded = the record uint4 {key, index, tk, mask} (the events of

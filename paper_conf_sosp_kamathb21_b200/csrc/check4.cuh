@@ -222,10 +222,6 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         // P4's lockstep clause will need this instruction's active mask when md is likely the
         // previous access, from another lane of the same warp, and the mask is partial: gather
         // it now so the trace read overlaps the scans (phase 1 re-checks the exact condition)
-        if (!MV && !head && !dev && !blk && !same_t && !(Z[j] >> 30)) {
-            M[j] = ld_event(P.ev, V[j]).w;
-            CSTAT(5);
-        }
     }
 
     // ---- warp aggregate in the packed state of check.cuh (state after the warp's last access) ----
@@ -386,20 +382,26 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                     break;
                 }
                 // P4 lockstep clause: md's lane in this instruction's active mask (tk bit 31: full
-                // warp; bit 30: own lane only; otherwise the mask itself, from the payload in MV
-                // mode, else gathered from the trace)
+                // warp; bit 30: own lane only; otherwise the mask itself: in the payload in MV
+                // mode, else read from the trace in phase 2 -- and only when no syncwarp separates
+                // md and the access, the other half of P4: gathering it up front was a random
+                // 32-byte read for 13 % of C5's accesses, 95 % of them then decided by the
+                // syncwarp (check counters, r02p))
                 if (same_w && unshared && (Z[j] >> 31)) {
                     CSTAT(4);
                     break;
                 }
+                bool defer_mask = false;
                 if (same_w && unshared && !(Z[j] >> 30)) {
-                    if (p == IGD_NONE32) p = tk_at(mdp) & 0xFFFFFFu;
-                    // prefetched unless md is an earlier writer (M[j] is the mask then only
-                    // if the previous access was also a same-warp candidate)
-                    const bool pre = MV || (prevMd && !(Z[j] >> 30));
-                    if (((pre ? M[j] : ld_event(P.ev, V[j]).w) >> lane_of(p)) & 1u) break;
+                    if (MV) {
+                        if (p == IGD_NONE32) p = tk_at(mdp) & 0xFFFFFFu;
+                        if ((M[j] >> lane_of(p)) & 1u) break;
+                    } else {
+                        defer_mask = true;
+                    }
                 }
                 fl = (same_w ? QF_SAME_W : 0u) | (same_b ? QF_SAME_B : 0u) | (dev ? QF_DEV : 0u) |
+                     (defer_mask ? QF_MASK : 0u) |
                      (blk ? QF_BLK : 0u);
                 if (as == IGD_SCOPE_BLOCK) {  // R1 candidate: block-scope atomic, writer elsewhere
                     const bool other =
@@ -485,6 +487,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             // 2^width (Fig. 4: WarpBarID 6, BlkBarID 8, DevFenceID 6, BlkFenceID 6 bits)
             const u32 gcnt = P.glo != P.ghi ? q_count(P.desc, P.sts, ks.grid, mdIdx, i) : 0u;
             if (p4w && (q_count(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i) & 63u)) continue;  // P4
+            if (p4w && (flags & QF_MASK) && ((ld_event(P.ev, i).w >> lane_of(p)) & 1u)) continue;  // P4 lockstep
             if (p5b && ((q_count(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i) + gcnt) & 255u)) continue;  // P5
             type = (flags & QF_R1) ? IGD_R1 : 0u;
             if (!type) {
@@ -503,6 +506,10 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         if (p4w && q_between(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i)) {  // P4: syncwarp
             CSTAT(12);
             continue;
+        }
+        if (p4w && (flags & QF_MASK)) {  // P4: lockstep, the mask read only now
+            CSTAT(5);
+            if ((ld_event(P.ev, i).w >> lane_of(p)) & 1u) continue;
         }
         const bool grid = q_grid(P, mdIdx, i);
         if (p5b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) {  // P5

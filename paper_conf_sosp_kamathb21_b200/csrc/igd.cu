@@ -141,7 +141,7 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
-    Buf off, ldesc, gtab, tcnt, tpts, tbits, skipb;
+    Buf off, ldesc, gtab, tcnt, tpts, tbits, fdev, skipb;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
     u64 rep_cap = 0;
@@ -818,6 +818,15 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lp.off = P_<u32>(ctx->off);
         lp.sts = P_<u32>(ctx->syn_v[scur]);
         lp.tcnt = P_<u32>(ctx->tcnt);
+        RET(ensure(ctx, ctx->fdev, n_sync + 64));
+        {
+            KTimer kt(ctx, KC_LOCK, 0);
+            syncx::k_fence_scopes<<<(g.T + 255) / 256, 256, 0, ctx->stream>>>(P_<u32>(ctx->off),
+                                                                             P_<u32>(ctx->syn_v[scur]), ks, g.T,
+                                                                             P_<uint8_t>(ctx->fdev));
+        }
+        CK(cudaGetLastError());
+        lp.fdev = P_<uint8_t>(ctx->fdev);
         const unsigned lblocks = (unsigned)(((u64)g.W * 32 + 255) / 256);
         {
             KTimer kt(ctx, KC_LOCK, 0);
@@ -1734,7 +1743,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
                   &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->tcnt,
-                  &ctx->tpts,         &ctx->tbits,    &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
+                  &ctx->tpts,         &ctx->tbits,    &ctx->fdev,     &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
                   &ctx->sh_cnt,       &ctx->sh_obase, &ctx->sh_send,  &ctx->sh_sidx_buf, &ctx->sh_sev_buf,
                   &ctx->cl_small,     &ctx->cl_mat,   &ctx->cl_recv,  &ctx->cl_sidx,  &ctx->cl_sev,

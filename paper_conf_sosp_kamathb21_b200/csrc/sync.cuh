@@ -95,7 +95,28 @@ struct LockParams {
     u64* tpts;            // thread change points (ts << 16 | bloom)
     const u32* gidx;      // sharded mode: global timestamps of the events in `ev` (sorted), else NULL
     u32 gn;
+    const uint8_t* fdev;  // per sorted sync record of an AnyF list: 1 = a device-scope fence
 };
+
+// Scope of every fence in the AnyF lists (1 = device or system): a merge of thread t's AnyF and
+// DevF lists (a device fence is on both, A12).  Lets the lock replay read a fence's scope from a
+// byte next to its timestamp instead of the trace or a second list cursor.
+__global__ void k_fence_scopes(const u32* __restrict__ off, const u32* __restrict__ sts, KeySpace ks, u32 T,
+                               uint8_t* __restrict__ fdev) {
+    const u32 t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= T) return;
+    u32 f = off[ks.any + t];
+    const u32 f_hi = off[ks.any + t + 1];
+    u32 d = off[ks.dev + t];
+    const u32 d_hi = off[ks.dev + t + 1];
+    u32 dts = d < d_hi ? sts[d] : IGD_NONE32;
+    for (; f < f_hi; f++) {
+        const u32 ts = sts[f];
+        const bool dev = dts == ts;
+        fdev[f] = dev ? 1 : 0;
+        if (dev) dts = ++d < d_hi ? sts[d] : IGD_NONE32;
+    }
+}
 
 // The event with timestamp ts: ev[ts] on one GPU; in sharded mode `ev` is the all-gathered
 // synchronization stream and its position is found by binary search on the timestamps.
@@ -113,10 +134,10 @@ __device__ __forceinline__ uint4 event_at(const LockParams& P, u32 ts) {
 
 // One warp per traced warp.  WRITE = false: count change points; true: write them.
 // The replay is a serial chain per traced warp (one iteration per lock / fence / grid event), so
-// every load it depends on is issued ahead: each lane keeps its next two fence timestamps and its
-// next device-fence timestamp (a fence is device scope iff it heads the thread's DevF list too --
-// no event load), and the warp holds a window of its next 32 lock events, loaded in parallel and
-// read by shuffles (sync-heavy C5: chained per-event loads made this kernel 43 ms).
+// every load it depends on is issued ahead: each lane keeps its next two fence timestamps with
+// their scopes (k_fence_scopes: no event load), and the warp holds a window of its next 32 lock
+// events, loaded in parallel and read by shuffles; fences that cannot activate anything are
+// skipped (sync-heavy C5: chained per-event loads and no-op fences made this kernel 43 ms).
 template <bool WRITE>
 __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     const u32 lane = threadIdx.x & 31u;
@@ -133,12 +154,10 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
         if (!WRITE && has_thread) P.tcnt[my_t] = 0;
         return;
     }
-    u32 f_lo = 0, f_hi = 0, d_lo = 0, d_hi = 0;
+    u32 f_lo = 0, f_hi = 0;
     if (has_thread) {
         f_lo = P.off[ks.any + my_t];
         f_hi = P.off[ks.any + my_t + 1];
-        d_lo = P.off[ks.dev + my_t];
-        d_hi = P.off[ks.dev + my_t + 1];
     }
     u32 g_lo = P.off[ks.grid], g_hi = P.off[ks.grid + 1];
     u32 k_lo = P.off[ks.kb], k_hi = P.off[ks.kb + 1];
@@ -152,8 +171,9 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
     u32 tout = (WRITE && has_thread) ? P.toff[my_t] : 0;
 
     auto ts_at = [&](u32 pos, u32 hi) -> u32 { return pos < hi ? __ldg(P.sts + pos) : IGD_NONE32; };
+    auto dev_at = [&](u32 pos, u32 hi) -> u32 { return pos < hi ? P.fdev[pos] : 0u; };
     u32 fA = ts_at(f_lo, f_hi), fB = ts_at(f_lo + 1, f_hi);  // this lane's next two fences
-    u32 dN = ts_at(d_lo, d_hi);                               // ... and next device fence
+    u32 sA = dev_at(f_lo, f_hi), sB = dev_at(f_lo + 1, f_hi);  // ... and their scopes (1 = device)
     // the warp's lock events come in bursts (a lock section's CAS / EXCH of every locked lane):
     // a window of the next 32, lane i holding event lk_lo + i, loaded in parallel
     u32 win = lk_lo;  // lock index held by lane 0
@@ -188,13 +208,17 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
         // section's later fences and release fences are the bulk of a lock-heavy warp's stream).
         const u32 next_rel = min(min(lA, g_next), k_next);
         if (fA < next_rel && !(isThread ? tt.pending() : wt.pending())) {
-            f_lo = fB >= next_rel ? f_lo + 1 : gallop(f_lo + 1, f_hi, next_rel);
-            fA = ts_at(f_lo, f_hi);
-            fB = ts_at(f_lo + 1, f_hi);
-            if (dN < next_rel) {
-                d_lo = gallop(d_lo, d_hi, next_rel);
-                dN = ts_at(d_lo, d_hi);
+            if (fB >= next_rel) {  // one fence to skip: the next one is in registers already
+                f_lo++;
+                fA = fB;
+                sA = sB;
+            } else {
+                f_lo = gallop(f_lo + 1, f_hi, next_rel);
+                fA = ts_at(f_lo, f_hi);
+                sA = dev_at(f_lo, f_hi);
             }
+            fB = ts_at(f_lo + 1, f_hi);
+            sB = dev_at(f_lo + 1, f_hi);
         }
         const u32 f_min = __reduce_min_sync(IGD_FULL, fA);
         const u32 ts = min(min(f_min, k_next), min(lA, g_next));
@@ -244,16 +268,16 @@ __global__ void __launch_bounds__(256) k_lock_infer(LockParams P) {
                 }
             }
         } else {
-            // a fence by the lane whose next fence is ts: device scope iff it also heads the lane's
-            // device-fence list (a device fence is on both lists, A12)
+            // a fence by the lane whose next fence is ts (its scope from the fdev byte)
             const u32 owner = __ffs(__ballot_sync(IGD_FULL, fA == ts)) - 1;
             u32 s = 0;
             if (lane == owner) {
-                s = (dN == ts) ? IGD_SCOPE_DEVICE : IGD_SCOPE_BLOCK;
-                if (dN == ts) dN = ts_at(++d_lo, d_hi);
+                s = sA ? IGD_SCOPE_DEVICE : IGD_SCOPE_BLOCK;
                 f_lo++;
                 fA = fB;
+                sA = sB;
                 fB = ts_at(f_lo + 1, f_hi);
+                sB = dev_at(f_lo + 1, f_hi);
             }
             s = __shfl_sync(IGD_FULL, s, owner);
             if (isThread) {
