@@ -455,7 +455,8 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_count_fused(Params
                 atomicAdd(&s_hacc[warp & 3u][key & 255u], 1u);
             }
             // digits 1..3: one set of atomics per distinct upper-24-bit value among the lanes
-            const u32 am = __ballot_sync(IGD_FULL, acc);
+            // (IGD_HIST_UP_LATE: histogrammed over the fused pass's keys instead)
+            const u32 am = IGD_HIST_UP_LATE ? 0u : __ballot_sync(IGD_FULL, acc);
             if (am) {
                 const u32 hi = key >> 8;
                 const u32 peers = __match_any_sync(IGD_FULL, acc ? hi : (0x1000000u | lane)) & am;

@@ -318,10 +318,28 @@ __global__ void k_lock_bits(const u32* __restrict__ toff, u32 T, u32* __restrict
 }
 
 // Lock sets of two (thread, time) pairs at once -- R5's L(c, i) and the last accessor's -- with
-// the two binary searches interleaved (independent L2 chains).
+// the two searches interleaved (independent L2 chains).  Short lists (<= 4 change points, most
+// threads) are scanned from independent loads instead of a dependent binary search.
+__device__ __forceinline__ u32 held_short(const u64* __restrict__ tpts, u32 lo, u32 hi, u32 i) {
+    u32 L = 0;
+#pragma unroll
+    for (u32 k = 0; k < 4; k++) {
+        if (lo + k < hi) {
+            const u64 v = __ldg(tpts + lo + k);
+            if ((u32)(v >> 16) < i) L = (u32)(v & 0xFFFFu);
+        }
+    }
+    return L;
+}
 __device__ __forceinline__ void held_before2(const LockView& V, u32 c0, u32 i0, u32 c1, u32 i1, u32& L0, u32& L1) {
     u32 lo0 = __ldg(V.toff + c0), hi0 = __ldg(V.toff + c0 + 1);
     u32 lo1 = __ldg(V.toff + c1), hi1 = __ldg(V.toff + c1 + 1);
+    const bool s0 = hi0 - lo0 <= 4u, s1 = hi1 - lo1 <= 4u;
+    if (s0 && s1) {
+        L0 = held_short(V.tpts, lo0, hi0, i0);
+        L1 = held_short(V.tpts, lo1, hi1, i1);
+        return;
+    }
     const u32 b0 = lo0, b1 = lo1;
     while (lo0 < hi0 || lo1 < hi1) {
         const u32 m0 = (lo0 + hi0) >> 1, m1 = (lo1 + hi1) >> 1;
