@@ -61,7 +61,15 @@ __device__ unsigned long long g_chk_stats[16];
     } while (0)
 
 // Is there an element x of entity e's list with a < x < b ?
-__device__ __noinline__ bool q_between(const uint4* __restrict__ desc, const u32* __restrict__ ts, u32 e, u32 a,
+#ifndef IGD_QB_INLINE
+#define IGD_QB_INLINE 0
+#endif
+#if IGD_QB_INLINE
+#define IGD_QB_ATTR __forceinline__
+#else
+#define IGD_QB_ATTR __noinline__
+#endif
+__device__ IGD_QB_ATTR bool q_between(const uint4* __restrict__ desc, const u32* __restrict__ ts, u32 e, u32 a,
                                        u32 b) {
     const uint4 d = __ldg(desc + e);
     CSTAT(7);
