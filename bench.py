@@ -318,6 +318,8 @@ def run_sharded(args, fam, rank, world, local):
                 "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                              "frac": achieved / peak, "peak_source": peak_kind, "traffic": None,
                              "launches_per_step": c / args.steps, "rank": 0},
+                "path": {"kernels": {k: {"launches": v[0] // args.steps, "ms": v[1] / args.steps}
+                                     for k, v in kstats.items() if v[0]}},
                 "cpu_baseline": None,
                 "e2e": {"value": n / e2e_s / 1e9 if e2e_times else None, "unit": "G events/s",
                         "h2d_bytes_per_step": n * 16, "d2h_bytes_per_step": int(len(out)) * 32 * world,

@@ -462,6 +462,11 @@ static int canon_reports(igd_ctx* ctx, const igd_report* in, u64 n, u64 n_time) 
     RET(ensure(ctx, ctx->rep_out, (n ? n : 1) * sizeof(igd_report)));
     if (n == 1 && in != P_<igd_report>(ctx->rep_out)) {
         CK(cudaMemcpyAsync(ctx->rep_out.p, in, sizeof(igd_report), cudaMemcpyDeviceToDevice, ctx->stream));
+    } else if (n > 1 && n <= (u64)check::SMALL_REP && n_time <= 0xFFFFFFFFull) {
+        // small sets (the latency-bound configs): one CTA, no host round trip
+        KTimer kt(ctx, KC_REPORT, 64.0 * (double)n);
+        check::k_report_sort_small<<<1, 1024, 0, ctx->stream>>>(in, (u32)n, P_<igd_report>(ctx->rep_out));
+        CK(cudaGetLastError());
     } else if (n > 1) {
         const int sms = sm_count(ctx);
         for (int b = 0; b < 2; b++) {
