@@ -129,7 +129,11 @@ typedef struct igd_ctx igd_ctx; /* opaque; owns every device buffer it allocates
    shared by the caller, e.g. a torch.distributed broadcast).  The call initialises an NCCL
    communicator (ncclCommInitRank: blocks until every rank joins) and makes igd_detect collective.
    nranks == 1 with a non-NULL id gives a one-rank communicator (the collective path on one GPU);
-   nranks == 1 with NULL is the single-GPU pipeline.  IGD_EINVAL: rank out of range, nranks > 1
+   nranks == 1 with NULL is the single-GPU pipeline.  An id whose first 8 bytes are "IGDLOOP:"
+   (followed by a NUL-terminated group name) selects the in-process loopback transport instead of
+   NCCL: the nranks contexts of one process, driven by one host thread each, exchange through
+   device copies with the same collectives (the test transport of one-GPU boxes, where NCCL
+   refuses two ranks on one device).  IGD_EINVAL: rank out of range, nranks > 1
    without an id, one of alloc_fn / free_fn NULL; IGD_ENCCL: libnccl unavailable or the
    communicator could not be created. */
 int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks, int rank,

@@ -27,6 +27,9 @@
 #include <nvtx3/nvToolsExt.h>
 #include <nccl.h>  // types and prototypes only: the library is resolved at run time (NcclApi)
 #include <algorithm>
+#include <condition_variable>
+#include <map>
+#include <mutex>
 #include <vector>
 
 #ifndef IGD_PASS0_GENERIC
@@ -34,6 +37,7 @@
 #endif
 
 namespace {
+struct LoopGroup;  // in-process loopback transport (defined with the collectives)
 
 enum KClass { KC_INGEST = 0, KC_SORT_SYNC, KC_CSR, KC_LOCK, KC_SORT_ACC, KC_CHECK, KC_REPORT, KC_MISC, KC_FUSED };
 
@@ -114,6 +118,7 @@ struct igd_ctx {
     // multi-GPU: an NCCL communicator makes igd_detect collective
     int nranks = 1, rank = 0;
     ncclComm_t comm = nullptr;
+    LoopGroup* loop = nullptr;  // in-process loopback transport (tests), instead of comm
     Buf cl_small, cl_mat, cl_recv, cl_sidx, cl_sev, cl_nrep, cl_rep;
     // per-kernel geometry (reading A34): the trace runs as segments between grid-changing
     // kernel boundaries, each on its own grid
@@ -1251,6 +1256,143 @@ static int stream_feed_impl(igd_ctx* ctx, const igd_event* events, u64 n, u32 ev
     return IGD_OK;
 }
 
+// ---------------- the collective transport ----------------
+// Four collectives carry the multi-GPU check.  With an NCCL communicator they are NCCL calls on
+// the context stream.  An id starting with "IGDLOOP:" instead selects the in-process loopback
+// transport: the P contexts of one process (driven by P host threads) meet at a barrier and copy
+// from each other's device buffers -- the same exchange pattern, testable on a one-GPU box, where
+// NCCL refuses two ranks on one device.
+namespace {
+struct LoopGroup {
+    int P = 0, refs = 0;
+    std::mutex m;
+    std::condition_variable cv;
+    int arrived = 0;
+    u64 gen = 0;
+    std::vector<const char*> base;      // per rank: the posted send buffer
+    std::vector<std::vector<u64>> off, len;  // per rank: per peer offset / bytes in that buffer
+    std::vector<u64> red;               // per rank x 8: all-reduce contributions
+};
+std::mutex g_loop_m;
+std::map<std::string, LoopGroup*> g_loops;
+
+LoopGroup* loop_join(const std::string& name, int P) {
+    std::lock_guard<std::mutex> lk(g_loop_m);
+    LoopGroup*& g = g_loops[name];
+    if (!g) {
+        g = new LoopGroup();
+        g->P = P;
+        g->base.assign(P, nullptr);
+        g->off.assign(P, std::vector<u64>(P, 0));
+        g->len.assign(P, std::vector<u64>(P, 0));
+        g->red.assign((size_t)P * 8, 0);
+    }
+    if (g->P != P) return nullptr;
+    g->refs++;
+    return g;
+}
+void loop_leave(LoopGroup* g) {
+    std::lock_guard<std::mutex> lk(g_loop_m);
+    if (--g->refs == 0) {
+        for (auto it = g_loops.begin(); it != g_loops.end(); ++it)
+            if (it->second == g) {
+                g_loops.erase(it);
+                break;
+            }
+        delete g;
+    }
+}
+void loop_barrier(LoopGroup* g) {
+    std::unique_lock<std::mutex> lk(g->m);
+    const u64 my = g->gen;
+    if (++g->arrived == g->P) {
+        g->arrived = 0;
+        g->gen++;
+        g->cv.notify_all();
+    } else {
+        g->cv.wait(lk, [&] { return g->gen != my; });
+    }
+}
+}  // namespace
+
+// min-all-reduce of n <= 8 u64 values in device memory (in place)
+static int coll_allreduce_min(igd_ctx* ctx, u64* dbuf, int n) {
+    if (ctx->comm) {
+        NK(nccl().AllReduce(dbuf, dbuf, n, ncclUint64, ncclMin, ctx->comm, ctx->stream));
+        return IGD_OK;
+    }
+    LoopGroup* g = ctx->loop;
+    u64 v[8];
+    CK(cudaMemcpyAsync(v, dbuf, n * sizeof(u64), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    for (int k = 0; k < n; k++) g->red[(size_t)ctx->rank * 8 + k] = v[k];
+    loop_barrier(g);
+    for (int k = 0; k < n; k++) {
+        u64 m = ~0ull;
+        for (int r = 0; r < g->P; r++) m = std::min(m, g->red[(size_t)r * 8 + k]);
+        v[k] = m;
+    }
+    loop_barrier(g);  // every rank has read the contributions
+    CK(cudaMemcpyAsync(dbuf, v, n * sizeof(u64), cudaMemcpyHostToDevice, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return IGD_OK;
+}
+
+// all-to-all(v): send[q] = bytes [soff[q], soff[q] + slen[q]) of sbase for rank q; the bytes from
+// rank q land at rbase + roff[q] (rlen[q] of them).  Every buffer is device memory.
+static int coll_alltoallv(igd_ctx* ctx, const void* sbase, const u64* soff, const u64* slen, void* rbase,
+                          const u64* roff, const u64* rlen) {
+    const int P = ctx->nranks, me = ctx->rank;
+    if (ctx->comm) {
+        NcclApi& N = nccl();
+        NK(N.GroupStart());
+        for (int q = 0; q < P; q++) {
+            if (slen[q]) NK(N.Send((const char*)sbase + soff[q], slen[q], ncclUint8, q, ctx->comm, ctx->stream));
+            if (rlen[q]) NK(N.Recv((char*)rbase + roff[q], rlen[q], ncclUint8, q, ctx->comm, ctx->stream));
+        }
+        NK(N.GroupEnd());
+        return IGD_OK;
+    }
+    LoopGroup* g = ctx->loop;
+    CK(cudaStreamSynchronize(ctx->stream));  // the send buffer is complete
+    g->base[me] = (const char*)sbase;
+    for (int q = 0; q < P; q++) {
+        g->off[me][q] = soff[q];
+        g->len[me][q] = slen[q];
+    }
+    loop_barrier(g);
+    int rc = IGD_OK;
+    for (int q = 0; q < P && rc == IGD_OK; q++) {
+        if (g->len[q][me] != rlen[q]) rc = IGD_ECUDA;  // counts disagree: a transport bug
+        else if (rlen[q] && cudaMemcpyAsync((char*)rbase + roff[q], g->base[q] + g->off[q][me], rlen[q],
+                                            cudaMemcpyDefault, ctx->stream) != cudaSuccess)
+            rc = IGD_ECUDA;
+    }
+    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) rc = IGD_ECUDA;
+    loop_barrier(g);  // every rank has copied out of the posted buffers
+    if (rc != IGD_OK) ctx->err = "loopback all-to-all failed";
+    return rc;
+}
+
+// all-gather(v): rank q's slen bytes at sbase land at rbase + roff[q] on every rank (rlen[q] each)
+static int coll_allgatherv(igd_ctx* ctx, const void* sbase, u64 slen, void* rbase, const u64* roff,
+                           const u64* rlen) {
+    const int P = ctx->nranks, me = ctx->rank;
+    if (ctx->comm) {
+        NcclApi& N = nccl();
+        NK(N.GroupStart());
+        for (int q = 0; q < P; q++) {
+            if (!rlen[q]) continue;
+            char* d = (char*)rbase + roff[q];
+            NK(N.Broadcast(q == me ? sbase : d, d, rlen[q], ncclUint8, q, ctx->comm, ctx->stream));
+        }
+        NK(N.GroupEnd());
+        return IGD_OK;
+    }
+    std::vector<u64> so(P, 0), sl(P, slen), ro(roff, roff + P), rl(rlen, rlen + P);
+    return coll_alltoallv(ctx, sbase, so.data(), sl.data(), rbase, ro.data(), rl.data());
+}
+
 // ---------------- multi-GPU collective check ----------------
 // Every rank holds the contiguous global range [first_event, first_event + n_events) of one trace.
 // 1. partition the chunk: access records grouped by owner rank fmix32(word) % P, and the
@@ -1266,9 +1408,7 @@ static int stream_feed_impl(igd_ctx* ctx, const igd_event* events, u64 n, u32 ev
 // Every rank returns the same global report set.  Errors found by any rank (bad event, word span,
 // a local allocation failure) are agreed through step 2, so no rank is left inside a collective.
 static int collective_detect(igd_ctx* ctx, u64* n_out) {
-    NcclApi& N = nccl();
     const u32 P = (u32)ctx->nranks, me = (u32)ctx->rank;
-    const ncclComm_t comm = ctx->comm;
     cudaStream_t st = ctx->stream;
     *n_out = 0;
     ctx->n_reports = 0;
@@ -1280,7 +1420,7 @@ static int collective_detect(igd_ctx* ctx, u64* n_out) {
     int lrc = shard_prepare_impl(ctx, P, counts.data(), &nsync, &bad, mm);
     u64 small[4] = {bad, mm[0], mm[0] == ~0ull ? ~0ull : ~mm[1], lrc == IGD_OK ? ~0ull : (u64)(-lrc)};
     CK(cudaMemcpyAsync(ctx->cl_small.p, small, sizeof(small), cudaMemcpyHostToDevice, st));
-    NK(N.AllReduce(ctx->cl_small.p, ctx->cl_small.p, 4, ncclUint64, ncclMin, comm, st));
+    RET(coll_allreduce_min(ctx, P_<u64>(ctx->cl_small), 4));
     CK(cudaMemcpyAsync(small, ctx->cl_small.p, sizeof(small), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (small[3] != ~0ull) {
@@ -1303,7 +1443,11 @@ static int collective_detect(igd_ctx* ctx, u64* n_out) {
     RET(ensure(ctx, ctx->cl_mat, (W * P + W) * sizeof(u64)));
     counts[P] = nsync;
     CK(cudaMemcpyAsync(P_<u64>(ctx->cl_mat) + W * P, counts.data(), W * sizeof(u64), cudaMemcpyHostToDevice, st));
-    NK(N.AllGather(P_<u64>(ctx->cl_mat) + W * P, ctx->cl_mat.p, W, ncclUint64, comm, st));
+    {
+        std::vector<u64> ro(P), rl(P, W * sizeof(u64));
+        for (u32 r = 0; r < P; r++) ro[r] = (u64)r * W * sizeof(u64);
+        RET(coll_allgatherv(ctx, P_<u64>(ctx->cl_mat) + W * P, W * sizeof(u64), ctx->cl_mat.p, ro.data(), rl.data()));
+    }
     std::vector<u64> M(W * P);
     CK(cudaMemcpyAsync(M.data(), ctx->cl_mat.p, W * P * sizeof(u64), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -1319,25 +1463,25 @@ static int collective_detect(igd_ctx* ctx, u64* n_out) {
     RET(ensure(ctx, ctx->cl_sidx, (nsy + 1) * sizeof(u32)));
     RET(ensure(ctx, ctx->cl_sev, (nsy + 1) * 16));
     {
-        // all-to-all of the access records (one grouped send / receive per peer, self included)
-        NK(N.GroupStart());
+        // all-to-all of the access records (received groups in source-rank order = trace order)
+        std::vector<u64> so(P), sl(P), rof(P), rl(P);
         for (u32 r = 0; r < P; r++) {
-            const u64 ns = M[me * W + r], nr = M[r * W + me];
-            if (ns) NK(N.Send((const char*)ctx->sh_send.p + soff[r] * 16, ns * 16, ncclUint8, (int)r, comm, st));
-            if (nr) NK(N.Recv((char*)ctx->cl_recv.p + roff[r] * 16, nr * 16, ncclUint8, (int)r, comm, st));
+            so[r] = soff[r] * 16;
+            sl[r] = M[me * W + r] * 16;
+            rof[r] = roff[r] * 16;
+            rl[r] = M[r * W + me] * 16;
         }
-        NK(N.GroupEnd());
+        RET(coll_alltoallv(ctx, ctx->sh_send.p, so.data(), sl.data(), ctx->cl_recv.p, rof.data(), rl.data()));
         // the synchronization streams, concatenated in rank order (a variable all-gather)
-        NK(N.GroupStart());
+        std::vector<u64> io(P), il(P), eo(P), el(P);
         for (u32 r = 0; r < P; r++) {
-            const u64 c = M[r * W + P];
-            if (!c) continue;
-            u32* di = P_<u32>(ctx->cl_sidx) + yoff[r];
-            char* de = (char*)ctx->cl_sev.p + yoff[r] * 16;
-            NK(N.Broadcast(r == me ? ctx->sh_sidx_buf.p : di, di, c, ncclUint32, (int)r, comm, st));
-            NK(N.Broadcast(r == me ? ctx->sh_sev_buf.p : de, de, c * 16, ncclUint8, (int)r, comm, st));
+            io[r] = yoff[r] * sizeof(u32);
+            il[r] = M[r * W + P] * sizeof(u32);
+            eo[r] = yoff[r] * 16;
+            el[r] = M[r * W + P] * 16;
         }
-        NK(N.GroupEnd());
+        RET(coll_allgatherv(ctx, ctx->sh_sidx_buf.p, nsync * sizeof(u32), ctx->cl_sidx.p, io.data(), il.data()));
+        RET(coll_allgatherv(ctx, ctx->sh_sev_buf.p, nsync * 16, ctx->cl_sev.p, eo.data(), el.data()));
     }
     RET(buf_free(ctx, ctx->sh_send));  // stream-ordered: after the sends
     // the words this rank owns
@@ -1356,7 +1500,12 @@ static int collective_detect(igd_ctx* ctx, u64* n_out) {
     RET(ensure(ctx, ctx->cl_nrep, 2 * P * sizeof(u64)));
     u64 mine[2] = {lrc == IGD_OK ? nloc : 0, lrc == IGD_OK ? 0 : (u64)(-lrc)};
     CK(cudaMemcpyAsync(P_<u64>(ctx->cl_nrep) + 2 * me, mine, sizeof(mine), cudaMemcpyHostToDevice, st));
-    NK(N.AllGather(P_<u64>(ctx->cl_nrep) + 2 * me, ctx->cl_nrep.p, 2, ncclUint64, comm, st));
+    {
+        std::vector<u64> ro(P), rl(P, 2 * sizeof(u64));
+        for (u32 r = 0; r < P; r++) ro[r] = (u64)r * 2 * sizeof(u64);
+        RET(coll_allgatherv(ctx, P_<u64>(ctx->cl_nrep) + 2 * me, 2 * sizeof(u64), ctx->cl_nrep.p, ro.data(),
+                            rl.data()));
+    }
     std::vector<u64> NR(2 * P);
     CK(cudaMemcpyAsync(NR.data(), ctx->cl_nrep.p, 2 * P * sizeof(u64), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -1365,20 +1514,17 @@ static int collective_detect(igd_ctx* ctx, u64* n_out) {
             if (lrc == IGD_OK) ctx->err = "rank " + std::to_string(r) + " failed in the check stage";
             return -(int)NR[2 * r + 1];
         }
-    u64 total = 0;
     std::vector<u64> off(P + 1, 0);
     for (u32 r = 0; r < P; r++) off[r + 1] = off[r] + NR[2 * r];
-    total = off[P];
+    const u64 total = off[P];
     if (P > 1) {
         RET(ensure(ctx, ctx->cl_rep, (total ? total : 1) * sizeof(igd_report)));
-        NK(N.GroupStart());
+        std::vector<u64> ro(P), rl(P);
         for (u32 r = 0; r < P; r++) {
-            const u64 c = NR[2 * r];
-            if (!c) continue;
-            char* d = (char*)ctx->cl_rep.p + off[r] * sizeof(igd_report);
-            NK(N.Broadcast(r == me ? ctx->rep_out.p : d, d, c * sizeof(igd_report), ncclUint8, (int)r, comm, st));
+            ro[r] = off[r] * sizeof(igd_report);
+            rl[r] = NR[2 * r] * sizeof(igd_report);
         }
-        NK(N.GroupEnd());
+        RET(coll_allgatherv(ctx, ctx->rep_out.p, nloc * sizeof(igd_report), ctx->cl_rep.p, ro.data(), rl.data()));
         RET(canon_reports(ctx, P_<igd_report>(ctx->cl_rep), total, ctx->sh_ntotal));
     }
     CK(cudaStreamSynchronize(st));
@@ -1440,7 +1586,17 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     }
     ctx->nranks = nranks;
     ctx->rank = rank;
-    if (nccl_unique_id) {
+    if (nccl_unique_id && memcmp(nccl_unique_id, "IGDLOOP:", 8) == 0) {
+        // in-process loopback transport (tests): ranks of one process meet by the id's name
+        char name[121];
+        memcpy(name, nccl_unique_id + 8, 120);
+        name[120] = 0;
+        ctx->loop = loop_join(name, nranks);
+        if (!ctx->loop) {
+            igd_ctx_destroy(ctx);
+            return IGD_EINVAL;
+        }
+    } else if (nccl_unique_id) {
         // a communicator (also for nranks == 1: the collective path on one GPU); blocks until
         // every rank has joined
         NcclApi& N = nccl();
@@ -1509,7 +1665,7 @@ int igd_detect(igd_ctx* ctx, uint32_t flags, uint64_t* n_reports_global) {
         ctx->err = "IGD_DETECT_LAST_K must be 1, 2, 4 or 8";
         return IGD_EINVAL;
     }
-    if (ctx->comm) {  // collective over the communicator's ranks
+    if (ctx->comm || ctx->loop) {  // collective over the communicator's ranks
         if (flags & IGD_DETECT_COALESCE) {  // reading A32: a group may straddle two ranks' chunks
             ctx->err = "IGD_DETECT_COALESCE is a single-context mode";
             return IGD_EINVAL;
@@ -1683,7 +1839,7 @@ int igd_kernel_stats(const igd_ctx* ctx, int kclass, const char** name, uint32_t
 
 int igd_stream_begin(igd_ctx* ctx, uint32_t n_blocks, uint32_t block_dim) {
     if (!ctx || n_blocks == 0 || block_dim == 0 || (u64)n_blocks * block_dim > (1ull << 24)) return IGD_EINVAL;
-    if (ctx->comm) {
+    if (ctx->comm || ctx->loop) {
         ctx->err = "streaming sessions are single-context";
         return IGD_EINVAL;
     }
@@ -1743,6 +1899,10 @@ void igd_ctx_destroy(igd_ctx* ctx) {
     if (ctx->comm) {
         nccl().CommDestroy(ctx->comm);
         ctx->comm = nullptr;
+    }
+    if (ctx->loop) {
+        loop_leave(ctx->loop);
+        ctx->loop = nullptr;
     }
     Buf* all[] = {&ctx->owned_events, &ctx->acc_k[0], &ctx->acc_k[1], &ctx->acc_v[0], &ctx->acc_v[1],
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,

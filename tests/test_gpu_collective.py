@@ -82,3 +82,83 @@ def test_collective_rejects_coalesce(cdet):
     with pytest.raises(igd.IgdError) as e:
         cdet.detect(coalesce=True)
     assert e.value.code == igd.igd.IGD_EINVAL
+
+
+# ---- P > 1 ranks through the collective C ABI on one GPU: the in-process loopback transport ----
+# ("IGDLOOP:<name>" ids; P contexts driven by P host threads exchange through device copies with
+# the same count matrix, all-to-all and all-gathers as the NCCL transport)
+def _loop_id(name):
+    return (b"IGDLOOP:" + name.encode()).ljust(128, b"\0")
+
+
+def run_ranks(ev, nb, bd, P, name, **kw):
+    import threading
+
+    import torch
+
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    n = len(ev)
+    out, errs = [None] * P, [None] * P
+
+    def rank(r):
+        try:
+            torch.cuda.set_device(0)
+            d = igd.Detector(0, stream=torch.cuda.Stream(0), nranks=P, rank=r, nccl_id=_loop_id(name))
+            lo, hi = n * r // P, n * (r + 1) // P
+            d.load(ev[lo:hi], nb, bd, first_event=lo, n_events_total=n)
+            d.detect(**kw)
+            out[r] = d.reports()
+            d.close()
+        except Exception as e:  # noqa: BLE001 -- reported by the caller
+            errs[r] = e
+
+    ts = [threading.Thread(target=rank, args=(r,)) for r in range(P)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(timeout=600)
+    return out, errs
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+def test_collective_loopback_ranks_vs_oracle(P):
+    w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    ev, nb, bd = _fast_random(40 + P, 150_000, 2_000, 6, 128, w)
+    want = oracle.run(ev, nb, bd)
+    out, errs = run_ranks(ev, nb, bd, P, f"ranks{P}")
+    assert errs == [None] * P
+    assert len(want) > 0
+    for r in range(P):
+        assert np.array_equal(out[r], want), f"rank {r}"
+
+
+def test_collective_loopback_lock_heavy_and_families():
+    import tracegen.families as F
+
+    w = [12, 10, 6, 10, 8, 12, 2, 2, 1, 1, 1, 1]
+    ev, nb, bd = _fast_random(50, 100_000, 300, 4, 64, w, lock_words=40)
+    out, errs = run_ranks(ev, nb, bd, 4, "locks4")
+    assert errs == [None] * 4 and all(np.array_equal(o, oracle.run(ev, nb, bd)) for o in out)
+    ev, nb, bd, led = F.generate(2)
+    out, errs = run_ranks(ev, nb, bd, 3, "c2x3")
+    assert errs == [None] * 3
+    assert [(r["addr"], r["cur"], r["prev"], r["type"]) for r in out[2]] == \
+           [(r["addr"], r["cur"], r["prev"], r["type"]) for r in led]
+
+
+def test_collective_loopback_paper_counters_and_sticky():
+    w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
+    ev, nb, bd = _fast_random(51, 80_000, 500, 3, 96, w)
+    for kw, nm in ((dict(paper_counters=True), "pc"), (dict(sticky_flags=True), "st")):
+        out, errs = run_ranks(ev, nb, bd, 2, nm, **kw)
+        assert errs == [None, None] and all(np.array_equal(o, oracle.run(ev, nb, bd, **kw)) for o in out)
+
+
+def test_collective_loopback_bad_event_agreed():
+    import paper_conf_sosp_kamathb21_b200 as igd
+
+    ev, nb, bd = _fast_random(52, 60_000, 100, 2, 64, [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1])
+    ev["tk"][45_001] = tg.pack_tk(0, 13, 0)   # on rank 2 of 3
+    out, errs = run_ranks(ev, nb, bd, 3, "bad3")
+    assert all(isinstance(e, igd.IgdError) and e.code == igd.igd.IGD_ETRACE and e.bad_index == 45_001 for e in errs)
