@@ -143,9 +143,25 @@ struct Params {
     u64 first_event; // global index offset (multi-rank)
     u32 addr_from_ev;  // tag-aliasing mode (A36): keys hold entry + tag, report addresses come from the trace
     u64* st_out;       // last-k mode (A37): per-access scan state out, no checks here (NULL otherwise)
+    const uint4* rec;  // sharded mode: the received records, ascending by index (active-mask lookups)
+    u32 nrec;
     u32 carry_before;  // streaming mode (f4): records with index < carry_before are carried state
     void* carry_out;   // streaming mode: 2 uint4 per access (carried pair at each word's last access)
 };
+
+// The active mask of the access with trace index i: from the trace on one GPU, else from the
+// received records of a sharded check (ascending by index: a binary search -- the mask is read
+// only when no syncwarp decides P4, rarely)
+__device__ __forceinline__ u32 mask_of(const Params& P, u32 i) {
+    if (!P.rec) return ld_event(P.ev, i).w;
+    u32 lo = 0, hi = P.nrec;
+    while (lo < hi) {
+        const u32 mid = (lo + hi) >> 1;
+        if (__ldg(&P.rec[mid].y) < i) lo = mid + 1;
+        else hi = mid;
+    }
+    return __ldg(&P.rec[lo].w);
+}
 
 // Streaming mode: keep the carried pairs written at each word's last access (compaction by
 // flag, exclusive scan, scatter; the survivors stay in key order)

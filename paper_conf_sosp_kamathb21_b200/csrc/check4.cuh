@@ -487,7 +487,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             // 2^width (Fig. 4: WarpBarID 6, BlkBarID 8, DevFenceID 6, BlkFenceID 6 bits)
             const u32 gcnt = P.glo != P.ghi ? q_count(P.desc, P.sts, ks.grid, mdIdx, i) : 0u;
             if (p4w && (q_count(P.desc, P.sts, ks.wb + warp_of(c), mdIdx, i) & 63u)) continue;  // P4
-            if (p4w && (flags & QF_MASK) && ((ld_event(P.ev, i).w >> lane_of(p)) & 1u)) continue;  // P4 lockstep
+            if (p4w && (flags & QF_MASK) && ((mask_of(P, i) >> lane_of(p)) & 1u)) continue;  // P4 lockstep
             if (p5b && ((q_count(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i) + gcnt) & 255u)) continue;  // P5
             type = (flags & QF_R1) ? IGD_R1 : 0u;
             if (!type) {
@@ -509,7 +509,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
         }
         if (p4w && (flags & QF_MASK)) {  // P4: lockstep, the mask read only now
             CSTAT(5);
-            if ((ld_event(P.ev, i).w >> lane_of(p)) & 1u) continue;
+            if ((mask_of(P, i) >> lane_of(p)) & 1u) continue;
         }
         const bool grid = q_grid(P, mdIdx, i);
         if (p5b && (grid || q_between(P.desc, P.sts, ks.bb + blk_of(c), mdIdx, i))) {  // P5

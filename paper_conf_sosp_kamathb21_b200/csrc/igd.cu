@@ -554,7 +554,11 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     RET(ensure(ctx, ctx->st_in_s, (in_tiles + 1) * sizeof(u32)));
     const u64 acc_cap = SH ? ctx->sh_nrec : n_ev;
     RET(ensure(ctx, ctx->gkb, 1024 * sizeof(u64)));
-    const int vbytes = SH ? 16 : 8;  // sorted payload: (index | tk) or {index, tk, mask, 0}
+    // sharded payload: the single-GPU (index | tk) u64 -- the received records stay resident for
+    // the rare active-mask lookups (SPLIT) -- or, in streaming sessions, the 16-byte record itself
+    // (its mask field carries the carried state)
+    const bool SPLIT = SH && !ctx->str_active;
+    const int vbytes = (SH && !SPLIT) ? 16 : 8;
     for (int b = 0; b < 2; b++) {
         RET(ensure(ctx, ctx->acc_k[b], acc_cap * sizeof(u32)));
         RET(ensure(ctx, ctx->acc_v[b], acc_cap * vbytes));
@@ -711,12 +715,21 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     }
     CK(cudaGetLastError());
     if (SH && n_acc > 0) {
-        // received records {key, index, tk, mask}: the sort keys and their digit histograms; the
-        // records themselves are the payload of the first radix pass
-        KTimer kt(ctx, KC_INGEST, 20.0 * (double)n_acc);
         const unsigned sb = (unsigned)std::min<u64>((n_acc + 255) / 256, (u64)sms * 8);
-        shard::k_record_keys<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
-                                                         P_<u32>(ctx->acc_k[0]), P_<u32>(ctx->hist));
+        if (SPLIT) {
+            // received records {key, index, tk, mask} -> sort keys + (index | tk) payload and the
+            // keys' digit histograms (12-byte sort elements, as on one GPU)
+            KTimer kt(ctx, KC_INGEST, 28.0 * (double)n_acc);
+            shard::k_record_split<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
+                                                              P_<u32>(ctx->acc_k[0]), P_<u64>(ctx->acc_v[0]),
+                                                              P_<u32>(ctx->hist));
+        } else {
+            // the sort keys and their digit histograms; the records themselves are the payload
+            // of the first radix pass
+            KTimer kt(ctx, KC_INGEST, 20.0 * (double)n_acc);
+            shard::k_record_keys<<<sb, 256, 0, ctx->stream>>>((const uint4*)ctx->sh_rec, (u32)n_acc,
+                                                             P_<u32>(ctx->acc_k[0]), P_<u32>(ctx->hist));
+        }
     }
     if (FUSED && IGD_HIST_UP_LATE && n_acc > 0) {
         KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);  // access-key digits 1..3
@@ -876,7 +889,8 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
                        bits_needed(ctx->h_stats[1] - kbase), &acur, vbytes, 1, 1, nullptr, 8));
     else
         RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc,
-                       TG ? TG : 32u, &acur, vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0, SH ? ctx->sh_rec : nullptr));
+                       TG ? TG : 32u, &acur, vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0,
+                       (SH && !SPLIT) ? ctx->sh_rec : nullptr));
     ctx->last_acur = acur;
     ctx->last_scur = scur;
     ctx->last_nsync = n_sync;
@@ -933,7 +947,11 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
                     cp.carry_before = (u32)ctx->str_n;
                     cp.carry_out = ctx->str_co.p;
                 }
-                launch_check(SH, cp.has_kb != 0,
+                if (SPLIT) {  // the active mask of an access, when needed, from the received records
+                    cp.rec = reinterpret_cast<const uint4*>(ctx->sh_rec);
+                    cp.nrec = (u32)n_acc;
+                }
+                launch_check(SH && !SPLIT, cp.has_kb != 0,
                              (ctx->paper_counters ? 1 : 0) | (ctx->sticky ? 2 : 0) | (LK > 1 ? 4 : 0) |
                                  (SH && ctx->str_active ? 8 : 0),
                              key64, (unsigned)tiles, ctx->stream, cp);

@@ -187,4 +187,30 @@ __global__ void __launch_bounds__(256) k_record_keys(const uint4* __restrict__ r
     }
 }
 
+// Received records -> the sort keys, the single-GPU payload (index | tk << 32) and the keys' 4 x
+// 8-bit digit histograms (warp-uniform digits aggregated into one shared atomic).
+__global__ void __launch_bounds__(256) k_record_split(const uint4* __restrict__ rec, u32 n, u32* __restrict__ keys,
+                                                      u64* __restrict__ vals, u32* __restrict__ hist) {
+    __shared__ u32 s[4][256];
+    const u32 lane = threadIdx.x & 31u;
+    for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) (&s[0][0])[i] = 0;
+    __syncthreads();
+    for (u32 i0 = blockIdx.x * blockDim.x; i0 < n; i0 += gridDim.x * blockDim.x) {
+        const u32 i = i0 + threadIdx.x;
+        const bool in = i < n;
+        const uint4 r = in ? __ldcs(rec + i) : make_uint4(0, 0, 0, 0);
+        if (in) {
+            keys[i] = r.x;
+            vals[i] = (u64)r.y | ((u64)r.z << 32);
+        }
+#pragma unroll
+        for (int p = 0; p < 4; p++) ingest::hist_add(s[p], (r.x >> (8 * p)) & 255u, in, lane);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < 4 * 256; i += blockDim.x) {
+        const u32 v = (&s[0][0])[i];
+        if (v) atomicAdd(&hist[i], v);
+    }
+}
+
 }  // namespace shard
