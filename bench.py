@@ -51,6 +51,26 @@ def log(*a):
     print(*a, file=sys.stderr, flush=True)
 
 
+_JSON_OUT = None
+
+
+def _claim_stdout():
+    """Keep fd 1 for the one JSON line: libraries print to stdout from C (NCCL's version banner
+    goes through printf when the communicator is created), so fd 1 is pointed at stderr for the
+    rest of the run and the line is written to a private duplicate of the original stdout."""
+    global _JSON_OUT
+    if _JSON_OUT is None:
+        sys.stdout.flush()
+        _JSON_OUT = os.fdopen(os.dup(1), "w")
+        os.dup2(2, 1)
+
+
+def emit(line):
+    out = _JSON_OUT if _JSON_OUT is not None else sys.stdout
+    out.write(json.dumps(line) + "\n")
+    out.flush()
+
+
 class ClockSampler:
     """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
 
@@ -199,7 +219,7 @@ def run_reference(args, fam, rank, world):
             "cpu_baseline": {"value": value, "unit": "G events/s", "cores": 1, "kind": "oracle",
                              "sample": sample_desc, "host": host_info()},
             "e2e": {"value": value, "unit": "G events/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 def run_sharded(args, fam, rank, world, local):
@@ -325,7 +345,7 @@ def run_sharded(args, fam, rank, world, local):
                         "h2d_bytes_per_step": n * 16, "d2h_bytes_per_step": int(len(out)) * 32 * world,
                         "ms_per_step": e2e_s * 1e3},
                 "gpu_launches": launches, "clocks": clk}
-        print(json.dumps(line), flush=True)
+        emit(line)
     det.close()
     dist.destroy_process_group()
 
@@ -382,7 +402,7 @@ def run_stream(args, fam):
                        "ledger_reports": int(len(lg)), "ledger_match": ledger_match,
                        "l2": "inputs larger than L2 (no flush)" if n * 16 > 126e6 else "inputs smaller than L2"},
             "roofline": None, "cpu_baseline": None, "e2e": None, "gpu_launches": None, "clocks": clk}
-    print(json.dumps(line), flush=True)
+    emit(line)
     det.close()
 
 
@@ -418,6 +438,7 @@ def ncu_traffic(workload, n, kclass):
 
 
 def main():
+    _claim_stdout()
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
@@ -624,7 +645,7 @@ def main():
                          "achieved_dram_frac": (path_bytes / (ms / 1e3) / 1e9 / peak) if path_bytes else None,
                          "stages_ms": stages, "kernels": breakdown},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk}
-        print(json.dumps(line), flush=True)
+        emit(line)
     if world > 1:
         dist.destroy_process_group()
 
