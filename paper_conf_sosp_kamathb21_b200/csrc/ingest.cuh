@@ -401,6 +401,108 @@ constexpr u64 kRules = 0x1ull | (0x1ull << 4) | (0x3ull << 8) | (0x3ull << 12) |
 constexpr u32 kSyncRecs = (1u << 6) | (1u << 8) | (1u << 10) | (1u << 12) | (1u << 14) | (1u << 16) |
                           (1u << 18) | (1u << 20) | (1u << 22) | (1u << 24);
 
+// The rule check folded into tables indexed by the event's top byte (kind | scope << 4 | the two
+// reserved bits << 6): kAllowed = the kind exists and its scope rule holds; the remaining rules
+// (lane in mask, addr 0, tid 0) are a 3-bit "needed" word per kind tested against the event's
+// facts; kNs0 / kNs1 = the number of sync records; kLockIdx = CAS / EXCH.
+constexpr u64 p0_allowed() {
+    u64 m = 0;
+    for (int i = 0; i < 64; i++) {
+        const int k = i & 15, sc = i >> 4;
+        const bool scoped = (kRules >> (4 * k)) & 2u;
+        if (k <= IGD_KERNEL_BOUNDARY && (scoped ? sc != 0 : sc == 0)) m |= 1ull << i;
+    }
+    return m;
+}
+constexpr u64 p0_ns(int bit) {
+    u64 m = 0;
+    for (int i = 0; i < 64; i++) {
+        const int k = i & 15, sc = i >> 4;
+        const u32 ns = k <= IGD_KERNEL_BOUNDARY ? ((kSyncRecs >> (2 * k)) & 3u) + (k == IGD_FENCE && sc >= 2 ? 1u : 0u) : 0u;
+        if ((ns >> bit) & 1u) m |= 1ull << i;
+    }
+    return m;
+}
+constexpr u64 p0_need() {
+    u64 m = 0;
+    for (int k = 0; k < 16; k++) m |= ((kRules >> (4 * k)) & 0xDull) << (4 * k);
+    return m;
+}
+constexpr u64 kAllowed = p0_allowed(), kNs0 = p0_ns(0), kNs1 = p0_ns(1), kNeed = p0_need();
+
+#ifndef IGD_P0_UNIF
+#define IGD_P0_UNIF 0  // 1: upper-digit histogram by a warp-uniform test + per-lane atomics (C5: 19.1 -> 22.6 ms, r02aa)
+#endif
+
+template <bool GEO2, bool COAL, bool FULL>
+__device__ __forceinline__ void count_tile(const Params& P, const Geo& g, u64 base, u32 tid, u32 lane, u32 warp,
+                                           u32 (*s_hacc)[256], u32 (*s_hup)[256], u64& wmin, u64& wmax,
+                                           u64& bad, u32& cnt_lock, u32& wsum) {
+    uint4 e[ITEMS];
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++) {
+        const u64 i = base + (u64)j * THREADS + tid;
+        e[j] = (FULL || i < P.n) ? ld_event_stream(P.ev, i) : make_uint4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int j = 0; j < ITEMS; j++) {
+        const u64 i = base + (u64)j * THREADS + tid;
+        const bool in = FULL || i < P.n;
+        const u32 t = e[j].z & 0xFFFFFFu, top = e[j].z >> 24, kind = top & 0xFu;
+        const bool addr0 = (e[j].x | e[j].y) == 0;
+        const u32 ln = GEO2 ? (t & 31u) : ((t - g.block(t) * g.D) & 31u);
+        const u32 facts = ((e[j].w >> ln) & 1u) | (addr0 ? 4u : 0u) | (t == 0u ? 8u : 0u);
+        const u32 need = (u32)(kNeed >> (4 * kind)) & 0xDu;
+        bool ok = in && top < 64u && ((kAllowed >> top) & 1u) && t < g.T && (need & ~facts) == 0u;
+        if (kind == IGD_KERNEL_BOUNDARY && ok && !addr0) {  // rare: another grid (A34)
+            ok = geo_code_ok(e[j].y, e[j].x);
+            if (ok) {
+                const unsigned long long slot = atomicAdd((unsigned long long*)&P.stats[6], 1ull);
+                if (slot < P.gkb_cap) P.gkb[slot] = i;
+            }
+        }
+        if (in && !ok) bad = min(bad, i);
+        bool acc = ok && kind <= IGD_EXCH;
+        if (COAL && acc && ((__ldg(P.skip_bits + (i >> 5)) >> (i & 31u)) & 1u)) acc = false;  // A32
+        const u32 ns = ok ? (u32)((kNs0 >> top) & 1u) | ((u32)((kNs1 >> top) & 1u) << 1) : 0u;
+        cnt_lock += (ok && (kind == IGD_CAS || kind == IGD_EXCH)) ? 1u : 0u;
+        const u32 key = (e[j].x >> 2) | (e[j].y << 30);
+        if (acc) {
+            const u64 word = ev_addr(e[j]) >> 2;
+            wmin = min(wmin, word);
+            wmax = max(wmax, word);
+            atomicAdd(&s_hacc[warp & 3u][key & 255u], 1u);
+        }
+        // digits 1..3 (IGD_HIST_UP_LATE: histogrammed over the fused pass's keys instead)
+        const u32 am = IGD_HIST_UP_LATE ? 0u : __ballot_sync(IGD_FULL, acc);
+        if (am) {
+            const u32 hi = key >> 8;
+            if (IGD_P0_UNIF) {
+                // one set of atomics when every access of the row shares the upper 24 bits (the
+                // common case for warp-contiguous words), else one per lane
+                const u32 src = __ffs(am) - 1;
+                const u32 h0 = __shfl_sync(IGD_FULL, hi, src);
+                const bool uni = __all_sync(IGD_FULL, !acc || hi == h0);
+                const u32 c = uni ? (lane == src ? __popc(am) : 0u) : (acc ? 1u : 0u);
+                if (c) {
+                    atomicAdd(&s_hup[0][hi & 255u], c);
+                    atomicAdd(&s_hup[1][(hi >> 8) & 255u], c);
+                    atomicAdd(&s_hup[2][hi >> 16], c);
+                }
+            } else {
+                const u32 peers = __match_any_sync(IGD_FULL, acc ? hi : (0x1000000u | lane)) & am;
+                const u32 c = (acc && lane == (u32)(__ffs(peers) - 1)) ? __popc(peers) : 0u;
+                if (c) {
+                    atomicAdd(&s_hup[0][hi & 255u], c);
+                    atomicAdd(&s_hup[1][(hi >> 8) & 255u], c);
+                    atomicAdd(&s_hup[2][hi >> 16], c);
+                }
+            }
+        }
+        wsum += __reduce_add_sync(IGD_FULL, (acc ? 1u : 0u) | (ns << 16));
+    }
+}
+
 template <bool GEO2, bool COAL>
 __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_count_fused(Params P) {
     __shared__ u32 s_hacc[4][256];
@@ -418,57 +520,11 @@ __global__ void __launch_bounds__(THREADS, IGD_INGEST_MINB) k_count_fused(Params
     const Geo g = P.g;
     for (u32 tile = blockIdx.x; tile < P.n_tiles; tile += gridDim.x) {
         const u64 base = (u64)tile * TILE;
-        uint4 e[ITEMS];
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            const u64 i = base + (u64)j * THREADS + tid;
-            e[j] = (i < P.n) ? ld_event_stream(P.ev, i) : make_uint4(0, 0, 0, 0);
-        }
         u32 wsum = 0;
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            const u64 i = base + (u64)j * THREADS + tid;
-            const bool in = i < P.n;
-            const u32 t = e[j].z & 0xFFFFFFu, kind = (e[j].z >> 24) & 0xFu, scope = (e[j].z >> 28) & 3u;
-            const bool addr0 = (e[j].x | e[j].y) == 0;
-            const u32 r = (u32)(kRules >> (4 * (kind & 15u))) & 15u;
-            const u32 ln = GEO2 ? (t & 31u) : ((t - g.block(t) * g.D) & 31u);
-            bool ok = (e[j].z >> 30) == 0 && kind <= IGD_KERNEL_BOUNDARY && t < g.T;
-            ok = ok && (!(r & 1u) || ((e[j].w >> ln) & 1u)) && ((r & 2u) ? scope != 0u : scope == 0u) &&
-                 (!(r & 4u) || addr0) && (!(r & 8u) || t == 0u) &&
-                 (kind != IGD_KERNEL_BOUNDARY || addr0 || geo_code_ok(e[j].y, e[j].x));
-            bool acc = in && ok && kind <= IGD_EXCH;
-            if (COAL && acc && ((__ldg(P.skip_bits + (i >> 5)) >> (i & 31u)) & 1u)) acc = false;  // A32
-            const u32 ns = (in && ok) ? ((kSyncRecs >> (2 * kind)) & 3u) + (kind == IGD_FENCE && scope >= 2u ? 1u : 0u)
-                                      : 0u;
-            if (in && !ok) bad = min(bad, i);
-            if (in && ok && kind == IGD_KERNEL_BOUNDARY && !addr0) {  // rare: another grid (A34)
-                const unsigned long long slot = atomicAdd((unsigned long long*)&P.stats[6], 1ull);
-                if (slot < P.gkb_cap) P.gkb[slot] = i;
-            }
-            cnt_lock += (in && ok && (kind == IGD_CAS || kind == IGD_EXCH)) ? 1u : 0u;
-            const u32 key = (e[j].x >> 2) | (e[j].y << 30);
-            if (acc) {
-                const u64 word = ev_addr(e[j]) >> 2;
-                wmin = min(wmin, word);
-                wmax = max(wmax, word);
-                atomicAdd(&s_hacc[warp & 3u][key & 255u], 1u);
-            }
-            // digits 1..3: one set of atomics per distinct upper-24-bit value among the lanes
-            // (IGD_HIST_UP_LATE: histogrammed over the fused pass's keys instead)
-            const u32 am = IGD_HIST_UP_LATE ? 0u : __ballot_sync(IGD_FULL, acc);
-            if (am) {
-                const u32 hi = key >> 8;
-                const u32 peers = __match_any_sync(IGD_FULL, acc ? hi : (0x1000000u | lane)) & am;
-                const u32 c = (acc && lane == (u32)(__ffs(peers) - 1)) ? __popc(peers) : 0u;
-                if (c) {
-                    atomicAdd(&s_hup[0][hi & 255u], c);
-                    atomicAdd(&s_hup[1][(hi >> 8) & 255u], c);
-                    atomicAdd(&s_hup[2][hi >> 16], c);
-                }
-            }
-            wsum += __reduce_add_sync(IGD_FULL, (acc ? 1u : 0u) | (ns << 16));
-        }
+        if (base + TILE <= P.n)
+            count_tile<GEO2, COAL, true>(P, g, base, tid, lane, warp, s_hacc, s_hup, wmin, wmax, bad, cnt_lock, wsum);
+        else
+            count_tile<GEO2, COAL, false>(P, g, base, tid, lane, warp, s_hacc, s_hup, wmin, wmax, bad, cnt_lock, wsum);
         if (lane == 0) s_wtot[warp] = wsum;
         __syncthreads();
         if (warp == 0) {
