@@ -100,12 +100,12 @@ __device__ __forceinline__ FDec fdecode(const uint4& e, const Geo& g, const KeyS
 }
 
 // the event tile (16 B per event), or the phase-2 buffers aliasing it if those are larger:
-// keys (KT), values (8 B), digits (1 B), per-warp digit counts
+// keys (KT), values (8 B), per-warp digit counts
 template <typename KT = u32>
 constexpr size_t smem_bytes() {
-    return (size_t)TILE * 16 > (size_t)TILE * (sizeof(KT) + 9) + WARPS * RADIX * 4
+    return (size_t)TILE * 16 > (size_t)TILE * (sizeof(KT) + 8) + WARPS * RADIX * 4
                ? (size_t)TILE * 16
-               : (size_t)TILE * (sizeof(KT) + 9) + WARPS * RADIX * 4;
+               : (size_t)TILE * (sizeof(KT) + 8) + WARPS * RADIX * 4;
 }
 
 // COAL: warp-coalesced mode (A32) -- a separate instantiation so the default path carries no
@@ -114,7 +114,6 @@ constexpr size_t smem_bytes() {
 // path of a4)
 template <bool COAL, typename KT = u32, bool GEO2 = false>
 __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params P) {
-    __shared__ u32 s_tile_excl[RADIX];
     __shared__ u32 s_gbase[RADIX];
     __shared__ u32 s_wsum[WARPS];
     __shared__ u32 s_wsync[WARPS];
@@ -124,12 +123,11 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     __shared__ u32 s_tile;
     extern __shared__ __align__(16) unsigned char s_dyn[];
     // phase 1: the event tile (64 KB).  Phase 2 (events dead), u32 keys: digit-sorted keys
-    // [0, 16K), values [16K, 48K), digit per position [48K, 52K), per-warp digit counts [52K, 60K).
+    // [0, 16K), values [16K, 48K), per-warp digit counts [48K, 56K).
     uint4* s_ev = reinterpret_cast<uint4*>(s_dyn);
     KT* s_k = reinterpret_cast<KT*>(s_dyn);
     u64* s_v = reinterpret_cast<u64*>(s_dyn + TILE * sizeof(KT));
-    uint8_t* s_dig = s_dyn + TILE * (sizeof(KT) + 8);
-    u32(*s_whist)[RADIX] = reinterpret_cast<u32(*)[RADIX]>(s_dyn + TILE * (sizeof(KT) + 9));
+    u32(*s_whist)[RADIX] = reinterpret_cast<u32(*)[RADIX]>(s_dyn + TILE * (sizeof(KT) + 8));
     KT* kout = reinterpret_cast<KT*>(P.kout);
 
     const u32 t = threadIdx.x, lane = t & 31u, warp = t >> 5;
@@ -250,21 +248,18 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     }
     __syncthreads();
 
-    // ---- per digit: exclusive over warps, tile count, publish the aggregate
-    u32 cnt;
+    // ---- per digit: tile count, exclusive scan over digits, every warp's tile position base
+    u32 cnt, tile_excl;
     {
         const u32 d = t;
-        u32 sum = 0;
+        u32 c[WARPS];
+        cnt = 0;
 #pragma unroll
         for (int w = 0; w < WARPS; w++) {
-            const u32 c = s_whist[w][d];
-            s_whist[w][d] = sum;
-            sum += c;
+            c[w] = s_whist[w][d];
+            cnt += c[w];
         }
-        cnt = sum;
         if (!IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
-    }
-    {
         u32 inc = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -277,8 +272,14 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
 #pragma unroll
         for (int w = 0; w < WARPS; w++)
             if ((u32)w < warp) wpre += s_wsum[w];
-        s_tile_excl[t] = wpre + inc - cnt;
+        tile_excl = wpre + inc - cnt;
         if (t == RADIX - 1) s_na = wpre + inc;  // accesses in this tile
+        u32 run = tile_excl;
+#pragma unroll
+        for (int w = 0; w < WARPS; w++) {
+            s_whist[w][d] = run;
+            run += c[w];
+        }
     }
     // ---- look-back for digit t (LB statuses per round trip, as rsort::k_onesweep)
     {
@@ -304,7 +305,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
             }
             st_relaxed(P.status + (u64)tile * RADIX + dg, ST_INC | (excl + cnt));
         }
-        s_gbase[dg] = P.digit_base[dg] + (u32)excl - s_tile_excl[dg];  // position = s_gbase[d] + i
+        s_gbase[dg] = P.digit_base[dg] + (u32)excl - tile_excl;  // position = s_gbase[d] + i
     }
     __syncthreads();
     // ---- records to their tile positions: key, payload (event index | tk << 32), digit
@@ -312,10 +313,9 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     for (int j = 0; j < ITEMS; j++) {
         if ((amask >> j) & 1u) {
             const u32 d = (u32)key[j] & 255u;
-            const u32 r = ((rank2[j / 2] >> (16 * (j & 1))) & 0xFFFFu) + s_tile_excl[d] + s_whist[warp][d];
+            const u32 r = ((rank2[j / 2] >> (16 * (j & 1))) & 0xFFFFu) + s_whist[warp][d];
             s_k[r] = key[j];
             s_v[r] = (base + wofs + j * 32 + lane) | ((u64)tk[j] << 32);
-            s_dig[r] = (uint8_t)d;
         }
     }
     __syncthreads();
@@ -325,9 +325,9 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     for (int k = 0; k < ITEMS; k++) {
         const u32 i = t + k * THREADS;
         if (i < na) {
-            const u32 d = s_dig[i];
-            const u32 o = s_gbase[d] + i;
-            __stcs(kout + o, s_k[i]);
+            const KT kk = s_k[i];
+            const u32 o = s_gbase[(u32)kk & 255u] + i;
+            __stcs(kout + o, kk);
             __stcs(P.vout + o, s_v[i]);
         }
     }

@@ -117,10 +117,10 @@ __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     }
 }
 
-// Dynamic shared memory of k_onesweep<VT, TAIL, KT>: staged keys, staged values, digit per position.
+// Dynamic shared memory of k_onesweep<VT, TAIL, KT>: staged keys, staged values.
 template <typename VT, typename KT = u32>
 constexpr size_t onesweep_smem() {
-    return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT) + TILE;
+    return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT);
 }
 
 #ifndef IGD_SORT_LB_EARLY
@@ -160,8 +160,7 @@ template <typename VT, bool TAIL, typename KT = u32>
 #define IGD_SORT_MINB 3
 #endif
 __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams P) {
-    __shared__ u32 s_whist[WARPS][RADIX];
-    __shared__ u32 s_tile_excl[RADIX];
+    __shared__ u32 s_whist[WARPS][RADIX];  // per-warp digit counts, then tile position bases
     __shared__ u32 s_gbase[RADIX];
     __shared__ u32 s_tile;
     __shared__ u32 s_wsum[WARPS];
@@ -170,7 +169,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     extern __shared__ __align__(16) unsigned char s_dyn[];
     KT* s_k = reinterpret_cast<KT*>(s_dyn);                           // keys in, then keys out
     VT* s_v = reinterpret_cast<VT*>(s_dyn + TILE * sizeof(KT));       // values in, then values out
-    uint8_t* s_dig = s_dyn + TILE * sizeof(KT) + TILE * sizeof(VT);   // digit of each output position
     const VT* vin = reinterpret_cast<const VT*>(P.vin);
     VT* vout = reinterpret_cast<VT*>(P.vout);
     const KT* kin = reinterpret_cast<const KT*>(P.kin);
@@ -256,22 +254,19 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         __syncwarp();
     }
     __syncthreads();
-    // per digit: exclusive over warps, tile count, publish
-    u32 cnt;
+    // per digit: tile count, exclusive scan over digits, then every warp's base for the digit
+    // (tile exclusive + earlier warps) in place of its count -- one shared load per rank below
+    u32 cnt, tile_excl;
     {
         const u32 d = t;  // THREADS == RADIX
-        u32 sum = 0;
+        u32 c[WARPS];
+        cnt = 0;
 #pragma unroll
         for (int w = 0; w < WARPS; w++) {
-            u32 c = s_whist[w][d];
-            s_whist[w][d] = sum;
-            sum += c;
+            c[w] = s_whist[w][d];
+            cnt += c[w];
         }
-        cnt = sum;
         if (!IGD_SORT_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
-    }
-    // block exclusive scan of cnt over digits
-    {
         u32 inc = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -284,7 +279,13 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
 #pragma unroll
         for (int w = 0; w < WARPS; w++)
             if ((u32)w < warp) wpre += s_wsum[w];
-        s_tile_excl[t] = wpre + inc - cnt;
+        tile_excl = wpre + inc - cnt;
+        u32 run = tile_excl;
+#pragma unroll
+        for (int w = 0; w < WARPS; w++) {
+            s_whist[w][d] = run;
+            run += c[w];
+        }
     }
     // Decoupled look-back for this digit: LB predecessor statuses are requested at once, so a
     // walk back over tiles that have published only their aggregate costs one L2 round trip per
@@ -301,14 +302,14 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         }
         // output position of tile position i with digit d = s_gbase[d] + i (u32 arithmetic wraps
         // back into range): one shared load per written element instead of two
-        s_gbase[d] = P.digit_base[d] + (u32)excl - s_tile_excl[d];
+        s_gbase[d] = P.digit_base[d] + (u32)excl - tile_excl;
     }
     __syncthreads();
     // keys: reorder in shared memory (rank[] becomes the tile position), write digit runs
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
         const u32 d = (u32)(key[j] >> shift) & dmask;
-        rank[j] += s_tile_excl[d] + s_whist[warp][d];
+        rank[j] += s_whist[warp][d];
         if (full || wbase + j * 32 + lane < P.n) s_k[rank[j]] = key[j];
     }
     __syncthreads();
@@ -319,7 +320,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         if (i < tile_n) {
             const KT kk = s_k[i];
             const u32 d = (u32)(kk >> shift) & dmask;
-            s_dig[i] = (uint8_t)d;
             __stcs(kout + (s_gbase[d] + i), kk);
         }
     }
@@ -345,7 +345,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
     for (int k = 0; k < ITEMS; k++) {
         const u32 i = t + k * THREADS;
         if (i < tile_n) {
-            const u32 d = s_dig[i];
+            const u32 d = (u32)(s_k[i] >> shift) & dmask;  // the staged keys are still in tile order
             __stcs(vout + (s_gbase[d] + i), s_v[i]);
         }
     }
