@@ -430,6 +430,23 @@ constexpr u64 p0_need() {
 }
 constexpr u64 kAllowed = p0_allowed(), kNs0 = p0_ns(0), kNs1 = p0_ns(1), kNeed = p0_need();
 
+// The field rules of include/igd.h for one event, from the tables above.  lane: the lane of the
+// event's tid (only meaningful when tid < T, which the rule also requires).  *grid: a kernel
+// boundary that carries the next kernel's grid (reading A34).
+__device__ __forceinline__ bool rules_ok(const uint4& e, u32 t, u32 lane, const Geo& g, bool* grid) {
+    const u32 top = e.z >> 24, kind = top & 0xFu;
+    const bool addr0 = (e.x | e.y) == 0;
+    const u32 facts = ((e.w >> lane) & 1u) | (addr0 ? 4u : 0u) | (t == 0u ? 8u : 0u);
+    const u32 need = (u32)(kNeed >> (4 * kind)) & 0xDu;
+    bool ok = top < 64u && ((kAllowed >> top) & 1u) && t < g.T && (need & ~facts) == 0u;
+    *grid = false;
+    if (kind == IGD_KERNEL_BOUNDARY && ok && !addr0) {  // rare
+        ok = geo_code_ok(e.y, e.x);
+        *grid = ok;
+    }
+    return ok;
+}
+
 #ifndef IGD_P0_UNIF
 #define IGD_P0_UNIF 0  // 1: upper-digit histogram by a warp-uniform test + per-lane atomics (C5: 19.1 -> 22.6 ms, r02aa)
 #endif
@@ -449,17 +466,12 @@ __device__ __forceinline__ void count_tile(const Params& P, const Geo& g, u64 ba
         const u64 i = base + (u64)j * THREADS + tid;
         const bool in = FULL || i < P.n;
         const u32 t = e[j].z & 0xFFFFFFu, top = e[j].z >> 24, kind = top & 0xFu;
-        const bool addr0 = (e[j].x | e[j].y) == 0;
         const u32 ln = GEO2 ? (t & 31u) : ((t - g.block(t) * g.D) & 31u);
-        const u32 facts = ((e[j].w >> ln) & 1u) | (addr0 ? 4u : 0u) | (t == 0u ? 8u : 0u);
-        const u32 need = (u32)(kNeed >> (4 * kind)) & 0xDu;
-        bool ok = in && top < 64u && ((kAllowed >> top) & 1u) && t < g.T && (need & ~facts) == 0u;
-        if (kind == IGD_KERNEL_BOUNDARY && ok && !addr0) {  // rare: another grid (A34)
-            ok = geo_code_ok(e[j].y, e[j].x);
-            if (ok) {
-                const unsigned long long slot = atomicAdd((unsigned long long*)&P.stats[6], 1ull);
-                if (slot < P.gkb_cap) P.gkb[slot] = i;
-            }
+        bool grid = false;
+        const bool ok = in && rules_ok(e[j], t, ln, g, &grid);
+        if (grid) {  // rare: another grid (A34)
+            const unsigned long long slot = atomicAdd((unsigned long long*)&P.stats[6], 1ull);
+            if (slot < P.gkb_cap) P.gkb[slot] = i;
         }
         if (in && !ok) bad = min(bad, i);
         bool acc = ok && kind <= IGD_EXCH;

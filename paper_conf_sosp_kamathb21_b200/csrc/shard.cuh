@@ -62,7 +62,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SHARD_MINB) k_shard(Params P) {
     const u32 tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const u32 lt = lanemask_lt();
     const Geo g = P.g;
-    const KeySpace ks = P.ks;
     const u32 NP = P.P;
     u64 wmin = ~0ull, wmax = 0, bad = ~0ull;
 
@@ -78,16 +77,19 @@ __global__ void __launch_bounds__(THREADS, IGD_SHARD_MINB) k_shard(Params P) {
             dst[j] = 0;
             tk[j] = 0;
             if (i < P.n) {
-                const ingest::Dec d = ingest::decode(e[j], g, ks);
-                if (d.flags & 16u) {
+                const u32 t = e[j].z & 0xFFFFFFu, kind = (e[j].z >> 24) & 0xFu;
+                const u32 ln = (t - g.block(t) * g.D) & 31u, lanebit = 1u << ln;
+                bool grid;
+                if (!ingest::rules_ok(e[j], t, ln, g, &grid)) {
                     bad = min(bad, P.first + i);
                 } else {
                     // a grid change (A34) is single-context only: counted, the host refuses it
-                    if (PASS == 0 && (d.flags & 32u)) atomicAdd((unsigned long long*)&P.stats[3], 1ull);
-                    const u32 kind = ev_kind(e[j]);
-                    if (d.flags & 1u) {
-                        dst[j] = 0x100u | (NP == 1 ? 0u : fmix32(d.key) % NP);
-                        tk[j] = d.tk;
+                    if (PASS == 0 && grid) atomicAdd((unsigned long long*)&P.stats[3], 1ull);
+                    if (kind <= IGD_EXCH) {
+                        const u32 key = (e[j].x >> 2) | (e[j].y << 30);
+                        dst[j] = 0x100u | (NP == 1 ? 0u : fmix32(key) % NP);
+                        // mask summaries for the check's lockstep clause (as ingest::decode)
+                        tk[j] = e[j].z | (e[j].w == IGD_FULL ? (1u << 31) : 0u) | (e[j].w == lanebit ? (1u << 30) : 0u);
                         const u64 word = ev_addr(e[j]) >> 2;
                         wmin = min(wmin, word);
                         wmax = max(wmax, word);
@@ -110,7 +112,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SHARD_MINB) k_shard(Params P) {
             }
         }
         __syncthreads();
-        if (PASS == 0) {
+        if constexpr (PASS == 0) {
             for (u32 o = tid; o <= NP; o += THREADS) {
                 u32 s = 0;
                 for (int j = 0; j < ITEMS; j++)
@@ -119,48 +121,50 @@ __global__ void __launch_bounds__(THREADS, IGD_SHARD_MINB) k_shard(Params P) {
             }
             __syncthreads();
             continue;
-        }
-        // exclusive offsets in (item, warp) order per destination
-        for (u32 o = tid; o <= NP; o += THREADS) {
-            u32 s = 0;
-            for (int j = 0; j < ITEMS; j++)
-                for (int w = 0; w < WARPS; w++) {
-                    const u32 c = s_wc[j][w][o];
-                    s_wc[j][w][o] = s;
-                    s += c;
+        } else {
+            // exclusive offsets in (item, warp) order per destination
+            for (u32 o = tid; o <= NP; o += THREADS) {
+                u32 s = 0;
+                for (int j = 0; j < ITEMS; j++)
+                    for (int w = 0; w < WARPS; w++) {
+                        const u32 c = s_wc[j][w][o];
+                        s_wc[j][w][o] = s;
+                        s += c;
+                    }
+            }
+            __syncthreads();
+#pragma unroll
+            for (int j = 0; j < ITEMS; j++) {
+                const u64 i = base + (u64)j * THREADS + tid;
+                if (i >= P.n) continue;
+                const u32 gi = (u32)(P.first + i);
+                if (dst[j] & 0x100u) {
+                    const u32 o = dst[j] & 0xFFu;
+                    const u64 pos = P.obase[o] + P.cnt[(u64)o * (P.n_tiles + 1) + tile] + s_wc[j][warp][o] + rk[j];
+                    const u32 key = (e[j].x >> 2) | (e[j].y << 30);
+                    P.send[pos] = make_uint4(key, gi, tk[j], e[j].w);
                 }
-        }
-        __syncthreads();
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            const u64 i = base + (u64)j * THREADS + tid;
-            if (i >= P.n) continue;
-            const u32 gi = (u32)(P.first + i);
-            if (dst[j] & 0x100u) {
-                const u32 o = dst[j] & 0xFFu;
-                const u64 pos = P.obase[o] + P.cnt[(u64)o * (P.n_tiles + 1) + tile] + s_wc[j][warp][o] + rk[j];
-                const u32 key = (e[j].x >> 2) | (e[j].y << 30);
-                P.send[pos] = make_uint4(key, gi, tk[j], e[j].w);
+                if (dst[j] >> 31) {
+                    const u64 pos = (u64)P.cnt[(u64)NP * (P.n_tiles + 1) + tile] + s_wc[j][warp][NP] + srk[j];
+                    P.sync_idx[pos] = gi;
+                    P.sync_ev[pos] = e[j];
+                }
             }
-            if (dst[j] >> 31) {
-                const u64 pos = (u64)P.cnt[(u64)NP * (P.n_tiles + 1) + tile] + s_wc[j][warp][NP] + srk[j];
-                P.sync_idx[pos] = gi;
-                P.sync_ev[pos] = e[j];
-            }
+            __syncthreads();
         }
-        __syncthreads();
     }
-    if (PASS != 0) return;
+    if constexpr (PASS == 0) {  // the chunk's word range and first invalid event
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        wmin = min(wmin, __shfl_xor_sync(IGD_FULL, wmin, o));
-        wmax = max(wmax, __shfl_xor_sync(IGD_FULL, wmax, o));
-        bad = min(bad, __shfl_xor_sync(IGD_FULL, bad, o));
-    }
-    if (lane == 0) {
-        if (wmin != ~0ull) atomicMin((unsigned long long*)&P.stats[0], (unsigned long long)wmin);
-        if (wmin != ~0ull) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
-        if (bad != ~0ull) atomicMin((unsigned long long*)&P.stats[2], (unsigned long long)bad);
+        for (int o = 16; o > 0; o >>= 1) {
+            wmin = min(wmin, __shfl_xor_sync(IGD_FULL, wmin, o));
+            wmax = max(wmax, __shfl_xor_sync(IGD_FULL, wmax, o));
+            bad = min(bad, __shfl_xor_sync(IGD_FULL, bad, o));
+        }
+        if (lane == 0) {
+            if (wmin != ~0ull) atomicMin((unsigned long long*)&P.stats[0], (unsigned long long)wmin);
+            if (wmin != ~0ull) atomicMax((unsigned long long*)&P.stats[1], (unsigned long long)wmax);
+            if (bad != ~0ull) atomicMin((unsigned long long*)&P.stats[2], (unsigned long long)bad);
+        }
     }
 }
 
