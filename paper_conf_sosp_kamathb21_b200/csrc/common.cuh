@@ -108,6 +108,20 @@ __device__ __forceinline__ u64 ld_relaxed(const u64* p) {
     return v;
 }
 
+// Digit statuses of the radix passes (rsort, fused) also carry the pass's epoch in bits 61..40,
+// values in bits 39..0: a status of an earlier pass reads as "not ready", so the per-(tile, digit)
+// buffer is never cleared between passes (it was ~2 GB of memset per pass at C5).
+#define DS_VAL_MASK ((1ull << 40) - 1)
+#define DS_EPOCH_MAX 0x3FFFFFu
+__device__ __forceinline__ u64 ds_make(u64 state, u32 epoch, u64 v) { return state | ((u64)epoch << 40) | v; }
+__device__ __forceinline__ bool ds_ready(u64 s, u32 epoch) {
+    return (s >> 62) != 0 && ((u32)(s >> 40) & DS_EPOCH_MAX) == epoch;
+}
+__device__ __forceinline__ u64 ds_spin(const u64* p, u64 s, u32 epoch) {
+    while (!ds_ready(s, epoch)) s = ld_relaxed(p);
+    return s;
+}
+
 // Wait until a look-back status word is published (non-zero state).  The back-off frees issue
 // slots for the other CTAs of the SM while a predecessor tile is still working.
 #ifndef IGD_SPIN_NS

@@ -49,7 +49,8 @@ struct Params {
     u32* sync_val;
     u64 sync_cap;
     const u32* digit_base;  // [256] exclusive global offsets of digit 0 of the access keys
-    u64* status;            // [n_tiles * 256], zeroed
+    u64* status;            // [n_tiles * 256] digit statuses tagged with `epoch` (see rsort::PassParams)
+    u32 epoch;
     u32* tile_ctr;          // zeroed: tile tickets (CTA start order, see rsort::k_onesweep)
     void* kout;             // access keys (u32 or u64, template KT), sorted by digit 0
     u64 kbase;              // KT = u64: key = word - kbase (kbase's low 8 bits are 0)
@@ -190,7 +191,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
     // The tile's digit counts are known before any ranking: publish them now, so successors
     // looking back rarely find this tile not ready (their spin was most of this kernel's issue
     // slots when the aggregate was published after ranking, ncu r01 v5)
-    if (IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
+    if (IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + t, ds_make(tile == 0 ? ST_INC : ST_AGG, P.epoch, s_cnt[t]));
 
     // ---- synchronization records, in trace order: base of this tile (ingest pass 0) + earlier
     // warps + earlier (item, lane) of this warp; keys from the event slots
@@ -259,7 +260,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
             c[w] = s_whist[w][d];
             cnt += c[w];
         }
-        if (!IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
+        if (!IGD_FUSED_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, ds_make(tile == 0 ? ST_INC : ST_AGG, P.epoch, cnt));
         u32 inc = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -292,18 +293,18 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
                 u64 s[IGD_SORT_LB];
 #pragma unroll
                 for (int q = 0; q < IGD_SORT_LB; q++)
-                    s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + dg) : ST_INC;
+                    s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + dg) : ds_make(ST_INC, P.epoch, 0);
 #pragma unroll
                 for (int q = 0; q < IGD_SORT_LB; q++) {
                     if (!done) {
-                        s[q] = spin_status(P.status + (u64)(tt - q) * RADIX + dg, s[q]);
-                        excl += s[q] & ST_VAL_MASK;
+                        s[q] = ds_spin(P.status + (u64)(tt - q) * RADIX + dg, s[q], P.epoch);
+                        excl += s[q] & DS_VAL_MASK;
                         done = (s[q] >> 62) == 2;
                     }
                 }
                 tt -= IGD_SORT_LB;
             }
-            st_relaxed(P.status + (u64)tile * RADIX + dg, ST_INC | (excl + cnt));
+            st_relaxed(P.status + (u64)tile * RADIX + dg, ds_make(ST_INC, P.epoch, excl + cnt));
         }
         s_gbase[dg] = P.digit_base[dg] + (u32)excl - tile_excl;  // position = s_gbase[d] + i
     }

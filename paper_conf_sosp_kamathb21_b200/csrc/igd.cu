@@ -146,6 +146,8 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
+    Buf dstatus;        // digit statuses of the radix passes, epoch-tagged (never cleared per pass)
+    u32 ds_epoch = 0;   // tag of the last radix pass
     Buf off, ldesc, gtab, tcnt, tpts, tbits, fdev, skipb;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
@@ -269,6 +271,20 @@ static int ensure(igd_ctx* ctx, Buf& b, size_t bytes) {
     return IGD_OK;
 }
 
+// The digit-status buffer for a radix pass over `tiles` tiles and the pass's epoch tag: cleared
+// only when (re)allocated or when the 22-bit epoch wraps.
+static int next_digit_epoch(igd_ctx* ctx, u64 tiles, u32* epoch) {
+    const size_t bytes = tiles * 256 * sizeof(u64);
+    const size_t old_cap = ctx->dstatus.cap;
+    RET(ensure(ctx, ctx->dstatus, bytes));
+    if (ctx->dstatus.cap != old_cap || ctx->ds_epoch >= 0x3FFFFFu) {
+        CK(cudaMemsetAsync(ctx->dstatus.p, 0, ctx->dstatus.cap, ctx->stream));
+        ctx->ds_epoch = 0;
+    }
+    *epoch = ++ctx->ds_epoch;
+    return IGD_OK;
+}
+
 template <class T>
 static T* P_(Buf& b) {
     return reinterpret_cast<T*>(b.p);
@@ -344,16 +360,15 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         rsort::k_digit_base<<<ndig, rsort::RADIX, 0, ctx->stream>>>(d_hist, P_<u32>(ctx->base));
     }
     const u64 tiles = (n + rsort::TILE - 1) / rsort::TILE;
-    RET(ensure(ctx, ctx->status, tiles * rsort::RADIX * sizeof(u64)));
     for (u32 p = first_pass; p < ndig; p++) {
         if (p * 8 >= max_bits) break;
         bool trivial = false;
         for (int d = 0; d < 256; d++)
             if (h_hist[p * 256 + d] == n) trivial = true;
         if (trivial) continue;
-        CK(cudaMemsetAsync(ctx->status.p, 0, tiles * rsort::RADIX * sizeof(u64), ctx->stream));
-        CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
         rsort::PassParams pp;
+        RET(next_digit_epoch(ctx, tiles, &pp.epoch));
+        CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
         pp.kin = k[cur].p;
         pp.vin = (!ran && vin_first) ? vin_first : v[cur].p;
         ran = true;
@@ -363,7 +378,7 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         pp.shift = p * 8;
         pp.dmask = max_bits >= p * 8 + 8 ? 255u : (1u << (max_bits - p * 8)) - 1u;
         pp.digit_base = P_<u32>(ctx->base) + p * 256;
-        pp.status = P_<u64>(ctx->status);
+        pp.status = P_<u64>(ctx->dstatus);
         pp.tile_ctr = P_<u32>(ctx->ctr);
         {
             KTimer kt(ctx, cls, 2.0 * (kbytes + vbytes) * (double)n);  // read + write the key and the value
@@ -670,10 +685,9 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
             KTimer kt(ctx, KC_MISC, 0);
             rsort::k_digit_base<<<1, rsort::RADIX, 0, ctx->stream>>>(P_<u32>(ctx->hist), P_<u32>(ctx->base));
         }
-        RET(ensure(ctx, ctx->status, ft * fused::RADIX * sizeof(u64)));
-        CK(cudaMemsetAsync(ctx->status.p, 0, ft * fused::RADIX * sizeof(u64), ctx->stream));
-        CK(cudaMemsetAsync(ctx->ctr.p, 0, sizeof(u32), ctx->stream));
         fused::Params fp;
+        RET(next_digit_epoch(ctx, ft, &fp.epoch));
+        CK(cudaMemsetAsync(ctx->ctr.p, 0, sizeof(u32), ctx->stream));
         fp.ev = src_ev;
         fp.n = n_src;
         fp.g = g;
@@ -683,7 +697,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         fp.sync_val = P_<u32>(ctx->syn_v[0]);
         fp.sync_cap = ctx->sync_cap;
         fp.digit_base = P_<u32>(ctx->base);
-        fp.status = P_<u64>(ctx->status);
+        fp.status = P_<u64>(ctx->dstatus);
         fp.tile_ctr = P_<u32>(ctx->ctr);
         fp.kout = ctx->acc_k[1].p;
         fp.kbase = kbase;
@@ -1924,7 +1938,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
     }
     Buf* all[] = {&ctx->owned_events, &ctx->acc_k[0], &ctx->acc_k[1], &ctx->acc_v[0], &ctx->acc_v[1],
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
-                  &ctx->st_in_s,      &ctx->status,   &ctx->stats,    &ctx->hist,     &ctx->base,
+                  &ctx->st_in_s,      &ctx->status,   &ctx->dstatus,  &ctx->stats,    &ctx->hist,     &ctx->base,
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->tcnt,
                   &ctx->tpts,         &ctx->tbits,    &ctx->fdev,     &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,

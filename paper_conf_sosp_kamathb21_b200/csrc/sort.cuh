@@ -96,7 +96,8 @@ struct PassParams {
     u32 shift;
     u32 dmask;              // 255, or fewer bits for the top digit of a masked key (tag mode, A36)
     const u32* digit_base;  // [256] exclusive global offsets of this pass's digits
-    u64* status;            // [n_tiles * 256], zeroed
+    u64* status;            // [n_tiles * 256] digit statuses (ds_make), tagged with `epoch`
+    u32 epoch;              // this pass's tag (1..DS_EPOCH_MAX): no clearing between passes
     u32* tile_ctr;          // zeroed before the pass: tile tickets (the TAIL launch follows the full one)
 };
 
@@ -138,12 +139,12 @@ __device__ __forceinline__ u64 lookback_digit(const PassParams& P, u32 tile, u32
         u64 s[IGD_SORT_LB];
 #pragma unroll
         for (int q = 0; q < IGD_SORT_LB; q++)
-            s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + d) : ST_INC;
+            s[q] = tt - q >= 0 ? ld_relaxed(P.status + (u64)(tt - q) * RADIX + d) : ds_make(ST_INC, P.epoch, 0);
 #pragma unroll
         for (int q = 0; q < IGD_SORT_LB; q++) {
             if (!done) {
-                s[q] = spin_status(P.status + (u64)(tt - q) * RADIX + d, s[q]);
-                excl += s[q] & ST_VAL_MASK;
+                s[q] = ds_spin(P.status + (u64)(tt - q) * RADIX + d, s[q], P.epoch);
+                excl += s[q] & DS_VAL_MASK;
                 done = (s[q] >> 62) == 2;
             }
         }
@@ -220,7 +221,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         for (int j = 0; j < ITEMS; j++)
             if (full || wbase + j * 32 + lane < P.n) atomicAdd(&s_cnt[(u32)(key[j] >> shift) & dmask], 1u);
         __syncthreads();
-        st_relaxed(P.status + (u64)tile * RADIX + t, (tile == 0 ? ST_INC : ST_AGG) | s_cnt[t]);
+        st_relaxed(P.status + (u64)tile * RADIX + t, ds_make(tile == 0 ? ST_INC : ST_AGG, P.epoch, s_cnt[t]));
     }
     u64 excl_early = 0;
     if (IGD_SORT_EARLY && IGD_SORT_LB_EARLY) {
@@ -228,7 +229,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         // published early, so successors' walks stop sooner (ncu r02h: look-back spins were a
         // quarter of the stall samples when it followed the ranking)
         excl_early = lookback_digit(P, tile, t);
-        if (tile > 0) st_relaxed(P.status + (u64)tile * RADIX + t, ST_INC | (excl_early + s_cnt[t]));
+        if (tile > 0) st_relaxed(P.status + (u64)tile * RADIX + t, ds_make(ST_INC, P.epoch, excl_early + s_cnt[t]));
     }
     u32 rank[ITEMS];
     const u32 lt = lanemask_lt();
@@ -266,7 +267,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             c[w] = s_whist[w][d];
             cnt += c[w];
         }
-        if (!IGD_SORT_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, (tile == 0 ? ST_INC : ST_AGG) | cnt);
+        if (!IGD_SORT_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, ds_make(tile == 0 ? ST_INC : ST_AGG, P.epoch, cnt));
         u32 inc = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -298,7 +299,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             excl = excl_early;
         } else if (tile > 0) {
             excl = lookback_digit(P, tile, d);
-            st_relaxed(P.status + (u64)tile * RADIX + d, ST_INC | (excl + cnt));
+            st_relaxed(P.status + (u64)tile * RADIX + d, ds_make(ST_INC, P.epoch, excl + cnt));
         }
         // output position of tile position i with digit d = s_gbase[d] + i (u32 arithmetic wraps
         // back into range): one shared load per written element instead of two
