@@ -318,23 +318,32 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
             m = am[j] & lt;
             const int la = m ? j * 32 + hib(m) : cA;
             const u32 las = m ? (((bsm[j] >> hib(m)) & 1u) ? IGD_SCOPE_BLOCK : IGD_SCOPE_DEVICE) : cAs;
-            m = dm[j] & le;
-            const int ldv = m ? j * 32 + hib(m) : cD;
-            m = bm[j] & le;
-            const int lbv = m ? j * 32 + hib(m) : cB;
             u32 lastW, as;
-            bool dev, blk;
             if (sH >= 0) {
                 lastW = lw >= sH ? wbase + (u32)lw : IGD_NONE32;
                 as = la >= sH ? las : 0u;
-                dev = ldv > sH;
-                blk = lbv > sH;
             } else {
                 lastW = lw >= 0 ? wbase + (u32)lw : st_lastW(carry);
                 as = la >= 0 ? las : st_as(carry);
-                dev = ldv >= 0 || st_dev(carry);
-                blk = lbv >= 0 || st_blk(carry);
             }
+            // the sharing flags: needed up front by the sticky / streaming / last-k modes, else
+            // only for the accesses that reach the queue (after the P2 / P3 / P6 / P4 exits)
+            auto sharing = [&](bool& dev, bool& blk) {
+                u32 mm = dm[j] & le;
+                const int ldv = mm ? j * 32 + hib(mm) : cD;
+                mm = bm[j] & le;
+                const int lbv = mm ? j * 32 + hib(mm) : cB;
+                if (sH >= 0) {
+                    dev = ldv > sH;
+                    blk = lbv > sH;
+                } else {
+                    dev = ldv >= 0 || st_dev(carry);
+                    blk = lbv >= 0 || st_blk(carry);
+                }
+            };
+            constexpr bool EAGER = STK || CARRY || LKO;
+            bool dev = false, blk = false;
+            if (EAGER) sharing(dev, blk);
             const u32 c = Z[j] & 0xFFFFFFu, kind = (Z[j] >> 24) & 0xFu;
             if (CARRY) {
                 cw_lastW = lastW;
@@ -400,6 +409,7 @@ __global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
                         defer_mask = true;
                     }
                 }
+                if (!EAGER) sharing(dev, blk);
                 fl = (same_w ? QF_SAME_W : 0u) | (same_b ? QF_SAME_B : 0u) | (dev ? QF_DEV : 0u) |
                      (defer_mask ? QF_MASK : 0u) |
                      (blk ? QF_BLK : 0u);
