@@ -17,7 +17,10 @@
 
 namespace rsort {
 
-constexpr int THREADS = 256;
+#ifndef IGD_SORT_THREADS
+#define IGD_SORT_THREADS 256  // a multiple of RADIX: threads >= RADIX own one digit in the per-digit steps
+#endif
+constexpr int THREADS = IGD_SORT_THREADS;
 constexpr int WARPS = THREADS / 32;
 #ifndef IGD_SORT_ITEMS
 #define IGD_SORT_ITEMS 16
@@ -34,6 +37,7 @@ constexpr int WARPS = THREADS / 32;
 constexpr int ITEMS = IGD_SORT_ITEMS;
 constexpr int TILE = THREADS * ITEMS;  // 4096
 constexpr int RADIX = 256;
+static_assert(THREADS % RADIX == 0, "one thread per digit in the per-digit steps");
 
 // Exclusive digit bases for every pass from the 4 x 256 histogram.
 __global__ void k_digit_base(const u32* __restrict__ hist, u32* __restrict__ base) {
@@ -124,9 +128,6 @@ constexpr size_t onesweep_smem() {
     return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT);
 }
 
-#ifndef IGD_SORT_LB_EARLY
-#define IGD_SORT_LB_EARLY 0  // 1: look-back before ranking (measured slower: C5 access sort 80.3 -> 86.7 ms, r02j)
-#endif
 // Decoupled look-back for digit d of `tile`: the sum of the digit's counts over all earlier tiles.
 // LB predecessor statuses are requested at once, so a walk back over tiles that have published
 // only their aggregate costs one L2 round trip per LB tiles instead of one per tile.
@@ -194,7 +195,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         }
     }
     for (int i = t; i < WARPS * RADIX; i += THREADS) (&s_whist[0][0])[i] = 0;
-    if (IGD_SORT_EARLY) s_cnt[t] = 0;
+    if (IGD_SORT_EARLY && t < RADIX) s_cnt[t] = 0;
     __syncthreads();
     const u32 tile = s_tile;
     const u32 base = tile * TILE;  // n <= 2^32 - 2^13 (checked by the host)
@@ -221,15 +222,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         for (int j = 0; j < ITEMS; j++)
             if (full || wbase + j * 32 + lane < P.n) atomicAdd(&s_cnt[(u32)(key[j] >> shift) & dmask], 1u);
         __syncthreads();
-        st_relaxed(P.status + (u64)tile * RADIX + t, ds_make(tile == 0 ? ST_INC : ST_AGG, P.epoch, s_cnt[t]));
-    }
-    u64 excl_early = 0;
-    if (IGD_SORT_EARLY && IGD_SORT_LB_EARLY) {
-        // the look-back right after the aggregate, before ranking: this tile's inclusive prefix is
-        // published early, so successors' walks stop sooner (ncu r02h: look-back spins were a
-        // quarter of the stall samples when it followed the ranking)
-        excl_early = lookback_digit(P, tile, t);
-        if (tile > 0) st_relaxed(P.status + (u64)tile * RADIX + t, ds_make(ST_INC, P.epoch, excl_early + s_cnt[t]));
+        if (t < RADIX) st_relaxed(P.status + (u64)tile * RADIX + t, ds_make(tile == 0 ? ST_INC : ST_AGG, P.epoch, s_cnt[t]));
     }
     u32 rank[ITEMS];
     const u32 lt = lanemask_lt();
@@ -255,30 +248,33 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         __syncwarp();
     }
     __syncthreads();
-    // per digit: tile count, exclusive scan over digits, then every warp's base for the digit
-    // (tile exclusive + earlier warps) in place of its count -- one shared load per rank below
-    u32 cnt, tile_excl;
-    {
-        const u32 d = t;  // THREADS == RADIX
-        u32 c[WARPS];
-        cnt = 0;
+    // per digit (threads < RADIX): tile count, exclusive scan over digits, then every warp's base
+    // for the digit (tile exclusive + earlier warps) in place of its count -- one shared load per
+    // rank below
+    constexpr int DW = RADIX / 32;  // warps that own digits
+    u32 cnt = 0, tile_excl = 0, inc = 0;
+    u32 c[WARPS];
+    const u32 d = t;
+    if (t < RADIX) {
 #pragma unroll
         for (int w = 0; w < WARPS; w++) {
             c[w] = s_whist[w][d];
             cnt += c[w];
         }
         if (!IGD_SORT_EARLY) st_relaxed(P.status + (u64)tile * RADIX + d, ds_make(tile == 0 ? ST_INC : ST_AGG, P.epoch, cnt));
-        u32 inc = cnt;
+        inc = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             u32 x = __shfl_up_sync(IGD_FULL, inc, o);
             if (lane >= (u32)o) inc += x;
         }
         if (lane == 31) s_wsum[warp] = inc;
-        __syncthreads();
+    }
+    __syncthreads();
+    if (t < RADIX) {
         u32 wpre = 0;
 #pragma unroll
-        for (int w = 0; w < WARPS; w++)
+        for (int w = 0; w < DW; w++)
             if ((u32)w < warp) wpre += s_wsum[w];
         tile_excl = wpre + inc - cnt;
         u32 run = tile_excl;
@@ -287,17 +283,11 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             s_whist[w][d] = run;
             run += c[w];
         }
-    }
-    // Decoupled look-back for this digit: LB predecessor statuses are requested at once, so a
-    // walk back over tiles that have published only their aggregate costs one L2 round trip per
-    // LB tiles instead of one per tile (C5: 127 -> 118 ms over 4 passes with LB = 4; issuing the
-    // first requests before the tile-local reorder to overlap them measured no further gain)
-    {
-        const u32 d = t;
+        // Decoupled look-back for this digit: LB predecessor statuses are requested at once, so a
+        // walk back over tiles that have published only their aggregate costs one L2 round trip
+        // per LB tiles instead of one per tile (C5: 127 -> 118 ms over 4 passes with LB = 4)
         u64 excl = 0;
-        if (IGD_SORT_EARLY && IGD_SORT_LB_EARLY) {
-            excl = excl_early;
-        } else if (tile > 0) {
+        if (tile > 0) {
             excl = lookback_digit(P, tile, d);
             st_relaxed(P.status + (u64)tile * RADIX + d, ds_make(ST_INC, P.epoch, excl + cnt));
         }
