@@ -16,14 +16,6 @@ extern "C" {
 int igd_debug_radix_sort(igd_ctx* ctx, uint32_t* d_keys, uint32_t* d_vals, uint64_t n, uint32_t max_bits, int mode,
                          float* ms);
 
-/* The wide-digit passes of the access sort (csrc/sortw.cuh) alone: n (u32 key, u64 value)
-   pairs in DEVICE memory sorted stably, in place, by key bits [8, 8 + w1 + w2) as two passes of
-   w1 and w2 bits (1 <= w1, w2 <= 11; bits 0..7 and above are ignored: in the detect pipeline the
-   fused ingest pass has already sorted by bits 0..7).  *ms = device time of the two passes.
-   Errors: IGD_EINVAL (bad widths, NULL pointers with n > 0), IGD_ETOOBIG (n >= 2^32 - 2^18). */
-int igd_debug_wide_sort(igd_ctx* ctx, uint32_t* d_keys, uint64_t* d_vals, uint64_t n, uint32_t w1, uint32_t w2,
-                        float* ms);
-
 /* a2 / a3 tables of the last igd_detect (single GPU).  sizes[0..3] = entities E, sync records,
    threads T, lock change points; then (any pointer may be NULL) off[E+1] = CSR offsets of the
    entity-sorted sync timestamps ts[n_sync] (entity layout: csrc/common.cuh KeySpace), and when

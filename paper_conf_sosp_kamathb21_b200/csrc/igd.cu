@@ -21,7 +21,6 @@
 #include "ingest.cuh"
 #include "lastk.cuh"
 #include "sort.cuh"
-#include "sortw.cuh"
 #include "shard.cuh"
 #include "sync.cuh"
 #include <dlfcn.h>
@@ -147,7 +146,6 @@ struct igd_ctx {
 
     Buf acc_k[2], acc_v[2], syn_k[2], syn_v[2];
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
-    Buf histw;          // wide-digit access sort (sortw.cuh): 2 x 2048 histogram, 2 x 2048 bases
     Buf dstatus;        // digit statuses of the radix passes, epoch-tagged (never cleared per pass)
     u32 ds_epoch = 0;   // tag of the last radix pass
     Buf off, ldesc, gtab, tcnt, tpts, tbits, fdev, skipb;
@@ -397,69 +395,6 @@ static int radix_sort(igd_ctx* ctx, int cls, Buf* k, Buf* v, u64 n, const u32* d
         CK(cudaMemcpyAsync(v[cur].p, vin_first, n * vbytes, cudaMemcpyDeviceToDevice, ctx->stream));
     *out_cur = cur;
     return IGD_OK;
-}
-
-// The access sort after the fused digit-0 pass as two wide-digit passes (sortw.cuh): digit 1 =
-// bits [8, 8 + w1), digit 2 = bits [8 + w1, 8 + w1 + w2), w1, w2 <= 11; keys and values in
-// acc_*[1] (the fused pass's output), result back in acc_*[1].  Digit bases from k_hist_w +
-// k_digit_base_w (launched after the fused pass).
-static int radix_sort_w(igd_ctx* ctx, u64 n, u32 w1, u32 w2, int* out_cur) {
-    int cur = 1;
-    *out_cur = cur;
-    if (n <= 1) return IGD_OK;
-    if (n > 0xFFFFFFFFull - 2ull * rsortw::CHUNK) return IGD_ETOOBIG;  // 32-bit chunk indexing
-    const u64 chunks = (n + rsortw::CHUNK - 1) / rsortw::CHUNK;
-    for (u32 p = 0; p < 2; p++) {
-        rsortw::Params pp;
-        RET(next_digit_epoch(ctx, chunks * (rsortw::RADIX / 256), &pp.epoch));
-        CK(cudaMemsetAsync(P_<u32>(ctx->ctr), 0, sizeof(u32), ctx->stream));
-        pp.kin = P_<u32>(ctx->acc_k[cur]);
-        pp.vin = P_<u64>(ctx->acc_v[cur]);
-        pp.kout = P_<u32>(ctx->acc_k[cur ^ 1]);
-        pp.vout = P_<u64>(ctx->acc_v[cur ^ 1]);
-        pp.n = (u32)n;
-        pp.shift = p == 0 ? 8u : 8u + w1;
-        pp.dmask = (1u << (p == 0 ? w1 : w2)) - 1u;
-        pp.digit_base = P_<u32>(ctx->histw) + 2 * rsortw::RADIX + p * rsortw::RADIX;
-        pp.status = P_<u64>(ctx->dstatus);
-        pp.tile_ctr = P_<u32>(ctx->ctr);
-        {
-            KTimer kt(ctx, KC_SORT_ACC, 24.0 * (double)n);  // read + write the key and the value
-            rsortw::k_sweep_w<<<(unsigned)chunks, rsortw::THREADS, rsortw::SMEM, ctx->stream>>>(pp);
-        }
-        CK(cudaGetLastError());
-        cur ^= 1;
-    }
-    *out_cur = cur;
-    return IGD_OK;
-}
-
-// Wide-digit split of the access keys after the fused digit-0 pass, from pass 0's 8-bit digit
-// histogram (host copy): used when three 8-bit passes would run (digits 1..3 non-trivial) and
-// the keys fit in 30 bits, i.e. 17..22 bits remain above digit 0.  Returns false otherwise.
-#ifndef IGD_SORT_WIDE
-#define IGD_SORT_WIDE 1
-#endif
-static bool wide_split(const u32* h_hist_acc, u64 n, u32* w1, u32* w2) {
-    if (!IGD_SORT_WIDE || n < 2) return false;
-    static int env = -1;
-    if (env < 0) {
-        const char* e = getenv("IGD_SORT_WIDE");
-        env = e ? atoi(e) : 1;
-    }
-    if (!env) return false;
-    for (int p = 1; p < 4; p++)
-        for (int d = 0; d < 256; d++)
-            if (h_hist_acc[p * 256 + d] == n) return false;  // a trivial digit: fewer 8-bit passes
-    int top = -1;
-    for (int d = 0; d < 256; d++)
-        if (h_hist_acc[3 * 256 + d]) top = d;
-    const u32 bits = 24 + bits_needed((u64)top);
-    if (top < 0 || bits > 30) return false;
-    const u32 rem = bits - 8;  // 17..22
-    *w1 = (rem + 1) / 2;
-    *w2 = rem - *w1;
-    return true;
 }
 
 // a6 kernel instantiation: sharded payload (MV), kernel boundaries (KB), paper-fidelity bits
@@ -725,9 +660,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         return IGD_EINVAL;
     }
     const u64 kbase = key64 ? (ctx->h_stats[0] & ~255ull) : 0;  // low digit unchanged: pass 0's histogram holds
-    // a5 with wide digits (sortw.cuh): 8 + w1 + w2 bits instead of four 8-bit digits
-    u32 ww1 = 0, ww2 = 0;
-    const bool wide = FUSED && !key64 && !TG && wide_split(ctx->h_hist, n_acc, &ww1, &ww2);
     if (key64) {
         if (!FUSED) {
             ctx->err = "word spans >= 2^32 words need the fused ingest pipeline (IGD_FUSED=1)";
@@ -835,23 +767,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 8);
         ingest::k_hist_keys<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[1]), (u32)n_acc, P_<u32>(ctx->hist), 1,
                                                          (u32)((1ull << TG) - 1));
-    }
-    if (wide) {
-        // the two wide digits' histograms over the keys the fused pass wrote, then their bases
-        RET(ensure(ctx, ctx->histw, 4 * rsortw::RADIX * sizeof(u32)));
-        CK(cudaMemsetAsync(ctx->histw.p, 0, 2 * rsortw::RADIX * sizeof(u32), ctx->stream));
-        {
-            KTimer kt(ctx, KC_INGEST, 4.0 * (double)n_acc);
-            const unsigned hb = (unsigned)std::min<u64>((n_acc / 4 + 255) / 256 + 1, (u64)sms * 4);
-            rsortw::k_hist_w<<<hb, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[1]), (u32)n_acc, 8u, (1u << ww1) - 1u,
-                                                          8u + ww1, (1u << ww2) - 1u, P_<u32>(ctx->histw));
-        }
-        {
-            KTimer kt(ctx, KC_MISC, 0);
-            rsortw::k_digit_base_w<<<2, rsortw::RADIX / 2, 0, ctx->stream>>>(
-                P_<u32>(ctx->histw), P_<u32>(ctx->histw) + 2 * rsortw::RADIX);
-        }
-        CK(cudaGetLastError());
     }
     if (FUSED && n_sync > 0) {
         // sync-key digit histograms over the records the fused pass wrote (trace order)
@@ -986,8 +901,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     if (key64)
         RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist) + 2048, h_hist64.data(),
                        bits_needed(ctx->h_stats[1] - kbase), &acur, vbytes, 1, 1, nullptr, 8));
-    else if (wide)
-        RET(radix_sort_w(ctx, n_acc, ww1, ww2, &acur));
     else
         RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc,
                        TG ? TG : 32u, &acur, vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0,
@@ -1686,7 +1599,6 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
     cudaFuncSetAttribute(fused::k_ingest_sort0<true, u64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)fused::smem_bytes<u64>());
     set_pass_smem<u32>();
-    cudaFuncSetAttribute(rsortw::k_sweep_w, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rsortw::SMEM);
     set_pass_smem<u64>();
     set_pass_smem<uint4>();
     set_pass_smem<u64, u64>();
@@ -2026,7 +1938,7 @@ void igd_ctx_destroy(igd_ctx* ctx) {
     }
     Buf* all[] = {&ctx->owned_events, &ctx->acc_k[0], &ctx->acc_k[1], &ctx->acc_v[0], &ctx->acc_v[1],
                   &ctx->syn_k[0],     &ctx->syn_k[1], &ctx->syn_v[0], &ctx->syn_v[1], &ctx->st_in_a,
-                  &ctx->st_in_s,      &ctx->status,   &ctx->dstatus,  &ctx->stats,    &ctx->hist,     &ctx->base,     &ctx->histw,
+                  &ctx->st_in_s,      &ctx->status,   &ctx->dstatus,  &ctx->stats,    &ctx->hist,     &ctx->base,
                   &ctx->ctr,          &ctx->off,      &ctx->ldesc,    &ctx->gtab,     &ctx->tcnt,
                   &ctx->tpts,         &ctx->tbits,    &ctx->fdev,     &ctx->skipb,    &ctx->rep_raw,  &ctx->rep_k[0], &ctx->rep_k[1],
                   &ctx->rep_v[0],     &ctx->rep_v[1], &ctx->rep_out,  &ctx->rep_ctr,  &ctx->rep_hist,
@@ -2155,45 +2067,6 @@ int igd_debug_radix_sort(igd_ctx* ctx, uint32_t* d_keys, uint32_t* d_vals, uint6
     if (rc != IGD_OK) return rc;
     CK(cudaMemcpyAsync(d_keys, ctx->acc_k[cur].p, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
     CK(cudaMemcpyAsync(d_vals, ctx->acc_v[cur].p, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
-    CK(cudaStreamSynchronize(ctx->stream));
-    return IGD_OK;
-}
-
-int igd_debug_wide_sort(igd_ctx* ctx, uint32_t* d_keys, uint64_t* d_vals, uint64_t n, uint32_t w1, uint32_t w2,
-                        float* ms) {
-    if (!ctx || w1 < 1 || w2 < 1 || w1 > (u32)rsortw::RBITS || w2 > (u32)rsortw::RBITS || (n && (!d_keys || !d_vals)))
-        return IGD_EINVAL;
-    if (n > 0xFFFFFFFFull - 2ull * rsortw::CHUNK) return IGD_ETOOBIG;
-    cudaSetDevice(ctx->device);
-    for (int b = 0; b < 2; b++) {
-        RET(ensure(ctx, ctx->acc_k[b], (n + 1) * sizeof(u32)));
-        RET(ensure(ctx, ctx->acc_v[b], (n + 1) * sizeof(u64)));
-    }
-    RET(ensure(ctx, ctx->histw, 4 * rsortw::RADIX * sizeof(u32)));
-    RET(ensure(ctx, ctx->ctr, 64));
-    CK(cudaMemcpyAsync(ctx->acc_k[1].p, d_keys, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
-    CK(cudaMemcpyAsync(ctx->acc_v[1].p, d_vals, n * 8, cudaMemcpyDeviceToDevice, ctx->stream));
-    CK(cudaMemsetAsync(ctx->histw.p, 0, 2 * rsortw::RADIX * sizeof(u32), ctx->stream));
-    const int sms = sm_count(ctx);
-    rsortw::k_hist_w<<<sms * 4, 256, 0, ctx->stream>>>(P_<u32>(ctx->acc_k[1]), (u32)n, 8u, (1u << w1) - 1u, 8u + w1,
-                                                      (1u << w2) - 1u, P_<u32>(ctx->histw));
-    rsortw::k_digit_base_w<<<2, rsortw::RADIX / 2, 0, ctx->stream>>>(P_<u32>(ctx->histw),
-                                                                     P_<u32>(ctx->histw) + 2 * rsortw::RADIX);
-    CK(cudaGetLastError());
-    cudaEvent_t a, b;
-    cudaEventCreate(&a);
-    cudaEventCreate(&b);
-    cudaEventRecord(a, ctx->stream);
-    int cur = 1;
-    const int rc = radix_sort_w(ctx, n, w1, w2, &cur);
-    cudaEventRecord(b, ctx->stream);
-    cudaEventSynchronize(b);
-    if (ms) cudaEventElapsedTime(ms, a, b);
-    cudaEventDestroy(a);
-    cudaEventDestroy(b);
-    if (rc != IGD_OK) return rc;
-    CK(cudaMemcpyAsync(d_keys, ctx->acc_k[cur].p, n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
-    CK(cudaMemcpyAsync(d_vals, ctx->acc_v[cur].p, n * 8, cudaMemcpyDeviceToDevice, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     return IGD_OK;
 }

@@ -153,9 +153,9 @@ def test_wide_keys_vs_oracle(det, seed, n, nb, bd, bits):
 
 @pytest.mark.parametrize("seed,n,nb,bd,bits,words", [(51, 300_000, 16, 128, 30, 3_000), (52, 100_003, 4, 64, 25, 500),
                                                      (53, 250_000, 8, 96, 27, 60_000), (54, 70_001, 2, 64, 29, 20)])
-def test_wide_digit_sort_vs_oracle(det, seed, n, nb, bd, bits, words):
-    # words spread over 2^25..2^30 words: the u32-key path with the access sort as two wide-digit
-    # passes after the fused digit-0 pass (sortw.cuh), several 32K-access chunks, ragged tails
+def test_30bit_word_span_vs_oracle(det, seed, n, nb, bd, bits, words):
+    # words spread over 2^25..2^30 words (C5's span): the u32-key path with every radix digit
+    # non-trivial, many tiles, ragged tails
     w = [20, 18, 10, 4, 3, 8, 3, 3, 1, 1, 1, 1]
     ev, nb, bd = _fast_random(seed, n, words, nb, bd, w, lock_words=12)
     rng = np.random.default_rng(seed)
@@ -166,7 +166,7 @@ def test_wide_digit_sort_vs_oracle(det, seed, n, nb, bd, bits, words):
     spread[0] = 0x3FF  # digits 1..3 all occupied by more than one bin
     spread[-1] = (1 << bits) - 1
     ev["addr"][acc] = (spread[inv] << np.uint64(2)) | (ev["addr"][acc] & np.uint64(3))
-    assert_same(det, ev, nb, bd, f"wide-digit seed {seed}")
+    assert_same(det, ev, nb, bd, f"30-bit span seed {seed}")
 
 
 @pytest.mark.parametrize("bad_at", [0, 5000, 99_999])

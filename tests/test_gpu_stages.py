@@ -53,47 +53,6 @@ def test_radix_sort_stable(det, mode, n, dist):
     assert np.array_equal(vs, vals[order])
 
 
-def gpu_wide_sort(det, keys, vals, w1, w2):
-    import torch
-
-    import paper_conf_sosp_kamathb21_b200 as igd
-
-    lib = igd.load_library()
-    lib.igd_debug_wide_sort.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
-                                        ctypes.c_uint32, ctypes.c_uint32, ctypes.POINTER(ctypes.c_float)]
-    k = torch.from_numpy(keys.view(np.int32)).cuda()
-    v = torch.from_numpy(vals.view(np.int64)).cuda()
-    ms = ctypes.c_float()
-    rc = lib.igd_debug_wide_sort(det.ctx, k.data_ptr(), v.data_ptr(), len(keys), w1, w2, ctypes.byref(ms))
-    assert rc == 0
-    return k.cpu().numpy().view(np.uint32), v.cpu().numpy().view(np.uint64), ms.value
-
-
-# a5 wide-digit passes (csrc/sortw.cuh): stable by bits [8, 8 + w1 + w2) == numpy stable argsort;
-# sizes span one sub-tile, one chunk (32768 keys) and several chunks with ragged tails
-@pytest.mark.parametrize("n,dist,w1,w2", [(1, "u", 11, 11), (5, "u", 11, 11), (4095, "u", 11, 11),
-                                          (32_768, "u", 11, 11), (32_769, "u", 9, 8), (1_000_003, "u", 11, 11),
-                                          (777_777, "skew", 11, 10), (300_000, "const", 11, 11),
-                                          (2_000_001, "hi", 11, 11), (500_000, "few", 10, 10)])
-def test_wide_sort_stable(det, n, dist, w1, w2):
-    rng = np.random.default_rng(n + 7 * w1 + w2)
-    if dist == "u":
-        keys = rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
-    elif dist == "skew":   # Zipf-like hot keys
-        keys = (rng.zipf(1.3, n) % (1 << 30)).astype(np.uint32)
-    elif dist == "const":
-        keys = np.full(n, 0x2345678, np.uint32)
-    elif dist == "few":    # a handful of distinct words
-        keys = rng.choice(np.array([7 << 8, 1 << 20, 3 << 27, 5], np.uint32), n)
-    else:                  # only the top wide digit varies
-        keys = (rng.integers(0, 2048, n).astype(np.uint32) << 19)
-    vals = rng.integers(0, 1 << 63, n, dtype=np.uint64)
-    ks, vs, _ = gpu_wide_sort(det, keys, vals, w1, w2)
-    order = np.argsort((keys >> 8) & np.uint32((1 << (w1 + w2)) - 1), kind="stable")
-    assert np.array_equal(ks, keys[order])
-    assert np.array_equal(vs, vals[order])
-
-
 # ---------------- a2: sync-epoch tables (CSR of per-entity timestamp lists) ----------------
 def _entities(ev, nb, bd):
     """Host restatement of the a2 record layout (csrc/common.cuh KeySpace): one (entity,
