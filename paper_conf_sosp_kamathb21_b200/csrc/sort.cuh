@@ -34,6 +34,9 @@ constexpr int WARPS = THREADS / 32;
 #ifndef IGD_SORT_LB
 #define IGD_SORT_LB 4
 #endif
+#ifndef IGD_SORT_GATHER
+#define IGD_SORT_GATHER 1  // output by gathering through a scattered source-position array (see below)
+#endif
 constexpr int ITEMS = IGD_SORT_ITEMS;
 constexpr int TILE = THREADS * ITEMS;  // 4096
 constexpr int RADIX = 256;
@@ -122,10 +125,11 @@ __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     }
 }
 
-// Dynamic shared memory of k_onesweep<VT, TAIL, KT>: staged keys, staged values.
+// Dynamic shared memory of k_onesweep<VT, TAIL, KT>: staged keys, staged values (+ the u16
+// source position of every output slot, IGD_SORT_GATHER).
 template <typename VT, typename KT = u32>
 constexpr size_t onesweep_smem() {
-    return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT);
+    return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT) + (IGD_SORT_GATHER ? (size_t)TILE * 2 : 0);
 }
 
 // Decoupled look-back for digit d of `tile`: the sum of the digit's counts over all earlier tiles.
@@ -214,6 +218,10 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         for (int j = 0; j < ITEMS; j++) {
             const u32 i = wbase + j * 32 + lane;
             key[j] = i < P.n ? __ldcs(kin + i) : KT(0);
+            if (IGD_SORT_GATHER) {  // the tail tile is staged by plain loads
+                s_k[wofs + j * 32 + lane] = key[j];
+                s_v[wofs + j * 32 + lane] = i < P.n ? __ldcs(vin + i) : VT{};
+            }
         }
     }
     if (IGD_SORT_EARLY) {
@@ -296,6 +304,34 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         s_gbase[d] = P.digit_base[d] + (u32)excl - tile_excl;
     }
     __syncthreads();
+#if IGD_SORT_GATHER
+    // Output by gathering: every input scatters only its tile position's source index (u16), and
+    // output slot i then reads its key and value from the staged input -- no key / value reorder
+    // buffers, no value registers, one barrier; 2 fewer shared-memory round trips per element
+    // than reordering keys and values through shared memory (the MIO pipe bounds this kernel)
+    {
+        u16* s_src = reinterpret_cast<u16*>(s_dyn + TILE * sizeof(KT) + TILE * sizeof(VT));
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const u32 d = (u32)(key[j] >> shift) & dmask;
+            if (full || wbase + j * 32 + lane < P.n) s_src[rank[j] + s_whist[warp][d]] = (u16)(wofs + j * 32 + lane);
+        }
+        __syncthreads();
+        if (full) mbar_wait(&s_mbar[1], 0);
+        const u32 tile_n = full ? (u32)TILE : P.n - base;
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            const u32 i = t + k * THREADS;
+            if (full || i < tile_n) {
+                const u32 src = s_src[i];
+                const KT kk = s_k[src];
+                const u32 o = s_gbase[(u32)(kk >> shift) & dmask] + i;
+                __stcs(kout + o, kk);
+                __stcs(vout + o, s_v[src]);
+            }
+        }
+    }
+#else
     // keys: reorder in shared memory (rank[] becomes the tile position), write digit runs
 #pragma unroll
     for (int j = 0; j < ITEMS; j++) {
@@ -340,6 +376,7 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             __stcs(vout + (s_gbase[d] + i), s_v[i]);
         }
     }
+#endif
 }
 
 }  // namespace rsort
