@@ -148,6 +148,13 @@ struct igd_ctx {
     Buf st_in_a, st_in_s, status, stats, hist, base, ctr;
     Buf dstatus;        // digit statuses of the radix passes, epoch-tagged (never cleared per pass)
     u32 ds_epoch = 0;   // tag of the last radix pass
+    // a2 / a3 run on a side stream concurrently with the a5 access sort (SideSection): their own
+    // scan / radix workspaces, swapped in for the section
+    cudaStream_t side = nullptr;
+    cudaEvent_t side_ev[2] = {nullptr, nullptr};
+    Buf sw_base, sw_dstatus, sw_status, sw_ctr;
+    u32 sw_epoch = 0;
+    bool in_side = false;
     Buf off, ldesc, gtab, tcnt, tpts, tbits, fdev, skipb;
     Buf rep_raw, rep_k[2], rep_v[2], rep_out, rep_ctr, rep_hist;
     u64 sync_cap = 0;
@@ -320,6 +327,61 @@ static void mark(igd_ctx* ctx, int stage) {
         ctx->nvtx_depth++;
     }
 }
+
+// a2 / a3 concurrently with a5: the host enqueues the access sort on the context stream, then
+// runs the a2 / a3 code with the side stream (forked from the context stream) as ctx->stream and
+// the scan / radix workspaces swapped for the side copies, so the two sorts never share a tile
+// counter, digit-status buffer or digit-base table; end() (or the destructor on an error path)
+// swaps back and joins: the context stream waits for everything the section enqueued.
+struct SideSection {
+    igd_ctx* ctx;
+    bool on = false;
+    explicit SideSection(igd_ctx* c) : ctx(c) {}
+    void swap_all() {
+        std::swap(ctx->stream, ctx->side);
+        std::swap(ctx->base, ctx->sw_base);
+        std::swap(ctx->dstatus, ctx->sw_dstatus);
+        std::swap(ctx->status, ctx->sw_status);
+        std::swap(ctx->ctr, ctx->sw_ctr);
+        std::swap(ctx->ds_epoch, ctx->sw_epoch);
+        ctx->in_side = !ctx->in_side;
+    }
+    // the fork point: recorded on the context stream before the work the section overlaps
+    bool use = false;
+    int fork(bool want) {
+        use = want && ctx->side;
+        if (use) CK(cudaEventRecord(ctx->side_ev[0], ctx->stream));
+        return IGD_OK;
+    }
+    int begin() {
+        if (!use) return IGD_OK;
+        CK(cudaStreamWaitEvent(ctx->side, ctx->side_ev[0], 0));
+        swap_all();
+        on = true;
+        // the side copies of the fixed-size workspaces (the others grow on demand)
+        RET(ensure(ctx, ctx->ctr, 64));
+        RET(ensure(ctx, ctx->base, 8 * 256 * sizeof(u32)));
+        return IGD_OK;
+    }
+    int end() {
+        if (!on) return IGD_OK;
+        on = false;
+        cudaError_t e = cudaEventRecord(ctx->side_ev[1], ctx->stream);  // the side stream
+        swap_all();
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(ctx->stream, ctx->side_ev[1], 0);
+        if (e != cudaSuccess) {
+            ctx->err = std::string("side stream join: ") + cudaGetErrorString(e);
+            return IGD_ECUDA;
+        }
+        return IGD_OK;
+    }
+    ~SideSection() {
+        if (on) {
+            cudaStreamSynchronize(ctx->stream);  // error path: the side work must not outlive its buffers' owner
+            end();
+        }
+    }
+};
 
 // One radix pass over n keys: the full tiles, then (if any) the partial last tile (same tile
 // counter: the tail's ticket is the last tile).
@@ -797,6 +859,32 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         memcpy(h_hist64.data(), ctx->h_hist + 2048, 2048 * sizeof(u32));
     }
 
+    // the a2 / a3 stages run concurrently with a5 (SideSection): their stage marks are taken
+    // here on the context stream, so the "a5" stage time covers a2 + a3 + a5 (the per-kernel
+    // class times still separate them)
+    mark(ctx, 2);
+    mark(ctx, 3);
+    // Overlap only when the lock replay is substantial (>= 1 lock event per 1024 events, e.g. the
+    // sync-heavy C5: 223 -> 216 ms): the overlapped kernels take SM slots from the sort, so for a
+    // light a2 / a3 (default C5: 0.05 % lock events) the gain is ~1 ms and the sort runs 5 % slower
+    // (r02s9); IGD_SIDE_STREAM=0 / 1 forces it off / on.
+    static int side_env = -2;
+    if (side_env == -2) {
+        const char* e = getenv("IGD_SIDE_STREAM");
+        side_env = e ? atoi(e) : -1;
+    }
+    SideSection side(ctx);
+    RET(side.fork(side_env >= 0 ? side_env != 0 : n_lock * 1024 >= n_src));
+    // ---------------- a5: accesses sorted by word, stable ----------------
+    int acur = 0;
+    if (key64)
+        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist) + 2048, h_hist64.data(),
+                       bits_needed(ctx->h_stats[1] - kbase), &acur, vbytes, 1, 1, nullptr, 8));
+    else
+        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc,
+                       TG ? TG : 32u, &acur, vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0,
+                       (SH && !SPLIT) ? ctx->sh_rec : nullptr));
+    RET(side.begin());
     // ---------------- a2: sync records sorted by entity, CSR offsets ----------------
     int scur = 0;
     ctx->last_nsync = 0;
@@ -806,7 +894,6 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
     // the check's 32-byte timestamp probes may read up to 64 entries past the last list: defined
     // values there (they are masked out of every decision; compute-sanitizer initcheck is clean)
     CK(cudaMemsetAsync(P_<u32>(ctx->syn_v[scur]) + n_sync, 0xFF, 64 * sizeof(u32), ctx->stream));
-    mark(ctx, 2);
     RET(ensure(ctx, ctx->off, ((u64)ks.E + 2) * sizeof(u32)));
     {
         u64 work = (u64)ks.E + 1;
@@ -895,16 +982,7 @@ static int detect_impl(igd_ctx* ctx, u64* n_out) {
         lv.tbits = P_<u32>(ctx->tbits);
         ctx->last_npts = tot;
     }
-    mark(ctx, 3);
-    // ---------------- a5: accesses sorted by word, stable ----------------
-    int acur = 0;
-    if (key64)
-        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist) + 2048, h_hist64.data(),
-                       bits_needed(ctx->h_stats[1] - kbase), &acur, vbytes, 1, 1, nullptr, 8));
-    else
-        RET(radix_sort(ctx, KC_SORT_ACC, ctx->acc_k, ctx->acc_v, n_acc, P_<u32>(ctx->hist), h_hist_acc,
-                       TG ? TG : 32u, &acur, vbytes, FUSED ? 1 : 0, FUSED ? 1 : 0,
-                       (SH && !SPLIT) ? ctx->sh_rec : nullptr));
+    RET(side.end());
     ctx->last_acur = acur;
     ctx->last_scur = scur;
     ctx->last_nsync = n_sync;
@@ -1609,6 +1687,17 @@ int igd_ctx_create(igd_ctx** out, int cuda_device, void* cuda_stream, int nranks
         return IGD_ENOMEM;
     }
     for (int i = 0; i <= IGD_N_STAGES; i++) cudaEventCreate(&ctx->ev[i]);
+    // the side stream at the greatest priority: its small a2 / a3 kernels take SM slots as the
+    // access sort's CTAs retire instead of queueing behind all of the sort's passes
+    int prio_lo = 0, prio_hi = 0;
+    cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+    if (cudaStreamCreateWithPriority(&ctx->side, cudaStreamNonBlocking, prio_hi) != cudaSuccess ||
+        cudaEventCreateWithFlags(&ctx->side_ev[0], cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&ctx->side_ev[1], cudaEventDisableTiming) != cudaSuccess) {
+        (void)cudaGetLastError();
+        igd_ctx_destroy(ctx);
+        return IGD_ECUDA;
+    }
     for (int i = 0; i < 2 * kMaxTimed; i++) cudaEventCreate(&ctx->kev[i]);
     for (int i = 0; i < IGD_N_STAGES; i++) ctx->stage_ms[i] = 0.f;
     for (int i = 0; i < IGD_N_KCLASS; i++) {
@@ -1946,9 +2035,16 @@ void igd_ctx_destroy(igd_ctx* ctx) {
                   &ctx->cl_small,     &ctx->cl_mat,   &ctx->cl_recv,  &ctx->cl_sidx,  &ctx->cl_sev,
                   &ctx->cl_nrep,      &ctx->cl_rep,   &ctx->gkb,      &ctx->seg_rep,  &ctx->lk_state,
                   &ctx->str_sidx,     &ctx->str_sev,  &ctx->str_carry[0], &ctx->str_carry[1], &ctx->str_rec,
-                  &ctx->str_co,       &ctx->str_flags};
+                  &ctx->str_co,       &ctx->str_flags, &ctx->sw_base, &ctx->sw_dstatus, &ctx->sw_status,
+                  &ctx->sw_ctr};
     for (Buf* b : all) buf_free(ctx, *b);
     cudaStreamSynchronize(ctx->stream);
+    if (ctx->side) {
+        cudaStreamSynchronize(ctx->side);
+        cudaStreamDestroy(ctx->side);
+    }
+    for (cudaEvent_t e : ctx->side_ev)
+        if (e) cudaEventDestroy(e);
     cudaFreeHost(ctx->h_stats);
     cudaFreeHost(ctx->h_hist);
     cudaFreeHost(ctx->h_small);
