@@ -29,7 +29,7 @@ namespace check {
 #define IGD_C4_ITEMS 4
 #endif
 #ifndef IGD_C4_MINB
-#define IGD_C4_MINB 6
+#define IGD_C4_MINB 7  // default mode: 32 registers (36 B of spills), 7 CTAs/SM: C5 check 53.5 -> 50.5 ms (r02s12; 8 equal, 5-6 slower)
 #endif
 #ifndef IGD_C4_MBAR
 #define IGD_C4_MBAR 1  // warps wait for the tile prefix on an mbarrier (0: poll a shared flag)
@@ -90,8 +90,10 @@ __device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, co
 // KT: u32 word keys (low 32 bits; spans < 2^32 words) or u64 keys (word - wbase, a4's wide path)
 // FID: paper-fidelity bits -- 1 = Fig. 4-width synchronization IDs (reading A33), 2 = sticky
 // sharing flags gate P3-P5 as Table 2 is written (reading A35), 4 = last-k state out (A37)
+// the default mode (single GPU, no fidelity bits, u32 keys) at IGD_C4_MINB CTAs per SM; the
+// other instantiations carry more state and spill more at 32 registers: 6 CTAs per SM (40)
 template <bool MV, bool KB, int FID, bool GEO2, typename KT = u32>
-__global__ void __launch_bounds__(C4_THREADS, IGD_C4_MINB) k_check4(Params P) {
+__global__ void __launch_bounds__(C4_THREADS, (!MV && FID == 0 && sizeof(KT) == 4) ? IGD_C4_MINB : 6) k_check4(Params P) {
     constexpr bool WRAP = (FID & 1) != 0;
     constexpr bool STK = (FID & 2) != 0;
     constexpr bool LKO = (FID & 4) != 0;  // last-k mode (A37): scan state out, decisions in k_lastk
