@@ -280,12 +280,9 @@ def run_sharded(args, fam, rank, world, local):
     e1 = torch.cuda.Event(enable_timing=True)
     kstats, launches = {}, 0
     e0.record(det.stream)
-    for _ in range(args.steps):
-        nrep = det.detect(timing=True)
+    for _ in range(args.steps):  # uninstrumented
+        nrep = det.detect()
         launches += det.launch_count()
-        for k, (c, ms_, b) in det.kernel_stats().items():
-            c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
-            kstats[k] = (c0 + c, m0 + ms_, b0 + b)
     e1.record(det.stream)
     torch.cuda.synchronize()
     dist.barrier()
@@ -296,6 +293,11 @@ def run_sharded(args, fam, rank, world, local):
     ms = float(t.item())
     value = n / (ms / 1e3) / 1e9
     rep = det.reports()
+    for _ in range(args.steps):  # per-kernel breakdown from instrumented steps after the timed region
+        det.detect(timing=True)
+        for k, (c, ms_, b) in det.kernel_stats().items():
+            c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
+            kstats[k] = (c0 + c, m0 + ms_, b0 + b)
     ledger_match = bool(len(lg) == len(rep) and np.array_equal(lg["addr"], rep["addr"])
                         and np.array_equal(lg["cur"], rep["cur"]) and np.array_equal(lg["prev"], rep["prev"])
                         and np.array_equal(lg["type"].astype(np.uint8), rep["type"]))
@@ -517,15 +519,11 @@ def main():
     torch.cuda.synchronize()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
-    kstats = {}
     launches = 0
     e0.record(stream)
-    for _ in range(args.steps):
-        nrep = det.detect(timing=True, coalesce=co, paper_counters=pc)
+    for _ in range(args.steps):  # uninstrumented: no per-kernel events inside the timed region
+        nrep = det.detect(coalesce=co, paper_counters=pc)
         launches += det.launch_count()
-        for k, (cnt, ms, b) in det.kernel_stats().items():
-            c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
-            kstats[k] = (c0 + cnt, m0 + ms, b0 + b)
     e1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -538,7 +536,16 @@ def main():
         ms = float(t.item())
     value = n * world / (ms / 1e3) / 1e9
     reports = det.reports()
+    # per-kernel breakdown (CUDA events on the context stream around every launch) and stage times
+    # from as many instrumented steps after the timed region
+    kstats = {}
+    for _ in range(args.steps):
+        det.detect(timing=True, coalesce=co, paper_counters=pc)
+        for k, (cnt, ms_, b) in det.kernel_stats().items():
+            c0, m0, b0 = kstats.get(k, (0, 0.0, 0.0))
+            kstats[k] = (c0 + cnt, m0 + ms_, b0 + b)
     stages = det.stage_times()
+    assert np.array_equal(det.reports(), reports), "instrumented and timed runs disagree"
 
     # ---------------- roofline of the dominant kernel class ----------------
     peak, peak_kind = peaks()
