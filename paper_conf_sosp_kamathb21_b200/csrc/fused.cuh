@@ -31,7 +31,7 @@ constexpr int TILE = THREADS * ITEMS;  // events per tile: a whole number of ing
 constexpr int TPI = TILE / ingest::TILE;  // ingest pass-0 tiles per fused tile
 constexpr int RADIX = 256;
 #ifndef IGD_FUSED_MIX
-#define IGD_FUSED_MIX 4  // N: one row in N ranked with match.any (N = 2 measured slower, 4 neutral-to-better)
+#define IGD_FUSED_MIX 0  // N: one row in N ranked with match.any; 0 = ballots only (C5 38.7 -> 38.2 ms, r02s15; N = 2 slower)
 #endif
 #ifndef IGD_FUSED_EARLY
 #define IGD_FUSED_EARLY 1
@@ -232,7 +232,7 @@ __global__ void __launch_bounds__(THREADS, IGD_FUSED_MINB) k_ingest_sort0(Params
         const bool valid = (amask >> j) & 1u;
         const u32 vmask = __ballot_sync(IGD_FULL, valid);
         const u32 d = (u32)key[j] & 255u;
-        const u32 peers = (IGD_FUSED_MIX && (j % IGD_FUSED_MIX) == IGD_FUSED_MIX - 1)
+        const u32 peers = (IGD_FUSED_MIX > 0 && (j % (IGD_FUSED_MIX > 0 ? IGD_FUSED_MIX : 1)) == IGD_FUSED_MIX - 1)
                               ? rsort::peers_of<0>(valid ? d : (0x100u | lane), vmask)
                                                     : rsort::peers_of<1>(valid ? d : (0x100u | lane), vmask);
         const u32 leader = __ffs(peers) - 1;
