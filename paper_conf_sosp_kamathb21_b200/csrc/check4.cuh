@@ -93,7 +93,7 @@ __device__ __forceinline__ bool q_between_inl(const uint4* __restrict__ desc, co
 // the default mode (single GPU, no fidelity bits, u32 keys) at IGD_C4_MINB CTAs per SM; the
 // other instantiations carry more state and spill more at 32 registers: 6 CTAs per SM (40)
 template <bool MV, bool KB, int FID, bool GEO2, typename KT = u32>
-__global__ void __launch_bounds__(C4_THREADS, (!MV && FID == 0 && sizeof(KT) == 4) ? IGD_C4_MINB : 6) k_check4(Params P) {
+__global__ void __launch_bounds__(C4_THREADS, (!MV && FID == 0 && sizeof(KT) == 4) ? IGD_C4_MINB : 1536 / C4_THREADS) k_check4(Params P) {
     constexpr bool WRAP = (FID & 1) != 0;
     constexpr bool STK = (FID & 2) != 0;
     constexpr bool LKO = (FID & 4) != 0;  // last-k mode (A37): scan state out, decisions in k_lastk
