@@ -123,7 +123,9 @@ typedef void (*igd_free_fn)(void* p, void* stream, void* user);
 typedef struct igd_ctx igd_ctx; /* opaque; owns every device buffer it allocates */
 
 /* Create a context on `cuda_device`, issuing all work on `cuda_stream` (a cudaStream_t;
-   NULL = the legacy default stream).
+   NULL = the legacy default stream).  The context also owns a greatest-priority side stream that
+   igd_detect forks from and joins back into `cuda_stream` (the a2 / a3 stages beside the access
+   sort on lock-heavy traces), so every result is ordered on `cuda_stream` as before.
    Multi-GPU: nranks > 1 processes (one per GPU) each create a context with their
    rank in [0, nranks) and the SAME 128-byte NCCL unique id (igd_nccl_unique_id on one rank,
    shared by the caller, e.g. a torch.distributed broadcast).  The call initialises an NCCL
