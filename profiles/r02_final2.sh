@@ -12,7 +12,7 @@ for c in C5 C4 C3; do
     python bench.py --config $c --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/${tag}_ncu_${c}.log 2>&1
   echo "ncu $c rc=$?"
   python profiles/summarize_launches.py gpurun_out/${tag}_launches_${c}.csv "$tag $c launch list" \
-    --traffic-json profiles/traffic_r02.json "$w" --detects 4 > gpurun_out/${tag}_launches_${c}_summary.txt
+    --traffic-json profiles/traffic_r02.json "$w" --detects 5 > gpurun_out/${tag}_launches_${c}_summary.txt
 done
 cp profiles/traffic_r02.json gpurun_out/traffic_r02.json
 for c in C1 C2 C3 C4 C5; do
