@@ -1,6 +1,6 @@
 // check4.cuh -- a6, ballot formulation: per-address segmented shadow-metadata pass + Table 2 check.
 //
-// Same contract as check::k_check (check.cuh) -- accesses sorted by (word, trace index); the
+// Input: accesses sorted by (word, trace index) (a5); the
 // shadow state the paper keeps per 4-byte word (Fig. 4; updates P:1000-1058) before
 // access j is a pure function of its word-segment prefix -- but the segmented
 // scan is done with warp ballots instead of a shuffle scan of a packed 64-bit state:
