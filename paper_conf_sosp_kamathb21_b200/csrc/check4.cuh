@@ -2,8 +2,9 @@
 //
 // Input: accesses sorted by (word, trace index) (a5); the
 // shadow state the paper keeps per 4-byte word (Fig. 4; updates P:1000-1058) before
-// access j is a pure function of its word-segment prefix -- but the segmented
-// scan is done with warp ballots instead of a shuffle scan of a packed 64-bit state:
+// access j is a pure function of its word-segment prefix.  Inside a warp the
+// segmented scan is done with warp ballots (the packed 64-bit state of check.cuh only crosses warps
+// and tiles):
 //
 //   A warp owns 32*ITEMS consecutive sorted accesses, striped: item j of lane l is position
 //   j*32 + l.  Six predicates per access are balloted (segment head, write, atomic, block-scoped
