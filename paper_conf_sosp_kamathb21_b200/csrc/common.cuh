@@ -198,31 +198,16 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, u32 bytes, 
 __device__ __forceinline__ void mbar_arrive(u64* mbar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(mbar)) : "memory");
 }
-#ifndef IGD_MBAR_HINT
-#define IGD_MBAR_HINT 0  // ns: suspend-time hint of the mbarrier waits (0: the system limit)
-#endif
 __device__ __forceinline__ void mbar_wait(u64* mbar, u32 phase) {
-    if (IGD_MBAR_HINT) {
-        asm volatile(
-            "{\n"
-            ".reg .pred p;\n"
-            "WAIT_%=:\n"
-            "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
-            "@!p bra WAIT_%=;\n"
-            "}\n" ::"r"(smem_u32(mbar)),
-            "r"(phase), "n"(IGD_MBAR_HINT)
-            : "memory");
-    } else {
-        asm volatile(
-            "{\n"
-            ".reg .pred p;\n"
-            "WAIT_%=:\n"
-            "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-            "@!p bra WAIT_%=;\n"
-            "}\n" ::"r"(smem_u32(mbar)),
-            "r"(phase)
-            : "memory");
-    }
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(mbar)),
+        "r"(phase)
+        : "memory");
 }
 
 __device__ __forceinline__ u32 lanemask_lt() {

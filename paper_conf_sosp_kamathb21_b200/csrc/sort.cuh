@@ -1,5 +1,6 @@
-// sort.cuh -- a5: stable LSD radix sort of (u32 key, u32 value) pairs, one kernel per 8-bit
-// digit ("onesweep": upfront digit histograms + per-tile decoupled look-back per digit).
+// sort.cuh -- a5: stable LSD radix sort of (u32 or u64 key, u32 / u64 / 16-byte value) pairs, one
+// kernel per 8-bit digit ("onesweep": upfront digit histograms + per-tile decoupled look-back per
+// digit).
 //
 // Stability: within a tile, each warp owns a contiguous run of 32*ITEMS inputs processed item
 // by item in input order; the rank of an input among equal digits is (earlier tiles via
@@ -7,11 +8,12 @@
 // input order.  Sorting accesses that arrive in trace order therefore yields (word, time)
 // order, the order the per-word shadow replay needs (SURVEY 8(c) C.3 "equivalent formulation").
 //
-// Per tile: keys are loaded (coalesced, warp-striped), ranked with a warp multisplit (eight
-// ballots give the mask of lanes holding the same digit -- no MATCH/MIO traffic), the tile's
-// digit counts are published and looked back, keys are reordered through shared memory and
-// written out in digit runs; values follow with the same ranks through the same buffer, so a
-// thread never holds keys and values at once (register budget -> 3-4 CTAs per SM).
+// Per tile: keys and values arrive in shared memory by one TMA bulk copy each; keys are ranked
+// with a warp multisplit (rows ranked alternately by eight ballots and match.any), the tile's
+// digit counts are published early and looked back, every input scatters its source position to
+// its tile position, and each output slot gathers its key and value from the staged tile and
+// writes them in digit runs (the kernel is bound by the shared-memory / MIO pipe: the gather
+// needs no reorder buffers and no value registers; 3 CTAs per SM).
 #pragma once
 #include "common.cuh"
 
@@ -33,9 +35,6 @@ constexpr int WARPS = THREADS / 32;
 #endif
 #ifndef IGD_SORT_LB
 #define IGD_SORT_LB 4
-#endif
-#ifndef IGD_SORT_GATHER
-#define IGD_SORT_GATHER 1  // output by gathering through a scattered source-position array (see below)
 #endif
 constexpr int ITEMS = IGD_SORT_ITEMS;
 constexpr int TILE = THREADS * ITEMS;  // 4096
@@ -125,11 +124,11 @@ __device__ __forceinline__ u32 peers_of(u32 d, u32 vmask) {
     }
 }
 
-// Dynamic shared memory of k_onesweep<VT, TAIL, KT>: staged keys, staged values (+ the u16
-// source position of every output slot, IGD_SORT_GATHER).
+// Dynamic shared memory of k_onesweep<VT, TAIL, KT>: staged keys, staged values, the u16 source
+// position of every output slot.
 template <typename VT, typename KT = u32>
 constexpr size_t onesweep_smem() {
-    return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT) + (IGD_SORT_GATHER ? (size_t)TILE * 2 : 0);
+    return (size_t)TILE * sizeof(KT) + (size_t)TILE * sizeof(VT) + (size_t)TILE * 2;
 }
 
 // Decoupled look-back for digit d of `tile`: the sum of the digit's counts over all earlier tiles.
@@ -218,10 +217,8 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         for (int j = 0; j < ITEMS; j++) {
             const u32 i = wbase + j * 32 + lane;
             key[j] = i < P.n ? __ldcs(kin + i) : KT(0);
-            if (IGD_SORT_GATHER) {  // the tail tile is staged by plain loads
-                s_k[wofs + j * 32 + lane] = key[j];
-                s_v[wofs + j * 32 + lane] = i < P.n ? __ldcs(vin + i) : VT{};
-            }
+            s_k[wofs + j * 32 + lane] = key[j];  // the tail tile is staged by plain loads
+            s_v[wofs + j * 32 + lane] = i < P.n ? __ldcs(vin + i) : VT{};
         }
     }
     if (IGD_SORT_EARLY) {
@@ -305,7 +302,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
         s_gbase[d] = P.digit_base[d] + (u32)excl - tile_excl;
     }
     __syncthreads();
-#if IGD_SORT_GATHER
     // Output by gathering: every input scatters only its tile position's source index (u16), and
     // output slot i then reads its key and value from the staged input -- no key / value reorder
     // buffers, no value registers, one barrier; 2 fewer shared-memory round trips per element
@@ -332,52 +328,6 @@ __global__ void __launch_bounds__(THREADS, IGD_SORT_MINB) k_onesweep(PassParams 
             }
         }
     }
-#else
-    // keys: reorder in shared memory (rank[] becomes the tile position), write digit runs
-#pragma unroll
-    for (int j = 0; j < ITEMS; j++) {
-        const u32 d = (u32)(key[j] >> shift) & dmask;
-        rank[j] += s_whist[warp][d];
-        if (full || wbase + j * 32 + lane < P.n) s_k[rank[j]] = key[j];
-    }
-    __syncthreads();
-    const u32 tile_n = full ? (u32)TILE : P.n - base;
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const u32 i = t + k * THREADS;
-        if (i < tile_n) {
-            const KT kk = s_k[i];
-            const u32 d = (u32)(kk >> shift) & dmask;
-            __stcs(kout + (s_gbase[d] + i), kk);
-        }
-    }
-    // values: same permutation, in place through the staged buffer
-    VT val[ITEMS];
-    if (full) {
-        mbar_wait(&s_mbar[1], 0);
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) val[j] = s_v[wofs + j * 32 + lane];
-    } else {
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            const u32 i = wbase + j * 32 + lane;
-            val[j] = i < P.n ? __ldcs(vin + i) : VT{};
-        }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < ITEMS; j++)
-        if (full || wbase + j * 32 + lane < P.n) s_v[rank[j]] = val[j];
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        const u32 i = t + k * THREADS;
-        if (i < tile_n) {
-            const u32 d = (u32)(s_k[i] >> shift) & dmask;  // the staged keys are still in tile order
-            __stcs(vout + (s_gbase[d] + i), s_v[i]);
-        }
-    }
-#endif
 }
 
 }  // namespace rsort
